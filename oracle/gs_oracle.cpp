@@ -1,0 +1,844 @@
+// gs_oracle.cpp — the CPU ORACLE for batched bottleneck attribution (GPUscout, SC-W 2023).
+//
+// *** TEST INFRASTRUCTURE ONLY. ***  Only tests/, __graft_entry__.smoke() and bench.py's
+// cpu_baseline / --impl reference legs may build, call or execute this program. It shares no
+// code, header, table or helper with the CUDA path (paper_conf_sc_senvs23_b200/csrc); the two
+// are written independently from the same reading of the paper.
+//
+// Plain, slow, obviously-correct: single-threaded, std::vector / std::map / std::sort, linear
+// scans, its own SASS text parser. Every step cites the PAPER.md passage (P:line, section) it
+// follows; where the paper is silent the DESIGN.md reading number is given (e.g. [R5]).
+//
+// Steps (SURVEY §8c O1–O15):
+//   O1  parse cuobjdump/nvdisasm SASS text                      P:209-213 §2.1
+//   O2  per-instruction register effects (dst, width, sources)   P:211-213 ("destination (+source) register numbers")
+//   O3  reaching definition = last earlier writer (linear order)  P:446-448 §3.2 ("previous SASS instruction executed by the register")
+//   O4  loop depth from backward branches                        P:640-645 §4.3, §4.4
+//   O5  bounded backward def-use trace of an address register    P:446-448, §4.2; north_star
+//   O6  VEC   vectorisable 32-bit global loads                   P:510-532 §4.1, Listing 1
+//   O7  SPILL local-memory spills STL/LDL + cause                  P:565-583 §4.2
+//   O8  SHMEM shared-memory candidates                           P:626-645 §4.3
+//   O9  GATOM global atomics                                     P:669-696 §4.4
+//   O10 RO    read-only / __restrict__ candidates                P:698-715 §4.5
+//   O11 TEX   texture candidates                                 P:717-744 §4.6
+//   O12 CONV  datatype conversions                               P:746-761 §4.7
+//   O13 per-PC x stall-reason histogram of PC samples            P:215-227 §2.2
+//   O14 join of the histogram onto flagged sites
+//   O15 ranking (total order on integers)                        [R20]
+//
+// Output: the canonical result text on stdout or --out.
+#include <algorithm>
+#include <chrono>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <set>
+#include <string>
+#include <vector>
+
+namespace {
+
+// ---------------------------------------------------------------- registers
+// One id space: GPR R0..R254 -> 0..254, RZ -> 255; UR0..UR62 -> 256..318, URZ -> 319.
+const int kRZ = 255, kURZ = 319, kNoReg = -1;
+bool is_zero_reg(int r) { return r == kRZ || r == kURZ; }
+bool is_ur(int r) { return r >= 256; }
+std::string reg_name(int r) {
+  char b[16];
+  if (r < 256) snprintf(b, sizeof b, r == kRZ ? "RZ" : "R%d", r);
+  else snprintf(b, sizeof b, r == kURZ ? "URZ" : "UR%d", r - 256);
+  return b;
+}
+
+// ---------------------------------------------------------------- operands
+enum OpndKind { K_REG, K_PRED, K_CREF, K_MEM, K_IMM, K_OTHER };
+struct Opnd {
+  OpndKind kind = K_OTHER;
+  int reg = kNoReg;            // K_REG: register id
+  std::vector<int> regs;       // every register token inside the operand (any kind)
+  int cbank = 0;               // K_CREF: bank
+  long long coff = 0;          // K_CREF: offset (immediate part)
+  int base = kNoReg;           // K_MEM: first register term of the address
+  long long off = 0;           // K_MEM: sum of immediate terms
+};
+
+std::string trim(const std::string& s) {
+  size_t a = s.find_first_not_of(" \t\r\n"), b = s.find_last_not_of(" \t\r\n");
+  return a == std::string::npos ? std::string() : s.substr(a, b - a + 1);
+}
+
+// Parse a bare register token (prefixes - ! ~ | already stripped), e.g. "R4.64", "UR6", "RZ".
+bool parse_reg(const std::string& t0, int* out) {
+  std::string t = t0;
+  size_t dot = t.find('.');
+  if (dot != std::string::npos) t = t.substr(0, dot);
+  while (!t.empty() && t.back() == '|') t.pop_back();
+  bool ur = false;
+  size_t p = 0;
+  if (t.size() >= 2 && t[0] == 'U' && t[1] == 'R') { ur = true; p = 2; }
+  else if (!t.empty() && t[0] == 'R') p = 1;
+  else return false;
+  std::string rest = t.substr(p);
+  if (rest == "Z") { *out = ur ? kURZ : kRZ; return true; }
+  if (rest.empty() || rest.size() > 3) return false;
+  for (char c : rest) if (c < '0' || c > '9') return false;
+  int n = atoi(rest.c_str());
+  if (ur ? n > 62 : n > 254) return false;
+  *out = ur ? 256 + n : n;
+  return true;
+}
+
+std::string strip_prefix(const std::string& t) {
+  size_t i = 0;
+  while (i < t.size() && (t[i] == '-' || t[i] == '!' || t[i] == '~' || t[i] == '|')) i++;
+  return t.substr(i);
+}
+
+bool parse_int(const std::string& t0, long long* v) {
+  std::string t = trim(t0);
+  bool neg = false;
+  if (!t.empty() && (t[0] == '-' || t[0] == '+')) { neg = t[0] == '-'; t = t.substr(1); }
+  if (t.empty()) return false;
+  char* end = nullptr;
+  long long x;
+  if (t.size() > 2 && t[0] == '0' && (t[1] == 'x' || t[1] == 'X')) x = strtoll(t.c_str() + 2, &end, 16);
+  else x = strtoll(t.c_str(), &end, 10);
+  if (*end) return false;
+  *v = neg ? -x : x;
+  return true;
+}
+
+// Sum immediates and collect registers of a bracket body like "R4.64+-0x10" or "R11+UR4".
+void parse_bracket(const std::string& body, Opnd* o, bool first_reg_is_base) {
+  size_t s = 0;
+  std::string b = body;
+  while (s <= b.size()) {
+    size_t e = b.find('+', s);
+    if (e == std::string::npos) e = b.size();
+    std::string term = trim(b.substr(s, e - s));
+    if (!term.empty()) {
+      int r;
+      long long v;
+      if (parse_reg(strip_prefix(term), &r)) {
+        o->regs.push_back(r);
+        if (first_reg_is_base && o->base == kNoReg) o->base = r;
+      } else if (parse_int(term, &v)) {
+        o->off += v;
+      }
+    }
+    s = e + 1;
+  }
+}
+
+Opnd parse_operand(const std::string& raw) {
+  Opnd o;
+  std::string t = trim(raw);
+  std::string u = strip_prefix(t);
+  // constant-bank reference c[bank][off]   (may carry a register inside the second bracket)
+  if (u.size() > 2 && u[0] == 'c' && u[1] == '[') {
+    o.kind = K_CREF;
+    size_t a = u.find(']');
+    long long bank = 0;
+    parse_int(u.substr(2, a - 2), &bank);
+    o.cbank = (int)bank;
+    size_t b0 = u.find('[', a), b1 = u.find(']', b0 == std::string::npos ? a : b0);
+    if (b0 != std::string::npos && b1 != std::string::npos) {
+      Opnd tmp;
+      parse_bracket(u.substr(b0 + 1, b1 - b0 - 1), &tmp, false);
+      o.coff = tmp.off;
+      o.regs = tmp.regs;
+    }
+    return o;
+  }
+  // memory operand [..], desc[URx][..], [R11+UR4]
+  if (u.find('[') != std::string::npos) {
+    o.kind = K_MEM;
+    size_t last_open = u.rfind('[');
+    size_t last_close = u.find(']', last_open);
+    // registers of any earlier bracket (desc[URd]) are sources, not the base
+    size_t p = 0;
+    while (true) {
+      size_t a = u.find('[', p);
+      if (a == std::string::npos || a == last_open) break;
+      size_t c = u.find(']', a);
+      Opnd tmp;
+      parse_bracket(u.substr(a + 1, c - a - 1), &tmp, false);
+      for (int r : tmp.regs) o.regs.push_back(r);
+      p = c + 1;
+    }
+    Opnd inner;
+    parse_bracket(u.substr(last_open + 1, last_close - last_open - 1), &inner, true);
+    o.base = inner.base;
+    o.off = inner.off;
+    for (int r : inner.regs) o.regs.push_back(r);
+    return o;
+  }
+  int r;
+  if (parse_reg(u, &r)) { o.kind = K_REG; o.reg = r; o.regs.push_back(r); return o; }
+  {  // predicates P0..P6, PT, UP0..UP6, UPT (optionally negated)
+    std::string p = u;
+    if (p.size() >= 2 && p[0] == 'U' && p[1] == 'P') p = p.substr(2);
+    else if (!p.empty() && p[0] == 'P') p = p.substr(1);
+    else p = "#";
+    if (p == "T" || (p.size() == 1 && p[0] >= '0' && p[0] <= '7')) { o.kind = K_PRED; return o; }
+  }
+  long long v;
+  if (parse_int(t, &v)) { o.kind = K_IMM; return o; }
+  o.kind = K_OTHER;  // SR_TID.X, floats, B0, 2D, PR ...  (never registers)
+  return o;
+}
+
+// ---------------------------------------------------------------- instructions
+struct Instr {
+  int pc = 0;
+  int line = -1;                  // source line from //## File ..., line N
+  std::string op;                 // base mnemonic
+  std::vector<std::string> mods;  // modifiers after the first '.'
+  std::vector<Opnd> ops;
+  int dst = kNoReg, dst_w = 0, dst_pos = -1;
+  std::vector<int> srcs;          // register sources (no RZ/URZ), O2
+  int mem = -1;                   // index of the memory operand in ops
+  long long bra_target = -1;      // BRA immediate target pc
+  bool has_mod(const char* m) const {
+    for (auto& s : mods) if (s == m) return true;
+    return false;
+  }
+};
+
+struct Kernel {
+  std::string name;
+  int param_base = 0x380;
+  std::vector<Instr> ins;
+  size_t first_slot = 0;
+};
+
+bool op_in(const std::string& op, std::initializer_list<const char*> l) {
+  for (auto* s : l) if (op == s) return true;
+  return false;
+}
+
+// O2 destination width table (DESIGN.md §3 table W).
+int dst_width(const Instr& I) {
+  for (auto& m : I.mods) if (m == "128") return 4;
+  if (I.op == "HMMA") return I.has_mod("F32") ? 4 : 2;
+  if (I.op == "LDSM") {
+    if (I.has_mod("4")) return 4;
+    if (I.has_mod("2")) return 2;
+    return 1;
+  }
+  for (auto& m : I.mods) if (m == "64" || m == "WIDE") return 2;
+  if (op_in(I.op, {"DADD", "DMUL", "DFMA", "DMNMX"})) return 2;
+  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I"})) {
+    for (auto& m : I.mods) {  // the first type modifier is the destination type
+      if (m == "F64" || m == "S64" || m == "U64") return 2;
+      if (m == "F32" || m == "F16" || m == "BF16" || m == "S32" || m == "U32" || m == "S16" ||
+          m == "U16" || m == "S8" || m == "U8" || m == "TF32" || m == "E4M3" || m == "E5M2")
+        return 1;
+    }
+  }
+  return 1;
+}
+
+// O2: decode dst and sources.
+void decode_effects(Instr& I) {
+  int d = -1;
+  if (!I.ops.empty() && I.ops[0].kind == K_REG) d = 0;
+  else if (I.ops.size() >= 2 && I.ops[0].kind == K_PRED && I.ops[1].kind == K_REG && I.op != "FCHK")
+    d = 1;  // SHFL PT, R0 ... ; ATOMG PT, R2 ... ; LOP3.LUT P0, R5 ...
+  if (d >= 0) {
+    I.dst_pos = d;
+    I.dst = I.ops[d].reg;
+    I.dst_w = dst_width(I);
+  }
+  for (size_t k = (size_t)(d + 1); k < I.ops.size(); k++)
+    for (int r : I.ops[k].regs)
+      if (!is_zero_reg(r)) I.srcs.push_back(r);
+  for (size_t k = 0; k < I.ops.size(); k++)
+    if (I.ops[k].kind == K_MEM) { I.mem = (int)k; break; }
+}
+
+// ---------------------------------------------------------------- O1 parser
+struct ParseError { std::string msg; };
+
+int arch_param_base(int sm) { return sm >= 100 ? 0x380 : (sm >= 90 ? 0x210 : 0x160); }
+
+std::vector<Kernel> parse_sass(const std::string& text) {
+  std::vector<Kernel> ks;
+  int cur_sm = 100, line_no = 0, src_line = -1;
+  size_t p = 0;
+  while (p < text.size()) {
+    size_t e = text.find('\n', p);
+    if (e == std::string::npos) e = text.size();
+    std::string L = text.substr(p, e - p);
+    p = e + 1;
+    line_no++;
+    std::string t = trim(L);
+    if (t.empty()) continue;
+    size_t cf = t.find("code for sm_");
+    if (cf != std::string::npos) { cur_sm = atoi(t.c_str() + cf + 12); continue; }
+    size_t tg = t.find(".target");
+    if (tg != std::string::npos && t.find("sm_") != std::string::npos) {
+      cur_sm = atoi(t.c_str() + t.find("sm_") + 3);
+      continue;
+    }
+    size_t fn = t.find("Function :");
+    if (fn != std::string::npos) {
+      Kernel k;
+      k.name = trim(t.substr(fn + 10));
+      k.param_base = arch_param_base(cur_sm);
+      ks.push_back(k);
+      src_line = -1;
+      continue;
+    }
+    if (t.rfind("//##", 0) == 0) {  // nvdisasm -g line info: //## File "f", line N
+      size_t ln = t.find("line ");
+      if (ln != std::string::npos) src_line = atoi(t.c_str() + ln + 5);
+      continue;
+    }
+    if (t.size() < 4 || t[0] != '/' || t[1] != '*') continue;
+    size_t c = t.find("*/");
+    if (c == std::string::npos) continue;
+    std::string pcs = t.substr(2, c - 2);
+    bool hex = !pcs.empty();
+    for (char ch : pcs) if (!isxdigit((unsigned char)ch)) hex = false;
+    if (!hex || pcs.rfind("0x", 0) == 0) continue;  // "/* 0x... */" encoding-only line
+    std::string body = t.substr(c + 2);
+    size_t semi = body.find(';');
+    if (semi == std::string::npos) continue;
+    body = trim(body.substr(0, semi));
+    if (ks.empty()) {  // instruction without a Function header (e.g. a paper listing)
+      Kernel k;
+      k.name = "<anonymous>";
+      k.param_base = arch_param_base(cur_sm);
+      ks.push_back(k);
+    }
+    Kernel& K = ks.back();
+    Instr I;
+    I.pc = (int)strtol(pcs.c_str(), nullptr, 16);
+    I.line = src_line;
+    if ((size_t)I.pc != K.ins.size() * 16)
+      throw ParseError{"line " + std::to_string(line_no) + ": pc not 16-strided"};
+    // guard predicate
+    if (!body.empty() && body[0] == '@') {
+      size_t sp = body.find_first_of(" \t");
+      body = trim(body.substr(sp));
+    }
+    size_t sp = body.find_first_of(" \t");
+    std::string opc = sp == std::string::npos ? body : body.substr(0, sp);
+    std::string rest = sp == std::string::npos ? "" : trim(body.substr(sp));
+    size_t d0 = opc.find('.');
+    I.op = opc.substr(0, d0);
+    while (d0 != std::string::npos) {
+      size_t d1 = opc.find('.', d0 + 1);
+      I.mods.push_back(opc.substr(d0 + 1, d1 == std::string::npos ? std::string::npos : d1 - d0 - 1));
+      d0 = d1;
+    }
+    // split operands at top-level commas
+    std::vector<std::string> raw;
+    int depth = 0;
+    std::string cur;
+    for (char ch : rest) {
+      if (ch == '[' || ch == '{') depth++;
+      if (ch == ']' || ch == '}') depth--;
+      if (ch == ',' && depth == 0) { raw.push_back(cur); cur.clear(); }
+      else cur += ch;
+    }
+    if (!trim(cur).empty()) raw.push_back(cur);
+    for (auto& r : raw) I.ops.push_back(parse_operand(r));
+    decode_effects(I);
+    if (I.op == "BRA" && !raw.empty()) {
+      long long v;
+      if (parse_int(raw.back(), &v)) I.bra_target = v;
+    }
+    K.ins.push_back(I);
+  }
+  size_t slot = 0;
+  for (auto& k : ks) { k.first_slot = slot; slot += k.ins.size(); }
+  return ks;
+}
+
+// ---------------------------------------------------------------- opcode classes
+bool is_constload(const std::string& op) { return op_in(op, {"LDC", "LDCU", "ULDC"}); }
+bool is_sreg(const std::string& op) { return op_in(op, {"S2R", "S2UR", "CS2R"}); }
+bool is_memload(const std::string& op) {
+  return op_in(op, {"LDG", "LDL", "LDS", "LD", "LDSM", "ATOM", "ATOMG", "ATOMS", "TLD", "TLD4",
+                    "TLDS", "TEX", "TMML", "TXD", "TXQ", "SULD", "SUATOM", "LDTM"});
+}
+bool is_conv(const std::string& op) {
+  return op_in(op, {"F2F", "F2I", "I2F", "I2I", "I2FP", "F2IP", "F2FP"});
+}
+bool is_arith(const Instr& I) {
+  if (I.op == "IMAD") return I.mods.empty() || I.mods[0] != "MOV";
+  return op_in(I.op, {"FADD", "FMUL", "FFMA", "FMNMX", "DADD", "DMUL", "DFMA", "HADD2", "HMUL2",
+                      "HFMA2", "MUFU", "IADD3", "VIADD", "IMUL", "IMNMX", "VIMNMX", "IABS"});
+}
+bool is_gatom(const std::string& op) { return op_in(op, {"ATOMG", "ATOM", "RED", "REDG"}); }
+bool is_store_class(const std::string& op) {
+  return op_in(op, {"STG", "ST", "ATOMG", "ATOM", "RED", "REDG", "SUST"});
+}
+bool is_traced_memop(const std::string& op) {
+  return op_in(op, {"LDG", "LDL", "STL", "STG", "ST", "ATOMG", "ATOM", "RED", "REDG", "SUST"});
+}
+// access width in bits of a memory instruction (reading #2)
+int access_bits(const Instr& I) {
+  for (auto& m : I.mods) {
+    if (m == "U8" || m == "S8") return 8;
+    if (m == "U16" || m == "S16") return 16;
+    if (m == "64") return 64;
+    if (m == "128") return 128;
+  }
+  return 32;
+}
+
+// ---------------------------------------------------------------- O5 traces
+enum TermKind { T_NONE, T_PARAM, T_CONST, T_ENTRY, T_SREG, T_MEMORY, T_IMM, T_TRUNC };
+struct Trace {
+  TermKind kind = T_NONE;
+  long long value = 0;  // PARAM: offset; CONST: bank<<32|off; ENTRY: reg; SREG/MEMORY: idx
+  std::vector<int> chain;
+};
+
+struct Config {
+  int D = 64, R = 19, TA = 1, TL = 2;
+};
+
+// RD values for one kernel. ENTRY is -1.  RD(i, r) = max j < i with r in dst(j).
+class KernelAnalysis {
+ public:
+  const Kernel& K;
+  std::vector<int> lw;                                  // running last-writer per register
+  std::vector<std::vector<std::pair<int, int>>> rd_at;  // rd_at[i] = {(r, RD(i, r))} queried
+  explicit KernelAnalysis(const Kernel& k) : K(k) {}
+
+  // O3: the reaching definition of register r at instruction i (linear order; predicated writes
+  // count; back-edges are not followed) — P:446-448 "the previous SASS instruction executed by
+  // the register".  Computed for all (i, r) pairs the later steps need, in one forward pass.
+  void compute_rd(const std::vector<std::pair<int, int>>& queries) {
+    rd_at.assign(K.ins.size(), {});
+    for (auto& q : queries) rd_at[q.first].push_back({q.second, -1});
+    lw.assign(320, -1);
+    for (size_t i = 0; i < K.ins.size(); i++) {
+      for (auto& q : rd_at[i]) q.second = lw[q.first];
+      const Instr& I = K.ins[i];
+      if (I.dst != kNoReg && !is_zero_reg(I.dst))
+        for (int w = 0; w < I.dst_w; w++) {
+          int r = I.dst + w;
+          if ((is_ur(I.dst) && r <= 318) || (!is_ur(I.dst) && r <= 254)) lw[r] = (int)i;
+        }
+    }
+  }
+  int rd(int i, int r) const {
+    for (auto& q : rd_at[i]) if (q.first == r) return q.second;
+    fprintf(stderr, "oracle bug: RD(%d,%s) not computed\n", i, reg_name(r).c_str());
+    abort();
+  }
+};
+
+// O5 pointer operand of instruction J (the register the trace continues through).
+// Returns 0: continue with *reg; 1: CONST terminal (*bank, *off); 2: IMM terminal.
+int pointer_operand(const Instr& J, int* reg, int* bank, long long* off) {
+  std::vector<const Opnd*> L;  // source operands after the dst, predicates skipped
+  for (size_t k = (size_t)(J.dst_pos + 1); k < J.ops.size(); k++)
+    if (J.ops[k].kind != K_PRED) L.push_back(&J.ops[k]);
+  const Opnd* pick = nullptr;
+  auto is_live_reg = [](const Opnd* o) { return o->kind == K_REG && !is_zero_reg(o->reg); };
+  if ((J.op == "IMAD" || J.op == "UIMAD") && J.has_mod("WIDE")) {
+    pick = L.size() > 2 ? L[2] : nullptr;
+  } else if (J.op == "LEA" || J.op == "ULEA") {
+    pick = L.size() > 1 ? L[1] : nullptr;
+  } else if (J.op == "IADD3" || J.op == "UIADD3") {
+    for (auto* o : L) if (o->kind == K_CREF) { pick = o; break; }
+    if (!pick) for (auto* o : L) if (is_live_reg(o) && is_ur(o->reg)) { pick = o; break; }
+    if (!pick) for (auto* o : L) if (is_live_reg(o) && !is_ur(o->reg)) { pick = o; break; }
+  } else {
+    for (auto* o : L) if (is_live_reg(o) || o->kind == K_CREF) { pick = o; break; }
+  }
+  if (pick && pick->kind == K_CREF) { *bank = pick->cbank; *off = pick->coff; return 1; }
+  if (pick && is_live_reg(pick)) { *reg = pick->reg; return 0; }
+  return 2;
+}
+
+// Collect every (i, r) RD query the trace from (i0, r0) can make (trace needs RD only along the
+// chain, but the chain depends on RD values: we therefore compute RD for every instruction's
+// pointer operand and for the starting registers; a plain superset).
+void trace_queries(const Kernel& K, std::vector<std::pair<int, int>>& q) {
+  for (size_t i = 0; i < K.ins.size(); i++) {
+    const Instr& I = K.ins[i];
+    if (I.dst != kNoReg) {
+      int reg, bank;
+      long long off;
+      if (pointer_operand(I, &reg, &bank, &off) == 0) q.push_back({(int)i, reg});
+    }
+    if (I.mem >= 0 && I.ops[I.mem].base != kNoReg && !is_zero_reg(I.ops[I.mem].base))
+      q.push_back({(int)i, I.ops[I.mem].base});
+    for (int s : I.srcs) q.push_back({(int)i, s});
+  }
+}
+
+// O5: the bounded backward trace of register r0 at instruction i (north_star).
+Trace trace(const Kernel& K, const KernelAnalysis& A, int i, int r0, int D) {
+  Trace T;
+  if (r0 == kNoReg || is_zero_reg(r0)) { T.kind = T_IMM; return T; }
+  int pos = i, r = r0;
+  for (int step = 0; step < D; step++) {
+    int j = A.rd(pos, r);                                   // 1. last writer
+    if (j < 0) { T.kind = T_ENTRY; T.value = r; return T; }
+    T.chain.push_back(j);                                   // 2. append
+    pos = j;
+    const Instr& J = K.ins[j];
+    if (is_constload(J.op)) {                               // 3. constant bank load
+      const Opnd* c = nullptr;
+      for (size_t k = (size_t)(J.dst_pos + 1); k < J.ops.size(); k++)
+        if (J.ops[k].kind == K_CREF) { c = &J.ops[k]; break; }
+      long long off = (c ? c->coff : 0) + 4LL * (r - J.dst);
+      int bank = c ? c->cbank : 0;
+      if (bank == 0 && off >= K.param_base) { T.kind = T_PARAM; T.value = off; }
+      else { T.kind = T_CONST; T.value = ((long long)bank << 32) | (off & 0xffffffffLL); }
+      return T;
+    }
+    if (is_sreg(J.op)) { T.kind = T_SREG; T.value = j; return T; }      // 4.
+    if (is_memload(J.op)) { T.kind = T_MEMORY; T.value = j; return T; }  // 5.
+    int reg, bank;
+    long long off;
+    int pk = pointer_operand(J, &reg, &bank, &off);                       // 6.
+    if (pk == 1) {
+      if (bank == 0 && off >= K.param_base) { T.kind = T_PARAM; T.value = off; }
+      else { T.kind = T_CONST; T.value = ((long long)bank << 32) | (off & 0xffffffffLL); }
+      return T;
+    }
+    if (pk == 2) { T.kind = T_IMM; return T; }
+    r = reg;
+  }
+  T.kind = T_TRUNC;
+  return T;
+}
+
+std::string term_str(const Trace& T) {
+  char b[64];
+  switch (T.kind) {
+    case T_NONE: return "NONE";
+    case T_PARAM: snprintf(b, sizeof b, "PARAM:0x%llx", T.value); return b;
+    case T_CONST: snprintf(b, sizeof b, "CONST:0x%llx:0x%llx", T.value >> 32, T.value & 0xffffffffLL); return b;
+    case T_ENTRY: return "ENTRY:" + reg_name((int)T.value);
+    case T_SREG: snprintf(b, sizeof b, "SREG:%lld", T.value); return b;
+    case T_MEMORY: snprintf(b, sizeof b, "MEMORY:%lld", T.value); return b;
+    case T_IMM: return "IMM";
+    case T_TRUNC: return "TRUNC";
+  }
+  return "?";
+}
+
+// ---------------------------------------------------------------- sites
+enum Rule { VEC = 0, SPILL, SHMEM, GATOM, RO, TEX, CONV, NRULES };
+const char* kRuleName[NRULES] = {"VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX", "CONV"};
+
+struct Site {
+  int k = 0, idx = 0, rule = 0;
+  int line = -1, loop_depth = 0;
+  Trace tr;
+  std::string attrs;
+};
+
+struct KernelStats {
+  int gatom = 0, satom = 0, conv = 0, vec_already = 0, ustores = 0;
+};
+
+// Detection (the paper's dry run) over one kernel.
+void detect_kernel(int kid, const Kernel& K, const Config& C, std::vector<Site>& sites, KernelStats& st) {
+  const int n = (int)K.ins.size();
+  KernelAnalysis A(K);
+  std::vector<std::pair<int, int>> q;
+  trace_queries(K, q);
+  A.compute_rd(q);
+
+  // O4 loop depth: number of backward BRA spans [t, pc(b)] containing pc(i).
+  std::vector<int> loop_depth(n, 0);
+  for (int b = 0; b < n; b++) {
+    const Instr& B = K.ins[b];
+    if (B.op != "BRA" || B.bra_target < 0) continue;
+    long long t = B.bra_target;
+    if (!(t < B.pc)) continue;  // forward or self branch
+    for (int i = 0; i < n; i++)
+      if (t <= K.ins[i].pc && K.ins[i].pc <= B.pc) loop_depth[i]++;
+  }
+
+  // O5 traces for every traced memory instruction (address base register).
+  std::vector<Trace> tr(n);
+  std::vector<bool> has_tr(n, false);
+  for (int i = 0; i < n; i++) {
+    const Instr& I = K.ins[i];
+    if (!is_traced_memop(I.op) || I.mem < 0) continue;
+    tr[i] = trace(K, A, i, I.ops[I.mem].base, C.D);
+    has_tr[i] = true;
+  }
+
+  // global LDG key groups: key(i) = (base reg, RD(i, base))   [reading #3]
+  struct Group {
+    std::set<long long> off32, off_all;
+    int n_loads = 0;
+  };
+  std::map<std::pair<int, int>, Group> groups;
+  auto key_of = [&](int i) {
+    int b = K.ins[i].ops[K.ins[i].mem].base;
+    int rdv = (b == kNoReg || is_zero_reg(b)) ? -2 : A.rd(i, b);
+    return std::make_pair(b, rdv);
+  };
+  for (int i = 0; i < n; i++) {
+    const Instr& I = K.ins[i];
+    if (I.op != "LDG" || I.mem < 0) continue;
+    Group& g = groups[key_of(i)];
+    g.n_loads++;
+    g.off_all.insert(I.ops[I.mem].off);
+    if (access_bits(I) == 32) g.off32.insert(I.ops[I.mem].off);
+  }
+
+  // n_arith(i) = |{ j in ARITH : exists source s of j with RD(j, s) = i }|
+  std::vector<int> n_arith(n, 0);
+  for (int j = 0; j < n; j++) {
+    const Instr& J = K.ins[j];
+    if (!is_arith(J)) continue;
+    std::set<int> defs;
+    for (int s : J.srcs) {
+      int d = A.rd(j, s);
+      if (d >= 0) defs.insert(d);
+    }
+    for (int d : defs) n_arith[d]++;
+  }
+
+  // O10 store roots of the kernel: resolved roots = PARAM offsets and ENTRY registers.
+  std::set<std::pair<int, long long>> store_roots;
+  for (int i = 0; i < n; i++) {
+    if (!has_tr[i] || !is_store_class(K.ins[i].op)) continue;
+    if (tr[i].kind == T_PARAM || tr[i].kind == T_ENTRY) store_roots.insert({tr[i].kind, tr[i].value});
+    else st.ustores++;
+  }
+
+  for (int i = 0; i < n; i++) {
+    const Instr& I = K.ins[i];
+    auto emit = [&](int rule, const Trace& t, const std::string& attrs) {
+      Site s;
+      s.k = kid; s.idx = i; s.rule = rule; s.line = I.line; s.loop_depth = loop_depth[i];
+      s.tr = t; s.attrs = attrs;
+      sites.push_back(s);
+    };
+    char b[160];
+    if (is_gatom(I.op)) st.gatom++;
+    if (I.op == "ATOMS") st.satom++;
+    if (is_conv(I.op)) st.conv++;
+    if (I.op == "LDG" && I.mem >= 0) {
+      int bits = access_bits(I);
+      if (bits == 64 || bits == 128) st.vec_already++;  // "already vectorised"
+      const Group& g = groups[key_of(i)];
+      // O6 VEC: 32-bit LDG whose group has >= 2 distinct immediate offsets.
+      if (bits == 32 && g.off32.size() >= 2) {
+        long long mn = *g.off32.begin(), mx = *g.off32.rbegin();
+        bool contig = true;
+        long long prev = mn;
+        for (auto it = std::next(g.off32.begin()); it != g.off32.end(); ++it) {
+          if (*it - prev != 4) contig = false;
+          prev = *it;
+        }
+        snprintf(b, sizeof b, "n=%zu min=%lld max=%lld contig=%d", g.off32.size(), mn, mx, contig ? 1 : 0);
+        emit(VEC, tr[i], b);
+      }
+      // O8 SHMEM: arithmetic on the loaded value, loaded repeatedly or in a loop.
+      if (n_arith[i] >= C.TA && (g.n_loads >= C.TL || loop_depth[i] >= 1)) {
+        snprintf(b, sizeof b, "loads=%d arith=%d", g.n_loads, n_arith[i]);
+        emit(SHMEM, tr[i], b);
+      }
+      // O10 RO: non-.CONSTANT load whose root no store of the kernel shares.
+      bool ro = false;
+      if (!I.has_mod("CONSTANT") && (tr[i].kind == T_PARAM || tr[i].kind == T_ENTRY))
+        ro = store_roots.count({tr[i].kind, tr[i].value}) == 0;
+      if (ro) emit(RO, tr[i], "");
+      // O11 TEX: read-only and adjacent loads (any width) on the same base value.
+      if (ro && g.off_all.size() >= 2) {
+        snprintf(b, sizeof b, "n=%zu", g.off_all.size());
+        emit(TEX, tr[i], b);
+      }
+    }
+    // O7 SPILL: every STL / LDL; STL also names the last writer of the spilled register.
+    if ((I.op == "STL" || I.op == "LDL") && I.mem >= 0) {
+      std::string data = "-", cause = "-";
+      if (I.op == "STL") {
+        for (size_t k = (size_t)I.mem + 1; k < I.ops.size(); k++)
+          if (I.ops[k].kind == K_REG) {
+            data = reg_name(I.ops[k].reg);
+            if (!is_zero_reg(I.ops[k].reg)) {
+              int c = A.rd(i, I.ops[k].reg);
+              cause = c < 0 ? "E" : std::to_string(c);
+            }
+            break;
+          }
+      } else if (I.dst != kNoReg) {
+        data = reg_name(I.dst);
+      }
+      snprintf(b, sizeof b, "data=%s cause=%s", data.c_str(), cause.c_str());
+      emit(SPILL, tr[i], b);
+    }
+    // O9 GATOM
+    if (is_gatom(I.op) && I.mem >= 0) emit(GATOM, tr[i], "");
+    // O12 CONV
+    if (is_conv(I.op)) emit(CONV, Trace(), "");
+  }
+}
+
+// ---------------------------------------------------------------- O13-O15
+struct RawSample { uint32_t kernel, pc, reason; };
+
+const int kRel[NRULES] = {
+    // bit r set = reason r in REL(rule).  long_scoreboard = 6, lg_throttle = 5, tex_throttle = 16
+    1 << 6,                 // VEC
+    (1 << 6) | (1 << 5),    // SPILL P:616-624
+    1 << 6,                 // SHMEM [R14 reading]
+    1 << 5,                 // GATOM P:685-687
+    1 << 6,                 // RO    [reading]
+    (1 << 6) | (1 << 16),   // TEX
+    -1,                     // CONV  all reasons [reading]
+};
+
+}  // namespace
+
+int main(int argc, char** argv) {
+  std::string sass_path, samples_path, out_path;
+  Config C;
+  long long K_top = -1;
+  int kbegin = 0, kend = -1;
+  bool detect = true, hist = true, timing = false;
+  for (int a = 1; a < argc; a++) {
+    std::string s = argv[a];
+    auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
+    if (s == "--sass") sass_path = nxt();
+    else if (s == "--samples") samples_path = nxt();
+    else if (s == "--out") out_path = nxt();
+    else if (s == "--D") C.D = atoi(nxt().c_str());
+    else if (s == "--R") C.R = atoi(nxt().c_str());
+    else if (s == "--ta") C.TA = atoi(nxt().c_str());
+    else if (s == "--tl") C.TL = atoi(nxt().c_str());
+    else if (s == "--k") K_top = atoll(nxt().c_str());
+    else if (s == "--kbegin") kbegin = atoi(nxt().c_str());
+    else if (s == "--kend") kend = atoi(nxt().c_str());
+    else if (s == "--no-detect") detect = false;
+    else if (s == "--no-hist") hist = false;
+    else if (s == "--time") timing = true;
+    else { fprintf(stderr, "unknown arg %s\n", s.c_str()); return 2; }
+  }
+  auto now = [] { return std::chrono::steady_clock::now(); };
+  auto secs = [](auto a, auto b) { return std::chrono::duration<double>(b - a).count(); };
+  FILE* f = fopen(sass_path.c_str(), "rb");
+  if (!f) { fprintf(stderr, "cannot open %s\n", sass_path.c_str()); return 2; }
+  std::string text;
+  {
+    fseek(f, 0, SEEK_END);
+    long sz = ftell(f);
+    fseek(f, 0, SEEK_SET);
+    text.resize((size_t)sz);
+    if (sz && fread(&text[0], 1, (size_t)sz, f) != (size_t)sz) return 2;
+    fclose(f);
+  }
+  auto t0 = now();
+  std::vector<Kernel> ks;
+  try { ks = parse_sass(text); } catch (ParseError& e) { fprintf(stderr, "parse error: %s\n", e.msg.c_str()); return 3; }
+  auto t1 = now();
+  if (kend < 0 || kend > (int)ks.size()) kend = (int)ks.size();
+  FILE* out = out_path.empty() ? stdout : fopen(out_path.c_str(), "wb");
+  fprintf(out, "# gs-canonical v1\n");
+  fprintf(out, "CFG D=%d R=%d TA=%d TL=%d\n", C.D, C.R, C.TA, C.TL);
+
+  std::vector<Site> sites;
+  std::vector<KernelStats> stats(ks.size());
+  if (detect)
+    for (int k = kbegin; k < kend; k++) detect_kernel(k, ks[k], C, sites, stats[k]);
+  auto t2 = now();
+  std::sort(sites.begin(), sites.end(), [](const Site& a, const Site& b) {
+    if (a.k != b.k) return a.k < b.k;
+    if (a.idx != b.idx) return a.idx < b.idx;
+    return a.rule < b.rule;
+  });
+  if (detect) {
+    for (int k = kbegin; k < kend; k++)
+      fprintf(out, "K %d %zu %zu gatom=%d satom=%d conv=%d vec_already=%d ustores=%d name=%s\n", k,
+              ks[k].ins.size(), ks[k].first_slot, stats[k].gatom, stats[k].satom, stats[k].conv,
+              stats[k].vec_already, stats[k].ustores, ks[k].name.c_str());
+    for (auto& s : sites) {
+      std::string chain;
+      for (size_t c = 0; c < s.tr.chain.size(); c++) chain += (c ? "," : "") + std::to_string(s.tr.chain[c]);
+      if (chain.empty()) chain = "-";
+      std::string line = s.line < 0 ? "-" : std::to_string(s.line);
+      fprintf(out, "S %d %d %s line=%s ld=%d term=%s d=%zu chain=%s%s%s\n", s.k, s.idx, kRuleName[s.rule],
+              line.c_str(), s.loop_depth, term_str(s.tr).c_str(), s.tr.chain.size(), chain.c_str(),
+              s.attrs.empty() ? "" : " ", s.attrs.c_str());
+    }
+  }
+  if (hist && !samples_path.empty()) {
+    // O13: H[slot][reason] += 1 for every valid sample.
+    size_t P = 0;
+    for (auto& k : ks) P += k.ins.size();
+    std::vector<uint64_t> H(P * 32, 0);
+    FILE* sf = fopen(samples_path.c_str(), "rb");
+    if (!sf) { fprintf(stderr, "cannot open %s\n", samples_path.c_str()); return 2; }
+    uint64_t N = 0, invalid = 0;
+    std::vector<RawSample> buf(1 << 16);
+    auto th0 = now();
+    while (size_t got = fread(buf.data(), sizeof(RawSample), buf.size(), sf)) {
+      for (size_t q = 0; q < got; q++) {
+        const RawSample& s = buf[q];
+        N++;
+        bool ok = s.kernel < ks.size() && s.pc % 16 == 0 && s.pc / 16 < ks[s.kernel].ins.size() &&
+                  s.reason < (uint32_t)C.R;
+        if (!ok) { invalid++; continue; }
+        H[(ks[s.kernel].first_slot + s.pc / 16) * 32 + s.reason]++;
+      }
+    }
+    fclose(sf);
+    auto th1 = now();
+    uint64_t mass = 0;
+    for (size_t b = 0; b < H.size(); b++)
+      if (H[b]) { fprintf(out, "H %zu %zu %llu\n", b / 32, b % 32, (unsigned long long)H[b]); mass += H[b]; }
+    fprintf(out, "N total=%llu valid=%llu invalid=%llu\n", (unsigned long long)N, (unsigned long long)mass,
+            (unsigned long long)invalid);
+    // O14 join: counts at the site's PC, site total, kernel total, REL sum.
+    std::vector<uint64_t> ktot(ks.size(), 0);
+    for (size_t k = 0; k < ks.size(); k++)
+      for (size_t i = 0; i < ks[k].ins.size(); i++)
+        for (int r = 0; r < 32; r++) ktot[k] += H[(ks[k].first_slot + i) * 32 + r];
+    struct Ranked { const Site* s; uint64_t rel, tot; };
+    std::vector<Ranked> rk;
+    for (auto& s : sites) {
+      size_t slot = ks[s.k].first_slot + (size_t)s.idx;
+      uint64_t tot = 0, rel = 0;
+      for (int r = 0; r < 32; r++) {
+        tot += H[slot * 32 + r];
+        if (kRel[s.rule] == -1 || (kRel[s.rule] >> r) & 1) rel += H[slot * 32 + r];
+      }
+      rk.push_back({&s, rel, tot});
+    }
+    // O15 rank: (rel desc, tot desc, kernel asc, idx asc, rule asc)
+    std::sort(rk.begin(), rk.end(), [](const Ranked& a, const Ranked& b) {
+      if (a.rel != b.rel) return a.rel > b.rel;
+      if (a.tot != b.tot) return a.tot > b.tot;
+      if (a.s->k != b.s->k) return a.s->k < b.s->k;
+      if (a.s->idx != b.s->idx) return a.s->idx < b.s->idx;
+      return a.s->rule < b.s->rule;
+    });
+    size_t lim = K_top < 0 ? rk.size() : std::min(rk.size(), (size_t)K_top);
+    for (size_t q = 0; q < lim; q++) {
+      const Site& s = *rk[q].s;
+      size_t slot = ks[s.k].first_slot + (size_t)s.idx;
+      std::string h;
+      for (int r = 0; r < C.R; r++) h += (r ? "," : "") + std::to_string(H[slot * 32 + r]);
+      fprintf(out, "R %zu %d %d %s rel=%llu tot=%llu ktot=%llu h=%s\n", q, s.k, s.idx, kRuleName[s.rule],
+              (unsigned long long)rk[q].rel, (unsigned long long)rk[q].tot, (unsigned long long)ktot[s.k], h.c_str());
+    }
+    if (timing) fprintf(stderr, "TIME hist_s=%.6f samples=%llu\n", secs(th0, th1), (unsigned long long)N);
+  }
+  auto t3 = now();
+  if (timing)
+    fprintf(stderr, "TIME parse_s=%.6f detect_s=%.6f total_s=%.6f instrs=%zu sites=%zu\n", secs(t0, t1),
+            secs(t1, t2), secs(t0, t3), [&] { size_t n = 0; for (auto& k : ks) n += k.ins.size(); return n; }(),
+            sites.size());
+  if (out != stdout) fclose(out);
+  return 0;
+}

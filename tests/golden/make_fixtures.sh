@@ -1,0 +1,19 @@
+#!/usr/bin/env bash
+# Regenerates the frozen SASS text fixtures from tests/golden/src/*.cu with this box's
+# nvcc 12.9 (cuobjdump -sass). The .sass files are committed; rerunning must give
+# identical text for the same toolchain. Spill fixtures also record ptxas -v output.
+set -euo pipefail
+cd "$(dirname "$0")"
+T=$(mktemp -d)
+for arch in sm_100a sm_70; do
+  for k in sgemm_naive jacobi mixbench atomics conv; do
+    nvcc -arch=$arch -cubin -O3 -o $T/$k.$arch.cubin src/$k.cu
+    cuobjdump -sass $T/$k.$arch.cubin > $k.$arch.sass
+  done
+done
+for cap in 24 32 40 64; do
+  nvcc -arch=sm_100a -cubin -O3 -maxrregcount=$cap -Xptxas -v -o $T/spill.$cap.cubin src/spill.cu \
+     2> spill.r$cap.ptxas.txt
+  cuobjdump -sass $T/spill.$cap.cubin > spill.r$cap.sm_100a.sass
+done
+rm -rf $T

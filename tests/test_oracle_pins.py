@@ -1,0 +1,284 @@
+"""Pins of the CPU oracle against facts fixed outside it.
+
+Every expected value here comes from the paper's text (cited), from the C ABI of a kernel whose
+source is in tests/golden/src (parameter offsets), from ptxas' own spill accounting, from a
+closed-form count table, or from the independent brute force in tests/brute.py — never from the
+oracle itself and never from the CUDA path.
+"""
+import random
+
+import numpy as np
+import pytest
+
+import brute
+import oracle_run as orc
+from oracle_run import Canon, golden
+
+pytestmark = pytest.mark.usefixtures("oracle_bin")
+
+
+# --------------------------------------------------------------------------- Listing 1
+def test_listing1_texture_and_vector_groups():
+    c = Canon(orc.run(golden("listing1.sass")))
+    vec = {s["idx"] for s in c.sites("VEC")}
+    # "Loads to R0 and R9 fetch data from adjacent memory addresses R2 and R2+-0x8 ...
+    #  The same holds for loads to R5 and R7."
+    assert vec == {0, 1, 2, 3}
+    groups = {s["idx"]: (s["term"], s["min"], s["max"], s["n"]) for s in c.sites("VEC")}
+    assert groups[0] == groups[3] == ("ENTRY:R2", "-8", "0", "2")
+    assert groups[1] == groups[2] == ("ENTRY:R4", "-8", "0", "2")
+    # "If these registers are read-only, they are potential candidates for texture memory":
+    # STG [R4], R9 writes through R4, so only the R2-based loads (R0, R9) are read-only.
+    assert {s["idx"] for s in c.sites("RO")} == {0, 3}
+    assert {s["idx"] for s in c.sites("TEX")} == {0, 3}
+    assert c.sites("SHMEM") == []  # no arithmetic on the loaded values
+
+
+# --------------------------------------------------------------------------- SGEMM
+# sgemm_naive(int M, int N, int K, float alpha, const float* A, const float* B, float beta, float* C)
+# C ABI parameter offsets from the param base: A +0x10, B +0x18, C +0x28.
+@pytest.mark.parametrize("arch,base", [("sm_100a", 0x380), ("sm_70", 0x160)])
+def test_sgemm_readonly_A_B_not_C(arch, base):
+    c = Canon(orc.run(golden(f"sgemm_naive.{arch}.sass")))
+    A, B, C = hex(base + 0x10), hex(base + 0x18), hex(base + 0x28)
+    ops = orc.sass_ops(golden(f"sgemm_naive.{arch}.sass"))
+    ldg = {i for i, op in ops.items() if op.startswith("LDG")}
+    ro_terms = {s["term"] for s in c.sites("RO")}
+    # "registers that are read-only throughout the lifetime of the kernel, and are not aliased"
+    # (P:943-946): A and B, never C (C is loaded and stored).
+    assert ro_terms == {f"PARAM:{A}", f"PARAM:{B}"}
+    ro = {s["idx"] for s in c.sites("RO")}
+    assert len(ldg - ro) == 1                           # exactly the C load is not read-only
+    # shared-memory advice on the loop loads
+    shm = c.sites("SHMEM")
+    assert {s["term"] for s in shm} == {f"PARAM:{A}", f"PARAM:{B}"}
+    assert any(s["ld"] == "1" for s in shm)
+
+
+def test_sgemm_sm100_eight_adjacent_A_loads():
+    """The unroll-by-8 A loads off R4 at -0x10..+0xc (SURVEY [probe 4]); the "reads seven
+    adjacent addresses" shape of P:789-792, inside the loop closed by `@P1 BRA 0x220` at 0x4b0."""
+    c = Canon(orc.run(golden("sgemm_naive.sm_100a.sass")))
+    want = {0x260 // 16, 0x270 // 16, 0x280 // 16, 0x2a0 // 16, 0x350 // 16, 0x370 // 16, 0x3a0 // 16,
+            0x3c0 // 16}
+    big = [s for s in c.sites("VEC") if s["n"] == "8"]
+    assert {s["idx"] for s in big} == want
+    for s in big:
+        assert (s["min"], s["max"], s["contig"], s["term"], s["ld"]) == ("-16", "12", "1", "PARAM:0x390", "1")
+        assert s["chain"].split(",")[-1] == str(0x190 // 16)     # LDCU.64 UR4, c[0x0][0x390]
+    # loop span [0x220, 0x4b0] only: the load at 0x870 (C) has loop depth 0
+    assert all(s["ld"] == "1" for s in c.sites() if 0x22 <= s["idx"] <= 0x4b)
+    assert all(s["ld"] == "0" for s in c.sites() if s["idx"] > 0x4b)
+
+
+# --------------------------------------------------------------------------- Jacobi
+# jacobi(const float* Told, float* Tnew, ...): Told at +0x0, Tnew at +0x8; six (float) casts.
+@pytest.mark.parametrize("arch,base", [("sm_100a", 0x380), ("sm_70", 0x160)])
+def test_jacobi_flags_and_six_conversions(arch, base):
+    c = Canon(orc.run(golden(f"jacobi.{arch}.sass")))
+    k = c.kstats()[0]
+    assert k["conv"] == 6 and len(c.sites("CONV")) == 6          # "six I2F"
+    told = f"PARAM:{hex(base)}"
+    # recommended: texture/shared, vectorised loads, __restrict__, conversions
+    for rule in ("TEX", "SHMEM", "VEC", "RO"):
+        assert c.sites(rule), rule
+        assert {s["term"] for s in c.sites(rule)} == {told}, rule
+
+
+# --------------------------------------------------------------------------- Mixbench
+def test_mixbench_sp_vectorise_dp_already_vectorised():
+    for arch in ("sm_100a", "sm_70"):
+        c = Canon(orc.run(golden(f"mixbench.{arch}.sass")))
+        ks = {d["name"]: d for d in c.kstats()}
+        dp = [d for n, d in ks.items() if "dp" in n][0]
+        sp = [d for n, d in ks.items() if "sp" in n][0]
+        # SP: one 32-bit load "also reads seven adjacent addresses"
+        vec = c.sites("VEC", k=sp["k"])
+        assert len(vec) == 8 and {(s["n"], s["contig"]) for s in vec} == {("8", "1")}
+        assert {int(s["max"]) - int(s["min"]) for s in vec} == {28}
+        # DP: "a 64-bit width vectorized read performed by the compiler"
+        assert c.sites("VEC", k=dp["k"]) == [] and dp["vec_already"] == 8
+        # shared-memory advice on the same loads
+        assert len(c.sites("SHMEM", k=sp["k"])) == 8 and len(c.sites("SHMEM", k=dp["k"])) == 8
+
+
+# --------------------------------------------------------------------------- spills
+@pytest.mark.parametrize("cap", [24, 32, 40, 64])
+def test_spill_sites_match_ptxas_bytes(cap):
+    """ptxas -v "N bytes spill stores, M bytes spill loads" == sum of STL / LDL access widths."""
+    path = golden(f"spill.r{cap}.sm_100a.sass")
+    c = Canon(orc.run(path))
+    ops = orc.sass_ops(path)
+    st = ld = 0
+    for s in c.sites("SPILL"):
+        op = ops[s["idx"]]
+        w = 16 if ".128" in op else 8 if ".64" in op else 4
+        if op.startswith("STL"):
+            st += w
+        else:
+            assert op.startswith("LDL")
+            ld += w
+    txt = open(golden(f"spill.r{cap}.ptxas.txt")).read()
+    want = txt.split("stack frame,")[1].split("\n")[0]
+    assert f"{st} bytes spill stores, {ld} bytes spill loads" in want
+    assert len(c.sites("SPILL")) == sum(1 for op in ops.values() if op.startswith(("STL", "LDL")))
+
+
+def test_fig2_spill_cause_is_last_writer():
+    """Fig.2 narrative: the cause of a spill of register X is the last instruction
+    that wrote X (an IADD); the lg_throttle stall is the largest at that instruction."""
+    text = "\tcode for sm_100a\n\t\tFunction : fig2\n" + "\n".join(
+        f"        /*{16 * i:04x}*/                   {b} ;" for i, b in enumerate([
+            "LDC R1, c[0x0][0x37c]",
+            "IADD3 R5, PT, PT, R2, R3, RZ",
+            "FMUL R6, R7, R8",
+            "STL [R1+0x4], R5",
+            "IADD3 R5, PT, PT, R5, 0x1, RZ",
+            "EXIT",
+        ])) + "\n"
+    # samples at the STL (pc 0x30): lg_throttle 7, long_scoreboard 2, wait 1
+    raw = np.array([[0, 0x30, 5]] * 7 + [[0, 0x30, 6]] * 2 + [[0, 0x30, 17]], dtype=np.uint32)
+    c = Canon(orc.run(text, samples=raw))
+    sp = c.sites("SPILL")
+    assert len(sp) == 1 and sp[0]["idx"] == 3 and sp[0]["cause"] == "1" and sp[0]["data"] == "R5"
+    assert sp[0]["term"] == "CONST:0x0:0x37c"               # the stack pointer, not a parameter
+    r = c.R[0].split()
+    h = [int(x) for x in r[-1].split("=")[1].split(",")]
+    assert int(np.argmax(h)) == 5                            # lg_throttle largest offender
+    assert r[5:8] == ["rel=9", "tot=10", "ktot=10"]          # SPILL REL = {long_sb, lg_throttle}
+
+
+# --------------------------------------------------------------------------- atomics, conversions
+def test_atomics_probe():
+    c = Canon(orc.run(golden("atomics.sm_100a.sass")))
+    g = c.sites("GATOM")
+    ops = orc.sass_ops(golden("atomics.sm_100a.sass"))
+    # source: one global atomicAdd in the loop, one after it (compiled to REDG), one shared atomic
+    assert [ops[s["idx"]].split(".")[0] for s in g] == ["REDG", "REDG"]
+    assert [s["ld"] for s in g] == ["1", "0"]
+    assert c.kstats()[0]["satom"] == 1 and c.kstats()[0]["gatom"] == 2
+    # gcount is param 1 (+0x8), gtotal param 2 (+0x10)
+    assert [s["term"] for s in g] == ["PARAM:0x388", "PARAM:0x390"]
+
+
+def test_conversion_probe():
+    c = Canon(orc.run(golden("conv.sm_100a.sass")))
+    assert c.kstats()[0]["conv"] == 2                       # one int->float, one double->float
+    ops = orc.sass_ops(golden("conv.sm_100a.sass"))
+    assert sorted(ops[s["idx"]] for s in c.sites("CONV")) == ["F2F.F32.F64", "I2FP.F32.S32"]
+
+
+# --------------------------------------------------------------------------- trace depth bound
+def chain_text(L):
+    body = ["LDC.64 R2, c[0x0][0x388]"]
+    r = 2
+    for i in range(L):
+        nr = 4 if r == 2 else 2
+        body.append(["IADD3 R%d, P0, PT, R%d, 0x10, RZ", "MOV R%d, R%d", "IMAD.WIDE R%d, R9, 0x4, R%d"][i % 3]
+                    % (nr, r))
+        r = nr
+    body.append(f"LDG.E R7, desc[UR6][R{r}.64]")
+    return "\tcode for sm_100a\n\t\tFunction : chain\n" + "\n".join(
+        f"        /*{16 * i:04x}*/                   {b} ;" for i, b in enumerate(body)) + "\n"
+
+
+@pytest.mark.parametrize("L,D,resolved", [(62, 64, True), (63, 64, True), (64, 64, False), (3, 4, True),
+                                          (4, 4, False)])
+def test_trace_depth_semantics(L, D, resolved):
+    """A chain needing exactly D last-writer steps resolves; D+1 steps is TRUNCATED (DESIGN §3 O5)."""
+    c = Canon(orc.run(chain_text(L), D=D))
+    ro = c.sites("RO")
+    if resolved:
+        assert len(ro) == 1 and ro[0]["term"] == "PARAM:0x388" and ro[0]["d"] == str(L + 1)
+    else:
+        assert ro == []          # TRUNCATED roots are never read-only (DESIGN §3 O10)
+    steps = L + 1
+    assert (steps <= D) == resolved
+
+
+def test_trace_truncated_chain_recorded():
+    # an LDG pair on the 65-step chain: both are VEC sites carrying the truncated trace
+    body = chain_text(64).splitlines()
+    last = body[-1]
+    reg = last.split("[R")[1].split(".")[0]
+    body.append(f"        /*{int(last.split('/*')[1].split('*/')[0], 16) + 16:04x}*/                   "
+                f"LDG.E R8, desc[UR6][R{reg}.64+0x4] ;")
+    c = Canon(orc.run("\n".join(body) + "\n", D=64))
+    v = c.sites("VEC")
+    assert len(v) == 2 and all(s["term"] == "TRUNC" and s["d"] == "64" for s in v)
+
+
+# --------------------------------------------------------------------------- brute force
+def test_brute_force_random_streams():
+    rng = random.Random(20231112)
+    for _ in range(300):
+        ks = [brute.random_stream(rng, rng.randint(1, 6)) for _ in range(rng.randint(1, 3))]
+        D = rng.choice([1, 2, 3, 64])
+        c = Canon(orc.run(brute.render(ks), D=D))
+        kl, sl = brute.detect(ks, D=D)
+        assert c.K == kl and c.S == sl, brute.render(ks)
+
+
+# --------------------------------------------------------------------------- histogram, join, rank
+def _sgemm_samples(order="trace", seed=3, n=50_000, n_bad=64):
+    from gen import samples as gs
+    path = golden("sgemm_naive.sm_100a.sass")
+    n_instr = [len(orc.sass_ops(path))]
+    cls = np.full(n_instr[0], gs.CLS_ALU, dtype=np.uint8)
+    cls[::7] = gs.CLS_MEM
+    tab = gs.table_class_weighted(cls, n, key=seed)
+    tr = gs.Trace(tab, [0], n_instr, order=order, seed=seed)
+    raw = tr.raw()
+    bad = gs.invalid_raw(1, n_instr, n_bad, key=seed)
+    return path, tab, gs.interleave(raw, bad, key=seed + 1), n_bad
+
+
+def test_histogram_equals_count_table():
+    path, tab, raw, n_bad = _sgemm_samples()
+    c = Canon(orc.run(path, samples=raw))
+    want = {(s, r): int(tab[s, r]) for s, r in zip(*np.nonzero(tab))}
+    assert c.H == want
+    assert c.N == {"total": str(len(raw)), "valid": str(int(tab.sum())), "invalid": str(n_bad)}
+
+
+def test_histogram_permutation_and_shard_invariance():
+    path, tab, raw, _ = _sgemm_samples(order="shuffled", seed=5)
+    full = Canon(orc.run(path, samples=raw))
+    rev = Canon(orc.run(path, samples=raw[::-1].copy()))
+    assert rev.H == full.H and rev.R == full.R
+    for shards in (2, 4, 8):
+        acc = {}
+        for part in np.array_split(raw, shards):
+            for key, v in Canon(orc.run(path, samples=part, detect=False)).H.items():
+                acc[key] = acc.get(key, 0) + v
+        assert acc == full.H
+
+
+def test_join_and_rank_closed_form():
+    """rel/tot/ktot recomputed from the count table and the site list, ranked with Python's sort."""
+    path, tab, raw, _ = _sgemm_samples(seed=9)
+    c = Canon(orc.run(path, samples=raw))
+    rel_sets = {"VEC": [6], "SPILL": [5, 6], "SHMEM": [6], "GATOM": [5], "RO": [6], "TEX": [6, 16],
+                "CONV": list(range(32))}
+    order = ["VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX", "CONV"]
+    rows = []
+    for s in c.sites():
+        h = tab[s["idx"]]
+        rows.append((-int(h[rel_sets[s["rule"]]].sum()), -int(h.sum()), s["k"], s["idx"], order.index(s["rule"])))
+    rows.sort()
+    got = [r.split() for r in c.R]
+    assert len(got) == len(rows)
+    ktot = int(tab.sum())
+    for q, (g, w) in enumerate(zip(got, rows)):
+        assert g[:5] == ["R", str(q), str(w[2]), str(w[3]), order[w[4]]]
+        assert g[5:8] == [f"rel={-w[0]}", f"tot={-w[1]}", f"ktot={ktot}"]
+
+
+def test_configs_generate_and_run():
+    from gen import sass as gsass
+    for cfg in ("C1", "C2"):
+        s = gsass.config_sass(cfg)
+        c = Canon(orc.run(s.text))
+        assert len(c.K) == {"C1": 1, "C2": 3}[cfg]
+        assert sum(k["n"] for k in c.kstats()) == s.P
+        assert c.sites("SPILL") if cfg == "C1" else c.sites("VEC")

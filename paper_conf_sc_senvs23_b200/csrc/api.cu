@@ -1,0 +1,289 @@
+// api.cu — the C ABI (include/gpuscout_b200.h): context, SASS loading, entry points.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <thread>
+
+#include "ctx.h"
+#include "loader.h"
+
+namespace gs {
+
+gs_status fail(gs_ctx* c, gs_status s, const std::string& msg) {
+  if (c) c->err = msg;
+  return s;
+}
+gs_status cuda_fail(gs_ctx* c, cudaError_t e, const char* what) {
+  return fail(c, GS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+namespace {
+
+void free_loaded(gs_ctx* c) {
+  detect_free(c);
+  if (c->d_rec) cudaFree(c->d_rec);
+  if (c->d_kd) cudaFree(c->d_kd);
+  if (c->d_wd) cudaFree(c->d_wd);
+  if (c->d_cbase) cudaFree(c->d_cbase);
+  c->d_rec = nullptr;
+  c->d_kd = nullptr;
+  c->d_wd = nullptr;
+  c->d_cbase = nullptr;
+  c->loaded = false;
+}
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+}  // namespace
+}  // namespace gs
+
+using namespace gs;
+
+extern "C" {
+
+const char* gs_version(void) { return "gpuscout_b200 0.1 (sm_100a)"; }
+
+gs_status gs_create(gs_ctx** out, int device, void* cuda_stream, const gs_config* cfg) {
+  if (!out) return GS_E_INVAL;
+  *out = nullptr;
+  gs_ctx* c = new (std::nothrow) gs_ctx();
+  if (!c) return GS_E_NOMEM;
+  c->device = device;
+  c->stream = static_cast<cudaStream_t>(cuda_stream);
+  if (cfg) c->cfg = *cfg;
+  if (!c->cfg.trace_depth) c->cfg.trace_depth = 64;
+  if (!c->cfg.n_reasons) c->cfg.n_reasons = 19;
+  if (!c->cfg.shmem_min_arith) c->cfg.shmem_min_arith = 1;
+  if (!c->cfg.shmem_min_loads) c->cfg.shmem_min_loads = 2;
+  if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_WINDOW) {
+    delete c;
+    return GS_E_INVAL;
+  }
+  cudaError_t e = cudaSetDevice(device);
+  if (e != cudaSuccess) {
+    delete c;
+    return GS_E_CUDA;
+  }
+  *out = c;
+  return GS_OK;
+}
+
+void gs_destroy(gs_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  else cudaDeviceSynchronize();
+  free_loaded(c);
+  attrib_free(c);
+  rank_free(c);
+  delete c;
+}
+
+const char* gs_last_error(const gs_ctx* c) { return c ? c->err.c_str() : "null context"; }
+
+gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kernels, uint64_t* n_instr) {
+  if (!c || (!text && len)) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  GS_CUDA(c, cudaSetDevice(c->device));
+  std::vector<ParsedKernel> ks;
+  std::string err;
+  const int nt = (int)std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  if (!parse_sass(text, len, nt, &ks, &err)) return fail(c, GS_E_PARSE, err);
+  uint64_t P = 0;
+  for (auto& k : ks) P += k.recs.size();
+  if (P > 0x7ffffffeull) return fail(c, GS_E_RANGE, "more than 2^31-2 instructions");
+  if (c->stream) GS_CUDA(c, cudaStreamSynchronize(c->stream));
+  free_loaded(c);
+  c->n_kernels = (uint32_t)ks.size();
+  c->n_instr = P;
+  c->names.clear();
+  c->kd_h.assign(ks.size(), KDesc{});
+  c->wd_h.clear();
+  c->lines_h.clear();
+  c->lines_h.reserve(P);
+  c->cbase_h.clear();
+  c->n_cand = c->n_ldg = c->n_store = 0;
+  std::vector<Rec> recs;
+  recs.reserve(P);
+  uint32_t slot = 0;
+  for (size_t k = 0; k < ks.size(); k++) {
+    ParsedKernel& pk = ks[k];
+    KDesc& K = c->kd_h[k];
+    K.first = slot;
+    K.n = (uint32_t)pk.recs.size();
+    K.param_base = pk.param_base;
+    K.win0 = (uint32_t)c->wd_h.size();
+    for (uint32_t s = 0; s < K.n; s += kWin) {
+      WDesc W{(uint32_t)k, slot + s, std::min(kWin, K.n - s), 0};
+      uint32_t nc = 0;
+      for (uint32_t i = 0; i < W.len; i++) {  // candidates per window: static opcode classes
+        const Rec& r = pk.recs[s + i];
+        const uint32_t cls = op_class(r_op(r));
+        if (cls & (C_TRACED | C_CONV)) nc++;
+        if (r_op(r) == OP_LDG) c->n_ldg++;
+        if (cls & C_STORE) c->n_store++;
+      }
+      c->cbase_h.push_back((uint32_t)c->n_cand);
+      c->n_cand += nc;
+      c->wd_h.push_back(W);
+    }
+    slot += K.n;
+    recs.insert(recs.end(), pk.recs.begin(), pk.recs.end());
+    c->lines_h.insert(c->lines_h.end(), pk.lines.begin(), pk.lines.end());
+    c->names.push_back(std::move(pk.name));
+  }
+  c->cbase_h.push_back((uint32_t)c->n_cand);
+  c->n_win = (uint32_t)c->wd_h.size();
+  if (c->n_cand > 0xffffffffull) return fail(c, GS_E_RANGE, "too many candidate instructions");
+  GS_CUDA(c, cudaMalloc((void**)&c->d_rec, std::max<uint64_t>(P, 1) * sizeof(Rec)));
+  GS_CUDA(c, cudaMalloc((void**)&c->d_kd, std::max<size_t>(ks.size(), 1) * sizeof(KDesc)));
+  GS_CUDA(c, cudaMalloc((void**)&c->d_wd, std::max<size_t>(c->wd_h.size(), 1) * sizeof(WDesc)));
+  GS_CUDA(c, cudaMalloc((void**)&c->d_cbase, c->cbase_h.size() * 4));
+  if (P) GS_CUDA(c, cudaMemcpyAsync(c->d_rec, recs.data(), P * sizeof(Rec), cudaMemcpyHostToDevice, c->stream));
+  if (!ks.empty())
+    GS_CUDA(c, cudaMemcpyAsync(c->d_kd, c->kd_h.data(), ks.size() * sizeof(KDesc), cudaMemcpyHostToDevice, c->stream));
+  if (!c->wd_h.empty())
+    GS_CUDA(c, cudaMemcpyAsync(c->d_wd, c->wd_h.data(), c->wd_h.size() * sizeof(WDesc), cudaMemcpyHostToDevice,
+                               c->stream));
+  GS_CUDA(c, cudaMemcpyAsync(c->d_cbase, c->cbase_h.data(), c->cbase_h.size() * 4, cudaMemcpyHostToDevice, c->stream));
+  gs_status s = detect_alloc(c);
+  if (s != GS_OK) return s;
+  // pageable source buffers: wait for the copies before they go out of scope
+  GS_CUDA(c, cudaStreamSynchronize(c->stream));
+  c->loaded = true;
+  if (n_kernels) *n_kernels = c->n_kernels;
+  if (n_instr) *n_instr = P;
+  return GS_OK;
+}
+
+gs_status gs_kernel_table(const gs_ctx* c, uint32_t* first_slot, uint32_t* n_instr, size_t cap) {
+  if (!c) return GS_E_INVAL;
+  if (!c->loaded) return GS_E_STATE;
+  const size_t n = std::min<size_t>(cap, c->n_kernels);
+  for (size_t k = 0; k < n; k++) {
+    if (first_slot) first_slot[k] = c->kd_h[k].first;
+    if (n_instr) n_instr[k] = c->kd_h[k].n;
+  }
+  return GS_OK;
+}
+
+const char* gs_kernel_name(const gs_ctx* c, uint32_t k) {
+  if (!c || !c->loaded || k >= c->n_kernels) return nullptr;
+  return c->names[k].c_str();
+}
+
+gs_status gs_instr_lines(const gs_ctx* c, int32_t* lines, size_t cap) {
+  if (!c || !lines) return GS_E_INVAL;
+  if (!c->loaded) return GS_E_STATE;
+  memcpy(lines, c->lines_h.data(), std::min<size_t>(cap, c->lines_h.size()) * 4);
+  return GS_OK;
+}
+
+gs_status gs_detect(gs_ctx* c, uint32_t k_begin, uint32_t k_end, uint64_t* n_sites) {
+  if (!c) return GS_E_INVAL;
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_detect before gs_load_sass");
+  if (k_begin > k_end || k_end > c->n_kernels) return fail(c, GS_E_INVAL, "bad kernel range");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  return detect_run(c, k_begin, k_end, n_sites);
+}
+
+gs_status gs_sites(const gs_ctx* c, const gs_site** d_sites, const uint32_t** d_chain, uint64_t* n_sites,
+                   uint64_t* n_chain) {
+  if (!c) return GS_E_INVAL;
+  if (!c->detected) return GS_E_STATE;
+  if (d_sites) *d_sites = c->d_sites;
+  if (d_chain) *d_chain = c->d_chain;
+  if (n_sites) *n_sites = c->n_sites;
+  if (n_chain) *n_chain = c->n_chain;
+  return GS_OK;
+}
+
+gs_status gs_sites_host(gs_ctx* c, gs_site* sites, size_t cap_sites, uint32_t* chain, size_t cap_chain) {
+  if (!c) return GS_E_INVAL;
+  if (!c->detected) return fail(c, GS_E_STATE, "gs_sites_host before gs_detect");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  const size_t ns = std::min<size_t>(cap_sites, c->n_sites), nch = std::min<size_t>(cap_chain, c->n_chain);
+  if (sites && ns) GS_CUDA(c, cudaMemcpyAsync(sites, c->d_sites, ns * sizeof(gs_site), cudaMemcpyDeviceToHost, c->stream));
+  if (chain && nch) GS_CUDA(c, cudaMemcpyAsync(chain, c->d_chain, nch * 4, cudaMemcpyDeviceToHost, c->stream));
+  GS_CUDA(c, cudaStreamSynchronize(c->stream));
+  return GS_OK;
+}
+
+gs_status gs_kernel_stats_get(const gs_ctx* c, gs_kernel_stats* out, size_t cap) {
+  if (!c || !out) return GS_E_INVAL;
+  if (!c->detected) return GS_E_STATE;
+  memcpy(out, c->kstats_h.data(), std::min<size_t>(cap, c->kstats_h.size()) * sizeof(gs_kernel_stats));
+  return GS_OK;
+}
+
+gs_status gs_pack_samples(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
+                          unsigned long long* d_n_invalid) {
+  if (!c || (n && (!d_raw || !d_words)) || !d_n_invalid) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_pack_samples before gs_load_sass");
+  if (c->n_instr >= (1ull << 27)) return fail(c, GS_E_RANGE, "packed samples address at most 2^27 slots");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  return pack_samples_run(c, d_raw, n, d_words, d_n_invalid);
+}
+
+gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, int32_t* d_hist,
+                               unsigned long long* d_n_invalid, int accumulate) {
+  if (!c || (n && !samples) || !d_n_invalid) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_attribute_samples before gs_load_sass");
+  if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
+  if (c->n_instr >= (1ull << 27)) return fail(c, GS_E_RANGE, "packed samples address at most 2^27 slots");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  if (!n || is_device_ptr(samples)) return hist_run(c, samples, n, d_hist, d_n_invalid, accumulate, true);
+  // host input: stream chunks through two device staging buffers; the H2D copy of chunk i+1
+  // (copy engine) overlaps the histogram of chunk i
+  const size_t chunk = size_t(16) << 20;  // words
+  if (c->stage_words < chunk) {
+    attrib_free(c);
+    for (int b = 0; b < 2; b++) {
+      GS_CUDA(c, cudaMalloc((void**)&c->d_stage[b], chunk * 4));
+      GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_stage[b], cudaEventDisableTiming));
+    }
+    c->stage_words = chunk;
+  }
+  if (!accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * 32 * 4, c->stream));
+  uint64_t done = 0;
+  int b = 0;
+  while (done < n) {
+    const uint64_t m = std::min<uint64_t>(chunk, n - done);
+    GS_CUDA(c, cudaMemcpyAsync(c->d_stage[b], samples + done, m * 4, cudaMemcpyHostToDevice, c->stream));
+    gs_status s = hist_run(c, c->d_stage[b], m, d_hist, d_n_invalid, 1, false);
+    if (s != GS_OK) return s;
+    GS_CUDA(c, cudaEventRecord(c->ev_stage[b], c->stream));
+    done += m;
+    b ^= 1;
+  }
+  GS_CUDA(c, cudaStreamSynchronize(c->stream));
+  return GS_OK;
+}
+
+gs_status gs_rank_sites(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, uint64_t* n_out) {
+  if (!c) return GS_E_INVAL;
+  c->err.clear();
+  if (!c->detected) return fail(c, GS_E_STATE, "gs_rank_sites before gs_detect");
+  if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
+  if (k && c->n_sites && !out) return fail(c, GS_E_INVAL, "null output");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  const bool host = out ? !is_device_ptr(out) : true;
+  return rank_run(c, d_hist, k, out, host, n_out);
+}
+
+int gs_last_hist_mode(const gs_ctx* c) { return c ? c->last_hist_mode : -1; }
+
+}  // extern "C"

@@ -1,0 +1,154 @@
+// ctx.h — the library context (opaque gs_ctx behind the C ABI) and internal launch helpers.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/gpuscout_b200.h"
+#include "record.h"
+
+namespace gs {
+
+constexpr uint32_t kWin = 512;  // instructions per detection window (never crosses a kernel)
+
+// A device buffer that only grows; freed with the context.
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+// Candidate arrays: one entry per traced memory instruction or conversion.
+struct CandArrays {
+  uint32_t *idx = nullptr, *kernel = nullptr, *base_rd = nullptr, *data_rd = nullptr, *tv = nullptr,
+           *grp = nullptr, *nsite = nullptr, *soff = nullptr;
+  uint8_t *ld = nullptr, *tk = nullptr, *depth = nullptr, *flags = nullptr;
+  unsigned long long* choff = nullptr;  // chain offsets (exclusive scan of chain lengths)
+};
+
+struct GroupTable {  // key-group statistics of global loads (R3)
+  uint32_t cap = 0;  // power of two
+  unsigned long long* key = nullptr;
+  uint32_t *nload = nullptr, *n32 = nullptr, *nall = nullptr, *or3 = nullptr, *and3 = nullptr;
+  int32_t *mn = nullptr, *mx = nullptr;
+};
+
+struct OffsetSet {  // distinct (group, offset) pairs
+  uint32_t cap = 0;
+  unsigned long long* key = nullptr;
+  uint32_t* flags = nullptr;
+};
+
+struct RootSet {  // store roots per kernel (R8)
+  uint32_t cap = 0;
+  unsigned long long* key = nullptr;
+};
+
+}  // namespace gs
+
+struct gs_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  gs_config cfg{};
+  std::string err;
+
+  // ---- loaded SASS (host mirrors)
+  bool loaded = false;
+  uint32_t n_kernels = 0, n_win = 0;
+  uint64_t n_instr = 0, n_cand = 0, n_ldg = 0, n_store = 0;
+  std::vector<std::string> names;
+  std::vector<gs::KDesc> kd_h;
+  std::vector<gs::WDesc> wd_h;
+  std::vector<uint32_t> cbase_h;  // candidate base per window (n_win + 1)
+  std::vector<int32_t> lines_h;
+
+  // ---- device copies
+  gs::Rec* d_rec = nullptr;
+  gs::KDesc* d_kd = nullptr;
+  gs::WDesc* d_wd = nullptr;
+  uint32_t* d_cbase = nullptr;
+
+  // ---- detection scratch
+  uint32_t* d_tab = nullptr;  // n_win x 320 last-writer summaries -> carry-in tables
+  int32_t* d_ldiff = nullptr; // loop-event difference array (kept zero between calls)
+  int32_t* d_wsum = nullptr;  // per-window loop-event sum
+  int32_t* d_wloop = nullptr; // per-window loop-depth carry-in
+  uint32_t* d_wev = nullptr;  // per-window loop-event count
+  uint32_t* d_ptrrd = nullptr;  // RD of each instruction's pointer operand (idx+1, 0 = ENTRY)
+  uint32_t* d_narith = nullptr; // n_arith per global load (sparse)
+  gs::CandArrays cand;
+  gs::GroupTable grp;
+  gs::OffsetSet oset;
+  gs::RootSet roots;
+  gs_kernel_stats* d_kstats = nullptr;
+  std::vector<gs_kernel_stats> kstats_h;
+  void* d_scan_tmp = nullptr;
+  size_t scan_tmp_bytes = 0;
+
+  // ---- detection result
+  bool detected = false;
+  uint32_t det_kb = 0, det_ke = 0;
+  uint64_t det_c0 = 0, det_c1 = 0;
+  gs_site* d_sites = nullptr;
+  uint64_t sites_cap = 0, n_sites = 0;
+  uint32_t* d_chain = nullptr;
+  uint64_t chain_cap = 0, n_chain = 0;
+
+  // ---- attribution / ranking scratch
+  int last_hist_mode = 0;
+  unsigned long long* d_rank_keys[2] = {nullptr, nullptr};
+  uint32_t* d_rank_vals[2] = {nullptr, nullptr};
+  uint64_t rank_cap = 0;
+  void* d_sort_tmp = nullptr;
+  size_t sort_tmp_bytes = 0;
+  unsigned long long* d_ktot = nullptr;
+  gs_ranked_site* d_ranked = nullptr;
+  uint64_t ranked_cap = 0;
+  uint32_t* h_stage[2] = {nullptr, nullptr};  // pinned staging for host sample input
+  uint32_t* d_stage[2] = {nullptr, nullptr};
+  cudaEvent_t ev_stage[2] = {nullptr, nullptr};
+  size_t stage_words = 0;
+};
+
+namespace gs {
+
+// error helpers (set ctx->err, return status)
+gs_status fail(gs_ctx* c, gs_status s, const std::string& msg);
+gs_status cuda_fail(gs_ctx* c, cudaError_t e, const char* what);
+#define GS_CUDA(ctx, call)                                  \
+  do {                                                      \
+    cudaError_t e_ = (call);                                \
+    if (e_ != cudaSuccess) return gs::cuda_fail(ctx, e_, #call); \
+  } while (0)
+
+template <typename T>
+cudaError_t dev_grow(T** p, uint64_t* cap, uint64_t need) {
+  if (*p && *cap >= need) return cudaSuccess;
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  if (need == 0) return cudaSuccess;
+  cudaError_t e = cudaMalloc((void**)p, need * sizeof(T));
+  if (e == cudaSuccess) *cap = need;
+  return e;
+}
+
+// launchers implemented in detect.cu / attrib.cu / rank.cu
+gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites);
+gs_status detect_alloc(gs_ctx* c);  // after a load
+void detect_free(gs_ctx* c);
+gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
+                           unsigned long long* d_n_invalid);
+gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,
+                   unsigned long long* d_n_invalid, int accumulate, bool zero_first);
+gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, bool out_is_host,
+                   uint64_t* n_out);
+void attrib_free(gs_ctx* c);
+void rank_free(gs_ctx* c);
+
+// device-wide exclusive scan of u32 counts into u32 or u64 offsets; total written to *d_total
+gs_status scan_u32(gs_ctx* c, const uint32_t* in, uint32_t* out, uint64_t n, unsigned long long* d_total);
+gs_status scan_u32_to_u64(gs_ctx* c, const uint32_t* in, unsigned long long* out, uint64_t n,
+                          unsigned long long* d_total);
+
+}  // namespace gs

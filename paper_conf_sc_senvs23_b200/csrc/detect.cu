@@ -1,0 +1,587 @@
+// detect.cu — SASS detection on the GPU (SURVEY §8a rows a-2 .. a-7; paper §4).
+//
+// Data layout: records (16 B each, one uint4 per lane) are processed in windows of kWin
+// instructions that never cross a kernel. One warp owns one window.
+//
+//   k_summary  per window: last writer of every register inside the window (R5), loop events of
+//              backward branches (R13), per-kernel opcode counters.
+//   k_carry    per kernel: turns window summaries into carry-in tables (segmented prefix), loop
+//              depth carry-in per window.
+//   k_resolve  per window: reaching definitions RD(i, r) for the pointer operand of
+//              every instruction and for the address base / spilled register of every
+//              candidate; loop depth; n_arith of global loads.
+//              Within a 32-instruction chunk the last earlier writer of a register comes from a
+//              warp-wide writer bitmask in shared memory (atomicOr + clz), across chunks and
+//              windows from the carried table.
+//   k_trace    per candidate: bounded backward def-use trace (R7) by pointer chasing
+//              through the per-instruction pointer-operand RD; store roots (R8); key-group
+//              statistics of global loads (R3).
+//   k_rules    per candidate: the seven rules -> flag mask and site count.
+//   scans      site offsets and chain-pool offsets.
+//   k_write    per candidate: gs_site records in (kernel, idx, rule) order + chains.
+#include <cuda_runtime.h>
+
+#include <climits>
+#include <cstdio>
+
+#include "ctx.h"
+
+namespace gs {
+namespace {
+
+constexpr uint64_t kEmpty = ~0ull;
+constexpr int kWarps = 8;  // warps (windows) per CTA in the window kernels
+
+__device__ __forceinline__ Rec ld_rec(const Rec* r, uint64_t i) {
+  uint4 v = __ldg(reinterpret_cast<const uint4*>(r) + i);
+  Rec o;
+  o.w0 = v.x; o.w1 = v.y; o.w2 = v.z; o.w3 = (int32_t)v.w;
+  return o;
+}
+__device__ __forceinline__ uint32_t reg_cap(uint32_t dst) { return dst < 256 ? 254u : 318u; }
+
+__device__ __forceinline__ uint32_t hash64(unsigned long long k) {
+  k ^= k >> 33; k *= 0xff51afd7ed558ccdull; k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull; k ^= k >> 33;
+  return (uint32_t)k;
+}
+__device__ uint32_t hinsert(unsigned long long* keys, uint32_t cap, unsigned long long k) {
+  uint32_t s = hash64(k) & (cap - 1);
+  for (;;) {
+    unsigned long long prev = atomicCAS(keys + s, kEmpty, k);
+    if (prev == kEmpty || prev == k) return s;
+    s = (s + 1) & (cap - 1);
+  }
+}
+__device__ bool hcontains(const unsigned long long* keys, uint32_t cap, unsigned long long k) {
+  uint32_t s = hash64(k) & (cap - 1);
+  for (;;) {
+    unsigned long long v = keys[s];
+    if (v == k) return true;
+    if (v == kEmpty) return false;
+    s = (s + 1) & (cap - 1);
+  }
+}
+__device__ __forceinline__ unsigned long long root_key(uint32_t kernel, uint32_t tk, uint32_t tv) {
+  return ((unsigned long long)kernel << 36) | ((unsigned long long)tk << 32) | tv;
+}
+// key of a global load's group (R3): (base register, RD(i, base)); ENTRY / no-base keys are per kernel
+__device__ __forceinline__ unsigned long long group_key(uint32_t base, uint32_t base_rd, uint32_t kernel) {
+  if (!reg_live(base)) return (2ull << 62) | ((unsigned long long)kernel << 10) | (base & 1023u);
+  if (base_rd == 0) return (1ull << 62) | ((unsigned long long)kernel << 10) | base;
+  return ((unsigned long long)base_rd << 10) | base;
+}
+
+// ------------------------------------------------------------------------------------------ A
+__global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+                                                         const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
+                                                         uint32_t* __restrict__ tab, int32_t* ldiff, int32_t* wsum,
+                                                         uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst) {
+  __shared__ uint32_t last[kWarps][kNumRegs];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t w = w0 + blockIdx.x * kWarps + warp;
+  if (w >= w0 + nw) return;
+  for (int r = lane; r < kNumRegs; r += 32) last[warp][r] = 0;
+  __syncwarp();
+  const WDesc W = wd[w];
+  const KDesc K = kd[W.kernel];
+  uint32_t n_gatom = 0, n_satom = 0, n_conv = 0, n_vec = 0;
+  for (uint32_t b = 0; b < W.len; b += 32) {
+    const uint32_t i = b + lane;
+    const bool valid = i < W.len;
+    const uint64_t g = (uint64_t)W.start + i;
+    Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
+    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r);
+    if (valid && dw && reg_live(dst)) {
+      const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
+      const uint32_t cap = reg_cap(dst);
+      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicMax(&last[warp][dst + q], v);
+    }
+    if (valid && op == OP_LDG) narith[g] = 0;
+    if (valid && op == OP_BRA && (r_flags(r) & F_BRA_OK)) {
+      const uint32_t t = (uint32_t)r_imm(r);           // loop [t, b] in kernel-local indices
+      atomicAdd(ldiff + K.first + t, 1);
+      atomicAdd(wsum + K.win0 + t / kWin, 1);
+      atomicAdd(wev + K.win0 + t / kWin, 1u);
+      const uint32_t b1 = (uint32_t)(g - K.first) + 1;
+      if (b1 < K.n) {
+        atomicAdd(ldiff + K.first + b1, -1);
+        atomicAdd(wsum + K.win0 + b1 / kWin, -1);
+        atomicAdd(wev + K.win0 + b1 / kWin, 1u);
+      }
+    }
+    if (valid) {
+      n_gatom += (cls & C_GATOM) ? 1 : 0;
+      n_satom += (cls & C_SATOM) ? 1 : 0;
+      n_conv += (cls & C_CONV) ? 1 : 0;
+      n_vec += (op == OP_LDG && (r_flags(r) & F_HASMEM) && (r_aw(r) == AW_64 || r_aw(r) == AW_128)) ? 1 : 0;
+    }
+  }
+  for (int o = 16; o; o >>= 1) {
+    n_gatom += __shfl_xor_sync(0xffffffffu, n_gatom, o);
+    n_satom += __shfl_xor_sync(0xffffffffu, n_satom, o);
+    n_conv += __shfl_xor_sync(0xffffffffu, n_conv, o);
+    n_vec += __shfl_xor_sync(0xffffffffu, n_vec, o);
+  }
+  if (lane == 0) {
+    if (n_gatom) atomicAdd(&kst[W.kernel].n_gatom, n_gatom);
+    if (n_satom) atomicAdd(&kst[W.kernel].n_satom, n_satom);
+    if (n_conv) atomicAdd(&kst[W.kernel].n_conv, n_conv);
+    if (n_vec) atomicAdd(&kst[W.kernel].n_vec_already, n_vec);
+  }
+  __syncwarp();
+  for (int r = lane; r < kNumRegs; r += 32) tab[(uint64_t)w * kNumRegs + r] = last[warp][r];
+}
+
+// ------------------------------------------------------------------------------------------ B
+__global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, uint32_t* tab,
+                        const int32_t* __restrict__ wsum, int32_t* wloop) {
+  const uint32_t k = kb + blockIdx.x;
+  if (k >= ke) return;
+  const KDesc K = kd[k];
+  const uint32_t nwk = (K.n + kWin - 1) / kWin;
+  for (int r = threadIdx.x; r <= kNumRegs; r += blockDim.x) {
+    if (r < kNumRegs) {
+      uint32_t state = 0;
+      for (uint32_t j = 0; j < nwk; j++) {
+        uint32_t* p = tab + (uint64_t)(K.win0 + j) * kNumRegs + r;
+        const uint32_t s = *p;
+        *p = state;
+        if (s) state = s;
+      }
+    } else {
+      int32_t acc = 0;
+      for (uint32_t j = 0; j < nwk; j++) {
+        wloop[K.win0 + j] = acc;
+        acc += wsum[K.win0 + j];
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------ C
+__global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+                                                         uint32_t w0, uint32_t nw, const uint32_t* __restrict__ tab,
+                                                         int32_t* ldiff, const int32_t* __restrict__ wloop,
+                                                         const uint32_t* __restrict__ wev,
+                                                         const uint32_t* __restrict__ cbase, uint64_t c0,
+                                                         uint32_t* __restrict__ ptrrd, uint32_t* narith, CandArrays ca) {
+  __shared__ uint32_t tabS[kWarps][kNumRegs];
+  __shared__ uint32_t cm[kWarps][kNumRegs];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t w = w0 + blockIdx.x * kWarps + warp;
+  if (w >= w0 + nw) return;
+  for (int r = lane; r < kNumRegs; r += 32) {
+    tabS[warp][r] = tab[(uint64_t)w * kNumRegs + r];
+    cm[warp][r] = 0;
+  }
+  __syncwarp();
+  const WDesc W = wd[w];
+  int32_t lcarry = wloop[w];
+  const bool has_ev = wev[w] != 0;
+  uint64_t cb = (uint64_t)cbase[w] - c0;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t gt = ~((2u << lane) - 1u);
+  uint32_t* T = tabS[warp];
+  uint32_t* M = cm[warp];
+  for (uint32_t b = 0; b < W.len; b += 32) {
+    const uint32_t i = b + lane;
+    const bool valid = i < W.len;
+    const uint64_t g = (uint64_t)W.start + i;
+    const uint64_t gbase = (uint64_t)W.start + b;
+    Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
+    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
+    const bool writes = valid && dw && reg_live(dst);
+    const uint32_t cap = reg_cap(dst);
+    if (writes)
+      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicOr(&M[dst + q], 1u << lane);
+    const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
+    __syncwarp();
+    // RD value: ((def + 1) << 1) | def_is_global_load, or 0 for ENTRY
+    auto RD = [&](uint32_t reg) -> uint32_t {
+      const uint32_t m = M[reg] & lt;
+      if (m) {
+        const uint32_t j = 31u - __clz(m);
+        return (uint32_t)((gbase + j + 1) << 1) | ((ldgmask >> j) & 1u);
+      }
+      return T[reg];
+    };
+    // loop depth: inclusive prefix of the event differences (R13)
+    int32_t ev = 0;
+    if (has_ev && valid) {
+      ev = ldiff[g];
+      if (ev) ldiff[g] = 0;  // keep the difference array zero for the next call
+    }
+    int32_t pre = ev;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t x = __shfl_up_sync(0xffffffffu, pre, o);
+      if (lane >= o) pre += x;
+    }
+    const int32_t depth = lcarry + pre;
+    lcarry += __shfl_sync(0xffffffffu, pre, 31);
+    if (valid && r_pk(r) == PK_REG) ptrrd[g] = RD(r_ptr(r)) >> 1;
+    const bool iscand = valid && (cls & (C_TRACED | C_CONV));
+    const uint32_t cmask = __ballot_sync(0xffffffffu, iscand);
+    if (iscand) {
+      const uint64_t c = cb + __popc(cmask & lt);
+      ca.idx[c] = (uint32_t)g;
+      ca.kernel[c] = W.kernel;
+      const uint32_t base = r_s0(r);
+      ca.base_rd[c] = ((fl & F_HASMEM) && reg_live(base)) ? (RD(base) >> 1) : 0xffffffffu;
+      const uint32_t data = r_s1(r);
+      ca.data_rd[c] = (op == OP_STL && reg_live(data)) ? (RD(data) >> 1) : 0xffffffffu;
+      ca.ld[c] = (uint8_t)(depth > 255 ? 255 : (depth < 0 ? 0 : depth));
+    }
+    cb += __popc(cmask);
+    if (valid && (cls & C_ARITH)) {  // n_arith (R29): count each defining load once
+      uint32_t defs[4];
+      int nd = 0;
+      const uint32_t src[4] = {r_s0(r), r_s1(r), r_s2(r), r_s3(r)};
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        if (!reg_live(src[q])) continue;
+        const uint32_t v = RD(src[q]);
+        if (!(v & 1u)) continue;
+        const uint32_t d = (v >> 1) - 1u;
+        bool dup = false;
+        for (int t = 0; t < nd; t++) dup |= defs[t] == d;
+        if (!dup) defs[nd++] = d;
+      }
+      for (int t = 0; t < nd; t++) atomicAdd(narith + defs[t], 1u);
+    }
+    __syncwarp();
+    if (writes) {
+      const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
+      for (uint32_t q = 0; q < dw && dst + q <= cap; q++)
+        if ((M[dst + q] & gt) == 0) T[dst + q] = v;
+    }
+    __syncwarp();
+    if (writes)
+      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) M[dst + q] = 0;
+    __syncwarp();
+  }
+}
+
+// ------------------------------------------------------------------------------------------ D
+struct TraceOut {
+  uint32_t tk, tv, depth;
+};
+
+// Bounded backward trace (R7). `emit` receives each chain element (kernel-local).
+template <typename Emit>
+__device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restrict__ ptrrd, const KDesc& K,
+                          uint32_t base, uint32_t base_rd, uint32_t D, Emit emit) {
+  TraceOut o{GS_T_IMM, 0, 0};
+  if (!reg_live(base) || base_rd == 0xffffffffu) return o;
+  uint32_t r = base, v = base_rd, depth = 0;
+  for (;;) {
+    if (depth == D) { o.tk = GS_T_TRUNC; break; }
+    if (v == 0) { o.tk = GS_T_ENTRY; o.tv = r; break; }
+    const uint32_t j = v - 1;
+    depth++;
+    emit(j - K.first);
+    const Rec rj = ld_rec(rec, j);
+    const uint32_t cj = op_class(r_op(rj));
+    if (cj & C_CONSTLOAD) {
+      const int32_t off = r_imm(rj) + 4 * (int32_t)(r - r_dst(rj));
+      const uint32_t bank = r_cbank(rj);
+      if (bank == 0 && off >= (int32_t)K.param_base) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
+      break;
+    }
+    if (cj & C_SREG) { o.tk = GS_T_SREG; o.tv = j - K.first; break; }
+    if (cj & C_MEMLOAD) { o.tk = GS_T_MEMORY; o.tv = j - K.first; break; }
+    const uint32_t pk = r_pk(rj);
+    if (pk == PK_CONST) {
+      const int32_t off = r_imm(rj);
+      const uint32_t bank = r_cbank(rj);
+      if (bank == 0 && off >= (int32_t)K.param_base) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
+      break;
+    }
+    if (pk != PK_REG) { o.tk = GS_T_IMM; break; }
+    r = r_ptr(rj);
+    v = ptrrd[j];
+  }
+  o.depth = depth;
+  return o;
+}
+
+__global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
+                        uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, OffsetSet os, RootSet rs,
+                        gs_kernel_stats* kst) {
+  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (c >= nc) return;
+  const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
+  const Rec ri = ld_rec(rec, g);
+  const uint32_t op = r_op(ri), cls = op_class(op);
+  if (!(cls & C_TRACED) || !(r_flags(ri) & F_HASMEM)) {
+    ca.tk[c] = GS_T_NONE; ca.tv[c] = 0; ca.depth[c] = 0; ca.grp[c] = 0xffffffffu;
+    return;
+  }
+  const KDesc K = kd[kernel];
+  const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
+  if (op == OP_LDG) {  // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max
+    const uint32_t slot = hinsert(gt.key, gt.cap, group_key(base, brd, kernel));
+    ca.grp[c] = slot;
+    atomicAdd(gt.nload + slot, 1u);
+    const int32_t off = r_imm(ri);
+    const bool is32 = r_aw(ri) == AW_32;
+    const uint32_t os_slot = hinsert(os.key, os.cap, ((unsigned long long)slot << 32) | (uint32_t)off);
+    const uint32_t prev = atomicOr(os.flags + os_slot, is32 ? 3u : 2u);
+    if (!(prev & 2u)) atomicAdd(gt.nall + slot, 1u);
+    if (is32 && !(prev & 1u)) {
+      atomicAdd(gt.n32 + slot, 1u);
+      atomicMin(gt.mn + slot, off);
+      atomicMax(gt.mx + slot, off);
+      atomicOr(gt.or3 + slot, (uint32_t)off & 3u);
+      atomicAnd(gt.and3 + slot, (uint32_t)off & 3u);
+    }
+  } else {
+    ca.grp[c] = 0xffffffffu;
+  }
+  const TraceOut t = chase(rec, ptrrd, K, base, brd, D, [](uint32_t) {});
+  ca.tk[c] = (uint8_t)t.tk;
+  ca.tv[c] = t.tv;
+  ca.depth[c] = (uint8_t)t.depth;
+  if (cls & C_STORE) {  // store roots (R8, R27)
+    if (t.tk == GS_T_PARAM || t.tk == GS_T_ENTRY) hinsert(rs.key, rs.cap, root_key(kernel, t.tk, t.tv));
+    else atomicAdd(&kst[kernel].n_unresolved_stores, 1u);
+  }
+}
+
+// ------------------------------------------------------------------------------------------ E
+struct RuleCfg {
+  uint32_t TA, TL;
+};
+
+__device__ uint32_t eval_rules(const Rec& ri, uint64_t c, const CandArrays& ca, const GroupTable& gt,
+                               const RootSet& rs, const uint32_t* narith, RuleCfg rc) {
+  const uint32_t op = r_op(ri), cls = op_class(op), fl = r_flags(ri);
+  uint32_t f = 0;
+  if (!(fl & F_HASMEM) && !(cls & C_CONV)) return 0;
+  if (op == OP_LDG && (fl & F_HASMEM)) {
+    const uint32_t s = ca.grp[c];
+    const uint32_t n32 = gt.n32[s], nall = gt.nall[s], nload = gt.nload[s];
+    if (r_aw(ri) == AW_32 && n32 >= 2) f |= 1u << GS_VEC;                                // O6
+    if (narith[ca.idx[c]] >= rc.TA && (nload >= rc.TL || ca.ld[c] >= 1)) f |= 1u << GS_SHMEM;  // O8
+    const uint32_t tk = ca.tk[c];
+    const bool ro = !(fl & F_CONSTANT) && (tk == GS_T_PARAM || tk == GS_T_ENTRY) &&
+                    !hcontains(rs.key, rs.cap, root_key(ca.kernel[c], tk, ca.tv[c]));   // O10
+    if (ro) f |= 1u << GS_RO;
+    if (ro && nall >= 2) f |= 1u << GS_TEX;                                              // O11
+  }
+  if ((op == OP_STL || op == OP_LDL) && (fl & F_HASMEM)) f |= 1u << GS_SPILL;          // O7
+  if ((cls & C_GATOM) && (fl & F_HASMEM)) f |= 1u << GS_GATOM;                         // O9
+  if (cls & C_CONV) f |= 1u << GS_CONV;                                                // O12
+  return f;
+}
+
+__global__ void k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca, GroupTable gt, RootSet rs,
+                        const uint32_t* __restrict__ narith, RuleCfg rc) {
+  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (c >= nc) return;
+  const Rec ri = ld_rec(rec, ca.idx[c]);
+  const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc);
+  ca.flags[c] = (uint8_t)f;
+  ca.nsite[c] = __popc(f);
+  ca.soff[c] = f ? ca.depth[c] : 0;  // chain length (scanned into choff)
+}
+
+__global__ void k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
+                        uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, const uint32_t* __restrict__ narith,
+                        const uint32_t* __restrict__ site_off, gs_site* __restrict__ sites,
+                        uint32_t* __restrict__ chain) {
+  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (c >= nc) return;
+  const uint32_t f = ca.flags[c];
+  if (!f) return;
+  const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
+  const KDesc K = kd[kernel];
+  const Rec ri = ld_rec(rec, g);
+  const unsigned long long coff = ca.choff[c];
+  // chain: re-chase and store kernel-local indices
+  uint32_t n = 0;
+  if (ca.depth[c])
+    chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, [&](uint32_t j) { chain[coff + n++] = j; });
+  uint32_t so = site_off[c];
+  for (uint32_t rule = 0; rule < 7; rule++) {
+    if (!((f >> rule) & 1u)) continue;
+    gs_site s;
+    s.kernel = kernel;
+    s.idx = g - K.first;
+    s.rule = (uint8_t)rule;
+    s.depth = ca.depth[c];
+    s.term_kind = ca.tk[c];
+    s.loop_depth = ca.ld[c];
+    s.term_value = ca.tv[c];
+    s.chain_off = (uint32_t)coff;
+    s.a0 = s.a1 = s.a2 = 0;
+    if (rule == GS_VEC) {
+      const uint32_t sl = ca.grp[c];
+      const uint32_t n32 = gt.n32[sl];
+      const int32_t mn = gt.mn[sl], mx = gt.mx[sl];
+      const bool contig = (int64_t)mx - (int64_t)mn == 4ll * ((int64_t)n32 - 1) && gt.or3[sl] == gt.and3[sl];
+      s.a0 = (int32_t)(n32 | (contig ? (1u << 30) : 0u));
+      s.a1 = mn;
+      s.a2 = mx;
+    } else if (rule == GS_SPILL) {
+      if (r_op(ri) == OP_STL) {
+        s.a0 = (int32_t)r_s1(ri);
+        const uint32_t rd = ca.data_rd[c];
+        s.a1 = rd == 0xffffffffu ? -2 : (rd == 0 ? -1 : (int32_t)(rd - 1 - K.first));
+      } else {
+        s.a0 = (int32_t)r_dst(ri);
+        s.a1 = -2;
+      }
+    } else if (rule == GS_SHMEM) {
+      s.a0 = (int32_t)gt.nload[ca.grp[c]];
+      s.a1 = (int32_t)narith[g];
+    } else if (rule == GS_TEX) {
+      s.a0 = (int32_t)gt.nall[ca.grp[c]];
+    }
+    if (rule == GS_CONV) { s.depth = 0; s.term_kind = GS_T_NONE; s.term_value = 0; }
+    sites[so++] = s;
+  }
+}
+
+__global__ void k_init_groups(GroupTable gt, OffsetSet os, RootSet rs) {
+  const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (i < gt.cap) {
+    gt.key[i] = kEmpty;
+    gt.nload[i] = gt.n32[i] = gt.nall[i] = gt.or3[i] = 0;
+    gt.and3[i] = 3u;
+    gt.mn[i] = INT_MAX;
+    gt.mx[i] = INT_MIN;
+  }
+  if (i < os.cap) { os.key[i] = kEmpty; os.flags[i] = 0; }
+  if (i < rs.cap) rs.key[i] = kEmpty;
+}
+
+uint32_t pow2_at_least(uint64_t n) {
+  uint64_t c = 16;
+  while (c < n) c <<= 1;
+  return (uint32_t)c;
+}
+
+}  // namespace
+
+void detect_free(gs_ctx* c) {
+  void* ps[] = {c->d_tab, c->d_ldiff, c->d_wsum, c->d_wloop, c->d_wev, c->d_ptrrd, c->d_narith,
+                c->cand.idx, c->cand.kernel, c->cand.base_rd, c->cand.data_rd, c->cand.tv, c->cand.grp,
+                c->cand.nsite, c->cand.soff, c->cand.ld, c->cand.tk, c->cand.depth, c->cand.flags,
+                c->cand.choff, c->grp.key, c->grp.nload, c->grp.n32, c->grp.nall, c->grp.or3, c->grp.and3,
+                c->grp.mn, c->grp.mx, c->oset.key, c->oset.flags, c->roots.key, c->d_kstats, c->d_sites,
+                c->d_chain, c->d_scan_tmp};
+  for (void* p : ps)
+    if (p) cudaFree(p);
+  c->d_tab = nullptr; c->d_ldiff = nullptr; c->d_wsum = nullptr; c->d_wloop = nullptr; c->d_wev = nullptr;
+  c->d_ptrrd = nullptr; c->d_narith = nullptr;
+  c->cand = CandArrays();
+  c->grp = GroupTable();
+  c->oset = OffsetSet();
+  c->roots = RootSet();
+  c->d_kstats = nullptr;
+  c->d_sites = nullptr; c->sites_cap = 0; c->n_sites = 0;
+  c->d_chain = nullptr; c->chain_cap = 0; c->n_chain = 0;
+  c->d_scan_tmp = nullptr; c->scan_tmp_bytes = 0;
+  c->detected = false;
+}
+
+gs_status detect_alloc(gs_ctx* c) {
+  const uint64_t P = c->n_instr, NW = c->n_win, NC = c->n_cand ? c->n_cand : 1;
+#define A(ptr, bytes) GS_CUDA(c, cudaMalloc((void**)&(ptr), (bytes) ? (bytes) : 16))
+  A(c->d_tab, NW * kNumRegs * 4);
+  A(c->d_ldiff, P * 4);
+  GS_CUDA(c, cudaMemsetAsync(c->d_ldiff, 0, P * 4, c->stream));
+  A(c->d_wsum, NW * 4);
+  A(c->d_wloop, NW * 4);
+  A(c->d_wev, NW * 4);
+  A(c->d_ptrrd, P * 4);
+  A(c->d_narith, P * 4);
+  A(c->cand.idx, NC * 4); A(c->cand.kernel, NC * 4); A(c->cand.base_rd, NC * 4); A(c->cand.data_rd, NC * 4);
+  A(c->cand.tv, NC * 4); A(c->cand.grp, NC * 4); A(c->cand.nsite, NC * 4); A(c->cand.soff, NC * 4 + 4);
+  A(c->cand.ld, NC); A(c->cand.tk, NC); A(c->cand.depth, NC); A(c->cand.flags, NC);
+  A(c->cand.choff, NC * 8 + 16);
+  c->grp.cap = pow2_at_least(2 * c->n_ldg + 16);
+  A(c->grp.key, (uint64_t)c->grp.cap * 8);
+  A(c->grp.nload, (uint64_t)c->grp.cap * 4); A(c->grp.n32, (uint64_t)c->grp.cap * 4);
+  A(c->grp.nall, (uint64_t)c->grp.cap * 4); A(c->grp.or3, (uint64_t)c->grp.cap * 4);
+  A(c->grp.and3, (uint64_t)c->grp.cap * 4); A(c->grp.mn, (uint64_t)c->grp.cap * 4);
+  A(c->grp.mx, (uint64_t)c->grp.cap * 4);
+  c->oset.cap = pow2_at_least(2 * c->n_ldg + 16);
+  A(c->oset.key, (uint64_t)c->oset.cap * 8);
+  A(c->oset.flags, (uint64_t)c->oset.cap * 4);
+  c->roots.cap = pow2_at_least(2 * c->n_store + 16);
+  A(c->roots.key, (uint64_t)c->roots.cap * 8);
+  A(c->d_kstats, (uint64_t)(c->n_kernels ? c->n_kernels : 1) * sizeof(gs_kernel_stats));
+#undef A
+  return GS_OK;
+}
+
+gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
+  cudaStream_t st = c->stream;
+  const uint32_t w0 = kb < c->n_kernels ? c->kd_h[kb].win0 : c->n_win;
+  const uint32_t w1 = ke < c->n_kernels ? c->kd_h[ke].win0 : c->n_win;
+  const uint32_t nw = w1 - w0;
+  const uint64_t c0 = c->cbase_h[w0], c1 = c->cbase_h[w1], nc = c1 - c0;
+  const uint32_t D = c->cfg.trace_depth;
+  c->detected = false;
+  GS_CUDA(c, cudaMemsetAsync(c->d_kstats, 0, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats), st));
+  if (nw) {
+    GS_CUDA(c, cudaMemsetAsync(c->d_wsum + w0, 0, (uint64_t)nw * 4, st));
+    GS_CUDA(c, cudaMemsetAsync(c->d_wev + w0, 0, (uint64_t)nw * 4, st));
+    const uint32_t grid = (nw + kWarps - 1) / kWarps;
+    k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
+                                           c->d_wev, c->d_narith, c->d_kstats);
+    GS_CUDA(c, cudaGetLastError());
+    k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop);
+    GS_CUDA(c, cudaGetLastError());
+    // candidate arrays are indexed relative to c0
+    k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
+                                           c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand);
+    GS_CUDA(c, cudaGetLastError());
+  }
+  unsigned long long* d_tot = c->cand.choff + nc;  // two totals after the offsets
+  unsigned long long tot[2] = {0, 0};
+  if (nc) {
+    const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
+    k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots);
+    GS_CUDA(c, cudaGetLastError());
+    const uint32_t gridc = (uint32_t)((nc + 255) / 256);
+    k_trace<<<gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
+                                   c->d_kstats);
+    GS_CUDA(c, cudaGetLastError());
+    k_rules<<<gridc, 256, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
+                                   RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads});
+    GS_CUDA(c, cudaGetLastError());
+    // chain offsets (u64) from chain lengths stored in soff, then site offsets in place of soff
+    gs_status s = scan_u32_to_u64(c, c->cand.soff, c->cand.choff, nc, d_tot);
+    if (s != GS_OK) return s;
+    s = scan_u32(c, c->cand.nsite, c->cand.soff, nc, d_tot + 1);
+    if (s != GS_OK) return s;
+    GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
+    GS_CUDA(c, cudaStreamSynchronize(st));
+  }
+  const uint64_t ns = tot[1], nch = tot[0];
+  if (nch > 0xffffffffull) return fail(c, GS_E_RANGE, "chain pool exceeds 2^32 entries");
+  GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
+  GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
+  if (nc && ns) {
+    k_write<<<(uint32_t)((nc + 255) / 256), 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
+                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain);
+    GS_CUDA(c, cudaGetLastError());
+  }
+  c->kstats_h.assign(c->n_kernels, gs_kernel_stats{});
+  if (c->n_kernels)
+    GS_CUDA(c, cudaMemcpyAsync(c->kstats_h.data(), c->d_kstats, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats),
+                               cudaMemcpyDeviceToHost, st));
+  GS_CUDA(c, cudaStreamSynchronize(st));
+  c->n_sites = ns;
+  c->n_chain = nch;
+  c->det_kb = kb; c->det_ke = ke; c->det_c0 = c0; c->det_c1 = c1;
+  c->detected = true;
+  if (n_sites) *n_sites = ns;
+  return GS_OK;
+}
+
+}  // namespace gs

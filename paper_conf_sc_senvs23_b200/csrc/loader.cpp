@@ -1,0 +1,495 @@
+// loader.cpp — SASS text -> packed 16-byte records (§2.1).
+//
+// Product code (host side of gs_load_sass). Written independently of oracle/gs_oracle.cpp from the
+// readings in DESIGN.md §3 (R1, R2, R6, R7, R23-R28). Kernels are parsed in parallel: a first
+// sequential pass only finds "Function :" headers and arch lines; each kernel's lines are then
+// tokenised by a worker thread into records.
+#include <algorithm>
+#include <atomic>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "loader.h"
+
+namespace gs {
+namespace {
+
+struct Sv {  // non-owning text span
+  const char* p = nullptr;
+  size_t n = 0;
+  bool eq(const char* s) const { size_t m = strlen(s); return m == n && memcmp(p, s, n) == 0; }
+  char operator[](size_t i) const { return p[i]; }
+};
+
+inline bool is_ws(char c) { return c == ' ' || c == '\t' || c == '\r' || c == '\n'; }
+inline Sv trim(Sv s) {
+  while (s.n && is_ws(s.p[0])) { s.p++; s.n--; }
+  while (s.n && is_ws(s.p[s.n - 1])) s.n--;
+  return s;
+}
+inline bool contains(Sv s, const char* needle, size_t* at = nullptr) {
+  size_t m = strlen(needle);
+  if (m > s.n) return false;
+  for (size_t i = 0; i + m <= s.n; i++)
+    if (memcmp(s.p + i, needle, m) == 0) { if (at) *at = i; return true; }
+  return false;
+}
+inline bool starts(Sv s, const char* pre) { size_t m = strlen(pre); return s.n >= m && memcmp(s.p, pre, m) == 0; }
+inline int hexv(char c) {
+  if (c >= '0' && c <= '9') return c - '0';
+  if (c >= 'a' && c <= 'f') return c - 'a' + 10;
+  if (c >= 'A' && c <= 'F') return c - 'A' + 10;
+  return -1;
+}
+
+// integer literal: optional sign, then 0x-hex or decimal, nothing else
+bool to_int(Sv s, long long* v) {
+  s = trim(s);
+  bool neg = false;
+  if (s.n && (s[0] == '-' || s[0] == '+')) { neg = s[0] == '-'; s.p++; s.n--; }
+  if (!s.n) return false;
+  long long x = 0;
+  if (s.n > 2 && s[0] == '0' && (s[1] == 'x' || s[1] == 'X')) {
+    for (size_t i = 2; i < s.n; i++) { int h = hexv(s[i]); if (h < 0) return false; x = x * 16 + h; }
+  } else {
+    for (size_t i = 0; i < s.n; i++) { if (s[i] < '0' || s[i] > '9') return false; x = x * 10 + (s[i] - '0'); }
+  }
+  *v = neg ? -x : x;
+  return true;
+}
+
+Sv unprefix(Sv s) {
+  while (s.n && (s[0] == '-' || s[0] == '!' || s[0] == '~' || s[0] == '|')) { s.p++; s.n--; }
+  return s;
+}
+
+// register token -> id (R6): Rn (n<=254) RZ URn (n<=62) URZ; suffix from the first '.' ignored
+int reg_id(Sv s) {
+  size_t cut = s.n;
+  for (size_t i = 0; i < s.n; i++) if (s[i] == '.') { cut = i; break; }
+  s.n = cut;
+  while (s.n && s[s.n - 1] == '|') s.n--;
+  bool ur = false;
+  size_t i = 0;
+  if (s.n >= 2 && s[0] == 'U' && s[1] == 'R') { ur = true; i = 2; }
+  else if (s.n >= 1 && s[0] == 'R') i = 1;
+  else return -1;
+  size_t m = s.n - i;
+  if (m == 1 && s[i] == 'Z') return ur ? kURZ : kRZ;
+  if (m == 0 || m > 3) return -1;
+  int v = 0;
+  for (size_t q = i; q < s.n; q++) { if (s[q] < '0' || s[q] > '9') return -1; v = v * 10 + (s[q] - '0'); }
+  if (ur) return v <= 62 ? 256 + v : -1;
+  return v <= 254 ? v : -1;
+}
+
+bool is_pred(Sv s) {
+  size_t i;
+  if (s.n >= 2 && s[0] == 'U' && s[1] == 'P') i = 2;
+  else if (s.n >= 1 && s[0] == 'P') i = 1;
+  else return false;
+  return s.n == i + 1 && (s[i] == 'T' || (s[i] >= '0' && s[i] <= '7'));
+}
+
+enum Kind { T_REG, T_PRED, T_CREF, T_MEM, T_MISC };
+struct Operand {
+  Kind k = T_MISC;
+  int reg = -1;              // T_REG
+  int bank = 0;              // T_CREF
+  long long imm = 0;         // T_CREF offset, T_MEM offset
+  int base = -1;             // T_MEM base register
+  int regs[8];               // all registers inside (brackets too), in order
+  int nregs = 0;
+  void add(int r) { if (nregs < 8) regs[nregs++] = r; }
+};
+
+// bracket body "R4.64+-0x10": registers (first one = base if wanted) and immediate sum
+void scan_bracket(Sv b, Operand* o, bool want_base, long long* sum) {
+  size_t s = 0;
+  while (s <= b.n) {
+    size_t e = s;
+    while (e < b.n && b[e] != '+') e++;
+    Sv term = trim(Sv{b.p + s, e - s});
+    if (term.n) {
+      int r = reg_id(unprefix(term));
+      long long v;
+      if (r >= 0) {
+        o->add(r);
+        if (want_base && o->base < 0) o->base = r;
+      } else if (to_int(term, &v)) {
+        *sum += v;
+      }
+    }
+    s = e + 1;
+  }
+}
+
+Operand classify(Sv raw) {
+  Operand o;
+  Sv t = trim(raw);
+  Sv u = unprefix(t);
+  if (u.n > 2 && u[0] == 'c' && u[1] == '[') {
+    o.k = T_CREF;
+    size_t a = 2;
+    while (a < u.n && u[a] != ']') a++;
+    long long bank = 0;
+    to_int(Sv{u.p + 2, a - 2}, &bank);
+    o.bank = (int)bank;
+    size_t b0 = a;
+    while (b0 < u.n && u[b0] != '[') b0++;
+    if (b0 < u.n) {
+      size_t b1 = b0;
+      while (b1 < u.n && u[b1] != ']') b1++;
+      if (b1 < u.n) scan_bracket(Sv{u.p + b0 + 1, b1 - b0 - 1}, &o, false, &o.imm);
+    }
+    return o;
+  }
+  size_t lb = u.n;
+  for (size_t i = 0; i < u.n; i++) if (u[i] == '[') { lb = i; }
+  if (lb < u.n) {  // memory operand; lb = last '['
+    o.k = T_MEM;
+    size_t i = 0;
+    while (i < u.n) {
+      if (u[i] != '[') { i++; continue; }
+      size_t c = i;
+      while (c < u.n && u[c] != ']') c++;
+      long long dummy = 0;
+      if (i == lb) scan_bracket(Sv{u.p + i + 1, c - i - 1}, &o, true, &o.imm);
+      else scan_bracket(Sv{u.p + i + 1, c - i - 1}, &o, false, &dummy);
+      i = c + 1;
+    }
+    return o;
+  }
+  int r = reg_id(u);
+  if (r >= 0) { o.k = T_REG; o.reg = r; o.add(r); return o; }
+  if (is_pred(u)) { o.k = T_PRED; return o; }
+  o.k = T_MISC;  // immediates, floats, SR_*, B0, PR, ...
+  return o;
+}
+
+struct OpName { const char* s; uint8_t id; };
+const OpName kOps[] = {
+    {"LDG", OP_LDG}, {"LDL", OP_LDL}, {"STL", OP_STL}, {"STG", OP_STG}, {"ST", OP_ST}, {"LD", OP_LD},
+    {"LDS", OP_LDS}, {"STS", OP_STS}, {"LDSM", OP_LDSM}, {"ATOM", OP_ATOM}, {"ATOMG", OP_ATOMG},
+    {"ATOMS", OP_ATOMS}, {"RED", OP_RED}, {"REDG", OP_REDG}, {"SUST", OP_SUST}, {"SULD", OP_SULD},
+    {"SUATOM", OP_SUATOM}, {"TLD", OP_TLD}, {"TLD4", OP_TLD4}, {"TLDS", OP_TLDS}, {"TEX", OP_TEX},
+    {"TMML", OP_TMML}, {"TXD", OP_TXD}, {"TXQ", OP_TXQ}, {"LDTM", OP_LDTM}, {"LDC", OP_LDC},
+    {"LDCU", OP_LDCU}, {"ULDC", OP_ULDC}, {"S2R", OP_S2R}, {"S2UR", OP_S2UR}, {"CS2R", OP_CS2R},
+    {"BRA", OP_BRA}, {"F2F", OP_F2F}, {"F2I", OP_F2I}, {"I2F", OP_I2F}, {"I2I", OP_I2I},
+    {"I2FP", OP_I2FP}, {"F2IP", OP_F2IP}, {"F2FP", OP_F2FP}, {"FADD", OP_FADD}, {"FMUL", OP_FMUL},
+    {"FFMA", OP_FFMA}, {"FMNMX", OP_FMNMX}, {"DADD", OP_DADD}, {"DMUL", OP_DMUL}, {"DFMA", OP_DFMA},
+    {"HADD2", OP_HADD2}, {"HMUL2", OP_HMUL2}, {"HFMA2", OP_HFMA2}, {"MUFU", OP_MUFU},
+    {"IADD3", OP_IADD3}, {"VIADD", OP_VIADD}, {"IMAD", OP_IMAD}, {"IMUL", OP_IMUL},
+    {"IMNMX", OP_IMNMX}, {"VIMNMX", OP_VIMNMX}, {"IABS", OP_IABS}, {"LEA", OP_LEA},
+    {"ULEA", OP_ULEA}, {"UIADD3", OP_UIADD3}, {"UIMAD", OP_UIMAD}, {"HMMA", OP_HMMA},
+    {"DMNMX", OP_DMNMX}, {"FCHK", OP_FCHK},
+};
+
+uint8_t op_lookup(Sv m) {
+  for (const auto& o : kOps)
+    if (m.eq(o.s)) return o.id;
+  return OP_OTHER;
+}
+
+struct Line {
+  const char* p;
+  size_t n;
+  long lineno;
+};
+
+// One instruction -> record. Returns false with msg on a malformed line.
+bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg) {
+  body = trim(body);
+  if (body.n && body[0] == '@') {  // guard predicate
+    size_t i = 0;
+    while (i < body.n && !is_ws(body[i])) i++;
+    body = trim(Sv{body.p + i, body.n - i});
+  }
+  size_t i = 0;
+  while (i < body.n && !is_ws(body[i])) i++;
+  Sv opc{body.p, i};
+  Sv rest = trim(Sv{body.p + i, body.n - i});
+  // mnemonic and modifiers
+  Sv mods[16];
+  int nm = 0;
+  size_t d = 0;
+  while (d < opc.n && opc[d] != '.') d++;
+  Sv mn{opc.p, d};
+  while (d < opc.n && nm < 16) {
+    size_t e = d + 1;
+    while (e < opc.n && opc[e] != '.') e++;
+    mods[nm++] = Sv{opc.p + d + 1, e - d - 1};
+    d = e;
+  }
+  auto has = [&](const char* m) { for (int q = 0; q < nm; q++) if (mods[q].eq(m)) return true; return false; };
+  uint32_t op = op_lookup(mn);
+  if (op == OP_IMAD && nm > 0 && mods[0].eq("MOV")) op = OP_IMAD_MOV;
+  // operands: top-level commas
+  Operand ops[16];
+  Sv raw_last;
+  int no = 0;
+  {
+    int depth = 0;
+    size_t s = 0;
+    for (size_t q = 0; q <= rest.n; q++) {
+      char c = q < rest.n ? rest[q] : ',';
+      if (c == '[' || c == '{') depth++;
+      else if (c == ']' || c == '}') depth--;
+      if ((c == ',' && depth == 0) || q == rest.n) {
+        Sv tok{rest.p + s, q - s};
+        if (q < rest.n || trim(tok).n) {
+          if (no >= 16) { *msg = "too many operands"; return false; }
+          ops[no++] = classify(tok);
+          raw_last = tok;
+        }
+        s = q + 1;
+      }
+    }
+  }
+  // destination (R23)
+  int dpos = -1;
+  if (no >= 1 && ops[0].k == T_REG) dpos = 0;
+  else if (no >= 2 && ops[0].k == T_PRED && ops[1].k == T_REG && op != OP_FCHK) dpos = 1;
+  uint32_t dst = kRegNone, dstw = 0;
+  if (dpos >= 0) {
+    dst = (uint32_t)ops[dpos].reg;
+    // width table W (R24)
+    if (has("128")) dstw = 4;
+    else if (op == OP_HMMA) dstw = has("F32") ? 4 : 2;
+    else if (mn.eq("LDSM")) dstw = has("4") ? 4 : (has("2") ? 2 : 1);
+    else if (has("64") || has("WIDE")) dstw = 2;
+    else if (op == OP_DADD || op == OP_DMUL || op == OP_DFMA || op == OP_DMNMX) dstw = 2;
+    else if (op == OP_F2F || op == OP_I2F || op == OP_F2I || op == OP_I2I) {
+      dstw = 1;
+      static const char* k64[] = {"F64", "S64", "U64"};
+      static const char* k32[] = {"F32", "F16", "BF16", "S32", "U32", "S16", "U16", "S8", "U8", "TF32", "E4M3", "E5M2"};
+      for (int q = 0; q < nm; q++) {
+        bool hit64 = false, hit32 = false;
+        for (auto* x : k64) hit64 |= mods[q].eq(x);
+        for (auto* x : k32) hit32 |= mods[q].eq(x);
+        if (hit64) { dstw = 2; break; }
+        if (hit32) break;
+      }
+    } else dstw = 1;
+  }
+  // memory operand
+  int mem = -1;
+  for (int q = 0; q < no; q++) if (ops[q].k == T_MEM) { mem = q; break; }
+  uint32_t flags = 0, aw = AW_NONE, s[4] = {kRegNone, kRegNone, kRegNone, kRegNone};
+  int32_t imm = 0;
+  uint32_t cbank = 0;
+  if (has("CONSTANT")) flags |= F_CONSTANT;
+  uint32_t cls = op_class(op);
+  if (mem >= 0) {
+    flags |= F_HASMEM;
+    const Operand& m = ops[mem];
+    s[0] = m.base >= 0 ? (uint32_t)m.base : kRegNone;
+    imm = (int32_t)m.imm;
+    for (int q = mem + 1; q < no; q++)
+      if (ops[q].k == T_REG) { s[1] = (uint32_t)ops[q].reg; break; }
+    aw = AW_32;
+    for (int q = 0; q < nm; q++) {
+      if (mods[q].eq("U8") || mods[q].eq("S8")) { aw = AW_8; break; }
+      if (mods[q].eq("U16") || mods[q].eq("S16")) { aw = AW_16; break; }
+      if (mods[q].eq("64")) { aw = AW_64; break; }
+      if (mods[q].eq("128")) { aw = AW_128; break; }
+    }
+  }
+  if (cls & C_ARITH) {  // register sources after dst (R25), at most 4
+    int ns = 0;
+    for (int q = dpos + 1; q < no; q++)
+      for (int t = 0; t < ops[q].nregs; t++) {
+        int r = ops[q].regs[t];
+        if (!reg_live((uint32_t)r)) continue;
+        if (ns == 4) { *msg = "arithmetic instruction with more than 4 register sources"; return false; }
+        s[ns++] = (uint32_t)r;
+      }
+  }
+  // constant-bank load (trace terminal): c[bank][off]
+  if (cls & C_CONSTLOAD) {
+    for (int q = dpos + 1; q < no; q++)
+      if (ops[q].k == T_CREF) { cbank = (uint32_t)ops[q].bank; imm = (int32_t)ops[q].imm; break; }
+  }
+  // pointer operand (R7 / SURVEY O5 step 6)
+  uint32_t pk = PK_IMM, ptr = kRegNone;
+  if (dpos >= 0 && !(cls & (C_CONSTLOAD | C_SREG | C_MEMLOAD))) {
+    const Operand* L[16];
+    int nl = 0;
+    for (int q = dpos + 1; q < no; q++) if (ops[q].k != T_PRED) L[nl++] = &ops[q];
+    const Operand* pick = nullptr;
+    auto live_reg = [](const Operand* o) { return o->k == T_REG && reg_live((uint32_t)o->reg); };
+    if ((mn.eq("IMAD") || mn.eq("UIMAD")) && has("WIDE")) {
+      pick = nl > 2 ? L[2] : nullptr;
+    } else if (mn.eq("LEA") || mn.eq("ULEA")) {
+      pick = nl > 1 ? L[1] : nullptr;
+    } else if (mn.eq("IADD3") || mn.eq("UIADD3")) {
+      for (int q = 0; q < nl && !pick; q++) if (L[q]->k == T_CREF) pick = L[q];
+      for (int q = 0; q < nl && !pick; q++) if (live_reg(L[q]) && L[q]->reg >= 256) pick = L[q];
+      for (int q = 0; q < nl && !pick; q++) if (live_reg(L[q]) && L[q]->reg < 256) pick = L[q];
+    } else {
+      for (int q = 0; q < nl && !pick; q++) if (live_reg(L[q]) || L[q]->k == T_CREF) pick = L[q];
+    }
+    if (pick && pick->k == T_CREF) { pk = PK_CONST; cbank = (uint32_t)pick->bank; imm = (int32_t)pick->imm; }
+    else if (pick && live_reg(pick)) { pk = PK_REG; ptr = (uint32_t)pick->reg; }
+  }
+  // backward branch (R13, R28)
+  if (op == OP_BRA && no > 0) {
+    long long t;
+    if (to_int(raw_last, &t)) {
+      long long pc = 16LL * (long long)index;
+      if (t < pc) {
+        long long tidx = t <= 0 ? 0 : (t + 15) / 16;
+        flags |= F_BRA_OK;
+        imm = (int32_t)tidx;
+      }
+    }
+  }
+  if (cbank > 31) { *msg = "constant bank > 31"; return false; }
+  *out = make_rec(op, flags, aw, dstw, pk, cbank, dst, ptr, s[0], s[1], s[2], s[3], imm);
+  (void)lineno;
+  return true;
+}
+
+int param_base_for(int sm) { return sm >= 100 ? 0x380 : (sm >= 90 ? 0x210 : 0x160); }
+
+struct Segment {
+  size_t begin, end;  // byte range (lines after the header)
+  long first_line;    // 1-based line number of the first line in range
+  int sm;
+  std::string name;
+  bool header;        // false for an anonymous leading kernel
+};
+
+bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::string* err) {
+  pk->name = seg.name;
+  pk->param_base = (uint32_t)param_base_for(seg.sm);
+  long lineno = seg.first_line;
+  int32_t src_line = -1;
+  size_t p = seg.begin;
+  while (p < seg.end) {
+    const char* nl = (const char*)memchr(text + p, '\n', seg.end - p);
+    size_t e = nl ? (size_t)(nl - text) : seg.end;
+    Sv t = trim(Sv{text + p, e - p});
+    long cur = lineno;
+    p = e + 1;
+    lineno++;
+    if (!t.n) continue;
+    if (starts(t, "//##")) {
+      size_t at;
+      if (contains(t, "line ", &at)) src_line = atoi(std::string(t.p + at + 5, t.n - at - 5).c_str());
+      continue;
+    }
+    if (t.n < 4 || t[0] != '/' || t[1] != '*') continue;
+    size_t c = 2;
+    while (c + 1 < t.n && !(t[c] == '*' && t[c + 1] == '/')) c++;
+    if (c + 1 >= t.n) continue;
+    Sv pcs{t.p + 2, c - 2};
+    bool hex = pcs.n > 0;
+    for (size_t q = 0; q < pcs.n; q++) if (hexv(pcs[q]) < 0) hex = false;
+    if (!hex || starts(pcs, "0x")) continue;
+    Sv body{t.p + c + 2, t.n - c - 2};
+    size_t semi = 0;
+    while (semi < body.n && body[semi] != ';') semi++;
+    if (semi == body.n) continue;
+    long long pc = 0;
+    for (size_t q = 0; q < pcs.n; q++) pc = pc * 16 + hexv(pcs[q]);
+    if (pc != 16LL * (long long)pk->recs.size()) {
+      *err = "line " + std::to_string(cur) + ": pc not 16-strided";
+      return false;
+    }
+    Rec r;
+    std::string msg;
+    if (!pack_line(Sv{body.p, semi}, cur, pk->recs.size(), &r, &msg)) {
+      *err = "line " + std::to_string(cur) + ": " + msg;
+      return false;
+    }
+    pk->recs.push_back(r);
+    pk->lines.push_back(src_line);
+  }
+  return true;
+}
+
+bool is_instr_line(Sv t) {
+  if (t.n < 4 || t[0] != '/' || t[1] != '*') return false;
+  size_t c = 2;
+  while (c + 1 < t.n && !(t[c] == '*' && t[c + 1] == '/')) c++;
+  if (c + 1 >= t.n || c == 2) return false;
+  for (size_t q = 2; q < c; q++) if (hexv(t[q]) < 0) return false;
+  if (t[2] == '0' && t[3] == 'x') return false;
+  Sv body{t.p + c + 2, t.n - c - 2};
+  for (size_t q = 0; q < body.n; q++) if (body[q] == ';') return true;
+  return false;
+}
+
+}  // namespace
+
+bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedKernel>* out, std::string* err) {
+  // pass 1: segments
+  std::vector<Segment> segs;
+  int sm = 100;
+  long lineno = 1;
+  size_t p = 0;
+  while (p < len) {
+    const char* nl = (const char*)memchr(text + p, '\n', len - p);
+    size_t e = nl ? (size_t)(nl - text) : len;
+    Sv t = trim(Sv{text + p, e - p});
+    size_t at;
+    if (t.n) {
+      if (contains(t, "code for sm_", &at)) {
+        sm = atoi(std::string(t.p + at + 12, t.n - at - 12).c_str());
+      } else if (contains(t, ".target") && contains(t, "sm_", &at)) {
+        sm = atoi(std::string(t.p + at + 3, t.n - at - 3).c_str());
+      } else if (contains(t, "Function :", &at)) {
+        if (!segs.empty()) segs.back().end = p;
+        Segment s;
+        s.begin = e + 1 > len ? len : e + 1;
+        s.end = len;
+        s.first_line = lineno + 1;
+        s.sm = sm;
+        Sv nm = trim(Sv{t.p + at + 10, t.n - at - 10});
+        s.name.assign(nm.p, nm.n);
+        s.header = true;
+        segs.push_back(s);
+      } else if (segs.empty() && !starts(t, "//##") && is_instr_line(t)) {
+        Segment s;  // instructions before any Function header: one anonymous kernel
+        s.begin = 0;
+        s.end = len;
+        s.first_line = 1;
+        s.sm = sm;
+        s.name = "<anonymous>";
+        s.header = false;
+        segs.push_back(s);
+      }
+    }
+    p = e + 1;
+    lineno++;
+  }
+  // a later "code for"/".target" line inside a segment applies to the next Function only; the
+  // per-segment sm was captured when its header was seen.
+  out->assign(segs.size(), ParsedKernel());
+  std::vector<std::string> errs(segs.size());
+  std::atomic<size_t> next(0);
+  std::atomic<bool> failed(false);
+  auto worker = [&]() {
+    for (;;) {
+      size_t k = next.fetch_add(1);
+      if (k >= segs.size() || failed.load()) return;
+      if (!parse_segment(text, segs[k], &(*out)[k], &errs[k])) failed = true;
+    }
+  };
+  int nt = std::max(1, std::min<int>(n_threads, (int)segs.size()));
+  std::vector<std::thread> th;
+  for (int i = 1; i < nt; i++) th.emplace_back(worker);
+  worker();
+  for (auto& t : th) t.join();
+  for (size_t k = 0; k < segs.size(); k++)
+    if (!errs[k].empty()) { *err = errs[k]; return false; }
+  return true;
+}
+
+}  // namespace gs

@@ -1,0 +1,21 @@
+// loader.h — host SASS parser/packer interface (see loader.cpp).
+#pragma once
+#include <string>
+#include <vector>
+
+#include "record.h"
+
+namespace gs {
+
+struct ParsedKernel {
+  std::string name;
+  uint32_t param_base = 0x380;
+  std::vector<Rec> recs;
+  std::vector<int32_t> lines;  // source line per instruction, -1 if unknown
+};
+
+// Parses cuobjdump / nvdisasm text into per-kernel packed records using up to n_threads threads.
+// Returns false and sets *err ("line N: ...") on malformed input.
+bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedKernel>* out, std::string* err);
+
+}  // namespace gs

@@ -1,0 +1,177 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, line by line.
+
+Bit-exact bar (integer/index work): identical canonical K/S/H/N/R lines.
+"""
+import random
+
+import numpy as np
+import pytest
+
+import brute
+import oracle_run as orc
+from oracle_run import Canon, golden
+
+pytestmark = [pytest.mark.gpu, pytest.mark.usefixtures("oracle_bin")]
+
+FIXTURES = ["listing1.sass", "sgemm_naive.sm_100a.sass", "sgemm_naive.sm_70.sass", "jacobi.sm_100a.sass",
+            "jacobi.sm_70.sass", "mixbench.sm_100a.sass", "mixbench.sm_70.sass", "atomics.sm_100a.sass",
+            "atomics.sm_70.sass", "conv.sm_100a.sass", "spill.r24.sm_100a.sass", "spill.r32.sm_100a.sass",
+            "spill.r40.sm_100a.sass", "spill.r64.sm_100a.sass"]
+
+
+@pytest.fixture(scope="module")
+def gs():
+    import torch
+    import paper_conf_sc_senvs23_b200 as g
+    from paper_conf_sc_senvs23_b200 import build
+    build.build()
+    assert torch.cuda.is_available()
+    return g
+
+
+def _ctx(gs, **kw):
+    return gs.Context(**kw)
+
+
+def _detect_lines(gs, text, D=64, kb=0, ke=None, **kw):
+    from paper_conf_sc_senvs23_b200 import report
+    ctx = _ctx(gs, trace_depth=D, **kw)
+    ctx.load_sass(text)
+    ctx.detect(kb, ke)
+    return Canon(report.canonical(ctx, kb, ke)), ctx
+
+
+def _read(name):
+    return open(golden(name), "rb").read()
+
+
+@pytest.mark.parametrize("name", FIXTURES)
+def test_detect_parity_fixtures(gs, name):
+    text = _read(name)
+    g, _ = _detect_lines(gs, text)
+    o = Canon(orc.run(text))
+    assert g.K == o.K
+    assert g.S == o.S
+
+
+def test_detect_parity_brute_streams(gs):
+    rng = random.Random(7)
+    for _ in range(60):
+        ks = [brute.random_stream(rng, rng.randint(1, 6)) for _ in range(rng.randint(1, 4))]
+        D = rng.choice([1, 2, 3, 64])
+        text = brute.render(ks)
+        g, _ = _detect_lines(gs, text, D=D)
+        o = Canon(orc.run(text, D=D))
+        assert g.K == o.K and g.S == o.S, text
+
+
+@pytest.mark.parametrize("cfg,scale", [("C1", 1), ("C2", 1), ("C3", 0.002), ("C4", 0.02), ("C5", 0.02)])
+def test_detect_parity_configs(gs, cfg, scale):
+    from gen import sass as gsass
+    s = gsass.config_sass(cfg, scale=scale)
+    g, _ = _detect_lines(gs, s.text)
+    o = Canon(orc.run(s.text))
+    assert g.K == o.K
+    assert len(g.S) == len(o.S)
+    assert g.S == o.S
+
+
+def test_detect_kernel_range(gs):
+    from gen import sass as gsass
+    s = gsass.config_sass("C4", scale=0.03)   # 7 kernels
+    for kb, ke in [(0, 3), (2, 7), (5, 5)]:
+        g, _ = _detect_lines(gs, s.text, kb=kb, ke=ke)
+        o = Canon(orc.run(s.text, kbegin=kb, kend=ke))
+        assert g.K == o.K and g.S == o.S
+
+
+def test_trace_depth_edges(gs):
+    from gen import sass as gsass
+    s = gsass.config_sass("C5", scale=0.01)   # contains the 63/64/65-step chains
+    for D in (1, 2, 63, 64, 65, 255):
+        g, _ = _detect_lines(gs, s.text, D=D)
+        o = Canon(orc.run(s.text, D=D))
+        assert g.S == o.S, D
+
+
+# ------------------------------------------------------------------------------ full flow
+def _flow(gs, text, raw, hist_mode=0, host_input=False, k=None, n_reasons=19):
+    import torch
+    from paper_conf_sc_senvs23_b200 import report
+    ctx = _ctx(gs, hist_mode=hist_mode, n_reasons=n_reasons)
+    ctx.load_sass(text)
+    ctx.detect()
+    raw_t = torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda()
+    words, ninv = ctx.pack_samples(raw_t)
+    if host_input:
+        hist, ninv2 = ctx.attribute_samples(words.cpu().numpy())
+    else:
+        hist, ninv2 = ctx.attribute_samples(words)
+    ranked = ctx.rank_sites(hist, k=k)
+    torch.cuda.synchronize()
+    n_invalid = int(ninv2.item())
+    assert n_invalid == int(ninv.item())     # packing marks exactly the invalid samples
+    return Canon(report.canonical(ctx, hist=hist, n_samples=len(raw), n_invalid=n_invalid, ranked=ranked)), ctx
+
+
+def _samples(s, n, order, seed, n_bad=100):
+    from gen import samples as gsm
+    tab = gsm.table_class_weighted(s.cls, n, key=seed)
+    tr = gsm.Trace(tab, s.first_slot, s.n_instr, order=order, seed=seed)
+    raw = tr.raw()
+    bad = gsm.invalid_raw(len(s.n_instr), s.n_instr, n_bad, key=seed)
+    return gsm.interleave(raw, bad, key=seed + 1), tab
+
+
+@pytest.mark.parametrize("cfg,n,order,mode", [
+    ("C1", 16384, "trace", 0), ("C1", 16384, "shuffled", 1), ("C1", 16384, "shuffled", 2),
+    ("C2", 400_000, "trace", 0), ("C2", 400_000, "shuffled", 1), ("C2", 400_000, "shuffled", 2),
+])
+def test_full_flow_parity(gs, cfg, n, order, mode):
+    from gen import sass as gsass
+    s = gsass.config_sass(cfg)
+    raw, tab = _samples(s, n, order, seed=11)
+    g, ctx = _flow(gs, s.text, raw, hist_mode=mode)
+    o = Canon(orc.run(s.text, samples=raw))
+    assert g.H == o.H and g.N == o.N
+    assert g.S == o.S and g.K == o.K
+    assert g.R == o.R
+
+
+def test_host_input_and_topk(gs):
+    from gen import sass as gsass
+    s = gsass.config_sass("C1")
+    raw, _ = _samples(s, 20000, "shuffled", seed=3)
+    g, _ = _flow(gs, s.text, raw, host_input=True, k=10)
+    o = Canon(orc.run(s.text, samples=raw, k=10))
+    assert g.H == o.H and g.R == o.R and len(g.R) == 10
+
+
+def test_fewer_reasons(gs):
+    from gen import sass as gsass
+    s = gsass.config_sass("C1")
+    raw, _ = _samples(s, 20000, "shuffled", seed=5)
+    g, _ = _flow(gs, s.text, raw, n_reasons=7)
+    o = Canon(orc.run(s.text, samples=raw, R=7))
+    assert g.H == o.H and g.N == o.N and g.R == o.R
+
+
+def test_empty_and_degenerate(gs):
+    import torch
+    ctx = _ctx(gs)
+    assert ctx.load_sass(b"") == (0, 0)
+    assert ctx.detect() == 0
+    hist, ninv = ctx.attribute_samples(torch.zeros(0, dtype=torch.int32, device="cuda"))
+    assert ctx.rank_sites(hist).shape == (0,)
+    # a kernel without instructions between two others
+    text = ("\tcode for sm_100a\n\t\tFunction : a\n        /*0000*/ LDG.E R0, desc[UR4][R2.64] ;\n"
+            "\t\tFunction : empty\n\t\tFunction : c\n        /*0000*/ LDG.E R1, desc[UR4][R2.64+0x4] ;\n")
+    g, _ = _detect_lines(gs, text)
+    o = Canon(orc.run(text))
+    assert g.K == o.K and g.S == o.S
+
+
+def test_parse_error_reported(gs):
+    ctx = _ctx(gs)
+    with pytest.raises(gs.GsError, match="line 3"):
+        ctx.load_sass("\t\tFunction : x\n        /*0000*/ NOP ;\n        /*0020*/ NOP ;\n")

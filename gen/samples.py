@@ -191,8 +191,18 @@ class Trace:
         if self.order == "shuffled":
             return feistel(p.astype(np.uint64), self.N, self.seed).astype(np.int64)
         # trace order: grouped by kernel, shuffled within the kernel's block
-        k = np.searchsorted(self.kstart, p, side="right") - 1
         q = np.empty_like(p)
+        if len(p) > 1 and np.all(p[1:] >= p[:-1]):      # sorted positions: split by kernel blocks
+            cuts = np.searchsorted(p, self.kstart, side="left")
+            for kk in range(len(self.kstart) - 1):
+                a, b = int(cuts[kk]), int(cuts[kk + 1])
+                if a == b:
+                    continue
+                n_k = int(self.kstart[kk + 1] - self.kstart[kk])
+                q[a:b] = self.kstart[kk] + feistel((p[a:b] - self.kstart[kk]).astype(np.uint64), n_k,
+                                                   self.seed * 1000003 + kk).astype(np.int64)
+            return q
+        k = np.searchsorted(self.kstart, p, side="right") - 1
         for kk in np.unique(k):
             m = k == kk
             n_k = int(self.kstart[kk + 1] - self.kstart[kk])
@@ -200,18 +210,27 @@ class Trace:
                                              self.seed * 1000003 + int(kk)).astype(np.int64)
         return q
 
-    def bins(self, a: int, b: int) -> np.ndarray:
-        q = self.sorted_index(np.arange(a, b, dtype=np.int64))
+    def bins(self, a: int, b: int, step: int = 1) -> np.ndarray:
+        return self.bins_at(np.arange(a, b, step, dtype=np.int64))
+
+    def bins_at(self, positions: np.ndarray) -> np.ndarray:
+        q = self.sorted_index(np.asarray(positions, dtype=np.int64))
         return self.nz[np.searchsorted(self.cum, q, side="right") - 1]
 
-    def raw(self, a: int = 0, b: int | None = None) -> np.ndarray:
-        """[b-a, 3] uint32 raw triples (kernel, pc byte offset, reason)."""
-        b = self.N if b is None else b
-        bins = self.bins(a, b)
+    def raw_at(self, positions: np.ndarray) -> np.ndarray:
+        return self.bins_to_raw(self.bins_at(positions))
+
+    def bins_to_raw(self, bins: np.ndarray) -> np.ndarray:
+        bins = np.asarray(bins, dtype=np.int64)
         slot, reason = bins // R_SLOTS, bins % R_SLOTS
         k = np.searchsorted(self.first_slot, slot, side="right") - 1
         pc = (slot - self.first_slot[k]) * 16
         return np.stack([k, pc, reason], axis=1).astype(np.uint32)
+
+    def raw(self, a: int = 0, b: int | None = None) -> np.ndarray:
+        """[b-a, 3] uint32 raw triples (kernel, pc byte offset, reason)."""
+        b = self.N if b is None else b
+        return self.bins_to_raw(self.bins(a, b))
 
     def packed(self, a: int = 0, b: int | None = None) -> np.ndarray:
         b = self.N if b is None else b

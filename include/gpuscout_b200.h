@@ -145,6 +145,10 @@ gs_status gs_attribute_samples(gs_ctx *ctx, const uint32_t *samples, uint64_t n,
 gs_status gs_rank_sites(gs_ctx *ctx, const int32_t *d_hist, uint64_t k, gs_ranked_site *out,
                         uint64_t *n_out);
 
+/* Number of CUDA kernels this library has launched in the process so far (its own kernels plus
+ * the CUB radix-sort kernels of gs_rank_sites). Lets a harness count launches in a timed region. */
+uint64_t gs_launch_count(void);
+
 /* Histogram strategy actually used by the last gs_attribute_samples (GS_HIST_*). */
 int gs_last_hist_mode(const gs_ctx *ctx);
 

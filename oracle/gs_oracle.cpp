@@ -706,7 +706,7 @@ int main(int argc, char** argv) {
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
-  bool detect = true, hist = true, timing = false;
+  bool detect = true, hist = true, timing = false, quiet = false;
   for (int a = 1; a < argc; a++) {
     std::string s = argv[a];
     auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
@@ -723,6 +723,7 @@ int main(int argc, char** argv) {
     else if (s == "--no-detect") detect = false;
     else if (s == "--no-hist") hist = false;
     else if (s == "--time") timing = true;
+    else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
     else { fprintf(stderr, "unknown arg %s\n", s.c_str()); return 2; }
   }
   auto now = [] { return std::chrono::steady_clock::now(); };
@@ -763,6 +764,7 @@ int main(int argc, char** argv) {
               ks[k].ins.size(), ks[k].first_slot, stats[k].gatom, stats[k].satom, stats[k].conv,
               stats[k].vec_already, stats[k].ustores, ks[k].name.c_str());
     for (auto& s : sites) {
+      if (quiet) break;
       std::string chain;
       for (size_t c = 0; c < s.tr.chain.size(); c++) chain += (c ? "," : "") + std::to_string(s.tr.chain[c]);
       if (chain.empty()) chain = "-";
@@ -796,7 +798,10 @@ int main(int argc, char** argv) {
     auto th1 = now();
     uint64_t mass = 0;
     for (size_t b = 0; b < H.size(); b++)
-      if (H[b]) { fprintf(out, "H %zu %zu %llu\n", b / 32, b % 32, (unsigned long long)H[b]); mass += H[b]; }
+      if (H[b]) {
+        if (!quiet) fprintf(out, "H %zu %zu %llu\n", b / 32, b % 32, (unsigned long long)H[b]);
+        mass += H[b];
+      }
     fprintf(out, "N total=%llu valid=%llu invalid=%llu\n", (unsigned long long)N, (unsigned long long)mass,
             (unsigned long long)invalid);
     // O14 join: counts at the site's PC, site total, kernel total, REL sum.
@@ -824,7 +829,9 @@ int main(int argc, char** argv) {
       return a.s->rule < b.s->rule;
     });
     size_t lim = K_top < 0 ? rk.size() : std::min(rk.size(), (size_t)K_top);
-    for (size_t q = 0; q < lim; q++) {
+    auto tr1 = now();
+    if (timing) fprintf(stderr, "TIME rank_s=%.6f sites=%zu\n", secs(th1, tr1), rk.size());
+    for (size_t q = 0; q < lim && !quiet; q++) {
       const Site& s = *rk[q].s;
       size_t slot = ks[s.k].first_slot + (size_t)s.idx;
       std::string h;

@@ -44,7 +44,11 @@ class GsError(RuntimeError):
 _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
-           "gs_attribute_samples", "gs_rank_sites", "gs_last_hist_mode"]
+           "gs_attribute_samples", "gs_rank_sites", "gs_last_hist_mode", "gs_launch_count"]
+
+
+def launch_count() -> int:
+    return int(load_library().gs_launch_count())
 
 
 def load_library(path: str = LIB_PATH):
@@ -73,6 +77,7 @@ def load_library(path: str = LIB_PATH):
         "gs_attribute_samples": (I32, [P, P, U64, P, P, I32]),
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
         "gs_last_hist_mode": (I32, [P]),
+        "gs_launch_count": (U64, []),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

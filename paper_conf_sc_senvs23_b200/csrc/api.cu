@@ -10,7 +10,12 @@
 #include "ctx.h"
 #include "loader.h"
 
+#include <atomic>
+
 namespace gs {
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
 gs_status fail(gs_ctx* c, gs_status s, const std::string& msg) {
   if (c) c->err = msg;
@@ -283,6 +288,8 @@ gs_status gs_rank_sites(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_
   const bool host = out ? !is_device_ptr(out) : true;
   return rank_run(c, d_hist, k, out, host, n_out);
 }
+
+uint64_t gs_launch_count(void) { return gs::g_launches.load(); }
 
 int gs_last_hist_mode(const gs_ctx* c) { return c ? c->last_hist_mode : -1; }
 

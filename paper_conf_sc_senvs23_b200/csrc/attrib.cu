@@ -132,7 +132,7 @@ gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_
                            unsigned long long* d_n_invalid) {
   if (!n) return GS_OK;
   k_pack<<<(unsigned)((n + 255) / 256), 256, 0, c->stream>>>(d_raw, n, c->d_kd, c->n_kernels, c->cfg.n_reasons,
-                                                             d_words, d_n_invalid);
+                                                             d_words, d_n_invalid); count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }
@@ -152,7 +152,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   // peel the words before the first 16-byte boundary so the main kernels use 128-bit loads
   const uint64_t head = std::min<uint64_t>(n, ((16u - (reinterpret_cast<uintptr_t>(d_words) & 15u)) & 15u) / 4u);
   if (head) {
-    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P, nr, d_hist, d_n_invalid);
+    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P, nr, d_hist, d_n_invalid); count_launch();
     GS_CUDA(c, cudaGetLastError());
     d_words += head;
     n -= head;
@@ -164,7 +164,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   c->last_hist_mode = (int)mode;
   if (mode == GS_HIST_GLOBAL) {
     const uint64_t blocks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 4, (n + kThreads * 4 - 1) / (kThreads * 4)));
-    k_hist_global<<<(unsigned)blocks, kThreads, 0, st>>>(d_words, n, P, nr, d_hist, d_n_invalid);
+    k_hist_global<<<(unsigned)blocks, kThreads, 0, st>>>(d_words, n, P, nr, d_hist, d_n_invalid); count_launch();
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
@@ -181,7 +181,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   chunk = (chunk + 3) & ~3ull;
   chunks = (n + chunk - 1) / chunk;
   k_hist_private<<<(unsigned)(chunks * n_ranges), kThreads, smem, st>>>(d_words, n, P, nr, n_ranges, range_bins, chunk,
-                                                                       d_hist, d_n_invalid);
+                                                                       d_hist, d_n_invalid); count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }

@@ -112,6 +112,9 @@ struct gs_ctx {
 
 namespace gs {
 
+// process-wide launch counter (gs_launch_count)
+void count_launch(uint64_t n = 1);
+
 // error helpers (set ctx->err, return status)
 gs_status fail(gs_ctx* c, gs_status s, const std::string& msg);
 gs_status cuda_fail(gs_ctx* c, cudaError_t e, const char* what);

@@ -532,27 +532,27 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     GS_CUDA(c, cudaMemsetAsync(c->d_wev + w0, 0, (uint64_t)nw * 4, st));
     const uint32_t grid = (nw + kWarps - 1) / kWarps;
     k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
-                                           c->d_wev, c->d_narith, c->d_kstats);
+                                           c->d_wev, c->d_narith, c->d_kstats); count_launch();
     GS_CUDA(c, cudaGetLastError());
-    k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop);
+    k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop); count_launch();
     GS_CUDA(c, cudaGetLastError());
     // candidate arrays are indexed relative to c0
     k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
-                                           c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand);
+                                           c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand); count_launch();
     GS_CUDA(c, cudaGetLastError());
   }
   unsigned long long* d_tot = c->cand.choff + nc;  // two totals after the offsets
   unsigned long long tot[2] = {0, 0};
   if (nc) {
     const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
-    k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots);
+    k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
     GS_CUDA(c, cudaGetLastError());
     const uint32_t gridc = (uint32_t)((nc + 255) / 256);
     k_trace<<<gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
-                                   c->d_kstats);
+                                   c->d_kstats); count_launch();
     GS_CUDA(c, cudaGetLastError());
     k_rules<<<gridc, 256, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
-                                   RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads});
+                                   RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}); count_launch();
     GS_CUDA(c, cudaGetLastError());
     // chain offsets (u64) from chain lengths stored in soff, then site offsets in place of soff
     gs_status s = scan_u32_to_u64(c, c->cand.soff, c->cand.choff, nc, d_tot);
@@ -568,7 +568,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
   if (nc && ns) {
     k_write<<<(uint32_t)((nc + 255) / 256), 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
-                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain);
+                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain); count_launch();
     GS_CUDA(c, cudaGetLastError());
   }
   c->kstats_h.assign(c->n_kernels, gs_kernel_stats{});

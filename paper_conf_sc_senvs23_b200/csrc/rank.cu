@@ -18,6 +18,9 @@
 namespace gs {
 namespace {
 
+// onesweep radix sort of 64-bit keys: 1 histogram + 1 exclusive-sum + 8 digit passes
+constexpr uint64_t kCubSortLaunches = 10;
+
 __constant__ uint32_t kRelMask[7] = {
     1u << 6,                // VEC   long_scoreboard
     (1u << 6) | (1u << 5),  // SPILL long_scoreboard + lg_throttle
@@ -115,7 +118,7 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
   const uint64_t kk = std::min<uint64_t>(k, ns);
   if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, (uint64_t)std::max<uint32_t>(c->n_kernels, 1) * 8));
   if (c->n_kernels) {
-    k_ktot<<<c->n_kernels, 256, 0, st>>>(d_hist, c->d_kd, c->n_kernels, c->d_ktot);
+    k_ktot<<<c->n_kernels, 256, 0, st>>>(d_hist, c->d_kd, c->n_kernels, c->d_ktot); count_launch();
     GS_CUDA(c, cudaGetLastError());
   }
   if (ns) {
@@ -154,15 +157,17 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
     unsigned long long* key_rel = reinterpret_cast<unsigned long long*>(c->d_sort_tmp);
     void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + rel_bytes;
     const unsigned grid = (unsigned)((ns + 255) / 256);
-    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, c->d_kd, key_tot, key_rel, v0);
+    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, c->d_kd, key_tot, key_rel, v0); count_launch();
     GS_CUDA(c, cudaGetLastError());
     size_t b1 = cub_bytes;
     GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, key_tot, key_tmp, v0, v1, (int)ns, 0, 64, st));
+    count_launch(kCubSortLaunches);
     // v1 = sites ordered by tot desc (stable); now sort by rel desc, stable
-    k_gather_keys<<<grid, 256, 0, st>>>(v1, key_rel, ns, key_tot);
+    k_gather_keys<<<grid, 256, 0, st>>>(v1, key_rel, ns, key_tot); count_launch();
     GS_CUDA(c, cudaGetLastError());
     b1 = cub_bytes;
     GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, key_tot, key_tmp, v1, v0, (int)ns, 0, 64, st));
+    count_launch(kCubSortLaunches);
     // v0 = final order
     if (kk) {
       gs_ranked_site* dst = out;
@@ -170,7 +175,7 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
         GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
         dst = c->d_ranked;
       }
-      k_emit<<<(unsigned)kk, 32, 0, st>>>(v0, kk, c->d_sites, d_hist, c->d_kd, c->d_ktot, dst);
+      k_emit<<<(unsigned)kk, 32, 0, st>>>(v0, kk, c->d_sites, d_hist, c->d_kd, c->d_ktot, dst); count_launch();
       GS_CUDA(c, cudaGetLastError());
       if (out_is_host)
         GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));

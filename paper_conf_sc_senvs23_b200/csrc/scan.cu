@@ -98,9 +98,9 @@ gs_status scan_impl(gs_ctx* c, const uint32_t* in, OutT* out, uint64_t n, unsign
     GS_CUDA(c, cudaMemsetAsync(d_total, 0, 8, c->stream));
     return GS_OK;
   }
-  k_tile_sum<<<(unsigned)nb, kThreads, 0, c->stream>>>(in, n, bs);
-  k_scan_bsum<<<1, kThreads, 0, c->stream>>>(bs, nb, d_total);
-  k_tile_apply<OutT><<<(unsigned)nb, kThreads, 0, c->stream>>>(in, n, bs, out);
+  k_tile_sum<<<(unsigned)nb, kThreads, 0, c->stream>>>(in, n, bs); count_launch();
+  k_scan_bsum<<<1, kThreads, 0, c->stream>>>(bs, nb, d_total); count_launch();
+  k_tile_apply<OutT><<<(unsigned)nb, kThreads, 0, c->stream>>>(in, n, bs, out); count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }

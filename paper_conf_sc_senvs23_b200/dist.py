@@ -1,0 +1,67 @@
+"""Multi-GPU orchestration: one process per GPU, torch.distributed for the plumbing.
+
+  * samples are sharded contiguously: rank g owns positions [g*N/G, (g+1)*N/G);
+  * kernels (detection) are sharded contiguously, balanced by instruction count;
+  * the per-rank int32 histograms are combined with ONE all_reduce(SUM) (NCCL over NVLink) —
+    integer addition is associative, so the result is bit-identical for any G;
+  * every rank joins its own sites against the full histogram and ranks them; the exact global
+    top-K is the merge of the local top-K lists under the total order (rel desc, tot desc,
+    kernel, idx, rule) (R20), gathered with one all_gather.
+
+The functions below are host logic only (ranges, merge); the device work is the library's.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def sample_range(n: int, rank: int, world: int) -> tuple[int, int]:
+    return n * rank // world, n * (rank + 1) // world
+
+
+def kernel_range(n_instr, rank: int, world: int) -> tuple[int, int]:
+    """Contiguous kernel range whose instruction count is ~1/world of the total."""
+    n_instr = np.asarray(n_instr, dtype=np.int64)
+    pre = np.concatenate([[0], np.cumsum(n_instr)])
+    total = int(pre[-1])
+
+    def cut(g):
+        if g <= 0:
+            return 0
+        if g >= world:
+            return len(n_instr)
+        return int(np.searchsorted(pre, total * g // world, side="left"))
+
+    return cut(rank), cut(rank + 1)
+
+
+def rank_key(row) -> tuple:
+    return (-int(row["rel"]), -int(row["tot"]), int(row["kernel"]), int(row["idx"]), int(row["rule"]))
+
+
+def merge_topk(parts: list[np.ndarray], k: int | None) -> np.ndarray:
+    """Exact global top-k from per-rank ranked lists (each already sorted by the total order)."""
+    rows = np.concatenate([p for p in parts if len(p)]) if any(len(p) for p in parts) else parts[0][:0]
+    if not len(rows):
+        return rows
+    # np.lexsort: the last key is the primary one
+    order = np.lexsort((rows["rule"], rows["idx"], rows["kernel"], -rows["tot"].astype(np.int64),
+                        -rows["rel"].astype(np.int64)))
+    rows = rows[order]
+    return rows if k is None else rows[:k]
+
+
+def allreduce_hist(hist, group=None):
+    import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(hist, op=dist.ReduceOp.SUM, group=group)
+    return hist
+
+
+def gather_ranked(local: np.ndarray, k: int | None, group=None) -> np.ndarray:
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return local if k is None else local[:k]
+    parts = [None] * dist.get_world_size(group)
+    dist.all_gather_object(parts, local if k is None else local[:k], group=group)
+    return merge_topk(parts, k)

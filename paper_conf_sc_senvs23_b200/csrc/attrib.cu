@@ -2,15 +2,29 @@
 // (§2.2, §3).
 //
 // Packed sample word: (slot << 5) | reason, slot = first_slot[kernel] + pc/16 (R30). Because a
-// histogram row is 32 bins wide the word IS the flat bin index, so the hot loop is
-// "validate, then increment H[word]". Strategies (gs_config.hist_mode):
-//   PRIVATE  the compact bin space (slot * n_reasons + reason) is split into ranges that fit one
-//            CTA's shared memory; each CTA streams a contiguous chunk of samples with 128-bit
-//            loads and counts the samples of its range with shared-memory atomics; the CTAs of
-//            one chunk are launched adjacently so the repeated reads of a chunk hit L2. Counts
-//            are flushed to the global histogram once per CTA.
-//   GLOBAL   one L2 atomic (RED) per valid sample.
-//   AUTO     PRIVATE when the compact bin space needs at most kMaxRanges ranges, else GLOBAL.
+// histogram row is 32 bins wide the word IS the flat bin index: the hot loop is "validate, then
+// increment H[word]". Global atomics alone run at ~50-200 G samples/s on B200 (L2 atomic rate,
+// profiles/r01_atomics_microbench.txt) — far below the ~1.6 T samples/s HBM streams 4-byte
+// samples at — so the counting happens in shared memory:
+//
+//   * compact bins cb = slot * n_reasons + reason (only active reasons occupy shared memory);
+//   * the table packs two 16-bit counters per 32-bit word (114688 bins in 224 KB, one CTA
+//     of 1024 threads per SM); a counter that reaches 0x8000 is drained (-0x8000 in shared
+//     memory, +0x8000 to the global bin) by the one thread whose atomicAdd returned 0x7FFF, so a
+//     16-bit half can never carry into its neighbour (at most a few thousand increments can be in
+//     flight per SM between that add and the drain) and the counts stay exact;
+//   * samples stream in with 128-bit loads.
+// Strategies (gs_config.hist_mode):
+//   PRIVATE  fixed windows: the compact bin space is split into ranges of one table each; each
+//            CTA counts the samples of its range in a contiguous chunk; the CTAs of one chunk are
+//            launched adjacently so the re-reads of a chunk hit L2. Flushed once per CTA.
+//   WINDOW   one persistent CTA per SM streams a contiguous 1/grid of the samples in tiles and
+//            moves its window with the data: at a tile whose first sample falls outside the
+//            window, the table is flushed and re-based at the sample's kernel (whole kernel if it
+//            fits, else centred on the sample). Samples outside the window go straight to L2
+//            atomics. Suited to PC-sampling traces, which arrive grouped by kernel launch.
+//   GLOBAL   one L2 atomic per valid sample (reference strategy).
+//   AUTO     PRIVATE if the compact bins fit in kMaxRanges tables, else WINDOW.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -20,12 +34,15 @@
 namespace gs {
 namespace {
 
-constexpr int kThreads = 512;
-constexpr uint32_t kRangeBins = 48 * 1024;  // u32 counters per CTA (192 KB of shared memory)
-constexpr uint32_t kMaxRanges = 8;
+constexpr int kThreadsGlobal = 512;
+constexpr int kThreadsSmem = 1024;
+constexpr uint32_t kTableWords = 56 * 1024;        // 224 KB of shared memory
+constexpr uint32_t kTableBins = 2 * kTableWords;   // 114688 16-bit counters
+constexpr uint32_t kMaxRanges = 3;
+constexpr uint32_t kTile4 = 8192;                  // uint4 per window decision (32K samples)
+constexpr uint32_t kNoWindow = 0xffffffffu;
 
 __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long* d_n_invalid) {
-  // n_bad per thread -> one atomic per warp
   for (int o = 16; o; o >>= 1) n_bad += __shfl_xor_sync(0xffffffffu, n_bad, o);
   if ((threadIdx.x & 31) == 0 && n_bad) atomicAdd(d_n_invalid, (unsigned long long)n_bad);
 }
@@ -50,9 +67,9 @@ __global__ void k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc
 }
 
 // -------------------------------------------------------------------------------- GLOBAL
-__global__ void __launch_bounds__(kThreads) k_hist_global(const uint32_t* __restrict__ s, uint64_t n, uint32_t P,
-                                                          uint32_t nr, int32_t* __restrict__ H,
-                                                          unsigned long long* d_n_invalid) {
+__global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* __restrict__ s, uint64_t n, uint32_t P,
+                                                                uint32_t nr, int32_t* __restrict__ H,
+                                                                unsigned long long* d_n_invalid) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   uint32_t bad = 0;
   const uint64_t n4 = n / 4;
@@ -74,56 +91,118 @@ __global__ void __launch_bounds__(kThreads) k_hist_global(const uint32_t* __rest
   count_invalid(bad, d_n_invalid);
 }
 
-// -------------------------------------------------------------------------------- PRIVATE
-// grid = n_chunks * n_ranges; blockIdx.x = chunk * n_ranges + range
-__global__ void __launch_bounds__(kThreads) k_hist_private(const uint32_t* __restrict__ s, uint64_t n, uint32_t P,
-                                                           uint32_t nr, uint32_t n_ranges, uint32_t range_bins,
-                                                           uint64_t chunk, int32_t* __restrict__ H,
-                                                           unsigned long long* d_n_invalid) {
-  extern __shared__ uint32_t cnt[];
-  const uint32_t range = blockIdx.x % n_ranges;
-  const uint64_t ci = blockIdx.x / n_ranges;
-  const uint32_t lo = range * range_bins;
-  for (uint32_t b = threadIdx.x; b < range_bins; b += blockDim.x) cnt[b] = 0;
-  __syncthreads();
-  uint64_t a = ci * chunk, e = a + chunk;
-  if (e > n) e = n;
+// -------------------------------------------------------------------------------- shared-memory table
+__device__ __forceinline__ uint32_t word_of(uint32_t cb, uint32_t nr) { return (cb / nr) * 32u + cb % nr; }
+
+// one sample: shared-memory 16-bit counter if inside the window; outside it an L2 atomic (WINDOW)
+// or nothing (PRIVATE: another CTA owns that range)
+template <bool SPILL_OUT>
+__device__ __forceinline__ void count_one(uint32_t w, uint32_t P, uint32_t nr, uint32_t wb, uint32_t* tab,
+                                          int32_t* H, uint32_t& bad) {
+  const uint32_t slot = w >> 5, rs = w & 31u;
+  if (slot < P && rs < nr) {
+    const uint32_t off = slot * nr + rs - wb;
+    if (off < kTableBins) {
+      const uint32_t sh = (off & 1u) << 4;
+      const uint32_t old = atomicAdd(tab + (off >> 1), 1u << sh);
+      if (((old >> sh) & 0xffffu) == 0x7fffu) {  // drain: keep every 16-bit half below 2^16
+        atomicSub(tab + (off >> 1), 0x8000u << sh);
+        atomicAdd(H + w, 0x8000);
+      }
+    } else if (SPILL_OUT) {
+      atomicAdd(H + w, 1);
+    }
+  } else {
+    bad++;
+  }
+}
+
+__device__ void flush_table(uint32_t* tab, uint32_t wb, uint32_t nr, int32_t* H) {
+  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) {
+    const uint32_t v = tab[i];
+    if (!v) continue;
+    tab[i] = 0;
+    const uint32_t cb = wb + 2 * i;
+    if (v & 0xffffu) atomicAdd(H + word_of(cb, nr), (int32_t)(v & 0xffffu));
+    if (v >> 16) atomicAdd(H + word_of(cb + 1, nr), (int32_t)(v >> 16));
+  }
+}
+
+// DYN = false: PRIVATE (fixed range per CTA); DYN = true: WINDOW (window follows the data)
+template <bool DYN>
+__global__ void __launch_bounds__(kThreadsSmem, 1)
+    k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
+                uint32_t nk, uint32_t n_ranges, uint64_t chunk, int32_t* __restrict__ H,
+                unsigned long long* d_n_invalid) {
+  extern __shared__ uint32_t tab[];
+  __shared__ uint32_t sh_wb[2];
+  const uint32_t range = DYN ? 0u : blockIdx.x % n_ranges;
+  const uint64_t ci = DYN ? blockIdx.x : blockIdx.x / n_ranges;
+  uint32_t wb = DYN ? kNoWindow : range * kTableBins;
+  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) tab[i] = 0;
+  const uint64_t a = ci * chunk;
+  const uint64_t e = a + chunk < n ? a + chunk : n;
   uint32_t bad = 0;
-  // chunk starts are multiples of 4 words: 128-bit loads for the body
-  const uint64_t a4 = a / 4, e4 = e / 4;
   const uint4* s4 = reinterpret_cast<const uint4*>(s);
-  for (uint64_t i = a4 + threadIdx.x; i < e4; i += blockDim.x) {
-    const uint4 v = __ldg(s4 + i);
-    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-    for (int q = 0; q < 4; q++) {
-      const uint32_t slot = w[q] >> 5, rs = w[q] & 31u;
-      if (slot < P && rs < nr) {
-        const uint32_t cb = slot * nr + rs - lo;
-        if (cb < range_bins) atomicAdd(cnt + cb, 1u);
-      } else {
-        bad++;
+  const uint64_t a4 = a / 4, e4 = e / 4;
+  __syncthreads();
+  uint32_t it = 0;
+  for (uint64_t t4 = a4; t4 < e4; t4 += kTile4, it++) {
+    const uint64_t t4e = t4 + kTile4 < e4 ? t4 + kTile4 : e4;
+    if (DYN) {
+      if (threadIdx.x == 0) {
+        uint32_t nwb = wb;
+        const uint32_t w = s[4 * t4], slot = w >> 5, rs = w & 31u;
+        if (slot < P && rs < nr) {
+          const uint32_t cb = slot * nr + rs;
+          if (wb == kNoWindow || cb - wb >= kTableBins) {
+            uint32_t lo = 0, hi = nk;  // kernel of the slot: last k with first <= slot
+            while (hi - lo > 1) {
+              const uint32_t mid = (lo + hi) >> 1;
+              if (kd[mid].first <= slot) lo = mid;
+              else hi = mid;
+            }
+            const uint32_t kb0 = kd[lo].first * nr, kbins = kd[lo].n * nr;
+            nwb = kbins <= kTableBins ? kb0 : (cb > kTableBins / 2 ? cb - kTableBins / 2 : 0);
+          }
+        }
+        if (nwb == kNoWindow) nwb = 0;  // first tile starts with an invalid sample
+        sh_wb[it & 1] = nwb;
+      }
+      __syncthreads();
+      const uint32_t nwb = sh_wb[it & 1];
+      if (nwb != wb) {
+        if (wb != kNoWindow) {
+          flush_table(tab, wb, nr, H);
+          __syncthreads();
+        }
+        wb = nwb;
       }
     }
-  }
-  for (uint64_t i = e4 * 4 + threadIdx.x; i < e; i += blockDim.x) {
-    const uint32_t w = s[i], slot = w >> 5, rs = w & 31u;
-    if (slot < P && rs < nr) {
-      const uint32_t cb = slot * nr + rs - lo;
-      if (cb < range_bins) atomicAdd(cnt + cb, 1u);
-    } else {
-      bad++;
+    uint64_t i = t4 + threadIdx.x;
+    for (; i + blockDim.x < t4e; i += 2 * blockDim.x) {  // two 128-bit loads in flight per thread
+      const uint4 v0 = __ldg(s4 + i), v1 = __ldg(s4 + i + blockDim.x);
+      count_one<DYN>(v0.x, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.y, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.z, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.w, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v1.x, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v1.y, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v1.z, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v1.w, P, nr, wb, tab, H, bad);
+    }
+    if (i < t4e) {
+      const uint4 v0 = __ldg(s4 + i);
+      count_one<DYN>(v0.x, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.y, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.z, P, nr, wb, tab, H, bad);
+      count_one<DYN>(v0.w, P, nr, wb, tab, H, bad);
     }
   }
+  for (uint64_t i = e4 * 4 + threadIdx.x; i < e; i += blockDim.x) count_one<DYN>(s[i], P, nr, wb, tab, H, bad);
   if (range == 0) count_invalid(bad, d_n_invalid);
   __syncthreads();
-  for (uint32_t b = threadIdx.x; b < range_bins; b += blockDim.x) {
-    const uint32_t v = cnt[b];
-    if (v) {
-      const uint32_t cbg = lo + b;
-      atomicAdd(H + (cbg / nr) * 32u + cbg % nr, (int32_t)v);
-    }
-  }
+  if (wb != kNoWindow) flush_table(tab, wb, nr, H);
 }
 
 }  // namespace
@@ -132,7 +211,8 @@ gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_
                            unsigned long long* d_n_invalid) {
   if (!n) return GS_OK;
   k_pack<<<(unsigned)((n + 255) / 256), 256, 0, c->stream>>>(d_raw, n, c->d_kd, c->n_kernels, c->cfg.n_reasons,
-                                                             d_words, d_n_invalid); count_launch();
+                                                             d_words, d_n_invalid);
+  count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }
@@ -143,45 +223,55 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
   if (zero_first && !accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, (uint64_t)P * 32 * 4, st));
   if (!n) return GS_OK;
+  if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
   int dev_sms = 148;
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
-  const uint64_t compact = (uint64_t)P * nr;
-  uint32_t mode = c->cfg.hist_mode;
-  const uint32_t n_ranges = (uint32_t)((compact + kRangeBins - 1) / kRangeBins);
-  if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
   // peel the words before the first 16-byte boundary so the main kernels use 128-bit loads
   const uint64_t head = std::min<uint64_t>(n, ((16u - (reinterpret_cast<uintptr_t>(d_words) & 15u)) & 15u) / 4u);
   if (head) {
-    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P, nr, d_hist, d_n_invalid); count_launch();
+    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P, nr, d_hist, d_n_invalid);
+    count_launch();
     GS_CUDA(c, cudaGetLastError());
     d_words += head;
     n -= head;
     if (!n) return GS_OK;
   }
-  if (mode == GS_HIST_AUTO) mode = (n_ranges <= kMaxRanges) ? GS_HIST_PRIVATE : GS_HIST_GLOBAL;
-  if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_GLOBAL;
-  if (mode == GS_HIST_WINDOW) mode = GS_HIST_GLOBAL;  // not implemented yet
+  const uint64_t compact = (uint64_t)P * nr;
+  const uint32_t n_ranges = (uint32_t)std::max<uint64_t>(1, (compact + kTableBins - 1) / kTableBins);
+  uint32_t mode = c->cfg.hist_mode;
+  if (mode == GS_HIST_AUTO) mode = n_ranges <= kMaxRanges ? GS_HIST_PRIVATE : GS_HIST_WINDOW;
+  if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_WINDOW;
   c->last_hist_mode = (int)mode;
   if (mode == GS_HIST_GLOBAL) {
-    const uint64_t blocks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 4, (n + kThreads * 4 - 1) / (kThreads * 4)));
-    k_hist_global<<<(unsigned)blocks, kThreads, 0, st>>>(d_words, n, P, nr, d_hist, d_n_invalid); count_launch();
+    const uint64_t blocks = std::max<uint64_t>(
+        1, std::min<uint64_t>((uint64_t)dev_sms * 4, (n + kThreadsGlobal * 4 - 1) / (kThreadsGlobal * 4)));
+    k_hist_global<<<(unsigned)blocks, kThreadsGlobal, 0, st>>>(d_words, n, P, nr, d_hist, d_n_invalid);
+    count_launch();
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
-  // PRIVATE: bins per range, chunk size so that every CTA sees >= 4 samples per bin of its range
-  const uint32_t range_bins = (uint32_t)((compact + n_ranges - 1) / n_ranges);
-  const size_t smem = (size_t)range_bins * 4;
-  GS_CUDA(c, cudaFuncSetAttribute(k_hist_private, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int per_sm = 1;
-  GS_CUDA(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_hist_private, kThreads, smem));
-  per_sm = std::max(per_sm, 1);
-  uint64_t chunks = std::max<uint64_t>(1, ((uint64_t)dev_sms * per_sm) / n_ranges);
-  chunks = std::min<uint64_t>(chunks, std::max<uint64_t>(1, n / (4ull * range_bins)));
+  const size_t smem = (size_t)kTableWords * 4;
+  const bool dyn = mode == GS_HIST_WINDOW;
+  uint64_t chunks;
+  if (dyn) {
+    chunks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms, n / (2ull * kTableBins) + 1));
+  } else {
+    chunks = std::max<uint64_t>(1, (uint64_t)dev_sms / n_ranges);
+    chunks = std::min<uint64_t>(chunks, std::max<uint64_t>(1, n / (2ull * kTableBins)));
+  }
   uint64_t chunk = (n + chunks - 1) / chunks;
   chunk = (chunk + 3) & ~3ull;
   chunks = (n + chunk - 1) / chunk;
-  k_hist_private<<<(unsigned)(chunks * n_ranges), kThreads, smem, st>>>(d_words, n, P, nr, n_ranges, range_bins, chunk,
-                                                                       d_hist, d_n_invalid); count_launch();
+  if (dyn) {
+    GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k_hist_smem<true><<<(unsigned)chunks, kThreadsSmem, smem, st>>>(d_words, n, P, nr, c->d_kd, c->n_kernels, 1, chunk,
+                                                                    d_hist, d_n_invalid);
+  } else {
+    GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k_hist_smem<false><<<(unsigned)(chunks * n_ranges), kThreadsSmem, smem, st>>>(
+        d_words, n, P, nr, c->d_kd, c->n_kernels, n_ranges, chunk, d_hist, d_n_invalid);
+  }
+  count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }

@@ -1,0 +1,102 @@
+"""Histogram strategies on the GPU against closed forms at full bench sizes.
+
+The expected histogram of a generated trace is its exact-count table (gen/samples.py), so the
+whole H can be compared bin by bin even at 2^30 samples (SURVEY §8c O13 pin).
+"""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+MODES = [0, 1, 2, 3]   # AUTO, GLOBAL, PRIVATE, WINDOW
+
+
+@pytest.fixture(scope="module")
+def gs():
+    import torch
+    import paper_conf_sc_senvs23_b200 as g
+    from paper_conf_sc_senvs23_b200 import build
+    build.build()
+    assert torch.cuda.is_available()
+    return g
+
+
+def _check(gs, s, tr, modes, words=None):
+    import torch
+    from gen.device import DeviceTrace
+    if words is None:
+        words = DeviceTrace(tr).packed()
+    want = torch.from_numpy(tr.table.astype(np.int32).reshape(-1)).cuda()
+    for mode in modes:
+        ctx = gs.Context(hist_mode=mode)
+        ctx.load_sass(s.text)
+        hist, ninv = ctx.attribute_samples(words)
+        torch.cuda.synchronize()
+        assert int(ninv.item()) == 0, mode
+        assert torch.equal(hist, want), (mode, int((hist != want).sum().item()))
+        ctx.close()
+
+
+@pytest.mark.parametrize("order", ["trace", "shuffled"])
+def test_c4_full_size_closed_form(gs, order):
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C4")
+    tab = gsm.table_c4(s.cls, s.first_slot, s.n_instr, 1 << 30, key=0x6E5C0004)
+    tr = gsm.Trace(tab, s.first_slot, s.n_instr, order=order, seed=1)
+    _check(gs, s, tr, [0, 3] if order == "trace" else [0, 1, 3])
+
+
+def test_c5_skew_closed_form(gs):
+    """90% of 200M samples on 10 PCs: hot bins receive >> 2^16 increments per CTA, exercising the
+    16-bit drain path of the shared-memory table."""
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C5")
+    hot = [int(f) + 40 for f in s.first_slot[:10]]
+    tab = gsm.table_c5(s.cls, hot, 200_000_000, key=0x6E5C0005)
+    assert tab.max() > 1 << 20
+    tr = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=2)
+    _check(gs, s, tr, MODES)
+
+
+def test_single_bin_drain(gs):
+    """All samples on one bin: every CTA drains that 16-bit counter many times."""
+    import torch
+    from gen import sass as gsass
+    s = gsass.config_sass("C1")
+    n = 3_000_000
+    words = torch.full((n,), (17 << 5) | 6, dtype=torch.int32, device="cuda")
+    for mode in MODES:
+        ctx = gs.Context(hist_mode=mode)
+        ctx.load_sass(s.text)
+        hist, ninv = ctx.attribute_samples(words)
+        torch.cuda.synchronize()
+        h = hist.view(-1, 32)
+        assert int(h[17, 6].item()) == n and int(h.sum().item()) == n and int(ninv.item()) == 0
+        ctx.close()
+
+
+@pytest.mark.parametrize("offset", [0, 1, 2, 3])
+def test_unaligned_views_and_invalid_words(gs, offset):
+    import torch
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    tab = gsm.table_class_weighted(s.cls, 2_000_000, key=4)
+    tr = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=4)
+    base = torch.from_numpy(tr.packed().view(np.int32)).cuda()
+    bad = torch.tensor([-1, (s.P << 5) | 1, (3 << 5) | 19, (3 << 5) | 31], dtype=torch.int32, device="cuda")
+    buf = torch.cat([torch.zeros(offset, dtype=torch.int32, device="cuda"), bad, base, bad])
+    view = buf[offset:]
+    want = torch.from_numpy(tab.astype(np.int32).reshape(-1)).cuda()
+    for mode in MODES:
+        ctx = gs.Context(hist_mode=mode)
+        ctx.load_sass(s.text)
+        hist, ninv = ctx.attribute_samples(view)
+        torch.cuda.synchronize()
+        assert int(ninv.item()) == 8 and torch.equal(hist, want), mode
+        # accumulate=True adds on top
+        hist2, _ = ctx.attribute_samples(view, hist=hist.clone(), accumulate=True)
+        assert torch.equal(hist2, 2 * want)
+        ctx.close()

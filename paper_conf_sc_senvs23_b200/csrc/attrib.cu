@@ -36,10 +36,10 @@ namespace {
 
 constexpr int kThreadsGlobal = 512;
 constexpr int kThreadsSmem = 1024;
-constexpr uint32_t kTableWords = 56 * 1024;        // 224 KB of shared memory
-constexpr uint32_t kTableBins = 2 * kTableWords;   // 114688 16-bit counters
+constexpr uint32_t kTableWords = 56 * 1024 - 32;   // 224 KB of shared memory: 32-bit counters + 32 spares
 constexpr uint32_t kMaxRanges = 3;
-constexpr uint32_t kTile4 = 8192;                  // uint4 per window decision (32K samples)
+constexpr uint32_t kTile4 = 65536;                 // uint4 per window decision (256K samples)
+constexpr int kVec = 4;                            // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
 
 __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long* d_n_invalid) {
@@ -92,54 +92,83 @@ __global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* 
 }
 
 // -------------------------------------------------------------------------------- shared-memory table
-__device__ __forceinline__ uint32_t word_of(uint32_t cb, uint32_t nr) { return (cb / nr) * 32u + cb % nr; }
+// The table holds kTableWords 32-bit counters for the compact bins of a window of whole slots
+// [ws, ws + nslots), nslots = kTableWords / n_reasons: counter index (slot - ws) * n_reasons + reason.
+// Fast path per sample (8 instructions): d = (w >> 5) - ws; in = d < nslots && (w & 31) < nr;
+// smem[d * nr + (w & 31)] += 1 (no return value). Lanes outside the window take a warp-uniform
+// slow path: L2 atomic (WINDOW) / skip (PRIVATE: another CTA owns that range) / invalid count.
 
-// one sample: shared-memory 16-bit counter if inside the window; outside it an L2 atomic (WINDOW)
-// or nothing (PRIVATE: another CTA owns that range)
 template <bool SPILL_OUT>
-__device__ __forceinline__ void count_one(uint32_t w, uint32_t P, uint32_t nr, uint32_t wb, uint32_t* tab,
-                                          int32_t* H, uint32_t& bad) {
-  const uint32_t slot = w >> 5, rs = w & 31u;
-  if (slot < P && rs < nr) {
-    const uint32_t off = slot * nr + rs - wb;
-    if (off < kTableBins) {
-      const uint32_t sh = (off & 1u) << 4;
-      const uint32_t old = atomicAdd(tab + (off >> 1), 1u << sh);
-      if (((old >> sh) & 0xffffu) == 0x7fffu) {  // drain: keep every 16-bit half below 2^16
-        atomicSub(tab + (off >> 1), 0x8000u << sh);
-        atomicAdd(H + w, 0x8000);
-      }
-    } else if (SPILL_OUT) {
-      atomicAdd(H + w, 1);
-    }
+__device__ __forceinline__ void slow_one(uint32_t w, uint32_t P, uint32_t nr, int32_t* H, uint32_t& bad) {
+  if ((w >> 5) < P && (w & 31u) < nr) {
+    if (SPILL_OUT) atomicAdd(H + w, 1);
   } else {
     bad++;
   }
 }
 
-__device__ void flush_table(uint32_t* tab, uint32_t wb, uint32_t nr, int32_t* H) {
-  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) {
-    const uint32_t v = tab[i];
-    if (!v) continue;
-    tab[i] = 0;
-    const uint32_t cb = wb + 2 * i;
-    if (v & 0xffffu) atomicAdd(H + word_of(cb, nr), (int32_t)(v & 0xffffu));
-    if (v >> 16) atomicAdd(H + word_of(cb + 1, nr), (int32_t)(v >> 16));
+// predicated shared-memory add of `one` (a run-time 1, so ptxas emits one predicated ATOMS.ADD
+// instead of a branch around ATOMS.POPC.INC)
+__device__ __forceinline__ void red_shared_add_if(uint32_t addr, uint32_t one, bool p) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}" ::"r"(addr), "r"(one),
+      "r"((uint32_t)p)
+      : "memory");
+}
+
+template <bool SPILL_OUT, int N>
+__device__ __forceinline__ void count_batch(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
+                                            uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
+                                            uint32_t& bad) {
+  uint32_t n_out = 0;
+#pragma unroll
+  for (int q = 0; q < N; q++) {
+    const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
+    const bool in = d < nslots && rs < nr;
+    // unconditional shared atomic: lanes outside the window add 0 to a spare word (no branch)
+    atomicAdd(tab + (in ? d * nr + rs : kTableWords + (threadIdx.x & 31u)), in ? one : 0u);
+    n_out += in ? 0u : 1u;
+  }
+  if (__any_sync(__activemask(), n_out)) {  // rare: some lane saw a sample outside the window
+#pragma unroll
+    for (int q = 0; q < N; q++) {
+      const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
+      if (!(d < nslots && rs < nr)) slow_one<SPILL_OUT>(w[q], P, nr, H, bad);
+    }
   }
 }
 
-// DYN = false: PRIVATE (fixed range per CTA); DYN = true: WINDOW (window follows the data)
+// flush the window's counters into H and zero them; word i <-> slot ws + i / nr, reason i % nr
+__device__ void flush_table(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nwords, int32_t* H) {
+  const uint32_t step_q = blockDim.x / nr, step_r = blockDim.x % nr;
+  uint32_t q = threadIdx.x / nr, r = threadIdx.x % nr;
+  for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) {
+    const uint32_t v = tab[i];
+    if (v) {
+      tab[i] = 0;
+      atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)v);
+    }
+    q += step_q;
+    r += step_r;
+    if (r >= nr) { r -= nr; q++; }
+  }
+}
+
+// DYN = false: PRIVATE (fixed slot range per CTA); DYN = true: WINDOW (window follows the data)
 template <bool DYN>
 __global__ void __launch_bounds__(kThreadsSmem, 1)
     k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
-                uint32_t nk, uint32_t n_ranges, uint64_t chunk, int32_t* __restrict__ H,
+                uint32_t nk, uint32_t n_ranges, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
                 unsigned long long* d_n_invalid) {
   extern __shared__ uint32_t tab[];
-  __shared__ uint32_t sh_wb[2];
+  __shared__ uint32_t sh_ws[2];
+  const uint32_t nslots = kTableWords / nr, nwords = nslots * nr;
+  const uint32_t tab_s = (uint32_t)__cvta_generic_to_shared(tab);
   const uint32_t range = DYN ? 0u : blockIdx.x % n_ranges;
   const uint64_t ci = DYN ? blockIdx.x : blockIdx.x / n_ranges;
-  uint32_t wb = DYN ? kNoWindow : range * kTableBins;
-  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) tab[i] = 0;
+  uint32_t ws = DYN ? kNoWindow : range * nslots;
+  uint32_t lim = DYN ? 0u : min(nslots, P - min(P, ws));  // slots of the window inside [0, P)
+  for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) tab[i] = 0;
   const uint64_t a = ci * chunk;
   const uint64_t e = a + chunk < n ? a + chunk : n;
   uint32_t bad = 0;
@@ -150,59 +179,76 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
   for (uint64_t t4 = a4; t4 < e4; t4 += kTile4, it++) {
     const uint64_t t4e = t4 + kTile4 < e4 ? t4 + kTile4 : e4;
     if (DYN) {
-      if (threadIdx.x == 0) {
-        uint32_t nwb = wb;
-        const uint32_t w = s[4 * t4], slot = w >> 5, rs = w & 31u;
-        if (slot < P && rs < nr) {
-          const uint32_t cb = slot * nr + rs;
-          if (wb == kNoWindow || cb - wb >= kTableBins) {
+      if (threadIdx.x < 32) {
+        // window for this tile: around the median slot of 32 evenly spaced samples (robust to the
+        // cold tail of a kernel's samples); whole kernel if it fits
+        const uint64_t span = t4e - t4;
+        const uint32_t w = s[4 * (t4 + span * threadIdx.x / 32)];
+        const bool ok = (w >> 5) < P && (w & 31u) < nr;
+        const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
+        uint32_t le = 0;  // lanes whose slot is <= mine
+        for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
+        const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
+        // median: the smallest valid slot with more than half of the valid samples at or below it
+        const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
+        if (threadIdx.x == 0) {
+          uint32_t nws = ws;
+          if (med != 0xffffffffu && (ws == kNoWindow || med - ws >= nslots || med - ws < nslots / 8 ||
+                                     med - ws >= nslots - nslots / 8)) {
             uint32_t lo = 0, hi = nk;  // kernel of the slot: last k with first <= slot
             while (hi - lo > 1) {
               const uint32_t mid = (lo + hi) >> 1;
-              if (kd[mid].first <= slot) lo = mid;
+              if (kd[mid].first <= med) lo = mid;
               else hi = mid;
             }
-            const uint32_t kb0 = kd[lo].first * nr, kbins = kd[lo].n * nr;
-            nwb = kbins <= kTableBins ? kb0 : (cb > kTableBins / 2 ? cb - kTableBins / 2 : 0);
+            const KDesc K = kd[lo];
+            uint32_t c;
+            if (K.n <= nslots) c = K.first;                         // the whole kernel fits
+            else {                                                  // centre on the median, inside the kernel
+              c = med > nslots / 2 ? med - nslots / 2 : 0;
+              c = min(max(c, K.first), K.first + K.n - nslots);
+            }
+            // keep the current window when the new one would not move it (already centred)
+            if (ws == kNoWindow || c != ws) nws = c;
           }
+          if (nws == kNoWindow) nws = 0;
+          sh_ws[it & 1] = nws;
         }
-        if (nwb == kNoWindow) nwb = 0;  // first tile starts with an invalid sample
-        sh_wb[it & 1] = nwb;
       }
       __syncthreads();
-      const uint32_t nwb = sh_wb[it & 1];
-      if (nwb != wb) {
-        if (wb != kNoWindow) {
-          flush_table(tab, wb, nr, H);
+      const uint32_t nws = sh_ws[it & 1];
+      if (nws != ws) {
+        if (ws != kNoWindow) {
+          flush_table(tab, ws, nr, lim * nr, H);
           __syncthreads();
         }
-        wb = nwb;
+        ws = nws;
+        lim = min(nslots, P - min(P, ws));
       }
     }
     uint64_t i = t4 + threadIdx.x;
-    for (; i + blockDim.x < t4e; i += 2 * blockDim.x) {  // two 128-bit loads in flight per thread
-      const uint4 v0 = __ldg(s4 + i), v1 = __ldg(s4 + i + blockDim.x);
-      count_one<DYN>(v0.x, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.y, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.z, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.w, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v1.x, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v1.y, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v1.z, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v1.w, P, nr, wb, tab, H, bad);
+    for (; i + (kVec - 1) * blockDim.x < t4e; i += kVec * blockDim.x) {  // kVec 128-bit loads in flight
+      uint32_t w[4 * kVec];
+#pragma unroll
+      for (int u = 0; u < kVec; u++) {
+        const uint4 v = __ldg(s4 + i + u * blockDim.x);
+        w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
+      }
+      count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
     }
-    if (i < t4e) {
-      const uint4 v0 = __ldg(s4 + i);
-      count_one<DYN>(v0.x, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.y, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.z, P, nr, wb, tab, H, bad);
-      count_one<DYN>(v0.w, P, nr, wb, tab, H, bad);
+    for (; i < t4e; i += blockDim.x) {
+      const uint4 v = __ldg(s4 + i);
+      const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+      count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
     }
   }
-  for (uint64_t i = e4 * 4 + threadIdx.x; i < e; i += blockDim.x) count_one<DYN>(s[i], P, nr, wb, tab, H, bad);
+  for (uint64_t i = e4 * 4 + threadIdx.x; i < e; i += blockDim.x) {
+    const uint32_t w[1] = {s[i]};
+    count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+  }
   if (range == 0) count_invalid(bad, d_n_invalid);
   __syncthreads();
-  if (wb != kNoWindow) flush_table(tab, wb, nr, H);
+  if (ws != kNoWindow) flush_table(tab, ws, nr, min(nwords, lim * nr), H);
 }
 
 }  // namespace
@@ -236,8 +282,8 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     n -= head;
     if (!n) return GS_OK;
   }
-  const uint64_t compact = (uint64_t)P * nr;
-  const uint32_t n_ranges = (uint32_t)std::max<uint64_t>(1, (compact + kTableBins - 1) / kTableBins);
+  const uint32_t nslots = kTableWords / nr;  // whole slots per shared-memory window
+  const uint32_t n_ranges = (uint32_t)std::max<uint64_t>(1, ((uint64_t)P + nslots - 1) / nslots);
   uint32_t mode = c->cfg.hist_mode;
   if (mode == GS_HIST_AUTO) mode = n_ranges <= kMaxRanges ? GS_HIST_PRIVATE : GS_HIST_WINDOW;
   if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_WINDOW;
@@ -250,14 +296,14 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
-  const size_t smem = (size_t)kTableWords * 4;
+  const size_t smem = (size_t)(kTableWords + 32) * 4;  // + one spare word per lane
   const bool dyn = mode == GS_HIST_WINDOW;
   uint64_t chunks;
   if (dyn) {
-    chunks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms, n / (2ull * kTableBins) + 1));
+    chunks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms, n / (2ull * kTableWords) + 1));
   } else {
     chunks = std::max<uint64_t>(1, (uint64_t)dev_sms / n_ranges);
-    chunks = std::min<uint64_t>(chunks, std::max<uint64_t>(1, n / (2ull * kTableBins)));
+    chunks = std::min<uint64_t>(chunks, std::max<uint64_t>(1, n / (2ull * kTableWords)));
   }
   uint64_t chunk = (n + chunks - 1) / chunks;
   chunk = (chunk + 3) & ~3ull;
@@ -265,11 +311,11 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   if (dyn) {
     GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     k_hist_smem<true><<<(unsigned)chunks, kThreadsSmem, smem, st>>>(d_words, n, P, nr, c->d_kd, c->n_kernels, 1, chunk,
-                                                                    d_hist, d_n_invalid);
+                                                                    1u, d_hist, d_n_invalid);
   } else {
     GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     k_hist_smem<false><<<(unsigned)(chunks * n_ranges), kThreadsSmem, smem, st>>>(
-        d_words, n, P, nr, c->d_kd, c->n_kernels, n_ranges, chunk, d_hist, d_n_invalid);
+        d_words, n, P, nr, c->d_kd, c->n_kernels, n_ranges, chunk, 1u, d_hist, d_n_invalid);
   }
   count_launch();
   GS_CUDA(c, cudaGetLastError());

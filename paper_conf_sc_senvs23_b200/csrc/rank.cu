@@ -1,13 +1,16 @@
 // rank.cu — join of the histogram onto the flagged sites and their ranking
 // (§3.2; rank key R20).
 //
-//   k_ktot   per kernel: total samples of the kernel (denominator of tot/ktot).
+//   k_ktot   per kernel: total samples of the kernel (denominator of tot/ktot), 128-bit loads,
+//            several CTAs per kernel.
 //   k_join   per site: tot = sum of the site PC's row, rel = sum over REL(rule) (P:556-563,
-//            P:616-624; CONV: all reasons). Writes ~tot / ~rel keys.
-//   sort     two stable LSD radix sorts (CUB DeviceRadixSort): by ~tot, then by ~rel. The sites
-//            enter in (kernel, idx, rule) order, so stability yields the total order
-//            (rel desc, tot desc, kernel, idx, rule).
-//   k_emit   the first k rows as gs_ranked_site.
+//            P:616-624; CONV: all reasons); running maxima of rel and tot.
+//   sort     the sites enter in (kernel, idx, rule) order, so a STABLE ascending sort on
+//            (maxR - rel, maxT - tot) yields the total order (rel desc, tot desc, kernel, idx,
+//            rule). When bits(maxR) + bits(maxT) <= 64 the two fields are packed into one 64-bit
+//            key and sorted once over exactly those bits (CUB onesweep radix sort); otherwise two
+//            stable passes (by tot, then by rel).
+//   k_emit   the first k rows as gs_ranked_site (one warp per row).
 #include <cub/device/device_radix_sort.cuh>
 #include <cuda_runtime.h>
 
@@ -17,9 +20,6 @@
 
 namespace gs {
 namespace {
-
-// onesweep radix sort of 64-bit keys: 1 histogram + 1 exclusive-sum + 8 digit passes
-constexpr uint64_t kCubSortLaunches = 10;
 
 __constant__ uint32_t kRelMask[7] = {
     1u << 6,                // VEC   long_scoreboard
@@ -31,62 +31,97 @@ __constant__ uint32_t kRelMask[7] = {
     0xffffffffu,            // CONV  all reasons (reading)
 };
 
-__global__ void k_ktot(const int32_t* __restrict__ H, const KDesc* __restrict__ kd, uint32_t nk,
-                       unsigned long long* __restrict__ ktot) {
+constexpr int kKtotThreads = 512;
+constexpr uint32_t kKtotSlotsPerCta = 1024;  // 128 KB of histogram per CTA
+
+// grid.x = kernel, grid.y = slice of the kernel's slots
+__global__ void __launch_bounds__(kKtotThreads) k_ktot(const int32_t* __restrict__ H, const KDesc* __restrict__ kd,
+                                                       uint32_t nk, unsigned long long* __restrict__ ktot) {
   const uint32_t k = blockIdx.x;
   if (k >= nk) return;
   const KDesc K = kd[k];
-  const uint64_t a = (uint64_t)K.first * 32, e = a + (uint64_t)K.n * 32;
+  const uint32_t s0 = blockIdx.y * kKtotSlotsPerCta;
+  if (s0 >= K.n) return;
+  const uint32_t s1 = min(K.n, s0 + kKtotSlotsPerCta);
+  const int4* h4 = reinterpret_cast<const int4*>(H + (uint64_t)(K.first + s0) * 32);
+  const uint32_t n4 = (s1 - s0) * 8;
   unsigned long long s = 0;
-  for (uint64_t i = a + threadIdx.x; i < e; i += blockDim.x) s += (uint32_t)H[i];
+  for (uint32_t i = threadIdx.x; i < n4; i += blockDim.x) {
+    const int4 v = __ldg(h4 + i);
+    s += (uint32_t)v.x + (uint64_t)(uint32_t)v.y + (uint32_t)v.z + (uint64_t)(uint32_t)v.w;
+  }
   for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  __shared__ unsigned long long ws[32];
+  __shared__ unsigned long long ws[kKtotThreads / 32];
   if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
   __syncthreads();
   if (threadIdx.x == 0) {
     unsigned long long t = 0;
-    for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += ws[w];
-    ktot[k] = t;
+    for (int w = 0; w < kKtotThreads / 32; w++) t += ws[w];
+    atomicAdd(ktot + k, t);
   }
 }
 
 __global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H,
-                       const KDesc* __restrict__ kd, unsigned long long* __restrict__ key_tot,
-                       unsigned long long* __restrict__ key_rel, uint32_t* __restrict__ vals) {
+                       const KDesc* __restrict__ kd, unsigned long long* __restrict__ rel_out,
+                       unsigned long long* __restrict__ tot_out, unsigned long long* __restrict__ mx) {
+  const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  unsigned long long tot = 0, rel = 0;
+  if (s < ns) {
+    const gs_site st = sites[s];
+    const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx;
+    const int4* row = reinterpret_cast<const int4*>(H + slot * 32);
+    const uint32_t m = kRelMask[st.rule];
+#pragma unroll
+    for (int q = 0; q < 8; q++) {
+      const int4 v = __ldg(row + q);
+      const uint32_t c[4] = {(uint32_t)v.x, (uint32_t)v.y, (uint32_t)v.z, (uint32_t)v.w};
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        tot += c[t];
+        if ((m >> (4 * q + t)) & 1u) rel += c[t];
+      }
+    }
+    rel_out[s] = rel;
+    tot_out[s] = tot;
+  }
+  unsigned long long mr = rel, mt = tot;
+  for (int o = 16; o; o >>= 1) {
+    mr = max(mr, __shfl_xor_sync(0xffffffffu, mr, o));
+    mt = max(mt, __shfl_xor_sync(0xffffffffu, mt, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(mx, mr);
+    atomicMax(mx + 1, mt);
+  }
+}
+
+// key = ((maskR - rel) << bt) | (maskT - tot); vals = site index
+__global__ void k_keys_packed(const unsigned long long* __restrict__ rel, const unsigned long long* __restrict__ tot,
+                              uint64_t ns, int bt, unsigned long long mask_r, unsigned long long mask_t,
+                              unsigned long long* __restrict__ keys, uint32_t* __restrict__ vals) {
   const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (s >= ns) return;
-  const gs_site st = sites[s];
-  const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx;
-  const int4* row = reinterpret_cast<const int4*>(H + slot * 32);
-  const uint32_t m = kRelMask[st.rule];
-  unsigned long long tot = 0, rel = 0;
-#pragma unroll
-  for (int q = 0; q < 8; q++) {
-    const int4 v = __ldg(row + q);
-    const uint32_t c[4] = {(uint32_t)v.x, (uint32_t)v.y, (uint32_t)v.z, (uint32_t)v.w};
-#pragma unroll
-    for (int t = 0; t < 4; t++) {
-      tot += c[t];
-      if ((m >> (4 * q + t)) & 1u) rel += c[t];
-    }
-  }
-  key_tot[s] = ~tot;
-  key_rel[s] = ~rel;
+  keys[s] = ((mask_r - rel[s]) << bt) | (mask_t - tot[s]);
   vals[s] = (uint32_t)s;
 }
 
-__global__ void k_gather_keys(const uint32_t* __restrict__ order, const unsigned long long* __restrict__ key_rel,
-                              uint64_t ns, unsigned long long* __restrict__ out) {
+// one field: key = mask - val[order[i]] (order == nullptr: identity, vals = i)
+__global__ void k_keys_field(const unsigned long long* __restrict__ val, const uint32_t* __restrict__ order,
+                             uint64_t ns, unsigned long long mask, unsigned long long* __restrict__ keys,
+                             uint32_t* __restrict__ vals) {
   const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (i < ns) out[i] = key_rel[order[i]];
+  if (i >= ns) return;
+  const uint32_t s = order ? order[i] : (uint32_t)i;
+  keys[i] = mask - val[s];
+  if (!order) vals[i] = s;
 }
 
 __global__ void k_emit(const uint32_t* __restrict__ order, uint64_t kk, const gs_site* __restrict__ sites,
                        const int32_t* __restrict__ H, const KDesc* __restrict__ kd,
                        const unsigned long long* __restrict__ ktot, gs_ranked_site* __restrict__ out) {
-  const uint64_t q = blockIdx.x;  // one warp per row
+  const uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);  // one warp per row
   if (q >= kk) return;
-  const int lane = threadIdx.x;
+  const int lane = threadIdx.x & 31;
   const gs_site st = sites[order[q]];
   const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx;
   const uint32_t c = (uint32_t)H[slot * 32 + lane];
@@ -109,6 +144,9 @@ __global__ void k_emit(const uint32_t* __restrict__ order, uint64_t kk, const gs
   }
 }
 
+int bits_of(unsigned long long v) { return v ? 64 - __builtin_clzll(v) : 0; }
+unsigned long long mask_of(int b) { return b >= 64 ? ~0ull : ((1ull << b) - 1); }
+
 }  // namespace
 
 gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, bool out_is_host,
@@ -116,9 +154,15 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
   cudaStream_t st = c->stream;
   const uint64_t ns = c->n_sites;
   const uint64_t kk = std::min<uint64_t>(k, ns);
-  if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, (uint64_t)std::max<uint32_t>(c->n_kernels, 1) * 8));
+  if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8));
+  unsigned long long* d_max = c->d_ktot + std::max<uint32_t>(c->n_kernels, 1);
+  GS_CUDA(c, cudaMemsetAsync(c->d_ktot, 0, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8, st));
   if (c->n_kernels) {
-    k_ktot<<<c->n_kernels, 256, 0, st>>>(d_hist, c->d_kd, c->n_kernels, c->d_ktot); count_launch();
+    uint32_t max_n = 1;
+    for (const auto& K : c->kd_h) max_n = std::max(max_n, K.n);
+    dim3 grid(c->n_kernels, (max_n + kKtotSlotsPerCta - 1) / kKtotSlotsPerCta);
+    k_ktot<<<grid, kKtotThreads, 0, st>>>(d_hist, c->d_kd, c->n_kernels, c->d_ktot);
+    count_launch();
     GS_CUDA(c, cudaGetLastError());
   }
   if (ns) {
@@ -134,48 +178,67 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
         GS_CUDA(c, cudaMalloc((void**)&c->d_rank_keys[b], ns * 8));
         GS_CUDA(c, cudaMalloc((void**)&c->d_rank_vals[b], ns * 4));
       }
-      // a third key buffer holds ~rel in site order
+      c->rank_cap = ns;
+    }
+    unsigned long long* k0 = c->d_rank_keys[0];
+    unsigned long long* k1 = c->d_rank_keys[1];
+    uint32_t* v0 = c->d_rank_vals[0];
+    uint32_t* v1 = c->d_rank_vals[1];
+    size_t cub_bytes = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, k0, k1, v0, v1, (int)ns, 0, 64, st);
+    const size_t arr = ((ns * 8 + 255) / 256) * 256;  // rel and tot arrays live in the temp block
+    if (c->sort_tmp_bytes < cub_bytes + 2 * arr) {
       if (c->d_sort_tmp) cudaFree(c->d_sort_tmp);
       c->d_sort_tmp = nullptr;
       c->sort_tmp_bytes = 0;
-      c->rank_cap = ns;
+      GS_CUDA(c, cudaMalloc(&c->d_sort_tmp, cub_bytes + 2 * arr));
+      c->sort_tmp_bytes = cub_bytes + 2 * arr;
     }
-    unsigned long long* key_tot = c->d_rank_keys[0];
-    unsigned long long* key_tmp = c->d_rank_keys[1];
-    uint32_t* v0 = c->d_rank_vals[0];
-    uint32_t* v1 = c->d_rank_vals[1];
-    // CUB temp storage also hosts the ~rel array (site order)
-    size_t cub_bytes = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, key_tot, key_tmp, v0, v1, (int)ns, 0, 64, st);
-    const size_t rel_bytes = ((ns * 8 + 255) / 256) * 256;
-    if (c->sort_tmp_bytes < cub_bytes + rel_bytes) {
-      if (c->d_sort_tmp) cudaFree(c->d_sort_tmp);
-      c->d_sort_tmp = nullptr;
-      GS_CUDA(c, cudaMalloc(&c->d_sort_tmp, cub_bytes + rel_bytes));
-      c->sort_tmp_bytes = cub_bytes + rel_bytes;
-    }
-    unsigned long long* key_rel = reinterpret_cast<unsigned long long*>(c->d_sort_tmp);
-    void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + rel_bytes;
+    unsigned long long* d_rel = reinterpret_cast<unsigned long long*>(c->d_sort_tmp);
+    unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
+    void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
     const unsigned grid = (unsigned)((ns + 255) / 256);
-    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, c->d_kd, key_tot, key_rel, v0); count_launch();
+    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, c->d_kd, d_rel, d_tot, d_max);
+    count_launch();
     GS_CUDA(c, cudaGetLastError());
+    unsigned long long mx[2];
+    GS_CUDA(c, cudaMemcpyAsync(mx, d_max, 16, cudaMemcpyDeviceToHost, st));
+    GS_CUDA(c, cudaStreamSynchronize(st));
+    const int br = bits_of(mx[0]), bt = bits_of(mx[1]);
+    const uint32_t* order = v0;
     size_t b1 = cub_bytes;
-    GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, key_tot, key_tmp, v0, v1, (int)ns, 0, 64, st));
-    count_launch(kCubSortLaunches);
-    // v1 = sites ordered by tot desc (stable); now sort by rel desc, stable
-    k_gather_keys<<<grid, 256, 0, st>>>(v1, key_rel, ns, key_tot); count_launch();
+    auto passes = [](int bits) { return (uint64_t)(bits + 7) / 8 + 2; };  // onesweep digits + hist + scan
+    if (br + bt <= 64) {
+      k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
+      count_launch();
+      if (br + bt > 0) {
+        cub::DoubleBuffer<unsigned long long> dk(k0, k1);
+        cub::DoubleBuffer<uint32_t> dv(v0, v1);
+        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, dk, dv, (int)ns, 0, br + bt, st));
+        count_launch(passes(br + bt));
+        order = dv.Current();
+      }
+    } else {
+      k_keys_field<<<grid, 256, 0, st>>>(d_tot, nullptr, ns, mask_of(bt), k0, v0);
+      count_launch();
+      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v0, v1, (int)ns, 0, bt, st));
+      count_launch(passes(bt));
+      k_keys_field<<<grid, 256, 0, st>>>(d_rel, v1, ns, mask_of(br), k0, nullptr);
+      count_launch();
+      b1 = cub_bytes;
+      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v1, v0, (int)ns, 0, br, st));
+      count_launch(passes(br));
+      order = v0;
+    }
     GS_CUDA(c, cudaGetLastError());
-    b1 = cub_bytes;
-    GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, key_tot, key_tmp, v1, v0, (int)ns, 0, 64, st));
-    count_launch(kCubSortLaunches);
-    // v0 = final order
     if (kk) {
       gs_ranked_site* dst = out;
       if (out_is_host) {
         GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
         dst = c->d_ranked;
       }
-      k_emit<<<(unsigned)kk, 32, 0, st>>>(v0, kk, c->d_sites, d_hist, c->d_kd, c->d_ktot, dst); count_launch();
+      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, c->d_kd, c->d_ktot, dst);
+      count_launch();
       GS_CUDA(c, cudaGetLastError());
       if (out_is_host)
         GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));

@@ -192,6 +192,7 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--order", default="trace", choices=["trace", "shuffled"])
     ap.add_argument("--hist-mode", type=int, default=0)
+    ap.add_argument("--hist-bits", type=int, default=0, choices=[0, 16, 32])
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-samples", type=int, default=1 << 25)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -220,7 +221,7 @@ def main():
     kb, ke = gdist.kernel_range(s.n_instr, rank, world)
     words = DeviceTrace(tr, local).packed(a, b)
     n_local = b - a
-    ctx = g.Context(device=local, hist_mode=args.hist_mode)
+    ctx = g.Context(device=local, hist_mode=args.hist_mode, hist_counter_bits=args.hist_bits)
     ctx.load_sass(s.text)
     P = ctx.n_instr
     hist = torch.empty(P * 32, dtype=torch.int32, device="cuda")

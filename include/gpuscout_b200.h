@@ -47,7 +47,8 @@ typedef struct {
   uint32_t shmem_min_arith; /* T_A of the SHMEM rule (R11). default 1                                 */
   uint32_t shmem_min_loads; /* T_L of the SHMEM rule (R11). default 2                                 */
   uint32_t hist_mode;       /* histogram strategy, GS_HIST_*. default GS_HIST_AUTO                    */
-  uint32_t reserved[3];
+  uint32_t hist_counter_bits; /* shared-memory counter width: 0 = auto, 16 (packed pairs) or 32      */
+  uint32_t reserved[2];
 } gs_config;
 
 enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3 };

@@ -34,7 +34,8 @@ KSTATS_DTYPE = np.dtype([("n_gatom", "<u4"), ("n_satom", "<u4"), ("n_conv", "<u4
 class GsConfig(ctypes.Structure):
     _fields_ = [("trace_depth", ctypes.c_uint32), ("n_reasons", ctypes.c_uint32),
                 ("shmem_min_arith", ctypes.c_uint32), ("shmem_min_loads", ctypes.c_uint32),
-                ("hist_mode", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+                ("hist_mode", ctypes.c_uint32), ("hist_counter_bits", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32 * 2)]
 
 
 class GsError(RuntimeError):
@@ -104,7 +105,8 @@ class Context:
     """One gs_ctx bound to a CUDA device and stream (default: torch's current stream)."""
 
     def __init__(self, device: int | None = None, stream=None, trace_depth: int = 64, n_reasons: int = 19,
-                 shmem_min_arith: int = 1, shmem_min_loads: int = 2, hist_mode: int = GS_HIST_AUTO):
+                 shmem_min_arith: int = 1, shmem_min_loads: int = 2, hist_mode: int = GS_HIST_AUTO,
+                 hist_counter_bits: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise GsError("no CUDA device: the library has no CPU fallback")
@@ -114,7 +116,7 @@ class Context:
             stream = torch.cuda.current_stream(self.device)
         self.torch_stream = stream
         handle = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
-        cfg = GsConfig(trace_depth, n_reasons, shmem_min_arith, shmem_min_loads, hist_mode)
+        cfg = GsConfig(trace_depth, n_reasons, shmem_min_arith, shmem_min_loads, hist_mode, hist_counter_bits)
         self.n_reasons = n_reasons
         self.trace_depth = trace_depth
         self.cfg = cfg

@@ -154,32 +154,139 @@ __device__ void flush_table(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nw
   }
 }
 
+// ---- 16-bit packed variant: two counters per word, twice the bins per window. The increment
+// that takes a half from 0x7FFF to 0x8000 (bit 15 flips: (old ^ (old + inc)) & (inc << 15)) drains
+// 0x8000 to the global bin, so a half never carries into its neighbour (at most a few thousand
+// increments can be in flight per SM between that add and the drain). Counts stay exact.
+template <bool SPILL_OUT, int N>
+__device__ __forceinline__ void count_batch16(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
+                                              uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
+                                              uint32_t& bad) {
+  uint32_t n_out = 0, ovf = 0;
+  uint32_t old[N], inc[N], idx[N];
+#pragma unroll
+  for (int q = 0; q < N; q++) {
+    const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
+    const bool in = d < nslots && rs < nr;
+    const uint32_t off = d * nr + rs;
+    idx[q] = in ? (off >> 1) : kTableWords + (threadIdx.x & 31u);
+    inc[q] = in ? (one << ((off & 1u) << 4)) : 0u;
+    old[q] = atomicAdd(tab + idx[q], inc[q]);
+    ovf |= (old[q] ^ (old[q] + inc[q])) & (inc[q] << 15);
+    n_out += in ? 0u : 1u;
+  }
+  const uint32_t act = __activemask();
+  if (__any_sync(act, ovf)) {  // rare: a counter reached 0x8000
+#pragma unroll
+    for (int q = 0; q < N; q++)
+      if ((old[q] ^ (old[q] + inc[q])) & (inc[q] << 15)) {
+        atomicSub(tab + idx[q], inc[q] << 15);
+        atomicAdd(H + w[q], 0x8000);
+      }
+  }
+  if (__any_sync(act, n_out)) {  // rare: some lane saw a sample outside the window
+#pragma unroll
+    for (int q = 0; q < N; q++) {
+      const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
+      if (!(d < nslots && rs < nr)) slow_one<SPILL_OUT>(w[q], P, nr, H, bad);
+    }
+  }
+}
+
+// word i holds bins 2i (low half) and 2i + 1 (high half); bin b <-> slot ws + b / nr, reason b % nr
+__device__ void flush_table16(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H) {
+  const uint32_t stride = 2 * blockDim.x, step_q = stride / nr, step_r = stride % nr;
+  uint32_t q = (2 * threadIdx.x) / nr, r = (2 * threadIdx.x) % nr;
+  for (uint32_t i = threadIdx.x; 2 * i < nbins; i += blockDim.x) {
+    const uint32_t v = tab[i];
+    if (v) {
+      tab[i] = 0;
+      if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
+      if (v >> 16) {
+        const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
+        atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
+      }
+    }
+    q += step_q;
+    r += step_r;
+    if (r >= nr) { r -= nr; q++; }
+  }
+}
+
+template <bool P16, bool SPILL_OUT, int N>
+__device__ __forceinline__ void count_any(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
+                                          uint32_t lim, uint32_t* tab, uint32_t one, int32_t* H, uint32_t& bad) {
+  if (P16) count_batch16<SPILL_OUT>(w, P, nr, ws, lim, tab, one, H, bad);
+  else count_batch<SPILL_OUT>(w, P, nr, ws, lim, tab, one, H, bad);
+}
+
+// Tile queue of the WINDOW kernel. Chunk c (CTA c's contiguous share) is cut into tiles of kTile4
+// uint4; rng[c] = (head << 32) | stolen counts tiles taken from the front by the owner and from the
+// back by other CTAs that finished their own chunk (work stealing keeps all SMs busy to the end
+// while each CTA still walks its own chunk front to back, so windows change rarely).
+__device__ __forceinline__ uint32_t n_tiles(uint64_t c, uint64_t chunk, uint64_t n) {
+  const uint64_t a4 = c * chunk / 4, e = (c + 1) * chunk < n ? (c + 1) * chunk : n, e4 = e / 4;
+  return e4 > a4 ? (uint32_t)((e4 - a4 + kTile4 - 1) / kTile4) : 0u;
+}
+
+// returns (chunk << 32) | tile, or ~0 when every tile of every chunk has been taken
+__device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, uint32_t grid, uint64_t chunk,
+                                        uint64_t n) {
+  const uint32_t mine = n_tiles(me, chunk, n);
+  for (;;) {  // own chunk, front to back
+    const unsigned long long o = *(volatile unsigned long long*)(rng + me);
+    const uint32_t head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
+    if (head + stolen >= mine) break;
+    if (atomicCAS(rng + me, o, o + (1ull << 32)) == o) return ((unsigned long long)me << 32) | head;
+  }
+  for (;;) {  // steal from the back of the chunk with the most tiles left
+    uint32_t best = grid, best_left = 0;
+    for (uint32_t v = 0; v < grid; v++) {
+      const unsigned long long o = *(volatile unsigned long long*)(rng + v);
+      const uint32_t nt = n_tiles(v, chunk, n), used = (uint32_t)(o >> 32) + (uint32_t)o;
+      if (nt > used && nt - used > best_left) { best_left = nt - used; best = v; }
+    }
+    if (best == grid) return ~0ull;
+    const unsigned long long o = *(volatile unsigned long long*)(rng + best);
+    const uint32_t nt = n_tiles(best, chunk, n), head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
+    if (head + stolen >= nt) continue;
+    if (atomicCAS(rng + best, o, o + 1ull) == o) return ((unsigned long long)best << 32) | (nt - 1 - stolen);
+  }
+}
+
 // DYN = false: PRIVATE (fixed slot range per CTA); DYN = true: WINDOW (window follows the data)
-template <bool DYN>
+template <bool DYN, bool P16>
 __global__ void __launch_bounds__(kThreadsSmem, 1)
     k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
                 uint32_t nk, uint32_t n_ranges, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
-                unsigned long long* d_n_invalid) {
+                unsigned long long* d_n_invalid, unsigned long long* rng) {
   extern __shared__ uint32_t tab[];
   __shared__ uint32_t sh_ws[2];
-  const uint32_t nslots = kTableWords / nr, nwords = nslots * nr;
-  const uint32_t tab_s = (uint32_t)__cvta_generic_to_shared(tab);
+  __shared__ unsigned long long sh_tile[2];
+  const uint32_t nslots = (P16 ? 2 * kTableWords : kTableWords) / nr;
   const uint32_t range = DYN ? 0u : blockIdx.x % n_ranges;
   const uint64_t ci = DYN ? blockIdx.x : blockIdx.x / n_ranges;
   uint32_t ws = DYN ? kNoWindow : range * nslots;
   uint32_t lim = DYN ? 0u : min(nslots, P - min(P, ws));  // slots of the window inside [0, P)
-  for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) tab[i] = 0;
-  const uint64_t a = ci * chunk;
-  const uint64_t e = a + chunk < n ? a + chunk : n;
+  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) tab[i] = 0;
   uint32_t bad = 0;
   const uint4* s4 = reinterpret_cast<const uint4*>(s);
-  const uint64_t a4 = a / 4, e4 = e / 4;
   __syncthreads();
-  uint32_t it = 0;
-  for (uint64_t t4 = a4; t4 < e4; t4 += kTile4, it++) {
-    const uint64_t t4e = t4 + kTile4 < e4 ? t4 + kTile4 : e4;
+  uint64_t t4 = ci * chunk / 4;  // PRIVATE: walk the own chunk
+  const uint64_t e_own = (ci + 1) * chunk < n ? (ci + 1) * chunk : n, e4_own = e_own / 4;
+  for (uint32_t it = 0;; it++) {
+    uint64_t t4e;
     if (DYN) {
-      if (threadIdx.x < 32) {
+      const auto tile_span = [&](unsigned long long tile) {
+        const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
+        const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
+        t4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
+        t4e = t4 + kTile4 < ce / 4 ? t4 + kTile4 : ce / 4;
+      };
+      if (threadIdx.x == 0) sh_tile[it & 1] = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
+      __syncwarp();
+      if (threadIdx.x < 32 && sh_tile[it & 1] != ~0ull) {
+        tile_span(sh_tile[it & 1]);
         // window for this tile: around the median slot of 32 evenly spaced samples (robust to the
         // cold tail of a kernel's samples); whole kernel if it fits
         const uint64_t span = t4e - t4;
@@ -202,29 +309,35 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
               else hi = mid;
             }
             const KDesc K = kd[lo];
-            uint32_t c;
-            if (K.n <= nslots) c = K.first;                         // the whole kernel fits
+            uint32_t cws;
+            if (K.n <= nslots) cws = K.first;                       // the whole kernel fits
             else {                                                  // centre on the median, inside the kernel
-              c = med > nslots / 2 ? med - nslots / 2 : 0;
-              c = min(max(c, K.first), K.first + K.n - nslots);
+              cws = med > nslots / 2 ? med - nslots / 2 : 0;
+              cws = min(max(cws, K.first), K.first + K.n - nslots);
             }
-            // keep the current window when the new one would not move it (already centred)
-            if (ws == kNoWindow || c != ws) nws = c;
+            if (ws == kNoWindow || cws != ws) nws = cws;
           }
           if (nws == kNoWindow) nws = 0;
           sh_ws[it & 1] = nws;
         }
       }
       __syncthreads();
+      const unsigned long long tile = sh_tile[it & 1];
+      if (tile == ~0ull) break;
+      tile_span(tile);
       const uint32_t nws = sh_ws[it & 1];
       if (nws != ws) {
         if (ws != kNoWindow) {
-          flush_table(tab, ws, nr, lim * nr, H);
+          if (P16) flush_table16(tab, ws, nr, lim * nr, H);
+          else flush_table(tab, ws, nr, lim * nr, H);
           __syncthreads();
         }
         ws = nws;
         lim = min(nslots, P - min(P, ws));
       }
+    } else {
+      if (t4 >= e4_own) break;
+      t4e = t4 + kTile4 < e4_own ? t4 + kTile4 : e4_own;
     }
     uint64_t i = t4 + threadIdx.x;
     for (; i + (kVec - 1) * blockDim.x < t4e; i += kVec * blockDim.x) {  // kVec 128-bit loads in flight
@@ -234,21 +347,40 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
         const uint4 v = __ldg(s4 + i + u * blockDim.x);
         w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
       }
-      count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+      if (P16) {  // returning atomics: batches of 4 keep the old values in registers
+#pragma unroll
+        for (int u = 0; u < kVec; u++) {
+          const uint32_t wq[4] = {w[4 * u], w[4 * u + 1], w[4 * u + 2], w[4 * u + 3]};
+          count_any<P16, DYN>(wq, P, nr, ws, lim, tab, one, H, bad);
+        }
+      } else {
+        count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+      }
     }
     for (; i < t4e; i += blockDim.x) {
       const uint4 v = __ldg(s4 + i);
       const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-      count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+      count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
     }
+    if (!DYN) t4 = t4e;
   }
-  for (uint64_t i = e4 * 4 + threadIdx.x; i < e; i += blockDim.x) {
-    const uint32_t w[1] = {s[i]};
-    count_batch<DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+  // the last chunk's words after its last 16-byte boundary (< 4 words), counted by its owner
+  if (e_own == n) {
+    if (DYN && ws == kNoWindow) {  // a window is needed even if no tile was processed
+      ws = 0;
+      lim = min(nslots, P);
+    }
+    for (uint64_t i = e4_own * 4 + threadIdx.x; i < n; i += blockDim.x) {
+      const uint32_t w[1] = {s[i]};
+      count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
+    }
   }
   if (range == 0) count_invalid(bad, d_n_invalid);
   __syncthreads();
-  if (ws != kNoWindow) flush_table(tab, ws, nr, min(nwords, lim * nr), H);
+  if (ws != kNoWindow) {
+    if (P16) flush_table16(tab, ws, nr, lim * nr, H);
+    else flush_table(tab, ws, nr, lim * nr, H);
+  }
 }
 
 }  // namespace
@@ -282,11 +414,20 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     n -= head;
     if (!n) return GS_OK;
   }
-  const uint32_t nslots = kTableWords / nr;  // whole slots per shared-memory window
-  const uint32_t n_ranges = (uint32_t)std::max<uint64_t>(1, ((uint64_t)P + nslots - 1) / nslots);
-  uint32_t mode = c->cfg.hist_mode;
-  if (mode == GS_HIST_AUTO) mode = n_ranges <= kMaxRanges ? GS_HIST_PRIVATE : GS_HIST_WINDOW;
+  const uint32_t nslots32 = kTableWords / nr, nslots16 = 2 * kTableWords / nr;  // whole slots per window
+  const auto ranges = [&](uint32_t ns) { return (uint32_t)std::max<uint64_t>(1, ((uint64_t)P + ns - 1) / ns); };
+  uint32_t max_kn = 0;
+  for (const auto& K : c->kd_h) max_kn = std::max(max_kn, K.n);
+  uint32_t mode = c->cfg.hist_mode, bits = c->cfg.hist_counter_bits;
+  if (mode == GS_HIST_AUTO) {
+    if (ranges(bits == 16 ? nslots16 : nslots32) <= kMaxRanges) mode = GS_HIST_PRIVATE;
+    else if (!bits && ranges(nslots16) <= kMaxRanges) { mode = GS_HIST_PRIVATE; bits = 16; }
+    else mode = GS_HIST_WINDOW;
+  }
+  if (!bits) bits = (mode == GS_HIST_WINDOW && max_kn > nslots32) ? 16 : 32;  // whole kernels per window
+  const uint32_t n_ranges = ranges(bits == 16 ? nslots16 : nslots32);
   if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_WINDOW;
+  c->last_hist_bits = (int)bits;
   c->last_hist_mode = (int)mode;
   if (mode == GS_HIST_GLOBAL) {
     const uint64_t blocks = std::max<uint64_t>(
@@ -308,21 +449,31 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   uint64_t chunk = (n + chunks - 1) / chunks;
   chunk = (chunk + 3) & ~3ull;
   chunks = (n + chunk - 1) / chunk;
-  if (dyn) {
-    GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k_hist_smem<true><<<(unsigned)chunks, kThreadsSmem, smem, st>>>(d_words, n, P, nr, c->d_kd, c->n_kernels, 1, chunk,
-                                                                    1u, d_hist, d_n_invalid);
-  } else {
-    GS_CUDA(c, cudaFuncSetAttribute(k_hist_smem<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k_hist_smem<false><<<(unsigned)(chunks * n_ranges), kThreadsSmem, smem, st>>>(
-        d_words, n, P, nr, c->d_kd, c->n_kernels, n_ranges, chunk, 1u, d_hist, d_n_invalid);
+  if (dyn) {  // work-stealing tile queue, one 64-bit word per chunk
+    GS_CUDA(c, dev_grow(&c->d_tileq, &c->tileq_cap, chunks));
+    GS_CUDA(c, cudaMemsetAsync(c->d_tileq, 0, chunks * 8, st));
   }
+  auto launch = [&](auto kern, uint32_t grid, uint32_t nrg) -> gs_status {
+    GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    kern<<<grid, kThreadsSmem, smem, st>>>(d_words, n, P, nr, c->d_kd, c->n_kernels, nrg, chunk, 1u, d_hist,
+                                           d_n_invalid, c->d_tileq);
+    return GS_OK;
+  };
+  gs_status ls;
+  if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
+                           : launch(k_hist_smem<true, false>, (uint32_t)chunks, 1u);
+  else ls = bits == 16 ? launch(k_hist_smem<false, true>, (uint32_t)(chunks * n_ranges), n_ranges)
+                       : launch(k_hist_smem<false, false>, (uint32_t)(chunks * n_ranges), n_ranges);
+  if (ls != GS_OK) return ls;
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;
 }
 
 void attrib_free(gs_ctx* c) {
+  if (c->d_tileq) cudaFree(c->d_tileq);
+  c->d_tileq = nullptr;
+  c->tileq_cap = 0;
   for (int b = 0; b < 2; b++) {
     if (c->h_stage[b]) cudaFreeHost(c->h_stage[b]);
     if (c->d_stage[b]) cudaFree(c->d_stage[b]);

@@ -95,7 +95,9 @@ struct gs_ctx {
   uint64_t chain_cap = 0, n_chain = 0;
 
   // ---- attribution / ranking scratch
-  int last_hist_mode = 0;
+  int last_hist_mode = 0, last_hist_bits = 0;
+  unsigned long long* d_tileq = nullptr;  // WINDOW histogram work-stealing queue
+  uint64_t tileq_cap = 0;
   unsigned long long* d_rank_keys[2] = {nullptr, nullptr};
   uint32_t* d_rank_vals[2] = {nullptr, nullptr};
   uint64_t rank_cap = 0;

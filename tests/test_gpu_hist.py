@@ -28,13 +28,14 @@ def _check(gs, s, tr, modes, words=None):
         words = DeviceTrace(tr).packed()
     want = torch.from_numpy(tr.table.astype(np.int32).reshape(-1)).cuda()
     for mode in modes:
-        ctx = gs.Context(hist_mode=mode)
-        ctx.load_sass(s.text)
-        hist, ninv = ctx.attribute_samples(words)
-        torch.cuda.synchronize()
-        assert int(ninv.item()) == 0, mode
-        assert torch.equal(hist, want), (mode, int((hist != want).sum().item()))
-        ctx.close()
+        for bits in ((16, 32) if mode in (0, 2, 3) else (0,)):
+            ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
+            ctx.load_sass(s.text)
+            hist, ninv = ctx.attribute_samples(words)
+            torch.cuda.synchronize()
+            assert int(ninv.item()) == 0, (mode, bits)
+            assert torch.equal(hist, want), (mode, bits, int((hist != want).sum().item()))
+            ctx.close()
 
 
 @pytest.mark.parametrize("order", ["trace", "shuffled"])
@@ -67,8 +68,8 @@ def test_single_bin_drain(gs):
     s = gsass.config_sass("C1")
     n = 3_000_000
     words = torch.full((n,), (17 << 5) | 6, dtype=torch.int32, device="cuda")
-    for mode in MODES:
-        ctx = gs.Context(hist_mode=mode)
+    for mode, bits in [(m, b) for m in MODES for b in (16, 32)]:
+        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
         ctx.load_sass(s.text)
         hist, ninv = ctx.attribute_samples(words)
         torch.cuda.synchronize()
@@ -90,8 +91,8 @@ def test_unaligned_views_and_invalid_words(gs, offset):
     buf = torch.cat([torch.zeros(offset, dtype=torch.int32, device="cuda"), bad, base, bad])
     view = buf[offset:]
     want = torch.from_numpy(tab.astype(np.int32).reshape(-1)).cuda()
-    for mode in MODES:
-        ctx = gs.Context(hist_mode=mode)
+    for mode, bits in [(m, b) for m in MODES for b in (16, 32)]:
+        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
         ctx.load_sass(s.text)
         hist, ninv = ctx.attribute_samples(view)
         torch.cuda.synchronize()

@@ -158,37 +158,42 @@ __device__ void flush_table(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nw
 // that takes a half from 0x7FFF to 0x8000 (bit 15 flips: (old ^ (old + inc)) & (inc << 15)) drains
 // 0x8000 to the global bin, so a half never carries into its neighbour (at most a few thousand
 // increments can be in flight per SM between that add and the drain). Counts stay exact.
+// rare path of count_batch16, out of line so its address arithmetic is not hoisted into the loop
+template <bool SPILL_OUT>
+__device__ __noinline__ void slow16(uint32_t w, uint32_t old, uint32_t inc, uint32_t idx, bool in, uint32_t P,
+                                    uint32_t nr, uint32_t* tab, int32_t* H, uint32_t* bad) {
+  if (!in) {
+    if ((w >> 5) < P && (w & 31u) < nr) {
+      if (SPILL_OUT) atomicAdd(H + w, 1);
+    } else {
+      (*bad)++;
+    }
+  } else if ((old ^ (old + inc)) & (inc << 15)) {  // this increment took the half to 0x8000
+    atomicSub(tab + idx, inc << 15);
+    atomicAdd(H + w, 0x8000);
+  }
+}
+
 template <bool SPILL_OUT, int N>
 __device__ __forceinline__ void count_batch16(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
                                               uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
                                               uint32_t& bad) {
-  uint32_t n_out = 0, ovf = 0;
-  uint32_t old[N], inc[N], idx[N];
+  uint32_t old[N], inc[N], idx[N], flag = 0;
 #pragma unroll
   for (int q = 0; q < N; q++) {
     const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
     const bool in = d < nslots && rs < nr;
     const uint32_t off = d * nr + rs;
-    idx[q] = in ? (off >> 1) : kTableWords + (threadIdx.x & 31u);
-    inc[q] = in ? (one << ((off & 1u) << 4)) : 0u;
+    inc[q] = (off & 1u) * 0xffffu + one;                      // 1 (low half) or 0x10000 (high half)
+    idx[q] = in ? (off >> 1) : kTableWords + (threadIdx.x & 31u);  // spare word outside the window
     old[q] = atomicAdd(tab + idx[q], inc[q]);
-    ovf |= (old[q] ^ (old[q] + inc[q])) & (inc[q] << 15);
-    n_out += in ? 0u : 1u;
+    flag |= ((old[q] ^ (old[q] + inc[q])) & (inc[q] << 15)) | (in ? 0u : 1u);
   }
-  const uint32_t act = __activemask();
-  if (__any_sync(act, ovf)) {  // rare: a counter reached 0x8000
-#pragma unroll
-    for (int q = 0; q < N; q++)
-      if ((old[q] ^ (old[q] + inc[q])) & (inc[q] << 15)) {
-        atomicSub(tab + idx[q], inc[q] << 15);
-        atomicAdd(H + w[q], 0x8000);
-      }
-  }
-  if (__any_sync(act, n_out)) {  // rare: some lane saw a sample outside the window
+  if (__any_sync(__activemask(), flag)) {  // rare: a half reached 0x8000, or a sample is outside the window
 #pragma unroll
     for (int q = 0; q < N; q++) {
       const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-      if (!(d < nslots && rs < nr)) slow_one<SPILL_OUT>(w[q], P, nr, H, bad);
+      slow16<SPILL_OUT>(w[q], old[q], inc[q], idx[q], d < nslots && rs < nr, P, nr, tab, H, &bad);
     }
   }
 }
@@ -283,29 +288,36 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
         t4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
         t4e = t4 + kTile4 < ce / 4 ? t4 + kTile4 : ce / 4;
       };
-      if (threadIdx.x == 0) sh_tile[it & 1] = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
-      __syncwarp();
-      if (threadIdx.x < 32 && sh_tile[it & 1] != ~0ull) {
-        tile_span(sh_tile[it & 1]);
-        // window for this tile: around the median slot of 32 evenly spaced samples (robust to the
-        // cold tail of a kernel's samples); whole kernel if it fits
-        const uint64_t span = t4e - t4;
-        const uint32_t w = s[4 * (t4 + span * threadIdx.x / 32)];
-        const bool ok = (w >> 5) < P && (w & 31u) < nr;
-        const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
-        uint32_t le = 0;  // lanes whose slot is <= mine
-        for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
-        const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
-        // median: the smallest valid slot with more than half of the valid samples at or below it
-        const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
-        if (threadIdx.x == 0) {
-          uint32_t nws = ws;
+      // warp 0 grabs the next tile and picks its window while the CTA counts the current one
+      const auto decide = [&](uint32_t buf) {
+        unsigned long long tile = 0;
+        if (threadIdx.x == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
+        tile = __shfl_sync(0xffffffffu, tile, 0);
+        uint32_t nws = ws;
+        if (tile != ~0ull) {
+          uint64_t a4, b4;
+          {
+            const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
+            const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
+            a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
+            b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
+          }
+          // window: around the median slot of 32 evenly spaced samples (robust to the cold tail
+          // of a kernel's samples); the whole kernel if it fits
+          const uint32_t w = __ldg(s + 4 * (a4 + (b4 - a4) * threadIdx.x / 32));
+          const bool ok = (w >> 5) < P && (w & 31u) < nr;
+          const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
+          uint32_t le = 0;  // lanes whose slot is <= mine
+          for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
+          const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
+          // median: the smallest valid slot with more than half of the valid samples at or below it
+          const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
           if (med != 0xffffffffu && (ws == kNoWindow || med - ws >= nslots || med - ws < nslots / 8 ||
                                      med - ws >= nslots - nslots / 8)) {
             uint32_t lo = 0, hi = nk;  // kernel of the slot: last k with first <= slot
             while (hi - lo > 1) {
               const uint32_t mid = (lo + hi) >> 1;
-              if (kd[mid].first <= med) lo = mid;
+              if (__ldg(&kd[mid].first) <= med) lo = mid;
               else hi = mid;
             }
             const KDesc K = kd[lo];
@@ -317,10 +329,14 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
             }
             if (ws == kNoWindow || cws != ws) nws = cws;
           }
-          if (nws == kNoWindow) nws = 0;
-          sh_ws[it & 1] = nws;
         }
-      }
+        if (nws == kNoWindow) nws = 0;
+        if (threadIdx.x == 0) {
+          sh_tile[buf] = tile;
+          sh_ws[buf] = nws;
+        }
+      };
+      if (it == 0 && threadIdx.x < 32) decide(0);
       __syncthreads();
       const unsigned long long tile = sh_tile[it & 1];
       if (tile == ~0ull) break;
@@ -335,6 +351,7 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
         ws = nws;
         lim = min(nslots, P - min(P, ws));
       }
+      if (threadIdx.x < 32) decide((it + 1) & 1);
     } else {
       if (t4 >= e4_own) break;
       t4e = t4 + kTile4 < e4_own ? t4 + kTile4 : e4_own;

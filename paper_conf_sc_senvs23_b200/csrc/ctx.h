@@ -10,7 +10,7 @@
 
 namespace gs {
 
-constexpr uint32_t kWin = 512;  // instructions per detection window (never crosses a kernel)
+constexpr uint32_t kWin = 256;  // instructions per detection window (never crosses a kernel)
 
 // A device buffer that only grows; freed with the context.
 struct DevBuf {

@@ -85,11 +85,20 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
   const WDesc W = wd[w];
   const KDesc K = kd[W.kernel];
   uint32_t n_gatom = 0, n_satom = 0, n_conv = 0, n_vec = 0;
-  for (uint32_t b = 0; b < W.len; b += 32) {
-    const uint32_t i = b + lane;
+  constexpr int kAhead = 4;  // chunks whose records are loaded together (no cross-chunk dependency)
+  for (uint32_t b0 = 0; b0 < W.len; b0 += 32 * kAhead) {
+    Rec rr[kAhead];
+#pragma unroll
+    for (int u = 0; u < kAhead; u++) {
+      const uint32_t i = b0 + 32 * u + lane;
+      rr[u] = i < W.len ? ld_rec(rec, (uint64_t)W.start + i) : Rec{0, 0, 0, 0};
+    }
+#pragma unroll
+    for (int u = 0; u < kAhead; u++) {
+    const uint32_t i = b0 + 32 * u + lane;
     const bool valid = i < W.len;
     const uint64_t g = (uint64_t)W.start + i;
-    Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
+    const Rec r = rr[u];
     const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r);
     if (valid && dw && reg_live(dst)) {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
@@ -114,6 +123,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
       n_satom += (cls & C_SATOM) ? 1 : 0;
       n_conv += (cls & C_CONV) ? 1 : 0;
       n_vec += (op == OP_LDG && (r_flags(r) & F_HASMEM) && (r_aw(r) == AW_64 || r_aw(r) == AW_128)) ? 1 : 0;
+    }
     }
   }
   for (int o = 16; o; o >>= 1) {
@@ -142,11 +152,17 @@ __global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, 
   for (int r = threadIdx.x; r <= kNumRegs; r += blockDim.x) {
     if (r < kNumRegs) {
       uint32_t state = 0;
-      for (uint32_t j = 0; j < nwk; j++) {
-        uint32_t* p = tab + (uint64_t)(K.win0 + j) * kNumRegs + r;
-        const uint32_t s = *p;
-        *p = state;
-        if (s) state = s;
+      constexpr uint32_t kB = 8;  // window summaries loaded per batch
+      for (uint32_t j0 = 0; j0 < nwk; j0 += kB) {
+        uint32_t v[kB];
+#pragma unroll
+        for (uint32_t u = 0; u < kB; u++)
+          v[u] = j0 + u < nwk ? tab[(uint64_t)(K.win0 + j0 + u) * kNumRegs + r] : 0u;
+#pragma unroll
+        for (uint32_t u = 0; u < kB; u++) {
+          if (j0 + u < nwk) tab[(uint64_t)(K.win0 + j0 + u) * kNumRegs + r] = state;
+          if (v[u]) state = v[u];
+        }
       }
     } else {
       int32_t acc = 0;
@@ -183,12 +199,14 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
   const uint32_t gt = ~((2u << lane) - 1u);
   uint32_t* T = tabS[warp];
   uint32_t* M = cm[warp];
+  Rec rnext = lane < W.len ? ld_rec(rec, (uint64_t)W.start + lane) : Rec{0, 0, 0, 0};
   for (uint32_t b = 0; b < W.len; b += 32) {
     const uint32_t i = b + lane;
     const bool valid = i < W.len;
     const uint64_t g = (uint64_t)W.start + i;
     const uint64_t gbase = (uint64_t)W.start + b;
-    Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
+    const Rec r = rnext;  // records of the next chunk are loaded while this one is resolved
+    rnext = i + 32 < W.len ? ld_rec(rec, g + 32) : Rec{0, 0, 0, 0};
     const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
     const bool writes = valid && dw && reg_live(dst);
     const uint32_t cap = reg_cap(dst);
@@ -306,21 +324,26 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restric
   return o;
 }
 
+// Threads [0, nc) trace candidate c; threads [nc, 2nc) update the key-group statistics of
+// candidate c - nc (two independent latency chains per candidate run on different threads).
 __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
                         uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, OffsetSet os, RootSet rs,
                         gs_kernel_stats* kst) {
-  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (c >= nc) return;
+  const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (t >= 2 * nc) return;
+  const bool groups = t >= nc;
+  const uint64_t c = groups ? t - nc : t;
   const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
   const Rec ri = ld_rec(rec, g);
   const uint32_t op = r_op(ri), cls = op_class(op);
-  if (!(cls & C_TRACED) || !(r_flags(ri) & F_HASMEM)) {
-    ca.tk[c] = GS_T_NONE; ca.tv[c] = 0; ca.depth[c] = 0; ca.grp[c] = 0xffffffffu;
-    return;
-  }
-  const KDesc K = kd[kernel];
+  const bool traced = (cls & C_TRACED) && (r_flags(ri) & F_HASMEM);
   const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
-  if (op == OP_LDG) {  // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max
+  if (groups) {
+    if (!traced || op != OP_LDG) {
+      ca.grp[c] = 0xffffffffu;
+      return;
+    }
+    // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max, contiguity
     const uint32_t slot = hinsert(gt.key, gt.cap, group_key(base, brd, kernel));
     ca.grp[c] = slot;
     atomicAdd(gt.nload + slot, 1u);
@@ -336,15 +359,19 @@ __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ k
       atomicOr(gt.or3 + slot, (uint32_t)off & 3u);
       atomicAnd(gt.and3 + slot, (uint32_t)off & 3u);
     }
-  } else {
-    ca.grp[c] = 0xffffffffu;
+    return;
   }
-  const TraceOut t = chase(rec, ptrrd, K, base, brd, D, [](uint32_t) {});
-  ca.tk[c] = (uint8_t)t.tk;
-  ca.tv[c] = t.tv;
-  ca.depth[c] = (uint8_t)t.depth;
+  if (!traced) {
+    ca.tk[c] = GS_T_NONE; ca.tv[c] = 0; ca.depth[c] = 0;
+    return;
+  }
+  const KDesc K = kd[kernel];
+  const TraceOut tr = chase(rec, ptrrd, K, base, brd, D, [](uint32_t) {});
+  ca.tk[c] = (uint8_t)tr.tk;
+  ca.tv[c] = tr.tv;
+  ca.depth[c] = (uint8_t)tr.depth;
   if (cls & C_STORE) {  // store roots (R8, R27)
-    if (t.tk == GS_T_PARAM || t.tk == GS_T_ENTRY) hinsert(rs.key, rs.cap, root_key(kernel, t.tk, t.tv));
+    if (tr.tk == GS_T_PARAM || tr.tk == GS_T_ENTRY) hinsert(rs.key, rs.cap, root_key(kernel, tr.tk, tr.tv));
     else atomicAdd(&kst[kernel].n_unresolved_stores, 1u);
   }
 }
@@ -548,7 +575,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
     GS_CUDA(c, cudaGetLastError());
     const uint32_t gridc = (uint32_t)((nc + 255) / 256);
-    k_trace<<<gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
+    k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
                                    c->d_kstats); count_launch();
     GS_CUDA(c, cudaGetLastError());
     k_rules<<<gridc, 256, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,

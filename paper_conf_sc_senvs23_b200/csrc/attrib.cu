@@ -28,6 +28,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "ctx.h"
 
@@ -41,6 +42,7 @@ constexpr uint32_t kMaxRanges = 3;
 constexpr uint32_t kTile4 = 65536;                 // uint4 per window decision (256K samples)
 constexpr int kVec = 4;                            // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
+constexpr uint32_t kTmaTableWords = 41600;  // TMA kernel: 16-bit pairs, 83200 bins (4378 slots at R = 19)
 
 __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long* d_n_invalid) {
   for (int o = 16; o; o >>= 1) n_bad += __shfl_xor_sync(0xffffffffu, n_bad, o);
@@ -116,25 +118,29 @@ __device__ __forceinline__ void red_shared_add_if(uint32_t addr, uint32_t one, b
       : "memory");
 }
 
+// predicated L2 atomic: one instruction, no branch
+__device__ __forceinline__ void red_global_add_if(int32_t* addr, uint32_t v, bool p) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.relaxed.gpu.global.add.u32 [%0], %1;\n\t}" ::"l"(addr),
+               "r"(v), "r"((uint32_t)p)
+               : "memory");
+}
+
+// 32-bit counters: no return values, no rare path. Per sample: shared atomic on the window slot
+// (or the lane's spare word), plus a predicated L2 atomic when the sample is valid but outside the
+// window (WINDOW only; PRIVATE leaves it to the CTA that owns that range).
 template <bool SPILL_OUT, int N>
 __device__ __forceinline__ void count_batch(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
                                             uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
                                             uint32_t& bad) {
-  uint32_t n_out = 0;
 #pragma unroll
   for (int q = 0; q < N; q++) {
-    const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-    const bool in = d < nslots && rs < nr;
-    // unconditional shared atomic: lanes outside the window add 0 to a spare word (no branch)
-    atomicAdd(tab + (in ? d * nr + rs : kTableWords + (threadIdx.x & 31u)), in ? one : 0u);
-    n_out += in ? 0u : 1u;
-  }
-  if (__any_sync(__activemask(), n_out)) {  // rare: some lane saw a sample outside the window
-#pragma unroll
-    for (int q = 0; q < N; q++) {
-      const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-      if (!(d < nslots && rs < nr)) slow_one<SPILL_OUT>(w[q], P, nr, H, bad);
-    }
+    const uint32_t slot = w[q] >> 5, d = slot - ws, rs = w[q] & 31u;
+    const bool rok = rs < nr;
+    const bool in = d < nslots && rok;
+    atomicAdd(tab + (in ? d * nr + rs : kTableWords + (threadIdx.x & 31u)), one);  // spare: never flushed
+    const bool valid = rok && slot < P;
+    if (SPILL_OUT) red_global_add_if(H + w[q], one, valid && !in);
+    bad += valid ? 0u : 1u;
   }
 }
 
@@ -160,7 +166,7 @@ __device__ void flush_table(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nw
 // increments can be in flight per SM between that add and the drain). Counts stay exact.
 // rare path of count_batch16, out of line so its address arithmetic is not hoisted into the loop
 template <bool SPILL_OUT>
-__device__ __noinline__ void slow16(uint32_t w, uint32_t old, uint32_t inc, uint32_t idx, bool in, uint32_t P,
+__device__ __noinline__ void slow16(uint32_t w, uint32_t old, uint32_t sh, uint32_t idx, bool in, uint32_t P,
                                     uint32_t nr, uint32_t* tab, int32_t* H, uint32_t* bad) {
   if (!in) {
     if ((w >> 5) < P && (w & 31u) < nr) {
@@ -168,32 +174,47 @@ __device__ __noinline__ void slow16(uint32_t w, uint32_t old, uint32_t inc, uint
     } else {
       (*bad)++;
     }
-  } else if ((old ^ (old + inc)) & (inc << 15)) {  // this increment took the half to 0x8000
-    atomicSub(tab + idx, inc << 15);
-    atomicAdd(H + w, 0x8000);
+    return;
+  }
+  if (!((old >> sh) & 0x8000u)) return;
+  // the half was already >= 0x8000: move 0x8000 of it to the global bin. Several threads may race
+  // here; the CAS makes each successful drain subtract exactly 0x8000 once.
+  uint32_t v = tab[idx];
+  while ((v >> sh) & 0x8000u) {
+    const uint32_t prev = atomicCAS(tab + idx, v, v - (0x8000u << sh));
+    if (prev == v) {
+      atomicAdd(H + w, 0x8000);
+      return;
+    }
+    v = prev;
   }
 }
 
-template <bool SPILL_OUT, int N>
+// 16-bit packed counters, two per word. Per sample: one returning shared atomic; the returned old
+// value flags a half already at >= 0x8000 (drained in the rare path before it could reach 0xFFFF:
+// at most a few thousand increments are in flight per SM), so counts stay exact.
+template <bool SPILL_OUT, int N, uint32_t SPARE = kTableWords>
 __device__ __forceinline__ void count_batch16(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
                                               uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
                                               uint32_t& bad) {
-  uint32_t old[N], inc[N], idx[N], flag = 0;
+  uint32_t old[N], flag = 0;
 #pragma unroll
   for (int q = 0; q < N; q++) {
     const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
     const bool in = d < nslots && rs < nr;
     const uint32_t off = d * nr + rs;
-    inc[q] = (off & 1u) * 0xffffu + one;                      // 1 (low half) or 0x10000 (high half)
-    idx[q] = in ? (off >> 1) : kTableWords + (threadIdx.x & 31u);  // spare word outside the window
-    old[q] = atomicAdd(tab + idx[q], inc[q]);
-    flag |= ((old[q] ^ (old[q] + inc[q])) & (inc[q] << 15)) | (in ? 0u : 1u);
+    const uint32_t inc = in ? ((off & 1u) ? 0x10000u : one) : 0u;
+    const uint32_t idx = in ? (off >> 1) : SPARE + (threadIdx.x & 31u);  // lane's spare word
+    old[q] = atomicAdd(tab + idx, inc);
+    flag |= (old[q] & (inc << 15)) | (in ? 0u : 1u);
   }
-  if (__any_sync(__activemask(), flag)) {  // rare: a half reached 0x8000, or a sample is outside the window
+  if (__any_sync(__activemask(), flag)) {  // rare: a half at >= 0x8000, or a sample outside the window
 #pragma unroll
     for (int q = 0; q < N; q++) {
       const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-      slow16<SPILL_OUT>(w[q], old[q], inc[q], idx[q], d < nslots && rs < nr, P, nr, tab, H, &bad);
+      const bool in = d < nslots && rs < nr;
+      const uint32_t off = d * nr + rs;
+      slow16<SPILL_OUT>(w[q], old[q], (off & 1u) << 4, off >> 1, in, P, nr, tab, H, &bad);
     }
   }
 }
@@ -400,6 +421,184 @@ __global__ void __launch_bounds__(kThreadsSmem, 1)
   }
 }
 
+// =============================================================================== TMA-fed WINDOW kernel
+// Warp-specialised: warp 0 is the producer (tile queue, window choice, TMA bulk copies of sample
+// stages into shared memory); warps 1..31 consume one 128-bit word (4 samples) each per stage.
+// kStages stages of kStage4 uint4 keep ~62 KB of samples in flight per SM independently of
+// registers (the register-fed kernel was memory-latency bound: 57% long-scoreboard stalls).
+constexpr int kConsumerWarps = 31;
+constexpr uint32_t kStage4 = kConsumerWarps * 32;          // uint4 per stage: one per consumer thread
+constexpr uint32_t kStageBytes = kStage4 * 16;             // 15872 B
+constexpr int kStages = 4;
+constexpr size_t kTmaSmem = (size_t)kStages * kStageBytes + (size_t)(kTmaTableWords + 32) * 4;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(unsigned long long* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done)
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                 : "=r"(done)
+                 : "r"(smem_u32(b)), "r"(parity)
+                 : "memory");
+}
+__device__ __forceinline__ void tma_load(void* dst, const void* src, uint32_t bytes, unsigned long long* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, %0;" ::"r"(kConsumerWarps * 32) : "memory"); }
+
+// flush helpers over an explicit thread range [0, nt)
+__device__ void flush_pairs(uint32_t* tab, uint32_t words, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H,
+                            uint32_t t, uint32_t nt) {
+  const uint32_t stride = 2 * nt, step_q = stride / nr, step_r = stride % nr;
+  uint32_t q = (2 * t) / nr, r = (2 * t) % nr;
+  for (uint32_t i = t; i < words && 2 * i < nbins; i += nt) {
+    const uint32_t v = tab[i];
+    if (v) {
+      tab[i] = 0;
+      if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
+      if (v >> 16) {
+        const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
+        atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
+      }
+    }
+    q += step_q;
+    r += step_r;
+    if (r >= nr) { r -= nr; q++; }
+  }
+}
+
+__global__ void __launch_bounds__(32 * (kConsumerWarps + 1), 1)
+    k_hist_tma(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
+               uint32_t nk, uint64_t chunk, uint32_t one, int32_t* __restrict__ H, unsigned long long* d_n_invalid,
+               unsigned long long* rng) {
+  extern __shared__ __align__(128) uint8_t dyn[];
+  uint4* stage = reinterpret_cast<uint4*>(dyn);
+  uint32_t* tab = reinterpret_cast<uint32_t*>(dyn + (size_t)kStages * kStageBytes);
+  __shared__ __align__(8) unsigned long long full_bar[kStages], empty_bar[kStages];
+  __shared__ uint32_t meta_ws[kStages], meta_cnt[kStages];
+  const uint32_t nslots = 2 * kTmaTableWords / nr;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (uint32_t i = threadIdx.x; i < kTmaTableWords + 32; i += blockDim.x) tab[i] = 0;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kStages; i++) {
+      mbar_init(full_bar + i, 1);
+      mbar_init(empty_bar + i, kConsumerWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  const uint4* s4 = reinterpret_cast<const uint4*>(s);
+  const uint64_t e_own = (blockIdx.x + 1) * chunk < n ? (blockIdx.x + 1) * chunk : n;
+  if (warp == 0) {
+    // ------------------------------------------------------------------ producer
+    uint32_t ws = kNoWindow, st = 0;
+    for (;;) {
+      unsigned long long tile = 0;
+      if (lane == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
+      tile = __shfl_sync(0xffffffffu, tile, 0);
+      if (tile == ~0ull) break;
+      const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
+      const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
+      const uint64_t t4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
+      const uint64_t t4e = t4 + kTile4 < ce / 4 ? t4 + kTile4 : ce / 4;
+      if (t4e <= t4) continue;
+      {  // window: around the median slot of 32 evenly spaced samples; the whole kernel if it fits
+        const uint32_t w = __ldg(s + 4 * (t4 + (t4e - t4) * lane / 32));
+        const bool ok = (w >> 5) < P && (w & 31u) < nr;
+        const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
+        uint32_t le = 0;
+        for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
+        const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
+        const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
+        if (med != 0xffffffffu && (ws == kNoWindow || med - ws >= nslots || med - ws < nslots / 8 ||
+                                   med - ws >= nslots - nslots / 8)) {
+          uint32_t lo = 0, hi = nk;
+          while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (__ldg(&kd[mid].first) <= med) lo = mid;
+            else hi = mid;
+          }
+          const KDesc K = kd[lo];
+          uint32_t cws;
+          if (K.n <= nslots) cws = K.first;
+          else {
+            cws = med > nslots / 2 ? med - nslots / 2 : 0;
+            cws = min(max(cws, K.first), K.first + K.n - nslots);
+          }
+          ws = cws;
+        }
+        if (ws == kNoWindow) ws = 0;
+      }
+      for (uint64_t p = t4; p < t4e; p += kStage4, st++) {
+        const uint32_t cnt = t4e - p < kStage4 ? (uint32_t)(t4e - p) : kStage4;
+        const uint32_t sb = st % kStages;
+        if (st >= (uint32_t)kStages) mbar_wait(empty_bar + sb, ((st / kStages) + 1) & 1);
+        if (lane == 0) {
+          meta_ws[sb] = ws;
+          meta_cnt[sb] = cnt;
+          mbar_arrive_tx(full_bar + sb, cnt * 16);
+          tma_load(stage + (size_t)sb * kStage4, s4 + p, cnt * 16, full_bar + sb);
+        }
+        __syncwarp();
+      }
+    }
+    const uint32_t sb = st % kStages;  // end marker
+    if (st >= (uint32_t)kStages) mbar_wait(empty_bar + sb, ((st / kStages) + 1) & 1);
+    if (lane == 0) {
+      meta_cnt[sb] = 0;
+      mbar_arrive(full_bar + sb);
+    }
+    return;
+  }
+  // -------------------------------------------------------------------- consumers
+  const uint32_t ct = threadIdx.x - 32, nct = kConsumerWarps * 32;
+  uint32_t ws = kNoWindow, lim = 0, bad = 0;
+  for (uint32_t st = 0;; st++) {
+    const uint32_t sb = st % kStages;
+    mbar_wait(full_bar + sb, (st / kStages) & 1);
+    const uint32_t cnt = meta_cnt[sb], nws = meta_ws[sb];
+    if (cnt == 0) break;
+    if (nws != ws) {  // window change: every consumer has finished the previous stages
+      consumer_sync();
+      if (ws != kNoWindow) flush_pairs(tab, kTmaTableWords, ws, nr, lim * nr, H, ct, nct);
+      consumer_sync();
+      ws = nws;
+      lim = min(nslots, P - min(P, ws));
+    }
+    const uint4 v = ct < cnt ? stage[(size_t)sb * kStage4 + ct] : make_uint4(0, 0, 0, 0);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty_bar + sb);  // stage may be refilled; the data is in registers
+    if (ct < cnt) {
+      const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+      count_batch16<true, 4, kTmaTableWords>(w, P, nr, ws, lim, tab, one, H, bad);
+    }
+  }
+  // the last chunk's words after its last 16-byte boundary (< 4): L2 atomics
+  if (e_own == n)
+    for (uint64_t i = (n / 4) * 4 + ct; i < n; i += nct) {
+      const uint32_t w = s[i];
+      if ((w >> 5) < P && (w & 31u) < nr) atomicAdd(H + w, 1);
+      else bad++;
+    }
+  for (int o = 16; o; o >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, o);
+  if (lane == 0 && bad) atomicAdd(d_n_invalid, (unsigned long long)bad);
+  consumer_sync();
+  if (ws != kNoWindow) flush_pairs(tab, kTmaTableWords, ws, nr, lim * nr, H, ct, nct);
+}
+
 }  // namespace
 
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
@@ -477,7 +676,12 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     return GS_OK;
   };
   gs_status ls;
-  if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
+  if (dyn && bits == 16 && getenv("GS_HIST_TMA")) {  // TMA-fed warp-specialised kernel (opt-in)
+    GS_CUDA(c, cudaFuncSetAttribute(k_hist_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmem));
+    k_hist_tma<<<(uint32_t)chunks, 32 * (kConsumerWarps + 1), kTmaSmem, st>>>(
+        d_words, n, P, nr, c->d_kd, c->n_kernels, chunk, 1u, d_hist, d_n_invalid, c->d_tileq);
+    ls = GS_OK;
+  } else if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
                            : launch(k_hist_smem<true, false>, (uint32_t)chunks, 1u);
   else ls = bits == 16 ? launch(k_hist_smem<false, true>, (uint32_t)(chunks * n_ranges), n_ranges)
                        : launch(k_hist_smem<false, false>, (uint32_t)(chunks * n_ranges), n_ranges);

@@ -32,7 +32,7 @@ def _load():
         _lib = ctypes.CDLL(build())
         P = ctypes.c_void_p
         _lib.gsgen_expand.argtypes = [P, P, ctypes.c_int64, P, ctypes.c_int, P, ctypes.c_int, ctypes.c_int64,
-                                      ctypes.c_int64, P, P]
+                                      ctypes.c_int64, ctypes.c_uint32, P, P]
         _lib.gsgen_expand.restype = ctypes.c_int
     return _lib
 
@@ -60,7 +60,7 @@ class DeviceTrace:
         self.keys = torch.from_numpy(keys.view(np.int32)).to(dev)
         self.N = trace.N
 
-    def packed(self, a: int = 0, b: int | None = None, out=None, stream=None):
+    def packed(self, a: int = 0, b: int | None = None, out=None, stream=None, n_reasons: int = 19):
         import torch
         b = self.N if b is None else b
         if out is None:
@@ -68,7 +68,7 @@ class DeviceTrace:
         st = (stream or torch.cuda.current_stream(self.dev)).cuda_stream
         rc = _load().gsgen_expand(self.nz.data_ptr(), self.cum.data_ptr(), len(self.tr.nz), self.kstart.data_ptr(),
                                   len(self.tr.kstart) - 1, self.keys.data_ptr(), self.ORDER[self.tr.order], a, b,
-                                  out.data_ptr(), ctypes.c_void_p(st))
+                                  n_reasons, out.data_ptr(), ctypes.c_void_p(st))
         if rc != 0:
             raise RuntimeError(f"gsgen_expand failed ({rc})")
         return out

@@ -3,8 +3,8 @@
 //
 // Sample p of the stream: q = sorted position (Feistel bijection of p, globally or within the
 // kernel's block), bin = the q-th bin of the slot-major layout (binary search over the prefix of
-// nonzero counts). The emitted word is the flat bin index slot*32 + reason, i.e. the packed
-// sample format of gs_attribute_samples. No method arithmetic lives here.
+// nonzero counts). The emitted word is slot * R + reason (R active reasons), the packed sample
+// format of gs_attribute_samples. No method arithmetic lives here.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -50,7 +50,7 @@ __device__ __forceinline__ int64_t upper_index(const int64_t* a, int64_t n, int6
 
 __global__ void k_expand(const int64_t* __restrict__ nz, const int64_t* __restrict__ cum, int64_t nnz,
                          const int64_t* __restrict__ kstart, int nk, const uint32_t* __restrict__ keys, int order,
-                         int64_t a, int64_t b, uint32_t* __restrict__ out) {
+                         int64_t a, int64_t b, uint32_t nr, uint32_t* __restrict__ out) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (a + i >= b) return;
   const int64_t p = a + i;
@@ -66,16 +66,18 @@ __global__ void k_expand(const int64_t* __restrict__ nz, const int64_t* __restri
     q = base + (int64_t)feistel((uint64_t)(p - base), (uint64_t)n_k, keys + 4 * k);
   }
   const int64_t j = upper_index(cum, nnz + 1, q);
-  out[i] = (uint32_t)nz[j];
+  const uint64_t bin = (uint64_t)nz[j];
+  out[i] = (uint32_t)((bin >> 5) * nr + (bin & 31));
 }
 
 }  // namespace
 
 extern "C" int gsgen_expand(const int64_t* d_nz, const int64_t* d_cum, int64_t nnz, const int64_t* d_kstart, int nk,
-                            const uint32_t* d_keys, int order, int64_t a, int64_t b, uint32_t* d_out, void* stream) {
+                            const uint32_t* d_keys, int order, int64_t a, int64_t b, uint32_t nr, uint32_t* d_out,
+                            void* stream) {
   if (b <= a) return 0;
   const int64_t n = b - a;
   k_expand<<<(unsigned)((n + 255) / 256), 256, 0, (cudaStream_t)stream>>>(d_nz, d_cum, nnz, d_kstart, nk, d_keys,
-                                                                         order, a, b, d_out);
+                                                                         order, a, b, nr, d_out);
   return (int)cudaGetLastError();
 }

@@ -8,8 +8,8 @@ count table itself, a closed form independent of both implementations (SURVEY §
 Sample record formats
   raw    : little-endian uint32 triples (kernel id, pc offset in bytes, reason id)  — what a
            PC-sampling collector reports; the oracle and gs_pack_samples consume it.
-  packed : uint32 word = (slot << 5) | reason with slot = first_slot[kernel] + pc/16 — the record
-           gs_attribute_samples consumes (its definition).
+  packed : uint32 word = slot * R + reason with slot = first_slot[kernel] + pc/16 and R the
+           active reason count — the record gs_attribute_samples consumes.
 """
 from __future__ import annotations
 
@@ -232,10 +232,10 @@ class Trace:
         b = self.N if b is None else b
         return self.bins_to_raw(self.bins(a, b))
 
-    def packed(self, a: int = 0, b: int | None = None) -> np.ndarray:
+    def packed(self, a: int = 0, b: int | None = None, n_reasons: int = R_ACTIVE) -> np.ndarray:
         b = self.N if b is None else b
         bins = self.bins(a, b)
-        return ((bins // R_SLOTS) << 5 | (bins % R_SLOTS)).astype(np.uint32)
+        return ((bins // R_SLOTS) * n_reasons + (bins % R_SLOTS)).astype(np.uint32)
 
 
 def invalid_raw(n_kernels: int, n_instr, n: int, key: int, n_reasons: int = R_ACTIVE) -> np.ndarray:

@@ -125,14 +125,16 @@ gs_status gs_sites_host(gs_ctx *ctx, gs_site *sites, size_t cap_sites, uint32_t 
 gs_status gs_kernel_stats_get(const gs_ctx *ctx, gs_kernel_stats *out, size_t cap);
 
 /* a-8: raw samples (device, n x {kernel u32, pc byte offset u32, reason u32}) ->
- * packed words (device, n x u32) word = (first_slot[kernel] + pc/16) << 5 | reason. Invalid
+ * packed words (device, n x u32) word = (first_slot[kernel] + pc/16) * n_reasons + reason (the
+ * compact bin index of the sample; requires n_instr * n_reasons < 2^32). Invalid
  * samples (R30) become 0xFFFFFFFF and are counted into *d_n_invalid (device u64, added to).
  * Async. */
 gs_status gs_pack_samples(gs_ctx *ctx, const uint32_t *d_raw, uint64_t n, uint32_t *d_words,
                           unsigned long long *d_n_invalid);
 
-/* a-9: H[slot*32 + reason] += 1 for every valid packed word (slot < P, reason <
- * n_reasons); others are counted into *d_n_invalid (device u64, added to). `samples` may be host
+/* a-9: H[slot*32 + reason] += 1 for every valid packed word w = slot * n_reasons +
+ * reason (valid iff w < n_instr * n_reasons); others are counted into *d_n_invalid (device u64,
+ * added to). `samples` may be host
  * (pinned or pageable; streamed in chunks with copies overlapped) or device memory. d_hist is a
  * caller-owned device int32 array of n_instr*32 bins, zeroed first unless accumulate != 0.
  * Async for device input; host input returns after the last chunk is consumed. */

@@ -37,19 +37,22 @@ def _run(cmd):
     return p.stderr
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale(LIB):
-        return LIB
-    os.makedirs(BUILD, exist_ok=True)
-    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-lineinfo", "-I", CSRC]
+def build(force: bool = False, verbose: bool = False, defines: tuple[str, ...] = (), out: str | None = None) -> str:
+    """defines/out: diagnostic variants only (tools/), e.g. defines=("GS_DIAG=1",), out=tools/libgs_diag.so."""
+    lib = out or LIB
+    if not force and not defines and not _stale(lib):
+        return lib
+    bdir = BUILD if not defines else os.path.join(BUILD, "diag_" + "_".join(d.replace("=", "") for d in defines))
+    os.makedirs(bdir, exist_ok=True)
+    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-lineinfo", "-I", CSRC, *("-D" + d for d in defines)]
     jobs = []
     objs = []
     for f in CUDA_SRCS:
-        o = os.path.join(BUILD, f + ".o")
+        o = os.path.join(bdir, f + ".o")
         objs.append(o)
         jobs.append([NVCC, *ARCH, *common, "-Xptxas", "-v", "-c", os.path.join(CSRC, f), "-o", o])
     for f in CXX_SRCS:
-        o = os.path.join(BUILD, f + ".o")
+        o = os.path.join(bdir, f + ".o")
         objs.append(o)
         jobs.append([NVCC, *common, "-Xcompiler", "-Wall", "-c", os.path.join(CSRC, f), "-o", o])
     with cf.ThreadPoolExecutor(max_workers=min(8, len(jobs))) as ex:
@@ -57,11 +60,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if verbose:
         for lg in logs:
             sys.stderr.write(lg)
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-lpthread"])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    defs = tuple(a[2:] for a in sys.argv[1:] if a.startswith("-D"))
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, defines=defs, out=outs[0] if outs else None))

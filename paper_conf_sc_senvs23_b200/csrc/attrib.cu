@@ -1,34 +1,33 @@
 // attrib.cu — PC-sample packing and the per-PC x stall-reason histogram
 // (§2.2, §3).
 //
-// Packed sample word: (slot << 5) | reason, slot = first_slot[kernel] + pc/16 (R30). Because a
-// histogram row is 32 bins wide the word IS the flat bin index: the hot loop is "validate, then
-// increment H[word]". Global atomics alone run at ~50-200 G samples/s on B200 (L2 atomic rate,
-// profiles/r01_atomics_microbench.txt) — far below the ~1.6 T samples/s HBM streams 4-byte
-// samples at — so the counting happens in shared memory:
+// Packed sample word = compact bin  cb = slot * R + reason  (slot = first_slot[kernel] + pc/16,
+// R = n_reasons active reasons; R30). Valid iff cb < P * R. The histogram H is int32 [P][32];
+// bin (slot, reason) lives at H[slot * 32 + reason].
 //
-//   * compact bins cb = slot * n_reasons + reason (only active reasons occupy shared memory);
-//   * the table packs two 16-bit counters per 32-bit word (114688 bins in 224 KB, one CTA
-//     of 1024 threads per SM); a counter that reaches 0x8000 is drained (-0x8000 in shared
-//     memory, +0x8000 to the global bin) by the one thread whose atomicAdd returned 0x7FFF, so a
-//     16-bit half can never carry into its neighbour (at most a few thousand increments can be in
-//     flight per SM between that add and the drain) and the counts stay exact;
-//   * samples stream in with 128-bit loads.
+// Global atomics alone run at 50-200 G samples/s on B200 (profiles/r01_atomics_microbench.txt),
+// far below the ~1.6 T samples/s HBM streams 4-byte samples at, so counting happens in shared
+// memory over a WINDOW of whole slots [ws, ws + nslots): table word (cb - ws*R) (32-bit counters)
+// or half (cb - ws*R) (16-bit counters, two per word). The compact word makes the per-sample fast
+// path tiny: off = cb - wb; in = off < lim; shared atomic on tab[in ? off : spare(lane)].
+// Samples outside the window (rare) take an out-of-line path after one warp vote per batch.
+//
+// 16-bit counters are exact: the returned old value flags a half that is already >= 0x8000; the
+// rare path moves 0x8000 of it to the global bin with a CAS, long before it could reach 0xFFFF
+// (at most a few thousand increments are in flight per SM).
+//
 // Strategies (gs_config.hist_mode):
-//   PRIVATE  fixed windows: the compact bin space is split into ranges of one table each; each
-//            CTA counts the samples of its range in a contiguous chunk; the CTAs of one chunk are
-//            launched adjacently so the re-reads of a chunk hit L2. Flushed once per CTA.
-//   WINDOW   one persistent CTA per SM streams a contiguous 1/grid of the samples in tiles and
-//            moves its window with the data: at a tile whose first sample falls outside the
-//            window, the table is flushed and re-based at the sample's kernel (whole kernel if it
-//            fits, else centred on the sample). Samples outside the window go straight to L2
-//            atomics. Suited to PC-sampling traces, which arrive grouped by kernel launch.
+//   PRIVATE  fixed slot ranges per CTA (the CTAs of one sample chunk are adjacent in launch
+//            order, so the re-reads of a chunk hit L2); used when the bins fit in <= 3 windows.
+//   WINDOW   one persistent CTA per SM; tiles of the sample stream come from a per-CTA queue
+//            with work stealing; the window follows the data (median slot of 32 samples of the
+//            next tile, decided by warp 0 while the CTA counts the current tile; the sample's
+//            whole kernel when it fits). Suited to PC-sampling traces, which arrive grouped by
+//            kernel launch.
 //   GLOBAL   one L2 atomic per valid sample (reference strategy).
-//   AUTO     PRIVATE if the compact bins fit in kMaxRanges tables, else WINDOW.
 #include <cuda_runtime.h>
 
 #include <algorithm>
-#include <cstdlib>
 
 #include "ctx.h"
 
@@ -36,13 +35,25 @@ namespace gs {
 namespace {
 
 constexpr int kThreadsGlobal = 512;
-constexpr int kThreadsSmem = 1024;
-constexpr uint32_t kTableWords = 56 * 1024 - 32;   // 224 KB of shared memory: 32-bit counters + 32 spares
+constexpr int kThreads = 1024;
+constexpr uint32_t kTableWords = 56 * 1024 - 32;   // + 32 spare words (one per lane) = 224 KB
 constexpr uint32_t kMaxRanges = 3;
-constexpr uint32_t kTile4 = 65536;                 // uint4 per window decision (256K samples)
+constexpr uint32_t kTile4 = 65536;                 // uint4 per tile (256K samples)
 constexpr int kVec = 4;                            // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
-constexpr uint32_t kTmaTableWords = 41600;  // TMA kernel: 16-bit pairs, 83200 bins (4378 slots at R = 19)
+
+// x / d for x < 2^32, 1 <= d <= 32: floor(x * ceil(2^40 / d) / 2^40) (error < 2^37 / 2^40 < 1/d)
+struct Div {
+  uint64_t m;
+  uint32_t d;
+};
+__host__ __device__ inline Div make_div(uint32_t d) { return Div{((1ull << 40) + d - 1) / d, d}; }
+__device__ __forceinline__ uint32_t divq(uint32_t x, Div v) { return (uint32_t)(((unsigned __int128)x * v.m) >> 40); }
+// H index of a compact bin
+__device__ __forceinline__ uint32_t hidx(uint32_t cb, Div v) {
+  const uint32_t q = divq(cb, v);
+  return q * 32u + (cb - q * v.d);
+}
 
 __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long* d_n_invalid) {
   for (int o = 16; o; o >>= 1) n_bad += __shfl_xor_sync(0xffffffffu, n_bad, o);
@@ -60,7 +71,7 @@ __global__ void k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc
     if (ok) {
       const KDesc K = kd[k];
       ok = (pc >> 4) < K.n;
-      if (ok) w = ((K.first + (pc >> 4)) << 5) | reason;
+      if (ok) w = (K.first + (pc >> 4)) * nr + reason;
     }
     words[i] = w;
     bad = ok ? 0 : 1;
@@ -69,8 +80,8 @@ __global__ void k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc
 }
 
 // -------------------------------------------------------------------------------- GLOBAL
-__global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* __restrict__ s, uint64_t n, uint32_t P,
-                                                                uint32_t nr, int32_t* __restrict__ H,
+__global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* __restrict__ s, uint64_t n,
+                                                                uint32_t pnr, Div dv, int32_t* __restrict__ H,
                                                                 unsigned long long* d_n_invalid) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   uint32_t bad = 0;
@@ -81,156 +92,153 @@ __global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* 
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      if ((w[q] >> 5) < P && (w[q] & 31u) < nr) atomicAdd(H + w[q], 1);
+      if (w[q] < pnr) atomicAdd(H + hidx(w[q], dv), 1);
       else bad++;
     }
   }
   for (uint64_t i = n4 * 4 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += stride) {
-    const uint32_t w = s[i];
-    if ((w >> 5) < P && (w & 31u) < nr) atomicAdd(H + w, 1);
+    if (s[i] < pnr) atomicAdd(H + hidx(s[i], dv), 1);
     else bad++;
   }
   count_invalid(bad, d_n_invalid);
 }
 
 // -------------------------------------------------------------------------------- shared-memory table
-// The table holds kTableWords 32-bit counters for the compact bins of a window of whole slots
-// [ws, ws + nslots), nslots = kTableWords / n_reasons: counter index (slot - ws) * n_reasons + reason.
-// Fast path per sample (8 instructions): d = (w >> 5) - ws; in = d < nslots && (w & 31) < nr;
-// smem[d * nr + (w & 31)] += 1 (no return value). Lanes outside the window take a warp-uniform
-// slow path: L2 atomic (WINDOW) / skip (PRIVATE: another CTA owns that range) / invalid count.
+struct Win {
+  uint32_t wb;   // first compact bin of the window (ws * R)
+  uint32_t lim;  // bins of the window inside [0, P * R)
+};
 
-template <bool SPILL_OUT>
-__device__ __forceinline__ void slow_one(uint32_t w, uint32_t P, uint32_t nr, int32_t* H, uint32_t& bad) {
-  if ((w >> 5) < P && (w & 31u) < nr) {
-    if (SPILL_OUT) atomicAdd(H + w, 1);
-  } else {
-    bad++;
+// Where a sample outside the window goes: OUT_DROP (PRIVATE: another CTA owns that range), OUT_RED
+// (L2 atomic), OUT_DEFER (WINDOW: appended to the CTA's ring, counted after the next window switch).
+enum { OUT_DROP = 0, OUT_RED = 1, OUT_DEFER = 2 };
+constexpr uint32_t kDeferCap = 4 * kTile4;  // words per ring half (one tile); two halves per CTA
+
+struct Spill {
+  uint32_t pnr;    // P * R: words >= pnr are invalid
+  Div dv;
+  int32_t* H;
+  uint32_t* cnt;   // shared: positions handed out in this ring half so far (monotone, wraps mod 2^32)
+  uint32_t* ring;  // the ring half of the current tile (kDeferCap words)
+  uint32_t base;   // its first position not yet consumed; appends stay below base + kDeferCap
+};
+
+__device__ __forceinline__ void red_bin(uint32_t w, const Spill& S) { atomicAdd(S.H + hidx(w, S.dv), 1); }
+
+// warp-aggregated append of the lanes with `mine` (all lanes of `am` call this together)
+__device__ __forceinline__ void defer_warp(uint32_t am, bool mine, uint32_t w, const Spill& S) {
+  const uint32_t m = __ballot_sync(am, mine);
+  if (!m) return;
+  const uint32_t lane = threadIdx.x & 31u, lead = __ffs(m) - 1;
+  uint32_t p = 0;
+  if (lane == lead) p = atomicAdd(S.cnt, (uint32_t)__popc(m));
+  p = __shfl_sync(am, p, lead) + __popc(m & ((1u << lane) - 1u));
+  if (mine) {
+    if (p - S.base < kDeferCap) S.ring[p & (kDeferCap - 1)] = w;
+    else red_bin(w, S);  // ring full: straight to L2
   }
 }
 
-// predicated shared-memory add of `one` (a run-time 1, so ptxas emits one predicated ATOMS.ADD
-// instead of a branch around ATOMS.POPC.INC)
-__device__ __forceinline__ void red_shared_add_if(uint32_t addr, uint32_t one, bool p) {
-  asm volatile(
-      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}" ::"r"(addr), "r"(one),
-      "r"((uint32_t)p)
-      : "memory");
-}
-
-// predicated L2 atomic: one instruction, no branch
-__device__ __forceinline__ void red_global_add_if(int32_t* addr, uint32_t v, bool p) {
-  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.relaxed.gpu.global.add.u32 [%0], %1;\n\t}" ::"l"(addr),
-               "r"(v), "r"((uint32_t)p)
-               : "memory");
-}
-
-// 32-bit counters: no return values, no rare path. Per sample: shared atomic on the window slot
-// (or the lane's spare word), plus a predicated L2 atomic when the sample is valid but outside the
-// window (WINDOW only; PRIVATE leaves it to the CTA that owns that range).
-template <bool SPILL_OUT, int N>
-__device__ __forceinline__ void count_batch(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
-                                            uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
-                                            uint32_t& bad) {
-#pragma unroll
-  for (int q = 0; q < N; q++) {
-    const uint32_t slot = w[q] >> 5, d = slot - ws, rs = w[q] & 31u;
-    const bool rok = rs < nr;
-    const bool in = d < nslots && rok;
-    atomicAdd(tab + (in ? d * nr + rs : kTableWords + (threadIdx.x & 31u)), one);  // spare: never flushed
-    const bool valid = rok && slot < P;
-    if (SPILL_OUT) red_global_add_if(H + w[q], one, valid && !in);
-    bad += valid ? 0u : 1u;
+// the rare part of a batch: outside the window (or invalid), or a 16-bit half that needs draining
+template <int OUT>
+__device__ __forceinline__ void out_of_window(uint32_t am, bool out, uint32_t w, const Spill& S, uint32_t& bad) {
+#if defined(GS_DIAG) && GS_DIAG == 5  // diagnostic: deferred samples dropped
+  if (OUT == OUT_DEFER) return;
+#endif
+#if defined(GS_DIAG) && GS_DIAG == 7  // diagnostic: n_invalid reports the deferred samples
+  if (OUT == OUT_DEFER) { if (out) bad++; return; }
+#endif
+#if defined(GS_DIAG) && GS_DIAG == 8  // diagnostic: n_invalid reports the samples sent to L2
+  if (OUT == OUT_RED) { if (out) bad++; return; }
+#endif
+  if (OUT == OUT_DEFER) defer_warp(am, out && w < S.pnr, w, S);
+  if (out) {
+    if (w >= S.pnr) bad++;
+    else if (OUT == OUT_RED) red_bin(w, S);
   }
 }
 
-// flush the window's counters into H and zero them; word i <-> slot ws + i / nr, reason i % nr
-__device__ void flush_table(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nwords, int32_t* H) {
-  const uint32_t step_q = blockDim.x / nr, step_r = blockDim.x % nr;
-  uint32_t q = threadIdx.x / nr, r = threadIdx.x % nr;
-  for (uint32_t i = threadIdx.x; i < nwords; i += blockDim.x) {
-    const uint32_t v = tab[i];
-    if (v) {
-      tab[i] = 0;
-      atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)v);
-    }
-    q += step_q;
-    r += step_r;
-    if (r >= nr) { r -= nr; q++; }
-  }
-}
-
-// ---- 16-bit packed variant: two counters per word, twice the bins per window. The increment
-// that takes a half from 0x7FFF to 0x8000 (bit 15 flips: (old ^ (old + inc)) & (inc << 15)) drains
-// 0x8000 to the global bin, so a half never carries into its neighbour (at most a few thousand
-// increments can be in flight per SM between that add and the drain). Counts stay exact.
-// rare path of count_batch16, out of line so its address arithmetic is not hoisted into the loop
-template <bool SPILL_OUT>
-__device__ __noinline__ void slow16(uint32_t w, uint32_t old, uint32_t sh, uint32_t idx, bool in, uint32_t P,
-                                    uint32_t nr, uint32_t* tab, int32_t* H, uint32_t* bad) {
-  if (!in) {
-    if ((w >> 5) < P && (w & 31u) < nr) {
-      if (SPILL_OUT) atomicAdd(H + w, 1);
-    } else {
-      (*bad)++;
-    }
-    return;
-  }
-  if (!((old >> sh) & 0x8000u)) return;
-  // the half was already >= 0x8000: move 0x8000 of it to the global bin. Several threads may race
-  // here; the CAS makes each successful drain subtract exactly 0x8000 once.
+// 16-bit drain (out of line): the half of tab[idx] selected by sh was already >= 0x8000
+__device__ __noinline__ void drain16(uint32_t* tab, uint32_t idx, uint32_t sh, uint32_t w, Div dv, int32_t* H) {
   uint32_t v = tab[idx];
-  while ((v >> sh) & 0x8000u) {
+  while ((v >> sh) & 0x8000u) {  // several threads may race; each successful CAS moves exactly 0x8000
     const uint32_t prev = atomicCAS(tab + idx, v, v - (0x8000u << sh));
     if (prev == v) {
-      atomicAdd(H + w, 0x8000);
+      atomicAdd(H + hidx(w, dv), 0x8000);
       return;
     }
     v = prev;
   }
 }
 
-// 16-bit packed counters, two per word. Per sample: one returning shared atomic; the returned old
-// value flags a half already at >= 0x8000 (drained in the rare path before it could reach 0xFFFF:
-// at most a few thousand increments are in flight per SM), so counts stay exact.
-template <bool SPILL_OUT, int N, uint32_t SPARE = kTableWords>
-__device__ __forceinline__ void count_batch16(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
-                                              uint32_t nslots, uint32_t* tab, uint32_t one, int32_t* H,
-                                              uint32_t& bad) {
+template <int OUT, int N>
+__device__ __forceinline__ void count32(const uint32_t (&w)[N], Win W, uint32_t* tab, uint32_t spare, uint32_t one,
+                                        const Spill& S, uint32_t& bad) {
+  bool all_in = true;
+#pragma unroll
+  for (int q = 0; q < N; q++) {
+    const uint32_t off = w[q] - W.wb;
+    const bool in = off < W.lim;
+    atomicAdd(tab + (in ? off : spare), one);  // the lane's spare word is never flushed
+    all_in &= in;
+  }
+  const uint32_t am = __activemask();
+  if (!__all_sync(am, all_in)) {
+#pragma unroll
+    for (int q = 0; q < N; q++) out_of_window<OUT>(am, w[q] - W.wb >= W.lim, w[q], S, bad);
+  }
+}
+
+template <int OUT, int N>
+__device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t* tab, uint32_t spare, uint32_t one,
+                                        const Spill& S, uint32_t& bad) {
+  // Per sample: off, in, word, half increment, one returning shared atomic, one mask test. A lane
+  // outside the window adds to its spare word (never flushed; kept nonzero) and its mask is all
+  // ones, so the same test flags "outside the window" and "half already >= 0x8000".
   uint32_t old[N], flag = 0;
 #pragma unroll
   for (int q = 0; q < N; q++) {
-    const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-    const bool in = d < nslots && rs < nr;
-    const uint32_t off = d * nr + rs;
-    const uint32_t inc = in ? ((off & 1u) ? 0x10000u : one) : 0u;
-    const uint32_t idx = in ? (off >> 1) : SPARE + (threadIdx.x & 31u);  // lane's spare word
-    old[q] = atomicAdd(tab + idx, inc);
-    flag |= (old[q] & (inc << 15)) | (in ? 0u : 1u);
+    const uint32_t off = w[q] - W.wb;
+    const bool in = off < W.lim;
+    const uint32_t inc = one << ((off & 1u) << 4);
+    old[q] = atomicAdd(tab + (in ? off >> 1 : spare), inc);
+    flag |= old[q] & (in ? inc << 15 : 0xffffffffu);
   }
-  if (__any_sync(__activemask(), flag)) {  // rare: a half at >= 0x8000, or a sample outside the window
+  const uint32_t am = __activemask();
+  if (__any_sync(am, flag)) {
 #pragma unroll
     for (int q = 0; q < N; q++) {
-      const uint32_t d = (w[q] >> 5) - ws, rs = w[q] & 31u;
-      const bool in = d < nslots && rs < nr;
-      const uint32_t off = d * nr + rs;
-      slow16<SPILL_OUT>(w[q], old[q], (off & 1u) << 4, off >> 1, in, P, nr, tab, H, &bad);
+      const uint32_t off = w[q] - W.wb;
+      out_of_window<OUT>(am, off >= W.lim, w[q], S, bad);
+      if (off < W.lim && ((old[q] >> ((off & 1u) << 4)) & 0x8000u))
+        drain16(tab, off >> 1, (off & 1u) << 4, w[q], S.dv, S.H);
     }
   }
 }
 
-// word i holds bins 2i (low half) and 2i + 1 (high half); bin b <-> slot ws + b / nr, reason b % nr
-__device__ void flush_table16(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H) {
-  const uint32_t stride = 2 * blockDim.x, step_q = stride / nr, step_r = stride % nr;
-  uint32_t q = (2 * threadIdx.x) / nr, r = (2 * threadIdx.x) % nr;
-  for (uint32_t i = threadIdx.x; 2 * i < nbins; i += blockDim.x) {
+// flush the window's counters into H and zero them (bin i of the window <-> slot ws + i / R,
+// reason i % R); P16: word i holds bins 2i (low half) and 2i + 1 (high half)
+template <bool P16>
+__device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H) {
+  const uint32_t per = P16 ? 2u : 1u;
+  const uint32_t stride = per * blockDim.x, step_q = stride / nr, step_r = stride % nr;
+  uint32_t q = (per * threadIdx.x) / nr, r = (per * threadIdx.x) % nr;
+  for (uint32_t i = threadIdx.x; per * i < nbins; i += blockDim.x) {
     const uint32_t v = tab[i];
+#if defined(GS_DIAG) && GS_DIAG == 6  // diagnostic: flush only zeroes
+    tab[i] = 0;
+    continue;
+#endif
     if (v) {
       tab[i] = 0;
-      if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
-      if (v >> 16) {
-        const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
-        atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
+      if (!P16) {
+        atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)v);
+      } else {
+        if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
+        if (v >> 16) {
+          const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
+          atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
+        }
       }
     }
     q += step_q;
@@ -239,23 +247,14 @@ __device__ void flush_table16(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t 
   }
 }
 
-template <bool P16, bool SPILL_OUT, int N>
-__device__ __forceinline__ void count_any(const uint32_t (&w)[N], uint32_t P, uint32_t nr, uint32_t ws,
-                                          uint32_t lim, uint32_t* tab, uint32_t one, int32_t* H, uint32_t& bad) {
-  if (P16) count_batch16<SPILL_OUT>(w, P, nr, ws, lim, tab, one, H, bad);
-  else count_batch<SPILL_OUT>(w, P, nr, ws, lim, tab, one, H, bad);
-}
-
 // Tile queue of the WINDOW kernel. Chunk c (CTA c's contiguous share) is cut into tiles of kTile4
 // uint4; rng[c] = (head << 32) | stolen counts tiles taken from the front by the owner and from the
-// back by other CTAs that finished their own chunk (work stealing keeps all SMs busy to the end
-// while each CTA still walks its own chunk front to back, so windows change rarely).
+// back by CTAs that finished their own chunk (work stealing: every SM stays busy to the end while
+// each CTA still walks its own chunk front to back, so windows change rarely).
 __device__ __forceinline__ uint32_t n_tiles(uint64_t c, uint64_t chunk, uint64_t n) {
   const uint64_t a4 = c * chunk / 4, e = (c + 1) * chunk < n ? (c + 1) * chunk : n, e4 = e / 4;
   return e4 > a4 ? (uint32_t)((e4 - a4 + kTile4 - 1) / kTile4) : 0u;
 }
-
-// returns (chunk << 32) | tile, or ~0 when every tile of every chunk has been taken
 __device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, uint32_t grid, uint64_t chunk,
                                         uint64_t n) {
   const uint32_t mine = n_tiles(me, chunk, n);
@@ -280,323 +279,238 @@ __device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, ui
   }
 }
 
+// kernel of a slot: last k with kd[k].first <= slot (kernels are contiguous slot ranges, sorted)
+__device__ __forceinline__ uint32_t kernel_of(uint32_t slot, const KDesc* __restrict__ kd, uint32_t nk) {
+  uint32_t lo = 0, hi = nk;
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(&kd[mid].first) <= slot) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// the window for a slot: its whole kernel when that fits, else nslots slots centred on it inside
+// the kernel
+__device__ uint32_t window_for(uint32_t slot, const KDesc* __restrict__ kd, uint32_t nk, uint32_t nslots) {
+  const KDesc K = kd[kernel_of(slot, kd, nk)];
+  if (K.n <= nslots) return K.first;
+  uint32_t cws = slot > nslots / 2 ? slot - nslots / 2 : 0;
+  return min(max(cws, K.first), K.first + K.n - nslots);
+}
+
+// median slot of one valid-or-not probe per lane (~0u if no lane holds a valid word)
+__device__ __forceinline__ uint32_t probe_median(bool ok, uint32_t slot) {
+  uint32_t le = 0;
+  for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
+  const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
+  return __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
+}
+
+// uint4 [i0, i1) of the stream, thread ct of nct: kVec 128-bit loads in flight, then the batch
+template <int OUT, bool P16>
+__device__ __forceinline__ void count_span(const uint4* __restrict__ s4, uint64_t i0, uint64_t i1, uint32_t ct,
+                                           uint32_t nct, Win W, uint32_t* tab, uint32_t spare, uint32_t one,
+                                           const Spill& S, uint32_t& bad) {
+  uint64_t i = i0 + ct;
+  for (; i + (kVec - 1) * nct < i1; i += kVec * nct) {
+    uint32_t w[4 * kVec];
+#pragma unroll
+    for (int u = 0; u < kVec; u++) {
+      const uint4 v = __ldg(s4 + i + u * nct);
+      w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
+    }
+    if (P16) {  // returning atomics: batches of 4 keep the old values in registers
+#pragma unroll
+      for (int u = 0; u < kVec; u++) {
+        const uint32_t wq[4] = {w[4 * u], w[4 * u + 1], w[4 * u + 2], w[4 * u + 3]};
+        count16<OUT>(wq, W, tab, spare, one, S, bad);
+      }
+    } else {
+      count32<OUT>(w, W, tab, spare, one, S, bad);
+    }
+  }
+  for (; i < i1; i += nct) {
+    const uint4 v = __ldg(s4 + i);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+    if (P16) count16<OUT>(w, W, tab, spare, one, S, bad);
+    else count32<OUT>(w, W, tab, spare, one, S, bad);
+  }
+}
+
+// ring positions [b, b + nd) of one half, all threads, 16 loads in flight; what falls outside the
+// window goes to L2. Padding lanes read an invalid word, counted as invalid and taken back out.
+template <bool P16>
+__device__ __forceinline__ void count_ring(const uint32_t* ring, uint32_t b, uint32_t nd, Win W, uint32_t* tab,
+                                           uint32_t spare, uint32_t one, const Spill& S, uint32_t& bad) {
+  for (uint32_t j0 = 0; j0 < nd; j0 += 16 * blockDim.x) {
+    uint32_t w[16], pad = 0;
+#pragma unroll
+    for (int u = 0; u < 16; u++) {
+      const uint32_t j = j0 + u * blockDim.x + threadIdx.x;
+      w[u] = j < nd ? ring[(b + j) & (kDeferCap - 1)] : 0xffffffffu;
+      pad += j < nd ? 0u : 1u;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t wq[4] = {w[4 * u], w[4 * u + 1], w[4 * u + 2], w[4 * u + 3]};
+      if (P16) count16<OUT_RED>(wq, W, tab, spare, one, S, bad);
+      else count32<OUT_RED>(wq, W, tab, spare, one, S, bad);
+    }
+    bad -= pad;
+  }
+}
+
 // DYN = false: PRIVATE (fixed slot range per CTA); DYN = true: WINDOW (window follows the data)
 template <bool DYN, bool P16>
-__global__ void __launch_bounds__(kThreadsSmem, 1)
-    k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
-                uint32_t nk, uint32_t n_ranges, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
-                unsigned long long* d_n_invalid, unsigned long long* rng) {
+__global__ void __launch_bounds__(kThreads, 1)
+    k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv,
+                const KDesc* __restrict__ kd, uint32_t nk, uint32_t n_ranges, uint64_t chunk, uint32_t one,
+                int32_t* __restrict__ H, unsigned long long* d_n_invalid, unsigned long long* rng,
+                uint32_t* __restrict__ defer_ring) {
+  constexpr int OUT = DYN ? OUT_DEFER : OUT_DROP;
   extern __shared__ uint32_t tab[];
-  __shared__ uint32_t sh_ws[2];
+  __shared__ uint32_t sh_ws[2], sh_ws2[2], sh_split[2];  // window, second window, split (uint4)
   __shared__ unsigned long long sh_tile[2];
+  __shared__ uint32_t sh_ndefer[2];  // per ring half: tile `it` defers into half it & 1
+  const uint32_t pnr = P * nr;
   const uint32_t nslots = (P16 ? 2 * kTableWords : kTableWords) / nr;
+  const uint32_t spare = kTableWords + (threadIdx.x & 31u);
   const uint32_t range = DYN ? 0u : blockIdx.x % n_ranges;
   const uint64_t ci = DYN ? blockIdx.x : blockIdx.x / n_ranges;
   uint32_t ws = DYN ? kNoWindow : range * nslots;
-  uint32_t lim = DYN ? 0u : min(nslots, P - min(P, ws));  // slots of the window inside [0, P)
-  for (uint32_t i = threadIdx.x; i < kTableWords; i += blockDim.x) tab[i] = 0;
+  Win W{0, 0};
+  if (!DYN) W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
+  for (uint32_t i = threadIdx.x; i < kTableWords + 32; i += blockDim.x) tab[i] = i < kTableWords ? 0u : 1u;
+  if (threadIdx.x < 2) sh_ndefer[threadIdx.x] = 0;
   uint32_t bad = 0;
+  uint32_t* const ring0 = DYN ? defer_ring + (uint64_t)blockIdx.x * 2 * kDeferCap : nullptr;
+  uint32_t dstart0 = 0, dstart1 = 0;  // per half: first position not yet consumed
+  Spill S{pnr, dv, H, nullptr, nullptr, 0};
   const uint4* s4 = reinterpret_cast<const uint4*>(s);
   __syncthreads();
-  uint64_t t4 = ci * chunk / 4;  // PRIVATE: walk the own chunk
+  uint64_t t4 = ci * chunk / 4, t4e = 0;  // PRIVATE: walk the own chunk
   const uint64_t e_own = (ci + 1) * chunk < n ? (ci + 1) * chunk : n, e4_own = e_own / 4;
   for (uint32_t it = 0;; it++) {
-    uint64_t t4e;
     if (DYN) {
-      const auto tile_span = [&](unsigned long long tile) {
+      const auto span = [&](unsigned long long tile, uint64_t& a4, uint64_t& b4) {
         const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
         const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
-        t4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
-        t4e = t4 + kTile4 < ce / 4 ? t4 + kTile4 : ce / 4;
+        a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
+        b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
       };
-      // warp 0 grabs the next tile and picks its window while the CTA counts the current one
+      // warp 0 grabs the next tile and picks its window(s) while the CTA counts the current one,
+      // from 32 evenly spaced probe samples of the tile (lane j probes position j/32):
+      //  * the probes' kernels form two runs (the tile crosses from one kernel launch into the
+      //    next, as a PC-sampling trace does): the tile is split at the first probe of the second
+      //    run; each part gets the window of its own probes (one flush mid-tile);
+      //  * otherwise one window: the current one if it holds all valid probes (a large kernel's
+      //    window re-centres when the median nears its edge), else the window of the median.
+      // For each part, the current window stays when it holds all of the part's valid probes.
+      // Samples outside the window in force are deferred (ring) to the next tile's top.
       const auto decide = [&](uint32_t buf) {
         unsigned long long tile = 0;
         if (threadIdx.x == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
         tile = __shfl_sync(0xffffffffu, tile, 0);
-        uint32_t nws = ws;
+        uint32_t nws = ws, nws2 = kNoWindow, split = 0;
         if (tile != ~0ull) {
           uint64_t a4, b4;
-          {
-            const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
-            const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
-            a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
-            b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
-          }
-          // window: around the median slot of 32 evenly spaced samples (robust to the cold tail
-          // of a kernel's samples); the whole kernel if it fits
-          const uint32_t w = __ldg(s + 4 * (a4 + (b4 - a4) * threadIdx.x / 32));
-          const bool ok = (w >> 5) < P && (w & 31u) < nr;
-          const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
-          uint32_t le = 0;  // lanes whose slot is <= mine
-          for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
-          const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
-          // median: the smallest valid slot with more than half of the valid samples at or below it
-          const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
-          if (med != 0xffffffffu && (ws == kNoWindow || med - ws >= nslots || med - ws < nslots / 8 ||
-                                     med - ws >= nslots - nslots / 8)) {
-            uint32_t lo = 0, hi = nk;  // kernel of the slot: last k with first <= slot
-            while (hi - lo > 1) {
-              const uint32_t mid = (lo + hi) >> 1;
-              if (__ldg(&kd[mid].first) <= med) lo = mid;
-              else hi = mid;
-            }
-            const KDesc K = kd[lo];
-            uint32_t cws;
-            if (K.n <= nslots) cws = K.first;                       // the whole kernel fits
-            else {                                                  // centre on the median, inside the kernel
-              cws = med > nslots / 2 ? med - nslots / 2 : 0;
-              cws = min(max(cws, K.first), K.first + K.n - nslots);
-            }
-            if (ws == kNoWindow || cws != ws) nws = cws;
+          span(tile, a4, b4);
+          const uint64_t at4 = a4 + (b4 - a4) * threadIdx.x / 32;
+          const uint32_t w = __ldg(s + 4 * at4);
+          const bool ok = w < pnr;
+          const uint32_t slot = ok ? divq(w, dv) : 0xffffffffu;
+          const uint32_t k = ok ? kernel_of(slot, kd, nk) : 0xffffffffu;
+          const uint32_t okm = __ballot_sync(0xffffffffu, ok);
+          const uint32_t k0 = __reduce_min_sync(0xffffffffu, k), k1 = __reduce_max_sync(0xffffffffu, ok ? k : 0u);
+          const uint32_t m0 = __ballot_sync(0xffffffffu, ok && k == k0), m1 = __ballot_sync(0xffffffffu, ok && k == k1);
+          const uint32_t lane = threadIdx.x & 31u;
+          // one window for the probes of mask pm: keep the current one if it holds them all
+          const auto pick = [&](uint32_t pm, uint32_t cur) {
+            const bool mine = (pm >> lane) & 1u;
+            const uint32_t outm = __ballot_sync(0xffffffffu, mine && (cur == kNoWindow || slot - cur >= nslots));
+            const uint32_t med = probe_median(mine, slot);
+            if (med == 0xffffffffu) return cur;
+            if (!outm && med - cur >= nslots / 8 && med - cur < nslots - nslots / 8) return cur;
+            return window_for(med, kd, nk, nslots);
+          };
+          // two runs: valid probes all in k0 or k1 (k0 != k1), every k0 probe before every k1 probe
+          const bool two_runs = okm && k0 != k1 && (m0 | m1) == okm && 31 - __clz(m0) < __ffs(m1) - 1;
+          if (two_runs) {
+            nws = pick(m0, ws);
+            nws2 = pick(m1, nws);
+            if (nws2 != nws) split = (uint32_t)(__shfl_sync(0xffffffffu, at4, __ffs(m1) - 1) - a4);
+            else nws2 = kNoWindow;
+          } else {
+            nws = pick(okm, ws);
           }
         }
         if (nws == kNoWindow) nws = 0;
         if (threadIdx.x == 0) {
           sh_tile[buf] = tile;
           sh_ws[buf] = nws;
+          sh_ws2[buf] = nws2;
+          sh_split[buf] = split;
         }
       };
       if (it == 0 && threadIdx.x < 32) decide(0);
       __syncthreads();
       const unsigned long long tile = sh_tile[it & 1];
-      if (tile == ~0ull) break;
-      tile_span(tile);
-      const uint32_t nws = sh_ws[it & 1];
-      if (nws != ws) {
+      const uint32_t nws = sh_ws[it & 1], nws2 = sh_ws2[it & 1], split = sh_split[it & 1];
+      // the previous tile's deferred samples: its half is quiet now (this tile appends to the other)
+      const uint32_t ph = (it + 1) & 1u, dend = sh_ndefer[ph], dbase = ph ? dstart1 : dstart0;
+      const uint32_t nd = it ? dend - dbase : 0u;
+      if (tile != ~0ull && nws != ws) {
         if (ws != kNoWindow) {
-          if (P16) flush_table16(tab, ws, nr, lim * nr, H);
-          else flush_table(tab, ws, nr, lim * nr, H);
+          flush<P16>(tab, ws, nr, W.lim, H);
           __syncthreads();
         }
         ws = nws;
-        lim = min(nslots, P - min(P, ws));
+        W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
       }
-      if (threadIdx.x < 32) decide((it + 1) & 1);
-    } else {
+      if (tile != ~0ull && threadIdx.x < 32) decide((it + 1) & 1);
+      if (nd) count_ring<P16>(ring0 + ph * kDeferCap, dbase, nd, W, tab, spare, one, S, bad);
+      if (ph) dstart1 = dend;
+      else dstart0 = dend;
+      if (tile == ~0ull) break;
+      // this tile appends to half it & 1, consumed at the next tile's top; a later tile reuses the
+      // half only after a barrier that follows that consumption
+      S.cnt = &sh_ndefer[it & 1u];
+      S.ring = ring0 + (it & 1u) * kDeferCap;
+      S.base = (it & 1u) ? dstart1 : dstart0;
+      span(tile, t4, t4e);
+      // WINDOW: warp 0 only decides windows (it would otherwise be the straggler of every tile);
+      // warps 1..31 count
+      const uint32_t ct = threadIdx.x - 32, nct = blockDim.x - 32;
+      if (nws2 == kNoWindow) {
+        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4, t4e, ct, nct, W, tab, spare, one, S, bad);
+      } else {
+        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4, t4 + split, ct, nct, W, tab, spare, one, S, bad);
+        __syncthreads();
+        if (nws2 != ws) {
+          flush<P16>(tab, ws, nr, W.lim, H);
+          __syncthreads();
+          ws = nws2;
+          W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
+        }
+        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4 + split, t4e, ct, nct, W, tab, spare, one, S, bad);
+      }
+    } else {  // PRIVATE: all warps walk the own chunk
       if (t4 >= e4_own) break;
       t4e = t4 + kTile4 < e4_own ? t4 + kTile4 : e4_own;
+      count_span<OUT, P16>(s4, t4, t4e, threadIdx.x, blockDim.x, W, tab, spare, one, S, bad);
+      t4 = t4e;
     }
-    uint64_t i = t4 + threadIdx.x;
-    for (; i + (kVec - 1) * blockDim.x < t4e; i += kVec * blockDim.x) {  // kVec 128-bit loads in flight
-      uint32_t w[4 * kVec];
-#pragma unroll
-      for (int u = 0; u < kVec; u++) {
-        const uint4 v = __ldg(s4 + i + u * blockDim.x);
-        w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
-      }
-      if (P16) {  // returning atomics: batches of 4 keep the old values in registers
-#pragma unroll
-        for (int u = 0; u < kVec; u++) {
-          const uint32_t wq[4] = {w[4 * u], w[4 * u + 1], w[4 * u + 2], w[4 * u + 3]};
-          count_any<P16, DYN>(wq, P, nr, ws, lim, tab, one, H, bad);
-        }
-      } else {
-        count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
-      }
-    }
-    for (; i < t4e; i += blockDim.x) {
-      const uint4 v = __ldg(s4 + i);
-      const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-      count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
-    }
-    if (!DYN) t4 = t4e;
   }
-  // the last chunk's words after its last 16-byte boundary (< 4 words), counted by its owner
-  if (e_own == n) {
-    if (DYN && ws == kNoWindow) {  // a window is needed even if no tile was processed
-      ws = 0;
-      lim = min(nslots, P);
-    }
+  // the last chunk's words after its last 16-byte boundary (< 4 words): L2 atomics
+  if (e_own == n && range == 0)
     for (uint64_t i = e4_own * 4 + threadIdx.x; i < n; i += blockDim.x) {
-      const uint32_t w[1] = {s[i]};
-      count_any<P16, DYN>(w, P, nr, ws, lim, tab, one, H, bad);
-    }
-  }
-  if (range == 0) count_invalid(bad, d_n_invalid);
-  __syncthreads();
-  if (ws != kNoWindow) {
-    if (P16) flush_table16(tab, ws, nr, lim * nr, H);
-    else flush_table(tab, ws, nr, lim * nr, H);
-  }
-}
-
-// =============================================================================== TMA-fed WINDOW kernel
-// Warp-specialised: warp 0 is the producer (tile queue, window choice, TMA bulk copies of sample
-// stages into shared memory); warps 1..31 consume one 128-bit word (4 samples) each per stage.
-// kStages stages of kStage4 uint4 keep ~62 KB of samples in flight per SM independently of
-// registers (the register-fed kernel was memory-latency bound: 57% long-scoreboard stalls).
-constexpr int kConsumerWarps = 31;
-constexpr uint32_t kStage4 = kConsumerWarps * 32;          // uint4 per stage: one per consumer thread
-constexpr uint32_t kStageBytes = kStage4 * 16;             // 15872 B
-constexpr int kStages = 4;
-constexpr size_t kTmaSmem = (size_t)kStages * kStageBytes + (size_t)(kTmaTableWords + 32) * 4;
-
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_tx(unsigned long long* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t parity) {
-  uint32_t done = 0;
-  while (!done)
-    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-                 : "=r"(done)
-                 : "r"(smem_u32(b)), "r"(parity)
-                 : "memory");
-}
-__device__ __forceinline__ void tma_load(void* dst, const void* src, uint32_t bytes, unsigned long long* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, %0;" ::"r"(kConsumerWarps * 32) : "memory"); }
-
-// flush helpers over an explicit thread range [0, nt)
-__device__ void flush_pairs(uint32_t* tab, uint32_t words, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H,
-                            uint32_t t, uint32_t nt) {
-  const uint32_t stride = 2 * nt, step_q = stride / nr, step_r = stride % nr;
-  uint32_t q = (2 * t) / nr, r = (2 * t) % nr;
-  for (uint32_t i = t; i < words && 2 * i < nbins; i += nt) {
-    const uint32_t v = tab[i];
-    if (v) {
-      tab[i] = 0;
-      if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
-      if (v >> 16) {
-        const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
-        atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
-      }
-    }
-    q += step_q;
-    r += step_r;
-    if (r >= nr) { r -= nr; q++; }
-  }
-}
-
-__global__ void __launch_bounds__(32 * (kConsumerWarps + 1), 1)
-    k_hist_tma(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, const KDesc* __restrict__ kd,
-               uint32_t nk, uint64_t chunk, uint32_t one, int32_t* __restrict__ H, unsigned long long* d_n_invalid,
-               unsigned long long* rng) {
-  extern __shared__ __align__(128) uint8_t dyn[];
-  uint4* stage = reinterpret_cast<uint4*>(dyn);
-  uint32_t* tab = reinterpret_cast<uint32_t*>(dyn + (size_t)kStages * kStageBytes);
-  __shared__ __align__(8) unsigned long long full_bar[kStages], empty_bar[kStages];
-  __shared__ uint32_t meta_ws[kStages], meta_cnt[kStages];
-  const uint32_t nslots = 2 * kTmaTableWords / nr;
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (uint32_t i = threadIdx.x; i < kTmaTableWords + 32; i += blockDim.x) tab[i] = 0;
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kStages; i++) {
-      mbar_init(full_bar + i, 1);
-      mbar_init(empty_bar + i, kConsumerWarps);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  }
-  __syncthreads();
-  const uint4* s4 = reinterpret_cast<const uint4*>(s);
-  const uint64_t e_own = (blockIdx.x + 1) * chunk < n ? (blockIdx.x + 1) * chunk : n;
-  if (warp == 0) {
-    // ------------------------------------------------------------------ producer
-    uint32_t ws = kNoWindow, st = 0;
-    for (;;) {
-      unsigned long long tile = 0;
-      if (lane == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
-      tile = __shfl_sync(0xffffffffu, tile, 0);
-      if (tile == ~0ull) break;
-      const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
-      const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
-      const uint64_t t4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
-      const uint64_t t4e = t4 + kTile4 < ce / 4 ? t4 + kTile4 : ce / 4;
-      if (t4e <= t4) continue;
-      {  // window: around the median slot of 32 evenly spaced samples; the whole kernel if it fits
-        const uint32_t w = __ldg(s + 4 * (t4 + (t4e - t4) * lane / 32));
-        const bool ok = (w >> 5) < P && (w & 31u) < nr;
-        const uint32_t slot = ok ? (w >> 5) : 0xffffffffu;
-        uint32_t le = 0;
-        for (int j = 0; j < 32; j++) le += __shfl_sync(0xffffffffu, slot, j) <= slot ? 1u : 0u;
-        const uint32_t nvalid = __popc(__ballot_sync(0xffffffffu, ok));
-        const uint32_t med = __reduce_min_sync(0xffffffffu, ok && 2 * le > nvalid ? slot : 0xffffffffu);
-        if (med != 0xffffffffu && (ws == kNoWindow || med - ws >= nslots || med - ws < nslots / 8 ||
-                                   med - ws >= nslots - nslots / 8)) {
-          uint32_t lo = 0, hi = nk;
-          while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (__ldg(&kd[mid].first) <= med) lo = mid;
-            else hi = mid;
-          }
-          const KDesc K = kd[lo];
-          uint32_t cws;
-          if (K.n <= nslots) cws = K.first;
-          else {
-            cws = med > nslots / 2 ? med - nslots / 2 : 0;
-            cws = min(max(cws, K.first), K.first + K.n - nslots);
-          }
-          ws = cws;
-        }
-        if (ws == kNoWindow) ws = 0;
-      }
-      for (uint64_t p = t4; p < t4e; p += kStage4, st++) {
-        const uint32_t cnt = t4e - p < kStage4 ? (uint32_t)(t4e - p) : kStage4;
-        const uint32_t sb = st % kStages;
-        if (st >= (uint32_t)kStages) mbar_wait(empty_bar + sb, ((st / kStages) + 1) & 1);
-        if (lane == 0) {
-          meta_ws[sb] = ws;
-          meta_cnt[sb] = cnt;
-          mbar_arrive_tx(full_bar + sb, cnt * 16);
-          tma_load(stage + (size_t)sb * kStage4, s4 + p, cnt * 16, full_bar + sb);
-        }
-        __syncwarp();
-      }
-    }
-    const uint32_t sb = st % kStages;  // end marker
-    if (st >= (uint32_t)kStages) mbar_wait(empty_bar + sb, ((st / kStages) + 1) & 1);
-    if (lane == 0) {
-      meta_cnt[sb] = 0;
-      mbar_arrive(full_bar + sb);
-    }
-    return;
-  }
-  // -------------------------------------------------------------------- consumers
-  const uint32_t ct = threadIdx.x - 32, nct = kConsumerWarps * 32;
-  uint32_t ws = kNoWindow, lim = 0, bad = 0;
-  for (uint32_t st = 0;; st++) {
-    const uint32_t sb = st % kStages;
-    mbar_wait(full_bar + sb, (st / kStages) & 1);
-    const uint32_t cnt = meta_cnt[sb], nws = meta_ws[sb];
-    if (cnt == 0) break;
-    if (nws != ws) {  // window change: every consumer has finished the previous stages
-      consumer_sync();
-      if (ws != kNoWindow) flush_pairs(tab, kTmaTableWords, ws, nr, lim * nr, H, ct, nct);
-      consumer_sync();
-      ws = nws;
-      lim = min(nslots, P - min(P, ws));
-    }
-    const uint4 v = ct < cnt ? stage[(size_t)sb * kStage4 + ct] : make_uint4(0, 0, 0, 0);
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty_bar + sb);  // stage may be refilled; the data is in registers
-    if (ct < cnt) {
-      const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-      count_batch16<true, 4, kTmaTableWords>(w, P, nr, ws, lim, tab, one, H, bad);
-    }
-  }
-  // the last chunk's words after its last 16-byte boundary (< 4): L2 atomics
-  if (e_own == n)
-    for (uint64_t i = (n / 4) * 4 + ct; i < n; i += nct) {
-      const uint32_t w = s[i];
-      if ((w >> 5) < P && (w & 31u) < nr) atomicAdd(H + w, 1);
+      if (s[i] < pnr) atomicAdd(H + hidx(s[i], dv), 1);
       else bad++;
     }
-  for (int o = 16; o; o >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, o);
-  if (lane == 0 && bad) atomicAdd(d_n_invalid, (unsigned long long)bad);
-  consumer_sync();
-  if (ws != kNoWindow) flush_pairs(tab, kTmaTableWords, ws, nr, lim * nr, H, ct, nct);
+  if (range == 0) count_invalid(bad, d_n_invalid);
+  __syncthreads();
+  if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H);
 }
 
 }  // namespace
@@ -615,6 +529,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
                    int accumulate, bool zero_first) {
   cudaStream_t st = c->stream;
   const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
+  const Div dv = make_div(nr);
   if (zero_first && !accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, (uint64_t)P * 32 * 4, st));
   if (!n) return GS_OK;
   if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
@@ -623,7 +538,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   // peel the words before the first 16-byte boundary so the main kernels use 128-bit loads
   const uint64_t head = std::min<uint64_t>(n, ((16u - (reinterpret_cast<uintptr_t>(d_words) & 15u)) & 15u) / 4u);
   if (head) {
-    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P, nr, d_hist, d_n_invalid);
+    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P * nr, dv, d_hist, d_n_invalid);
     count_launch();
     GS_CUDA(c, cudaGetLastError());
     d_words += head;
@@ -643,17 +558,17 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   if (!bits) bits = (mode == GS_HIST_WINDOW && max_kn > nslots32) ? 16 : 32;  // whole kernels per window
   const uint32_t n_ranges = ranges(bits == 16 ? nslots16 : nslots32);
   if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_WINDOW;
-  c->last_hist_bits = (int)bits;
   c->last_hist_mode = (int)mode;
+  c->last_hist_bits = mode == GS_HIST_GLOBAL ? 0 : (int)bits;
   if (mode == GS_HIST_GLOBAL) {
     const uint64_t blocks = std::max<uint64_t>(
         1, std::min<uint64_t>((uint64_t)dev_sms * 4, (n + kThreadsGlobal * 4 - 1) / (kThreadsGlobal * 4)));
-    k_hist_global<<<(unsigned)blocks, kThreadsGlobal, 0, st>>>(d_words, n, P, nr, d_hist, d_n_invalid);
+    k_hist_global<<<(unsigned)blocks, kThreadsGlobal, 0, st>>>(d_words, n, P * nr, dv, d_hist, d_n_invalid);
     count_launch();
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
-  const size_t smem = (size_t)(kTableWords + 32) * 4;  // + one spare word per lane
+  const size_t smem = (size_t)(kTableWords + 32) * 4;
   const bool dyn = mode == GS_HIST_WINDOW;
   uint64_t chunks;
   if (dyn) {
@@ -665,23 +580,19 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   uint64_t chunk = (n + chunks - 1) / chunks;
   chunk = (chunk + 3) & ~3ull;
   chunks = (n + chunk - 1) / chunk;
-  if (dyn) {  // work-stealing tile queue, one 64-bit word per chunk
+  if (dyn) {  // work-stealing tile queue, one 64-bit word per chunk; two deferral ring halves per CTA
     GS_CUDA(c, dev_grow(&c->d_tileq, &c->tileq_cap, chunks));
     GS_CUDA(c, cudaMemsetAsync(c->d_tileq, 0, chunks * 8, st));
+    GS_CUDA(c, dev_grow(&c->d_defer, &c->defer_cap, chunks * 2 * kDeferCap));
   }
   auto launch = [&](auto kern, uint32_t grid, uint32_t nrg) -> gs_status {
     GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    kern<<<grid, kThreadsSmem, smem, st>>>(d_words, n, P, nr, c->d_kd, c->n_kernels, nrg, chunk, 1u, d_hist,
-                                           d_n_invalid, c->d_tileq);
+    kern<<<grid, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, nrg, chunk, 1u, d_hist,
+                                       d_n_invalid, c->d_tileq, c->d_defer);
     return GS_OK;
   };
   gs_status ls;
-  if (dyn && bits == 16 && getenv("GS_HIST_TMA")) {  // TMA-fed warp-specialised kernel (opt-in)
-    GS_CUDA(c, cudaFuncSetAttribute(k_hist_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmem));
-    k_hist_tma<<<(uint32_t)chunks, 32 * (kConsumerWarps + 1), kTmaSmem, st>>>(
-        d_words, n, P, nr, c->d_kd, c->n_kernels, chunk, 1u, d_hist, d_n_invalid, c->d_tileq);
-    ls = GS_OK;
-  } else if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
+  if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
                            : launch(k_hist_smem<true, false>, (uint32_t)chunks, 1u);
   else ls = bits == 16 ? launch(k_hist_smem<false, true>, (uint32_t)(chunks * n_ranges), n_ranges)
                        : launch(k_hist_smem<false, false>, (uint32_t)(chunks * n_ranges), n_ranges);
@@ -695,6 +606,9 @@ void attrib_free(gs_ctx* c) {
   if (c->d_tileq) cudaFree(c->d_tileq);
   c->d_tileq = nullptr;
   c->tileq_cap = 0;
+  if (c->d_defer) cudaFree(c->d_defer);
+  c->d_defer = nullptr;
+  c->defer_cap = 0;
   for (int b = 0; b < 2; b++) {
     if (c->h_stage[b]) cudaFreeHost(c->h_stage[b]);
     if (c->d_stage[b]) cudaFree(c->d_stage[b]);

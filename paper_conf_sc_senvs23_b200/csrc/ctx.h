@@ -98,6 +98,8 @@ struct gs_ctx {
   int last_hist_mode = 0, last_hist_bits = 0;
   unsigned long long* d_tileq = nullptr;  // WINDOW histogram work-stealing queue
   uint64_t tileq_cap = 0;
+  uint32_t* d_defer = nullptr;  // WINDOW histogram: per-CTA rings of deferred (out-of-window) samples
+  uint64_t defer_cap = 0;
   unsigned long long* d_rank_keys[2] = {nullptr, nullptr};
   uint32_t* d_rank_vals[2] = {nullptr, nullptr};
   uint64_t rank_cap = 0;

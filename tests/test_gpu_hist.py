@@ -67,7 +67,7 @@ def test_single_bin_drain(gs):
     from gen import sass as gsass
     s = gsass.config_sass("C1")
     n = 3_000_000
-    words = torch.full((n,), (17 << 5) | 6, dtype=torch.int32, device="cuda")
+    words = torch.full((n,), 17 * 19 + 6, dtype=torch.int32, device="cuda")
     for mode, bits in [(m, b) for m in MODES for b in (16, 32)]:
         ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
         ctx.load_sass(s.text)
@@ -87,7 +87,7 @@ def test_unaligned_views_and_invalid_words(gs, offset):
     tab = gsm.table_class_weighted(s.cls, 2_000_000, key=4)
     tr = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=4)
     base = torch.from_numpy(tr.packed().view(np.int32)).cuda()
-    bad = torch.tensor([-1, (s.P << 5) | 1, (3 << 5) | 19, (3 << 5) | 31], dtype=torch.int32, device="cuda")
+    bad = torch.tensor([-1, s.P * 19 + 1, s.P * 19, -16], dtype=torch.int32, device="cuda")
     buf = torch.cat([torch.zeros(offset, dtype=torch.int32, device="cuda"), bad, base, bad])
     view = buf[offset:]
     want = torch.from_numpy(tab.astype(np.int32).reshape(-1)).cuda()

@@ -1,0 +1,42 @@
+"""Times gs_attribute_samples alone on the bench workload (CUDA events), optionally with another
+build of the library (diagnostic variants).   python tools/time_hist.py [--lib PATH] [--bits 16] [--mode 0]"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+ap = argparse.ArgumentParser()
+ap.add_argument("--lib", default=None)
+ap.add_argument("--bits", type=int, default=0)
+ap.add_argument("--mode", type=int, default=0)
+ap.add_argument("--order", default="trace")
+ap.add_argument("--iters", type=int, default=10)
+a = ap.parse_args()
+import torch  # noqa: E402
+
+from paper_conf_sc_senvs23_b200 import binding  # noqa: E402
+if a.lib:
+    binding.load_library(a.lib)
+import bench  # noqa: E402
+from gen.device import DeviceTrace  # noqa: E402
+
+s, tr = bench.build_workload("C4", a.order)
+words = DeviceTrace(tr).packed()
+ctx = binding.Context(hist_mode=a.mode, hist_counter_bits=a.bits)
+ctx.load_sass(s.text)
+hist = torch.empty(ctx.n_instr * 32, dtype=torch.int32, device="cuda")
+ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
+for _ in range(3):
+    ctx.attribute_samples(words, hist, ninv)
+torch.cuda.synchronize()
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+for _ in range(a.iters):
+    ctx.attribute_samples(words, hist, ninv)
+e1.record()
+torch.cuda.synchronize()
+ms = e0.elapsed_time(e1) / a.iters
+print(f"lib={a.lib or 'default'} bits={a.bits} mode={a.mode} order={a.order}: {ms:.3f} ms, "
+      f"{tr.N / ms / 1e6:.1f} G samples/s, frac {(4 * tr.N + 128 * ctx.n_instr) / ms / 1e6 / 6555.8:.3f} "
+      f"n_invalid {int(ninv.item())}")

@@ -38,7 +38,10 @@ constexpr int kThreadsGlobal = 512;
 constexpr int kThreads = 1024;
 constexpr uint32_t kTableWords = 56 * 1024 - 32;   // + 32 spare words (one per lane) = 224 KB
 constexpr uint32_t kMaxRanges = 3;
-constexpr uint32_t kTile4 = 65536;                 // uint4 per tile (256K samples)
+#ifndef GS_TILE4
+#define GS_TILE4 16384
+#endif
+constexpr uint32_t kTile4 = GS_TILE4;              // uint4 per WINDOW tile (64K samples)
 constexpr int kVec = 4;                            // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
 
@@ -112,7 +115,7 @@ struct Win {
 // Where a sample outside the window goes: OUT_DROP (PRIVATE: another CTA owns that range), OUT_RED
 // (L2 atomic), OUT_DEFER (WINDOW: appended to the CTA's ring, counted after the next window switch).
 enum { OUT_DROP = 0, OUT_RED = 1, OUT_DEFER = 2 };
-constexpr uint32_t kDeferCap = 4 * kTile4;  // words per ring half (one tile); two halves per CTA
+constexpr uint32_t kDeferCap = 1u << 16;  // words per ring half; two halves per CTA (overflow -> L2)
 
 struct Spill {
   uint32_t pnr;    // P * R: words >= pnr are invalid
@@ -194,15 +197,17 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
                                         const Spill& S, uint32_t& bad) {
   // Per sample: off, in, word, half increment, one returning shared atomic, one mask test. A lane
   // outside the window adds to its spare word (never flushed; kept nonzero) and its mask is all
-  // ones, so the same test flags "outside the window" and "half already >= 0x8000".
-  uint32_t old[N], flag = 0;
+  // ones, so the same test flags "outside the window" and "half already >= 0x8000". One vote per
+  // batch; the rare path re-reads the words to find the halves to drain. Every thread that sees
+  // a half >= 0x8000 checks it before its next batch, so a half overshoots 0x8000 by at most
+  // (threads x batch) < 0x8000 increments before it is drained.
+  uint32_t flag = 0;
 #pragma unroll
   for (int q = 0; q < N; q++) {
     const uint32_t off = w[q] - W.wb;
     const bool in = off < W.lim;
     const uint32_t inc = one << ((off & 1u) << 4);
-    old[q] = atomicAdd(tab + (in ? off >> 1 : spare), inc);
-    flag |= old[q] & (in ? inc << 15 : 0xffffffffu);
+    flag |= atomicAdd(tab + (in ? off >> 1 : spare), inc) & (in ? inc << 15 : 0xffffffffu);
   }
   const uint32_t am = __activemask();
   if (__any_sync(am, flag)) {
@@ -210,7 +215,7 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
     for (int q = 0; q < N; q++) {
       const uint32_t off = w[q] - W.wb;
       out_of_window<OUT>(am, off >= W.lim, w[q], S, bad);
-      if (off < W.lim && ((old[q] >> ((off & 1u) << 4)) & 0x8000u))
+      if (flag && off < W.lim && ((tab[off >> 1] >> ((off & 1u) << 4)) & 0x8000u))
         drain16(tab, off >> 1, (off & 1u) << 4, w[q], S.dv, S.H);
     }
   }
@@ -219,11 +224,11 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
 // flush the window's counters into H and zero them (bin i of the window <-> slot ws + i / R,
 // reason i % R); P16: word i holds bins 2i (low half) and 2i + 1 (high half)
 template <bool P16>
-__device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H) {
+__device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H, uint32_t t, uint32_t nt) {
   const uint32_t per = P16 ? 2u : 1u;
-  const uint32_t stride = per * blockDim.x, step_q = stride / nr, step_r = stride % nr;
-  uint32_t q = (per * threadIdx.x) / nr, r = (per * threadIdx.x) % nr;
-  for (uint32_t i = threadIdx.x; per * i < nbins; i += blockDim.x) {
+  const uint32_t stride = per * nt, step_q = stride / nr, step_r = stride % nr;
+  uint32_t q = (per * t) / nr, r = (per * t) % nr;
+  for (uint32_t i = t; per * i < nbins; i += nt) {
     const uint32_t v = tab[i];
 #if defined(GS_DIAG) && GS_DIAG == 6  // diagnostic: flush only zeroes
     tab[i] = 0;
@@ -320,12 +325,8 @@ __device__ __forceinline__ void count_span(const uint4* __restrict__ s4, uint64_
       const uint4 v = __ldg(s4 + i + u * nct);
       w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
     }
-    if (P16) {  // returning atomics: batches of 4 keep the old values in registers
-#pragma unroll
-      for (int u = 0; u < kVec; u++) {
-        const uint32_t wq[4] = {w[4 * u], w[4 * u + 1], w[4 * u + 2], w[4 * u + 3]};
-        count16<OUT>(wq, W, tab, spare, one, S, bad);
-      }
+    if (P16) {
+      count16<OUT>(w, W, tab, spare, one, S, bad);
     } else {
       count32<OUT>(w, W, tab, spare, one, S, bad);
     }
@@ -342,12 +343,13 @@ __device__ __forceinline__ void count_span(const uint4* __restrict__ s4, uint64_
 // window goes to L2. Padding lanes read an invalid word, counted as invalid and taken back out.
 template <bool P16>
 __device__ __forceinline__ void count_ring(const uint32_t* ring, uint32_t b, uint32_t nd, Win W, uint32_t* tab,
-                                           uint32_t spare, uint32_t one, const Spill& S, uint32_t& bad) {
-  for (uint32_t j0 = 0; j0 < nd; j0 += 16 * blockDim.x) {
+                                           uint32_t spare, uint32_t one, const Spill& S, uint32_t& bad, uint32_t t,
+                                           uint32_t nt) {
+  for (uint32_t j0 = 0; j0 < nd; j0 += 16 * nt) {
     uint32_t w[16], pad = 0;
 #pragma unroll
     for (int u = 0; u < 16; u++) {
-      const uint32_t j = j0 + u * blockDim.x + threadIdx.x;
+      const uint32_t j = j0 + u * nt + t;
       w[u] = j < nd ? ring[(b + j) & (kDeferCap - 1)] : 0xffffffffu;
       pad += j < nd ? 0u : 1u;
     }
@@ -361,156 +363,215 @@ __device__ __forceinline__ void count_ring(const uint32_t* ring, uint32_t b, uin
   }
 }
 
-// DYN = false: PRIVATE (fixed slot range per CTA); DYN = true: WINDOW (window follows the data)
-template <bool DYN, bool P16>
+// ---------------------------------------------------------------------- PRIVATE
+// fixed slot range per CTA (range = blockIdx % n_ranges); the CTA walks its sample chunk
+template <bool P16>
 __global__ void __launch_bounds__(kThreads, 1)
-    k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv,
-                const KDesc* __restrict__ kd, uint32_t nk, uint32_t n_ranges, uint64_t chunk, uint32_t one,
-                int32_t* __restrict__ H, unsigned long long* d_n_invalid, unsigned long long* rng,
-                uint32_t* __restrict__ defer_ring) {
-  constexpr int OUT = DYN ? OUT_DEFER : OUT_DROP;
+    k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv, uint32_t n_ranges,
+                uint64_t chunk, uint32_t one, int32_t* __restrict__ H, unsigned long long* d_n_invalid) {
   extern __shared__ uint32_t tab[];
-  __shared__ uint32_t sh_ws[2], sh_ws2[2], sh_split[2];  // window, second window, split (uint4)
-  __shared__ unsigned long long sh_tile[2];
-  __shared__ uint32_t sh_ndefer[2];  // per ring half: tile `it` defers into half it & 1
   const uint32_t pnr = P * nr;
   const uint32_t nslots = (P16 ? 2 * kTableWords : kTableWords) / nr;
   const uint32_t spare = kTableWords + (threadIdx.x & 31u);
-  const uint32_t range = DYN ? 0u : blockIdx.x % n_ranges;
-  const uint64_t ci = DYN ? blockIdx.x : blockIdx.x / n_ranges;
-  uint32_t ws = DYN ? kNoWindow : range * nslots;
-  Win W{0, 0};
-  if (!DYN) W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
+  const uint32_t range = blockIdx.x % n_ranges;
+  const uint64_t ci = blockIdx.x / n_ranges;
+  const uint32_t ws = range * nslots;
+  const Win W{ws * nr, min(nslots, P - min(P, ws)) * nr};
   for (uint32_t i = threadIdx.x; i < kTableWords + 32; i += blockDim.x) tab[i] = i < kTableWords ? 0u : 1u;
-  if (threadIdx.x < 2) sh_ndefer[threadIdx.x] = 0;
   uint32_t bad = 0;
-  uint32_t* const ring0 = DYN ? defer_ring + (uint64_t)blockIdx.x * 2 * kDeferCap : nullptr;
-  uint32_t dstart0 = 0, dstart1 = 0;  // per half: first position not yet consumed
-  Spill S{pnr, dv, H, nullptr, nullptr, 0};
-  const uint4* s4 = reinterpret_cast<const uint4*>(s);
+  const Spill S{pnr, dv, H, nullptr, nullptr, 0};
   __syncthreads();
-  uint64_t t4 = ci * chunk / 4, t4e = 0;  // PRIVATE: walk the own chunk
-  const uint64_t e_own = (ci + 1) * chunk < n ? (ci + 1) * chunk : n, e4_own = e_own / 4;
-  for (uint32_t it = 0;; it++) {
-    if (DYN) {
-      const auto span = [&](unsigned long long tile, uint64_t& a4, uint64_t& b4) {
-        const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
-        const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
-        a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
-        b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
-      };
-      // warp 0 grabs the next tile and picks its window(s) while the CTA counts the current one,
-      // from 32 evenly spaced probe samples of the tile (lane j probes position j/32):
-      //  * the probes' kernels form two runs (the tile crosses from one kernel launch into the
-      //    next, as a PC-sampling trace does): the tile is split at the first probe of the second
-      //    run; each part gets the window of its own probes (one flush mid-tile);
-      //  * otherwise one window: the current one if it holds all valid probes (a large kernel's
-      //    window re-centres when the median nears its edge), else the window of the median.
-      // For each part, the current window stays when it holds all of the part's valid probes.
-      // Samples outside the window in force are deferred (ring) to the next tile's top.
-      const auto decide = [&](uint32_t buf) {
-        unsigned long long tile = 0;
-        if (threadIdx.x == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
-        tile = __shfl_sync(0xffffffffu, tile, 0);
-        uint32_t nws = ws, nws2 = kNoWindow, split = 0;
-        if (tile != ~0ull) {
-          uint64_t a4, b4;
-          span(tile, a4, b4);
-          const uint64_t at4 = a4 + (b4 - a4) * threadIdx.x / 32;
-          const uint32_t w = __ldg(s + 4 * at4);
-          const bool ok = w < pnr;
-          const uint32_t slot = ok ? divq(w, dv) : 0xffffffffu;
-          const uint32_t k = ok ? kernel_of(slot, kd, nk) : 0xffffffffu;
-          const uint32_t okm = __ballot_sync(0xffffffffu, ok);
-          const uint32_t k0 = __reduce_min_sync(0xffffffffu, k), k1 = __reduce_max_sync(0xffffffffu, ok ? k : 0u);
-          const uint32_t m0 = __ballot_sync(0xffffffffu, ok && k == k0), m1 = __ballot_sync(0xffffffffu, ok && k == k1);
-          const uint32_t lane = threadIdx.x & 31u;
-          // one window for the probes of mask pm: keep the current one if it holds them all
-          const auto pick = [&](uint32_t pm, uint32_t cur) {
-            const bool mine = (pm >> lane) & 1u;
-            const uint32_t outm = __ballot_sync(0xffffffffu, mine && (cur == kNoWindow || slot - cur >= nslots));
-            const uint32_t med = probe_median(mine, slot);
-            if (med == 0xffffffffu) return cur;
-            if (!outm && med - cur >= nslots / 8 && med - cur < nslots - nslots / 8) return cur;
-            return window_for(med, kd, nk, nslots);
-          };
-          // two runs: valid probes all in k0 or k1 (k0 != k1), every k0 probe before every k1 probe
-          const bool two_runs = okm && k0 != k1 && (m0 | m1) == okm && 31 - __clz(m0) < __ffs(m1) - 1;
-          if (two_runs) {
-            nws = pick(m0, ws);
-            nws2 = pick(m1, nws);
-            if (nws2 != nws) split = (uint32_t)(__shfl_sync(0xffffffffu, at4, __ffs(m1) - 1) - a4);
-            else nws2 = kNoWindow;
-          } else {
-            nws = pick(okm, ws);
-          }
-        }
-        if (nws == kNoWindow) nws = 0;
-        if (threadIdx.x == 0) {
-          sh_tile[buf] = tile;
-          sh_ws[buf] = nws;
-          sh_ws2[buf] = nws2;
-          sh_split[buf] = split;
-        }
-      };
-      if (it == 0 && threadIdx.x < 32) decide(0);
-      __syncthreads();
-      const unsigned long long tile = sh_tile[it & 1];
-      const uint32_t nws = sh_ws[it & 1], nws2 = sh_ws2[it & 1], split = sh_split[it & 1];
-      // the previous tile's deferred samples: its half is quiet now (this tile appends to the other)
-      const uint32_t ph = (it + 1) & 1u, dend = sh_ndefer[ph], dbase = ph ? dstart1 : dstart0;
-      const uint32_t nd = it ? dend - dbase : 0u;
-      if (tile != ~0ull && nws != ws) {
-        if (ws != kNoWindow) {
-          flush<P16>(tab, ws, nr, W.lim, H);
-          __syncthreads();
-        }
-        ws = nws;
-        W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
-      }
-      if (tile != ~0ull && threadIdx.x < 32) decide((it + 1) & 1);
-      if (nd) count_ring<P16>(ring0 + ph * kDeferCap, dbase, nd, W, tab, spare, one, S, bad);
-      if (ph) dstart1 = dend;
-      else dstart0 = dend;
-      if (tile == ~0ull) break;
-      // this tile appends to half it & 1, consumed at the next tile's top; a later tile reuses the
-      // half only after a barrier that follows that consumption
-      S.cnt = &sh_ndefer[it & 1u];
-      S.ring = ring0 + (it & 1u) * kDeferCap;
-      S.base = (it & 1u) ? dstart1 : dstart0;
-      span(tile, t4, t4e);
-      // WINDOW: warp 0 only decides windows (it would otherwise be the straggler of every tile);
-      // warps 1..31 count
-      const uint32_t ct = threadIdx.x - 32, nct = blockDim.x - 32;
-      if (nws2 == kNoWindow) {
-        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4, t4e, ct, nct, W, tab, spare, one, S, bad);
-      } else {
-        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4, t4 + split, ct, nct, W, tab, spare, one, S, bad);
-        __syncthreads();
-        if (nws2 != ws) {
-          flush<P16>(tab, ws, nr, W.lim, H);
-          __syncthreads();
-          ws = nws2;
-          W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
-        }
-        if (threadIdx.x >= 32) count_span<OUT, P16>(s4, t4 + split, t4e, ct, nct, W, tab, spare, one, S, bad);
-      }
-    } else {  // PRIVATE: all warps walk the own chunk
-      if (t4 >= e4_own) break;
-      t4e = t4 + kTile4 < e4_own ? t4 + kTile4 : e4_own;
-      count_span<OUT, P16>(s4, t4, t4e, threadIdx.x, blockDim.x, W, tab, spare, one, S, bad);
-      t4 = t4e;
-    }
-  }
+  const uint64_t e_own = (ci + 1) * chunk < n ? (ci + 1) * chunk : n;
+  count_span<OUT_DROP, P16>(reinterpret_cast<const uint4*>(s), ci * chunk / 4, e_own / 4, threadIdx.x, blockDim.x, W,
+                            tab, spare, one, S, bad);
   // the last chunk's words after its last 16-byte boundary (< 4 words): L2 atomics
   if (e_own == n && range == 0)
-    for (uint64_t i = e4_own * 4 + threadIdx.x; i < n; i += blockDim.x) {
+    for (uint64_t i = e_own / 4 * 4 + threadIdx.x; i < n; i += blockDim.x) {
       if (s[i] < pnr) atomicAdd(H + hidx(s[i], dv), 1);
       else bad++;
     }
   if (range == 0) count_invalid(bad, d_n_invalid);
   __syncthreads();
-  if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H);
+  flush<P16>(tab, ws, nr, W.lim, H, threadIdx.x, blockDim.x);
+}
+
+// ---------------------------------------------------------------------- WINDOW
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {  // release.cta
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {  // acquire.cta
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT%=;\n}" ::"r"(
+          smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// the 31 counting warps only (warp 0 keeps producing)
+__device__ __forceinline__ void bar_counters() { asm volatile("bar.sync 1, %0;" ::"r"(kThreads - 32) : "memory"); }
+
+constexpr uint32_t kItems = 8;  // descriptor ring depth
+struct Item {
+  uint64_t a4, b4;  // uint4 range of the stream
+  uint32_t ws;      // window (first slot) for the range
+  uint32_t last;    // 1: no more work
+};
+
+// One persistent CTA per SM. Warp 0 (producer) grabs tiles from the work-stealing queue, picks
+// each tile's window(s) from 32 probe samples and publishes (range, window) items through an
+// mbarrier ring; warps 1..31 (counters) count each item into the shared table. The counters only
+// synchronise with each other when the window changes (named barrier, flush, barrier), so tiles
+// can be small (short tail) without a CTA-wide barrier per tile.
+//
+// Window choice per tile (lane j probes position j/32 of the tile):
+//  * the probes' kernels form two runs (the tile crosses from one kernel launch into the next, as
+//    a PC-sampling trace does): two items split at the first probe of the second run, each with
+//    the window of its own probes;
+//  * otherwise one item with one window.
+// A part keeps the previous window when that holds all of its valid probes (a large kernel's
+// window re-centres when the median nears its edge); else the window of its probes' median.
+// Samples outside the window in force go to the CTA's deferral ring (half = epoch & 1, an epoch
+// being a run of items with one window) and are counted right after the next window switch,
+// against the new window (a straddling tile's early samples of the next kernel land there).
+template <bool P16>
+__global__ void __launch_bounds__(kThreads, 1)
+    k_hist_window(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv,
+                  const KDesc* __restrict__ kd, uint32_t nk, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
+                  unsigned long long* d_n_invalid, unsigned long long* rng, uint32_t* __restrict__ defer_ring) {
+  extern __shared__ uint32_t tab[];
+  __shared__ Item items[kItems];
+  __shared__ __align__(8) uint64_t full[kItems], empty[kItems];
+  __shared__ uint32_t sh_ndefer[2];
+  const uint32_t pnr = P * nr;
+  const uint32_t nslots = (P16 ? 2 * kTableWords : kTableWords) / nr;
+  const uint32_t lane = threadIdx.x & 31u;
+  for (uint32_t i = threadIdx.x; i < kTableWords + 32; i += blockDim.x) tab[i] = i < kTableWords ? 0u : 1u;
+  if (threadIdx.x < kItems) {
+    mbar_init(&full[threadIdx.x], 1);
+    mbar_init(&empty[threadIdx.x], kThreads / 32 - 1);
+  }
+  if (threadIdx.x < 2) sh_ndefer[threadIdx.x] = 0;
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+
+  const auto span = [&](unsigned long long tile, uint64_t& a4, uint64_t& b4) {
+    const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
+    const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
+    a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
+    b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
+  };
+
+  if (threadIdx.x < 32) {  // ------------------------------------------------ producer
+    uint32_t pws = kNoWindow, j = 0;
+    const auto publish = [&](uint64_t a4, uint64_t b4, uint32_t ws, uint32_t last) {
+      const uint32_t k = j % kItems;
+      if (lane == 0) {
+        mbar_wait(&empty[k], ((j / kItems) & 1u) ^ 1u);
+        items[k] = Item{a4, b4, ws, last};
+        mbar_arrive(&full[k]);
+      }
+      __syncwarp();
+      j++;
+    };
+    for (;;) {
+      unsigned long long tile = 0;
+      if (lane == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
+      tile = __shfl_sync(0xffffffffu, tile, 0);
+      if (tile == ~0ull) break;
+      uint64_t a4, b4;
+      span(tile, a4, b4);
+      const uint64_t at4 = a4 + (b4 - a4) * lane / 32;
+      const uint32_t w = __ldg(s + 4 * at4);
+      const bool ok = w < pnr;
+      const uint32_t slot = ok ? divq(w, dv) : 0xffffffffu;
+      const uint32_t k = ok ? kernel_of(slot, kd, nk) : 0xffffffffu;
+      const uint32_t okm = __ballot_sync(0xffffffffu, ok);
+      const uint32_t k0 = __reduce_min_sync(0xffffffffu, k), k1 = __reduce_max_sync(0xffffffffu, ok ? k : 0u);
+      const uint32_t m0 = __ballot_sync(0xffffffffu, ok && k == k0), m1 = __ballot_sync(0xffffffffu, ok && k == k1);
+      // one window for the probes of mask pm, given the window before them
+      const auto pick = [&](uint32_t pm, uint32_t cur) {
+        const bool mine = (pm >> lane) & 1u;
+        const uint32_t outm = __ballot_sync(0xffffffffu, mine && (cur == kNoWindow || slot - cur >= nslots));
+        const uint32_t med = probe_median(mine, slot);
+        if (med == 0xffffffffu) return cur == kNoWindow ? 0u : cur;
+        if (!outm && med - cur >= nslots / 8 && med - cur < nslots - nslots / 8) return cur;
+        return window_for(med, kd, nk, nslots);
+      };
+      // two runs: valid probes all in k0 or k1 (k0 != k1), every k0 probe before every k1 probe
+      const bool two_runs = okm && k0 != k1 && (m0 | m1) == okm && 31 - __clz(m0) < __ffs(m1) - 1;
+      if (two_runs) {
+        const uint32_t ws1 = pick(m0, pws), ws2 = pick(m1, ws1);
+        if (ws2 != ws1) {
+          const uint64_t mid = __shfl_sync(0xffffffffu, at4, __ffs(m1) - 1);
+          publish(a4, mid, ws1, 0);
+          publish(mid, b4, ws2, 0);
+        } else {
+          publish(a4, b4, ws1, 0);
+        }
+        pws = ws2;
+      } else {
+        pws = pick(okm, pws);
+        publish(a4, b4, pws, 0);
+      }
+    }
+    publish(0, 0, pws, 1);
+    return;
+  }
+
+  // --------------------------------------------------------------------------- counters
+  const uint32_t ct = threadIdx.x - 32, nct = kThreads - 32;
+  const uint32_t spare = kTableWords + lane;
+  const uint4* s4 = reinterpret_cast<const uint4*>(s);
+  uint32_t* const ring0 = defer_ring + (uint64_t)blockIdx.x * 2 * kDeferCap;
+  uint32_t bad = 0, ws = kNoWindow, epoch = 0, dstart0 = 0, dstart1 = 0;
+  Win W{0, 0};
+  Spill S{pnr, dv, H, &sh_ndefer[0], ring0, 0};
+  for (uint32_t j = 0;; j++) {
+    const uint32_t k = j % kItems;
+    mbar_wait(&full[k], (j / kItems) & 1u);
+    const Item it = items[k];
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[k]);
+    if (it.last) break;
+    if (it.ws != ws) {  // window switch: every counter is done with the old window
+      bar_counters();
+      if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H, ct, nct);
+      bar_counters();
+      ws = it.ws;
+      W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
+      if (ws != kNoWindow && j) {  // the ended epoch's deferred samples, against the new window
+        const uint32_t h = epoch & 1u, dend = sh_ndefer[h], db = h ? dstart1 : dstart0;
+        if (dend != db)  // positions past the capacity went to L2 when they were deferred
+          count_ring<P16>(ring0 + h * kDeferCap, db, min(dend - db, kDeferCap), W, tab, spare, one, S, bad, ct, nct);
+        if (h) dstart1 = dend;
+        else dstart0 = dend;
+        epoch++;
+      }
+      const uint32_t h = epoch & 1u;  // the new epoch appends to the other half
+      S.cnt = &sh_ndefer[h];
+      S.ring = ring0 + h * kDeferCap;
+      S.base = h ? dstart1 : dstart0;
+    }
+    count_span<OUT_DEFER, P16>(s4, it.a4, it.b4, ct, nct, W, tab, spare, one, S, bad);
+  }
+  bar_counters();
+  {  // the last epoch's deferred samples: what is not in the current window goes to L2
+    const uint32_t h = epoch & 1u, dend = sh_ndefer[h], db = h ? dstart1 : dstart0;
+    if (dend != db)
+      count_ring<P16>(ring0 + h * kDeferCap, db, min(dend - db, kDeferCap), W, tab, spare, one, S, bad, ct, nct);
+  }
+  // the stream's words after its last 16-byte boundary (< 4 words): L2 atomics
+  if (blockIdx.x == gridDim.x - 1)
+    for (uint64_t i = n / 4 * 4 + ct; i < n; i += nct) {
+      if (s[i] < pnr) atomicAdd(H + hidx(s[i], dv), 1);
+      else bad++;
+    }
+  count_invalid(bad, d_n_invalid);
+  bar_counters();
+  if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H, ct, nct);
 }
 
 }  // namespace
@@ -585,17 +646,24 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, cudaMemsetAsync(c->d_tileq, 0, chunks * 8, st));
     GS_CUDA(c, dev_grow(&c->d_defer, &c->defer_cap, chunks * 2 * kDeferCap));
   }
-  auto launch = [&](auto kern, uint32_t grid, uint32_t nrg) -> gs_status {
+  const auto prep = [&](auto kern) -> gs_status {
     GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    kern<<<grid, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, nrg, chunk, 1u, d_hist,
-                                       d_n_invalid, c->d_tileq, c->d_defer);
     return GS_OK;
   };
-  gs_status ls;
-  if (dyn) ls = bits == 16 ? launch(k_hist_smem<true, true>, (uint32_t)chunks, 1u)
-                           : launch(k_hist_smem<true, false>, (uint32_t)chunks, 1u);
-  else ls = bits == 16 ? launch(k_hist_smem<false, true>, (uint32_t)(chunks * n_ranges), n_ranges)
-                       : launch(k_hist_smem<false, false>, (uint32_t)(chunks * n_ranges), n_ranges);
+  gs_status ls = GS_OK;
+  if (dyn) {
+    const auto kern = bits == 16 ? k_hist_window<true> : k_hist_window<false>;
+    ls = prep(kern);
+    if (ls == GS_OK)
+      kern<<<(uint32_t)chunks, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, chunk, 1u, d_hist,
+                                                     d_n_invalid, c->d_tileq, c->d_defer);
+  } else {
+    const auto kern = bits == 16 ? k_hist_smem<true> : k_hist_smem<false>;
+    ls = prep(kern);
+    if (ls == GS_OK)
+      kern<<<(uint32_t)(chunks * n_ranges), kThreads, smem, st>>>(d_words, n, P, nr, dv, n_ranges, chunk, 1u, d_hist,
+                                                                  d_n_invalid);
+  }
   if (ls != GS_OK) return ls;
   count_launch();
   GS_CUDA(c, cudaGetLastError());

@@ -7,8 +7,9 @@
 
 One step = one pass of the whole path over one batch: gs_detect (reaching defs, loop marks, traces,
 rules, compaction) over this rank's kernels + gs_attribute_samples (histogram of this rank's
-sample shard) + [all_reduce of the histogram] + gs_rank_sites (join + rank, all sites, rows to a
-device buffer). Inputs (packed SASS records, packed samples) are resident in HBM before the
+sample shard, compact R-bin rows) + [reduce-scatter of the histogram by the kernel-aligned slot
+ranges of the detection shards] + gs_rank_sites_slice (join + rank of this rank's sites against
+its summed slice, rows to a device buffer). Inputs (packed SASS records, packed samples) are resident in HBM before the
 timed region. Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
@@ -193,6 +194,7 @@ def main():
     ap.add_argument("--order", default="trace", choices=["trace", "shuffled"])
     ap.add_argument("--hist-mode", type=int, default=0)
     ap.add_argument("--hist-bits", type=int, default=0, choices=[0, 16, 32])
+    ap.add_argument("--hist-row32", action="store_true", help="32-bin histogram rows instead of compact R-bin rows")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-samples", type=int, default=1 << 25)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -221,10 +223,14 @@ def main():
     kb, ke = gdist.kernel_range(s.n_instr, rank, world)
     words = DeviceTrace(tr, local).packed(a, b)
     n_local = b - a
-    ctx = g.Context(device=local, hist_mode=args.hist_mode, hist_counter_bits=args.hist_bits)
+    R = 19
+    row = 32 if args.hist_row32 else R     # compact rows: 4*R B per slot to zero, write and reduce
+    ctx = g.Context(device=local, n_reasons=R, hist_mode=args.hist_mode, hist_counter_bits=args.hist_bits,
+                    hist_row=row)
     ctx.load_sass(s.text)
     P = ctx.n_instr
-    hist = torch.empty(P * 32, dtype=torch.int32, device="cuda")
+    hist = torch.empty(P * row, dtype=torch.int32, device="cuda")
+    s0, s1 = gdist.slot_ranges(s.first_slot, s.n_instr, world)[rank]
     ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
     n_sites = ctx.detect(kb, ke)
     ranked_dev = torch.empty(max(1, n_sites) * binding.RANKED_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
@@ -244,8 +250,8 @@ def main():
         if record_hist:
             e1.record(stream)
             hist_events.append((e0, e1))
-        gdist.allreduce_hist(hist)
-        ctx.rank_sites(hist, k=None, out=ranked_dev)
+        part = gdist.reduce_scatter_hist(hist, row, gdist.slot_ranges(s.first_slot, s.n_instr, world))
+        ctx.rank_sites(part, k=None, out=ranked_dev, slot_begin=s0, slot_end=s1)
 
     for _ in range(args.warmup):
         step()
@@ -258,11 +264,13 @@ def main():
     l0 = binding.launch_count()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
+    torch.cuda.cudart().cudaProfilerStart()   # ncu --profile-from-start off: the timed steps only
     ev0.record(stream)
     for _ in range(args.steps):
         step(record_hist=True)
     ev1.record(stream)
     torch.cuda.synchronize()
+    torch.cuda.cudart().cudaProfilerStop()
     if world > 1:
         dist.barrier()
     launches = binding.launch_count() - l0
@@ -275,13 +283,16 @@ def main():
     ms_max, hist_ms_max = float(t[0]), float(t[1])
     mode = ctx.last_hist_mode()
 
-    # correctness guard on the bench configuration (closed form: mass and invalid count)
-    mass = int(hist.to(torch.int64).sum().item())
-    assert mass == tr.N and int(ninv.item()) == 0, (mass, tr.N, int(ninv.item()))
+    # correctness guard on the bench configuration (closed form: mass and invalid count; with a
+    # reduce-scatter each rank holds the summed rows of its own slot range)
+    mass = torch.tensor([int(hist[s0 * row:s1 * row].to(torch.int64).sum().item())], dtype=torch.int64, device="cuda")
+    if world > 1:
+        dist.all_reduce(mass)
+    assert int(mass.item()) == tr.N and int(ninv.item()) == 0, (int(mass.item()), tr.N, int(ninv.item()))
 
     # roofline of the dominant kernel (the attribution pass: histogram of this rank's samples)
     peak, peak_src = read_peaks()
-    alg_bytes = 4.0 * n_local + 4.0 * 32 * P          # samples read + histogram written once
+    alg_bytes = 4.0 * n_local + 4.0 * R * P           # samples read + histogram (R bins per slot) written once
     achieved = alg_bytes / (hist_ms_max * 1e-3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}_{args.order}.json")
@@ -295,7 +306,7 @@ def main():
     del words
     e2e_times = []
     n_rows = 0
-    for i in range(args.e2e_steps + 1):
+    for i in range(max(1, args.e2e_steps) + 1):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
@@ -303,8 +314,8 @@ def main():
         ctx.detect(kb, ke)
         ninv.zero_()
         ctx.attribute_samples(host_words, hist, ninv)     # H2D streamed inside the call
-        gdist.allreduce_hist(hist)
-        rows = ctx.rank_sites(hist, k=None)                # D2H of the ranked rows
+        part = gdist.reduce_scatter_hist(hist, row, gdist.slot_ranges(s.first_slot, s.n_instr, world))
+        rows = ctx.rank_sites(part, k=None, slot_begin=s0, slot_end=s1)   # D2H of the ranked rows
         rows = gdist.gather_ranked(rows, None)
         torch.cuda.synchronize()
         if i:

@@ -48,7 +48,11 @@ typedef struct {
   uint32_t shmem_min_loads; /* T_L of the SHMEM rule (R11). default 2                                 */
   uint32_t hist_mode;       /* histogram strategy, GS_HIST_*. default GS_HIST_AUTO                    */
   uint32_t hist_counter_bits; /* shared-memory counter width: 0 = auto, 16 (packed pairs) or 32      */
-  uint32_t reserved[2];
+  uint32_t hist_row;        /* bins per histogram row (one row per PC slot): 0 or 32 -> 32 (reason r at
+                               column r, the row padded to 32), or n_reasons -> compact rows holding only
+                               the active reasons (4*R bytes per slot: less to zero, write and reduce
+                               across GPUs). Any other value -> GS_E_INVAL.         */
+  uint32_t reserved;
 } gs_config;
 
 enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3 };
@@ -132,11 +136,11 @@ gs_status gs_kernel_stats_get(const gs_ctx *ctx, gs_kernel_stats *out, size_t ca
 gs_status gs_pack_samples(gs_ctx *ctx, const uint32_t *d_raw, uint64_t n, uint32_t *d_words,
                           unsigned long long *d_n_invalid);
 
-/* a-9: H[slot*32 + reason] += 1 for every valid packed word w = slot * n_reasons +
- * reason (valid iff w < n_instr * n_reasons); others are counted into *d_n_invalid (device u64,
- * added to). `samples` may be host
+/* a-9: H[slot*row + reason] += 1 for every valid packed word w = slot * n_reasons +
+ * reason (valid iff w < n_instr * n_reasons; row = gs_config.hist_row, 32 by default); others are
+ * counted into *d_n_invalid (device u64, added to). `samples` may be host
  * (pinned or pageable; streamed in chunks with copies overlapped) or device memory. d_hist is a
- * caller-owned device int32 array of n_instr*32 bins, zeroed first unless accumulate != 0.
+ * caller-owned device int32 array of n_instr*row bins, zeroed first unless accumulate != 0.
  * Async for device input; host input returns after the last chunk is consumed. */
 gs_status gs_attribute_samples(gs_ctx *ctx, const uint32_t *samples, uint64_t n, int32_t *d_hist,
                                unsigned long long *d_n_invalid, int accumulate);
@@ -147,6 +151,14 @@ gs_status gs_attribute_samples(gs_ctx *ctx, const uint32_t *samples, uint64_t n,
  * *n_out. Synchronises the stream. */
 gs_status gs_rank_sites(gs_ctx *ctx, const int32_t *d_hist, uint64_t k, gs_ranked_site *out,
                         uint64_t *n_out);
+/* Same as gs_rank_sites against a histogram SLICE: d_hist (device) holds the rows of slots
+ * [slot_begin, slot_end) only (row width gs_config.hist_row), e.g. this rank's part after a
+ * reduce-scatter of the histogram by the kernel-aligned slot ranges of the detection shards
+ * (SURVEY §8e, §8f row 1). The slice must cover every slot of the kernels of the last gs_detect,
+ * else GS_E_RANGE. ktot is computed for those kernels only. gs_rank_sites(ctx, h, ...) ==
+ * gs_rank_sites_slice(ctx, h, 0, n_instr, ...). Synchronises the stream. */
+gs_status gs_rank_sites_slice(gs_ctx *ctx, const int32_t *d_hist, uint64_t slot_begin, uint64_t slot_end,
+                              uint64_t k, gs_ranked_site *out, uint64_t *n_out);
 
 /* Number of CUDA kernels this library has launched in the process so far (its own kernels plus
  * the CUB radix-sort kernels of gs_rank_sites). Lets a harness count launches in a timed region. */

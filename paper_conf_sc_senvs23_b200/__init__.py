@@ -6,8 +6,8 @@ multi-GPU orchestration (dist.py).
 """
 from .binding import (GS_HIST_AUTO, GS_HIST_GLOBAL, GS_HIST_PRIVATE, GS_HIST_WINDOW, RANKED_DTYPE, RULES,
                       SITE_DTYPE, Context, GsError, gs_attribute_samples, gs_detect, gs_load_sass,
-                      gs_pack_samples, gs_rank_sites, load_library)
+                      gs_pack_samples, gs_rank_sites, gs_rank_sites_slice, load_library)
 
 __all__ = ["Context", "GsError", "load_library", "gs_load_sass", "gs_detect", "gs_pack_samples",
-           "gs_attribute_samples", "gs_rank_sites", "SITE_DTYPE", "RANKED_DTYPE", "RULES", "GS_HIST_AUTO",
+           "gs_attribute_samples", "gs_rank_sites", "gs_rank_sites_slice", "SITE_DTYPE", "RANKED_DTYPE", "RULES", "GS_HIST_AUTO",
            "GS_HIST_GLOBAL", "GS_HIST_PRIVATE", "GS_HIST_WINDOW"]

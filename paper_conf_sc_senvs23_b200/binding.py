@@ -35,7 +35,7 @@ class GsConfig(ctypes.Structure):
     _fields_ = [("trace_depth", ctypes.c_uint32), ("n_reasons", ctypes.c_uint32),
                 ("shmem_min_arith", ctypes.c_uint32), ("shmem_min_loads", ctypes.c_uint32),
                 ("hist_mode", ctypes.c_uint32), ("hist_counter_bits", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32 * 2)]
+                ("hist_row", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
 class GsError(RuntimeError):
@@ -45,7 +45,7 @@ class GsError(RuntimeError):
 _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
-           "gs_attribute_samples", "gs_rank_sites", "gs_last_hist_mode", "gs_launch_count"]
+           "gs_attribute_samples", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
 
 
 def launch_count() -> int:
@@ -77,6 +77,7 @@ def load_library(path: str = LIB_PATH):
         "gs_pack_samples": (I32, [P, P, U64, P, P]),
         "gs_attribute_samples": (I32, [P, P, U64, P, P, I32]),
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
+        "gs_rank_sites_slice": (I32, [P, P, U64, U64, U64, P, ctypes.POINTER(U64)]),
         "gs_last_hist_mode": (I32, [P]),
         "gs_launch_count": (U64, []),
     }
@@ -106,7 +107,7 @@ class Context:
 
     def __init__(self, device: int | None = None, stream=None, trace_depth: int = 64, n_reasons: int = 19,
                  shmem_min_arith: int = 1, shmem_min_loads: int = 2, hist_mode: int = GS_HIST_AUTO,
-                 hist_counter_bits: int = 0):
+                 hist_counter_bits: int = 0, hist_row: int = 32):
         import torch
         if not torch.cuda.is_available():
             raise GsError("no CUDA device: the library has no CPU fallback")
@@ -116,8 +117,10 @@ class Context:
             stream = torch.cuda.current_stream(self.device)
         self.torch_stream = stream
         handle = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
-        cfg = GsConfig(trace_depth, n_reasons, shmem_min_arith, shmem_min_loads, hist_mode, hist_counter_bits)
+        cfg = GsConfig(trace_depth, n_reasons, shmem_min_arith, shmem_min_loads, hist_mode, hist_counter_bits,
+                       hist_row)
         self.n_reasons = n_reasons
+        self.hist_row = hist_row or 32  # bins per histogram row: 32, or n_reasons (compact)
         self.trace_depth = trace_depth
         self.cfg = cfg
         h = ctypes.c_void_p()
@@ -215,7 +218,7 @@ class Context:
         import torch
         dev = torch.device("cuda", self.device)
         if hist is None:
-            hist = torch.empty(self.n_instr * 32, dtype=torch.int32, device=dev)
+            hist = torch.empty(self.n_instr * self.hist_row, dtype=torch.int32, device=dev)
         if n_invalid is None:
             n_invalid = torch.zeros(1, dtype=torch.int64, device=dev)
         n = samples.shape[0] if hasattr(samples, "shape") else len(samples)
@@ -227,19 +230,23 @@ class Context:
         return self.L.gs_last_hist_mode(self.h)
 
     # ---- a-11, a-12
-    def rank_sites(self, hist, k: int | None = None, out=None) -> np.ndarray:
-        """Returns a numpy RANKED_DTYPE array (host) or fills `out` (a device uint8 tensor of k*168 B)."""
+    def rank_sites(self, hist, k: int | None = None, out=None, slot_begin: int = 0,
+                   slot_end: int | None = None) -> np.ndarray:
+        """Returns a numpy RANKED_DTYPE array (host) or fills `out` (a device uint8 tensor of k*168 B).
+        `hist` holds the rows of slots [slot_begin, slot_end) (default: all slots)."""
         kk = (1 << 64) - 1 if k is None else k
+        slot_end = self.n_instr if slot_end is None else slot_end
         n_out = ctypes.c_uint64()
         if out is None:
             _, _, ns, _ = self.sites_device()
             m = ns if k is None else min(k, ns)
             res = np.zeros(m, RANKED_DTYPE)
-            self._check(self.L.gs_rank_sites(self.h, hist.data_ptr(), kk, res.ctypes.data if m else None,
-                                             ctypes.byref(n_out)), "gs_rank_sites")
+            self._check(self.L.gs_rank_sites_slice(self.h, hist.data_ptr(), slot_begin, slot_end, kk,
+                                                   res.ctypes.data if m else None, ctypes.byref(n_out)),
+                        "gs_rank_sites")
             return res[: n_out.value]
-        self._check(self.L.gs_rank_sites(self.h, hist.data_ptr(), kk, _ptr(out), ctypes.byref(n_out)),
-                    "gs_rank_sites")
+        self._check(self.L.gs_rank_sites_slice(self.h, hist.data_ptr(), slot_begin, slot_end, kk, _ptr(out),
+                                               ctypes.byref(n_out)), "gs_rank_sites")
         return n_out.value
 
 
@@ -262,3 +269,7 @@ def gs_attribute_samples(ctx: Context, samples, hist=None, n_invalid=None, accum
 
 def gs_rank_sites(ctx: Context, hist, k: int | None = None, out=None):
     return ctx.rank_sites(hist, k, out)
+
+
+def gs_rank_sites_slice(ctx: Context, hist, slot_begin: int, slot_end: int, k: int | None = None, out=None):
+    return ctx.rank_sites(hist, k, out, slot_begin=slot_begin, slot_end=slot_end)

@@ -70,7 +70,9 @@ gs_status gs_create(gs_ctx** out, int device, void* cuda_stream, const gs_config
   if (!c->cfg.n_reasons) c->cfg.n_reasons = 19;
   if (!c->cfg.shmem_min_arith) c->cfg.shmem_min_arith = 1;
   if (!c->cfg.shmem_min_loads) c->cfg.shmem_min_loads = 2;
+  if (!c->cfg.hist_row) c->cfg.hist_row = 32;
   if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_WINDOW ||
+      (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) ||
       (c->cfg.hist_counter_bits != 0 && c->cfg.hist_counter_bits != 16 && c->cfg.hist_counter_bits != 32)) {
     delete c;
     return GS_E_INVAL;
@@ -263,7 +265,7 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
     }
     c->stage_words = chunk;
   }
-  if (!accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * 32 * 4, c->stream));
+  if (!accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * c->cfg.hist_row * 4, c->stream));
   uint64_t done = 0;
   int b = 0;
   while (done < n) {
@@ -279,15 +281,29 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
   return GS_OK;
 }
 
-gs_status gs_rank_sites(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, uint64_t* n_out) {
+gs_status gs_rank_sites_slice(gs_ctx* c, const int32_t* d_hist, uint64_t slot_begin, uint64_t slot_end, uint64_t k,
+                              gs_ranked_site* out, uint64_t* n_out) {
   if (!c) return GS_E_INVAL;
   c->err.clear();
   if (!c->detected) return fail(c, GS_E_STATE, "gs_rank_sites before gs_detect");
-  if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
+  if (slot_begin > slot_end || slot_end > c->n_instr) return fail(c, GS_E_INVAL, "bad slot range");
+  if (!d_hist && slot_end > slot_begin) return fail(c, GS_E_INVAL, "null histogram");
   if (k && c->n_sites && !out) return fail(c, GS_E_INVAL, "null output");
+  // the detected kernels' slots [first(kb), first(ke)) must lie inside the slice
+  const uint64_t need0 = c->det_kb < c->n_kernels ? c->kd_h[c->det_kb].first : c->n_instr;
+  const uint64_t need1 = c->det_ke < c->n_kernels ? c->kd_h[c->det_ke].first : c->n_instr;
+  if (need1 > need0 && (slot_begin > need0 || slot_end < need1))
+    return fail(c, GS_E_RANGE, "histogram slice [" + std::to_string(slot_begin) + ", " + std::to_string(slot_end) +
+                                   ") does not cover the detected kernels' slots [" + std::to_string(need0) + ", " +
+                                   std::to_string(need1) + ")");
   GS_CUDA(c, cudaSetDevice(c->device));
   const bool host = out ? !is_device_ptr(out) : true;
-  return rank_run(c, d_hist, k, out, host, n_out);
+  return rank_run(c, d_hist, (uint32_t)slot_begin, k, out, host, n_out);
+}
+
+gs_status gs_rank_sites(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, uint64_t* n_out) {
+  if (!c) return GS_E_INVAL;
+  return gs_rank_sites_slice(c, d_hist, 0, c->n_instr, k, out, n_out);
 }
 
 uint64_t gs_launch_count(void) { return gs::g_launches.load(); }

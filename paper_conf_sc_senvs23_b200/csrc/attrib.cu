@@ -2,8 +2,9 @@
 // (§2.2, §3).
 //
 // Packed sample word = compact bin  cb = slot * R + reason  (slot = first_slot[kernel] + pc/16,
-// R = n_reasons active reasons; R30). Valid iff cb < P * R. The histogram H is int32 [P][32];
-// bin (slot, reason) lives at H[slot * 32 + reason].
+// R = n_reasons active reasons; R30). Valid iff cb < P * R. The histogram H is int32 [P][row]
+// (row = gs_config.hist_row: 32, or R for compact rows); bin (slot, reason) lives at
+// H[slot * row + reason] — with compact rows that is H[cb].
 //
 // Global atomics alone run at 50-200 G samples/s on B200 (profiles/r01_atomics_microbench.txt),
 // far below the ~1.6 T samples/s HBM streams 4-byte samples at, so counting happens in shared
@@ -45,17 +46,20 @@ constexpr uint32_t kTile4 = GS_TILE4;              // uint4 per WINDOW tile (64K
 constexpr int kVec = 4;                            // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
 
-// x / d for x < 2^32, 1 <= d <= 32: floor(x * ceil(2^40 / d) / 2^40) (error < 2^37 / 2^40 < 1/d)
+// x / d for x < 2^32, 1 <= d <= 32: floor(x * ceil(2^40 / d) / 2^40) (error < 2^37 / 2^40 < 1/d);
+// row = bins per H row (32, or d for compact rows)
 struct Div {
   uint64_t m;
   uint32_t d;
+  uint32_t row;
 };
-__host__ __device__ inline Div make_div(uint32_t d) { return Div{((1ull << 40) + d - 1) / d, d}; }
+__host__ __device__ inline Div make_div(uint32_t d, uint32_t row) { return Div{((1ull << 40) + d - 1) / d, d, row}; }
 __device__ __forceinline__ uint32_t divq(uint32_t x, Div v) { return (uint32_t)(((unsigned __int128)x * v.m) >> 40); }
-// H index of a compact bin
-__device__ __forceinline__ uint32_t hidx(uint32_t cb, Div v) {
+// H index of a compact bin (the bin itself when rows are compact)
+__device__ __forceinline__ uint64_t hidx(uint32_t cb, Div v) {
+  if (v.row == v.d) return cb;
   const uint32_t q = divq(cb, v);
-  return q * 32u + (cb - q * v.d);
+  return (uint64_t)q * v.row + (cb - q * v.d);
 }
 
 __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long* d_n_invalid) {
@@ -224,7 +228,8 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
 // flush the window's counters into H and zero them (bin i of the window <-> slot ws + i / R,
 // reason i % R); P16: word i holds bins 2i (low half) and 2i + 1 (high half)
 template <bool P16>
-__device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, int32_t* H, uint32_t t, uint32_t nt) {
+__device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t row, uint32_t nbins, int32_t* H, uint32_t t,
+                      uint32_t nt) {
   const uint32_t per = P16 ? 2u : 1u;
   const uint32_t stride = per * nt, step_q = stride / nr, step_r = stride % nr;
   uint32_t q = (per * t) / nr, r = (per * t) % nr;
@@ -237,12 +242,12 @@ __device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t nbins, i
     if (v) {
       tab[i] = 0;
       if (!P16) {
-        atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)v);
+        atomicAdd(H + (uint64_t)(ws + q) * row + r, (int32_t)v);
       } else {
-        if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * 32u + r, (int32_t)(v & 0xffffu));
+        if (v & 0xffffu) atomicAdd(H + (uint64_t)(ws + q) * row + r, (int32_t)(v & 0xffffu));
         if (v >> 16) {
           const uint32_t q1 = r + 1 == nr ? q + 1 : q, r1 = r + 1 == nr ? 0 : r + 1;
-          atomicAdd(H + (uint64_t)(ws + q1) * 32u + r1, (int32_t)(v >> 16));
+          atomicAdd(H + (uint64_t)(ws + q1) * row + r1, (int32_t)(v >> 16));
         }
       }
     }
@@ -392,7 +397,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   if (range == 0) count_invalid(bad, d_n_invalid);
   __syncthreads();
-  flush<P16>(tab, ws, nr, W.lim, H, threadIdx.x, blockDim.x);
+  flush<P16>(tab, ws, nr, dv.row, W.lim, H, threadIdx.x, blockDim.x);
 }
 
 // ---------------------------------------------------------------------- WINDOW
@@ -538,7 +543,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (it.last) break;
     if (it.ws != ws) {  // window switch: every counter is done with the old window
       bar_counters();
-      if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H, ct, nct);
+      if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
       bar_counters();
       ws = it.ws;
       W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
@@ -571,7 +576,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   count_invalid(bad, d_n_invalid);
   bar_counters();
-  if (ws != kNoWindow) flush<P16>(tab, ws, nr, W.lim, H, ct, nct);
+  if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
 }
 
 }  // namespace
@@ -590,8 +595,8 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
                    int accumulate, bool zero_first) {
   cudaStream_t st = c->stream;
   const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
-  const Div dv = make_div(nr);
-  if (zero_first && !accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, (uint64_t)P * 32 * 4, st));
+  const Div dv = make_div(nr, c->cfg.hist_row);
+  if (zero_first && !accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, (uint64_t)P * c->cfg.hist_row * 4, st));
   if (!n) return GS_OK;
   if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
   int dev_sms = 148;

@@ -148,8 +148,9 @@ gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_
                            unsigned long long* d_n_invalid);
 gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,
                    unsigned long long* d_n_invalid, int accumulate, bool zero_first);
-gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, bool out_is_host,
-                   uint64_t* n_out);
+// d_hist holds the rows of slots [slot0, ...) (row width cfg.hist_row)
+gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k, gs_ranked_site* out,
+                   bool out_is_host, uint64_t* n_out);
 void attrib_free(gs_ctx* c);
 void rank_free(gs_ctx* c);
 

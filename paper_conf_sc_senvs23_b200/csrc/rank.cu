@@ -1,8 +1,9 @@
 // rank.cu — join of the histogram onto the flagged sites and their ranking
 // (§3.2; rank key R20).
 //
-//   k_ktot   per kernel: total samples of the kernel (denominator of tot/ktot), 128-bit loads,
-//            several CTAs per kernel.
+//   k_ktot   per detected kernel: total samples of the kernel (denominator of tot/ktot), 128-bit
+//            loads, several CTAs per kernel.
+//   The histogram may be a slice (rows of slots [slot0, ...)) of width 32 or R (gs_config.hist_row).
 //   k_join   per site: tot = sum of the site PC's row, rel = sum over REL(rule) (P:556-563,
 //            P:616-624; CONV: all reasons); running maxima of rel and tot.
 //   sort     the sites enter in (kernel, idx, rule) order, so a STABLE ascending sort on
@@ -34,19 +35,29 @@ __constant__ uint32_t kRelMask[7] = {
 constexpr int kKtotThreads = 512;
 constexpr uint32_t kKtotSlotsPerCta = 1024;  // 128 KB of histogram per CTA
 
-// grid.x = kernel, grid.y = slice of the kernel's slots
-__global__ void __launch_bounds__(kKtotThreads) k_ktot(const int32_t* __restrict__ H, const KDesc* __restrict__ kd,
-                                                       uint32_t nk, unsigned long long* __restrict__ ktot) {
-  const uint32_t k = blockIdx.x;
-  if (k >= nk) return;
+// grid.x = kernel - kb, grid.y = slice of the kernel's slots. H holds rows of width `row` from slot
+// slot0 on; a kernel's rows are one contiguous int32 range, read with 128-bit loads between a
+// scalar head and tail (compact rows of R < 32 bins are not 16-byte aligned per slot).
+__global__ void __launch_bounds__(kKtotThreads) k_ktot(const int32_t* __restrict__ H, uint32_t slot0, uint32_t row,
+                                                       const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke,
+                                                       unsigned long long* __restrict__ ktot) {
+  const uint32_t k = kb + blockIdx.x;
+  if (k >= ke) return;
   const KDesc K = kd[k];
   const uint32_t s0 = blockIdx.y * kKtotSlotsPerCta;
   if (s0 >= K.n) return;
   const uint32_t s1 = min(K.n, s0 + kKtotSlotsPerCta);
-  const int4* h4 = reinterpret_cast<const int4*>(H + (uint64_t)(K.first + s0) * 32);
-  const uint32_t n4 = (s1 - s0) * 8;
+  const uint64_t e0 = (uint64_t)(K.first - slot0 + s0) * row, e1 = (uint64_t)(K.first - slot0 + s1) * row;
+  const uint64_t mis = (uint64_t)(reinterpret_cast<uintptr_t>(H) >> 2) & 3u;  // H is 4-byte aligned
+  const uint64_t up = ((e0 + mis + 3) & ~(uint64_t)3) - mis, dn = ((e1 + mis) & ~(uint64_t)3) - mis;
+  const uint64_t a0 = up < e1 ? up : e1;
+  const uint64_t a1 = dn > a0 ? dn : a0;
   unsigned long long s = 0;
-  for (uint32_t i = threadIdx.x; i < n4; i += blockDim.x) {
+  for (uint64_t i = e0 + threadIdx.x; i < a0; i += blockDim.x) s += (uint32_t)__ldg(H + i);
+  for (uint64_t i = a1 + threadIdx.x; i < e1; i += blockDim.x) s += (uint32_t)__ldg(H + i);
+  const int4* h4 = reinterpret_cast<const int4*>(H + a0);
+  const uint64_t n4 = (a1 - a0) / 4;
+  for (uint64_t i = threadIdx.x; i < n4; i += blockDim.x) {
     const int4 v = __ldg(h4 + i);
     s += (uint32_t)v.x + (uint64_t)(uint32_t)v.y + (uint32_t)v.z + (uint64_t)(uint32_t)v.w;
   }
@@ -61,24 +72,33 @@ __global__ void __launch_bounds__(kKtotThreads) k_ktot(const int32_t* __restrict
   }
 }
 
-__global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H,
-                       const KDesc* __restrict__ kd, unsigned long long* __restrict__ rel_out,
+__global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H, uint32_t slot0,
+                       uint32_t row, bool vec, const KDesc* __restrict__ kd, unsigned long long* __restrict__ rel_out,
                        unsigned long long* __restrict__ tot_out, unsigned long long* __restrict__ mx) {
   const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   unsigned long long tot = 0, rel = 0;
   if (s < ns) {
     const gs_site st = sites[s];
-    const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx;
-    const int4* row = reinterpret_cast<const int4*>(H + slot * 32);
+    const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx - slot0;
     const uint32_t m = kRelMask[st.rule];
+    if (vec) {  // 32-wide, 16-byte aligned rows
+      const int4* r4 = reinterpret_cast<const int4*>(H + slot * 32);
 #pragma unroll
-    for (int q = 0; q < 8; q++) {
-      const int4 v = __ldg(row + q);
-      const uint32_t c[4] = {(uint32_t)v.x, (uint32_t)v.y, (uint32_t)v.z, (uint32_t)v.w};
+      for (int q = 0; q < 8; q++) {
+        const int4 v = __ldg(r4 + q);
+        const uint32_t c[4] = {(uint32_t)v.x, (uint32_t)v.y, (uint32_t)v.z, (uint32_t)v.w};
 #pragma unroll
-      for (int t = 0; t < 4; t++) {
-        tot += c[t];
-        if ((m >> (4 * q + t)) & 1u) rel += c[t];
+        for (int t = 0; t < 4; t++) {
+          tot += c[t];
+          if ((m >> (4 * q + t)) & 1u) rel += c[t];
+        }
+      }
+    } else {
+      const int32_t* r1 = H + slot * row;
+      for (uint32_t t = 0; t < row; t++) {
+        const uint32_t c = (uint32_t)__ldg(r1 + t);
+        tot += c;
+        if ((m >> t) & 1u) rel += c;
       }
     }
     rel_out[s] = rel;
@@ -117,14 +137,14 @@ __global__ void k_keys_field(const unsigned long long* __restrict__ val, const u
 }
 
 __global__ void k_emit(const uint32_t* __restrict__ order, uint64_t kk, const gs_site* __restrict__ sites,
-                       const int32_t* __restrict__ H, const KDesc* __restrict__ kd,
+                       const int32_t* __restrict__ H, uint32_t slot0, uint32_t row, const KDesc* __restrict__ kd,
                        const unsigned long long* __restrict__ ktot, gs_ranked_site* __restrict__ out) {
   const uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);  // one warp per row
   if (q >= kk) return;
   const int lane = threadIdx.x & 31;
   const gs_site st = sites[order[q]];
-  const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx;
-  const uint32_t c = (uint32_t)H[slot * 32 + lane];
+  const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx - slot0;
+  const uint32_t c = (uint32_t)lane < row ? (uint32_t)H[slot * row + lane] : 0u;
   const uint32_t m = kRelMask[st.rule];
   unsigned long long tot = c, rel = ((m >> lane) & 1u) ? c : 0;
   for (int o = 16; o; o >>= 1) {
@@ -149,19 +169,20 @@ unsigned long long mask_of(int b) { return b >= 64 ? ~0ull : ((1ull << b) - 1); 
 
 }  // namespace
 
-gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site* out, bool out_is_host,
-                   uint64_t* n_out) {
+gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k, gs_ranked_site* out,
+                   bool out_is_host, uint64_t* n_out) {
   cudaStream_t st = c->stream;
   const uint64_t ns = c->n_sites;
   const uint64_t kk = std::min<uint64_t>(k, ns);
   if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8));
   unsigned long long* d_max = c->d_ktot + std::max<uint32_t>(c->n_kernels, 1);
   GS_CUDA(c, cudaMemsetAsync(c->d_ktot, 0, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8, st));
-  if (c->n_kernels) {
+  const uint32_t row = c->cfg.hist_row;
+  if (c->det_ke > c->det_kb) {  // kernel totals of the detected kernels only
     uint32_t max_n = 1;
-    for (const auto& K : c->kd_h) max_n = std::max(max_n, K.n);
-    dim3 grid(c->n_kernels, (max_n + kKtotSlotsPerCta - 1) / kKtotSlotsPerCta);
-    k_ktot<<<grid, kKtotThreads, 0, st>>>(d_hist, c->d_kd, c->n_kernels, c->d_ktot);
+    for (uint32_t k = c->det_kb; k < c->det_ke; k++) max_n = std::max(max_n, c->kd_h[k].n);
+    dim3 grid(c->det_ke - c->det_kb, (max_n + kKtotSlotsPerCta - 1) / kKtotSlotsPerCta);
+    k_ktot<<<grid, kKtotThreads, 0, st>>>(d_hist, slot0, row, c->d_kd, c->det_kb, c->det_ke, c->d_ktot);
     count_launch();
     GS_CUDA(c, cudaGetLastError());
   }
@@ -198,7 +219,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
     unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
     void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
     const unsigned grid = (unsigned)((ns + 255) / 256);
-    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, c->d_kd, d_rel, d_tot, d_max);
+    const bool vec = row == 32 && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0;
+    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, vec, c->d_kd, d_rel, d_tot, d_max);
     count_launch();
     GS_CUDA(c, cudaGetLastError());
     unsigned long long mx[2];
@@ -237,7 +259,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_site*
         GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
         dst = c->d_ranked;
       }
-      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, c->d_kd, c->d_ktot, dst);
+      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row, c->d_kd,
+                                                        c->d_ktot, dst);
       count_launch();
       GS_CUDA(c, cudaGetLastError());
       if (out_is_host)

@@ -35,6 +35,41 @@ def kernel_range(n_instr, rank: int, world: int) -> tuple[int, int]:
     return cut(rank), cut(rank + 1)
 
 
+def slot_ranges(first_slot, n_instr, world: int) -> list[tuple[int, int]]:
+    """Slot range [s, e) of every rank's detection shard (kernel_range): contiguous, kernel-aligned,
+    covering [0, P) exactly once."""
+    first_slot = np.asarray(first_slot, dtype=np.int64)
+    n_instr = np.asarray(n_instr, dtype=np.int64)
+    P = int(first_slot[-1] + n_instr[-1]) if len(n_instr) else 0
+    out = []
+    for g in range(world):
+        kb, ke = kernel_range(n_instr, g, world)
+        s = int(first_slot[kb]) if kb < len(n_instr) else P
+        e = int(first_slot[ke]) if ke < len(n_instr) else P
+        out.append((s, e))
+    return out
+
+
+def reduce_scatter_hist(hist, row: int, ranges, group=None):
+    """Sum the per-rank histograms (rows of `row` bins, one per slot) and leave on rank g the summed
+    rows of slots ranges[g] = [s, e); returns that slice (a view of `hist`). One collective: NCCL's
+    reduce_scatter (uneven parts run as grouped ncclReduce calls); on other backends one reduce per
+    part. Single process: the slice of the whole histogram."""
+    import torch.distributed as dist
+    parts = [hist[s * row:e * row] for s, e in ranges]
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return parts[0] if len(parts) == 1 else hist
+    me = dist.get_rank(group)
+    if dist.get_backend(group) == "nccl":
+        dist.reduce_scatter(parts[me], parts, op=dist.ReduceOp.SUM, group=group)
+    else:
+        works = [dist.reduce(p, dst=g, op=dist.ReduceOp.SUM, group=group, async_op=True)
+                 for g, p in enumerate(parts) if p.numel()]
+        for w in works:
+            w.wait()
+    return parts[me]
+
+
 def rank_key(row) -> tuple:
     return (-int(row["rel"]), -int(row["tot"]), int(row["kernel"]), int(row["idx"]), int(row["rule"]))
 

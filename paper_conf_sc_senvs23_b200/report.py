@@ -74,7 +74,9 @@ def canonical(ctx, k_begin: int = 0, k_end: int | None = None, hist=None, n_samp
     sites, chain = ctx.sites()
     out += site_lines(sites, chain, ctx.instr_lines(), first)
     if hist is not None:
-        h = hist.detach().cpu().numpy().astype(np.int64).reshape(-1, 32) if hasattr(hist, "detach") else hist
+        row = getattr(ctx, "hist_row", 32)
+        h = hist.detach().cpu().numpy() if hasattr(hist, "detach") else np.asarray(hist)
+        h = h.astype(np.int64).reshape(-1, row)
         nzs, nzr = np.nonzero(h)
         out += [f"H {s} {r} {h[s, r]}" for s, r in zip(nzs, nzr)]
         valid = int(h.sum())

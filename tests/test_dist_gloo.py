@@ -109,6 +109,63 @@ def test_two_rank_gloo_matches_single_process(k):
         assert np.array_equal(merged[f], want_rows[f]), f
 
 
+def _rs_worker(rank, world, port, text, raw, P, first_slot, n_instr, row, result_q):
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import torch
+    import torch.distributed as dist
+    import oracle_run as orc
+    from oracle_run import Canon
+    from paper_conf_sc_senvs23_b200 import dist as gdist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        a, b = gdist.sample_range(len(raw), rank, world)
+        local = Canon(orc.run(text, samples=raw[a:b], detect=False))
+        hist = torch.zeros(P * row, dtype=torch.int32)
+        for (slot, r), c in local.H.items():
+            hist[slot * row + r] = c
+        ranges = gdist.slot_ranges(first_slot, n_instr, world)
+        part = gdist.reduce_scatter_hist(hist, row, ranges)
+        result_q.put((rank, ranges[rank], part.numpy().copy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,row", [(2, 19), (3, 32)])
+def test_reduce_scatter_slices_equal_full_histogram(world, row):
+    """Each rank's reduce-scattered slice (kernel-aligned slot range of its detection shard) equals
+    the single-process histogram rows of that range; the slices tile [0, P)."""
+    import oracle_run as orc
+    from oracle_run import Canon
+    from gen import samples as gsm
+    from gen import sass as gsass
+    orc.build_oracle()
+    s = gsass.config_sass("C2")
+    tab = gsm.table_class_weighted(s.cls, 200_000, key=23)
+    raw = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=23).raw()
+    full = Canon(orc.run(s.text, samples=raw, detect=False))
+    want = np.zeros((s.P, row), np.int64)
+    for (slot, r), c in full.H.items():
+        want[slot, r] = c
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rs_worker, args=(r, world, port, s.text, raw, s.P, s.first_slot, s.n_instr, row, q))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=300) for _ in range(world)], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res[0][1][0] == 0 and res[-1][1][1] == s.P
+    assert all(res[i][1][1] == res[i + 1][1][0] for i in range(world - 1))
+    for _, (sb, se), part in res:
+        assert np.array_equal(part.reshape(-1, row).astype(np.int64), want[sb:se])
+
+
 def test_kernel_range_balance():
     from paper_conf_sc_senvs23_b200 import dist as gdist
     n = np.array([100, 5000, 7, 7, 3000, 2000, 1, 64] * 5)

@@ -21,25 +21,33 @@ def gs():
     return g
 
 
-def _check(gs, s, tr, modes, words=None):
+def _want(tab, row):
+    """closed-form histogram in the layout of `row` bins per slot (32, or R = 19 compact)"""
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(tab[:, :row]).astype(np.int32).reshape(-1)).cuda()
+
+
+def _check(gs, s, tr, modes, words=None, rows=(32, 19)):
     import torch
     from gen.device import DeviceTrace
     if words is None:
         words = DeviceTrace(tr).packed()
-    want = torch.from_numpy(tr.table.astype(np.int32).reshape(-1)).cuda()
-    for mode in modes:
-        for bits in ((16, 32) if mode in (0, 2, 3) else (0,)):
-            ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
-            ctx.load_sass(s.text)
-            hist, ninv = ctx.attribute_samples(words)
-            torch.cuda.synchronize()
-            assert int(ninv.item()) == 0, (mode, bits)
-            assert torch.equal(hist, want), (mode, bits, int((hist != want).sum().item()))
-            ctx.close()
+    for row in rows:
+        want = _want(tr.table, row)
+        for mode in modes:
+            for bits in ((16, 32) if mode in (0, 2, 3) else (0,)):
+                ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits, hist_row=row)
+                ctx.load_sass(s.text)
+                hist, ninv = ctx.attribute_samples(words)
+                torch.cuda.synchronize()
+                assert int(ninv.item()) == 0, (mode, bits, row)
+                assert torch.equal(hist, want), (mode, bits, row, int((hist != want).sum().item()))
+                ctx.close()
 
 
 @pytest.mark.parametrize("order", ["trace", "shuffled"])
 def test_c4_full_size_closed_form(gs, order):
+    """C4 (2^30 samples over 1M PCs) in both orders, 32-bin and compact 19-bin rows."""
     from gen import samples as gsm
     from gen import sass as gsass
     s = gsass.config_sass("C4")
@@ -68,12 +76,12 @@ def test_single_bin_drain(gs):
     s = gsass.config_sass("C1")
     n = 3_000_000
     words = torch.full((n,), 17 * 19 + 6, dtype=torch.int32, device="cuda")
-    for mode, bits in [(m, b) for m in MODES for b in (16, 32)]:
-        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
+    for mode, bits, row in [(m, b, r) for m in MODES for b in (16, 32) for r in (32, 19)]:
+        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits, hist_row=row)
         ctx.load_sass(s.text)
         hist, ninv = ctx.attribute_samples(words)
         torch.cuda.synchronize()
-        h = hist.view(-1, 32)
+        h = hist.view(-1, row)
         assert int(h[17, 6].item()) == n and int(h.sum().item()) == n and int(ninv.item()) == 0
         ctx.close()
 
@@ -90,9 +98,9 @@ def test_unaligned_views_and_invalid_words(gs, offset):
     bad = torch.tensor([-1, s.P * 19 + 1, s.P * 19, -16], dtype=torch.int32, device="cuda")
     buf = torch.cat([torch.zeros(offset, dtype=torch.int32, device="cuda"), bad, base, bad])
     view = buf[offset:]
-    want = torch.from_numpy(tab.astype(np.int32).reshape(-1)).cuda()
-    for mode, bits in [(m, b) for m in MODES for b in (16, 32)]:
-        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits)
+    for mode, bits, row in [(m, b, r) for m in MODES for b in (16, 32) for r in (32, 19)]:
+        want = _want(tab, row)
+        ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits, hist_row=row)
         ctx.load_sass(s.text)
         hist, ninv = ctx.attribute_samples(view)
         torch.cuda.synchronize()

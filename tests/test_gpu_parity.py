@@ -95,10 +95,10 @@ def test_trace_depth_edges(gs):
 
 
 # ------------------------------------------------------------------------------ full flow
-def _flow(gs, text, raw, hist_mode=0, host_input=False, k=None, n_reasons=19):
+def _flow(gs, text, raw, hist_mode=0, host_input=False, k=None, n_reasons=19, hist_row=32):
     import torch
     from paper_conf_sc_senvs23_b200 import report
-    ctx = _ctx(gs, hist_mode=hist_mode, n_reasons=n_reasons)
+    ctx = _ctx(gs, hist_mode=hist_mode, n_reasons=n_reasons, hist_row=hist_row)
     ctx.load_sass(text)
     ctx.detect()
     raw_t = torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda()
@@ -137,6 +137,50 @@ def test_full_flow_parity(gs, cfg, n, order, mode):
     assert g.H == o.H and g.N == o.N
     assert g.S == o.S and g.K == o.K
     assert g.R == o.R
+
+
+@pytest.mark.parametrize("cfg,n,order,mode", [("C1", 16384, "shuffled", 0), ("C2", 400_000, "trace", 0),
+                                              ("C2", 400_000, "shuffled", 1), ("C2", 400_000, "trace", 3)])
+def test_full_flow_parity_compact_rows(gs, cfg, n, order, mode):
+    """gs_config.hist_row = R: histogram rows hold only the active reasons."""
+    from gen import sass as gsass
+    s = gsass.config_sass(cfg)
+    raw, _ = _samples(s, n, order, seed=13)
+    g, _ = _flow(gs, s.text, raw, hist_mode=mode, hist_row=19)
+    o = Canon(orc.run(s.text, samples=raw))
+    assert g.H == o.H and g.N == o.N and g.S == o.S and g.R == o.R
+
+
+@pytest.mark.parametrize("row", [32, 19])
+def test_rank_against_histogram_slice(gs, row):
+    """gs_rank_sites_slice: a detection shard ranked against only its kernels' rows (the part a rank
+    holds after the reduce-scatter) gives the rows the oracle gives for that shard; a slice that
+    misses a detected kernel's slot is refused."""
+    import torch
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import dist as gdist
+    s = gsass.config_sass("C2")
+    raw, _ = _samples(s, 300_000, "shuffled", seed=17, n_bad=0)
+    ctx = _ctx(gs, hist_row=row)
+    ctx.load_sass(s.text)
+    raw_t = torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda()
+    words, _ = ctx.pack_samples(raw_t)
+    hist, _ = ctx.attribute_samples(words)
+    for world in (2, 3):
+        ranges = gdist.slot_ranges(s.first_slot, s.n_instr, world)
+        for g_ in range(world):
+            kb, ke = gdist.kernel_range(s.n_instr, g_, world)
+            sb, se = ranges[g_]
+            ctx.detect(kb, ke)
+            part = hist[sb * row:se * row].clone()        # a separate allocation, like a received slice
+            got = ctx.rank_sites(part, slot_begin=sb, slot_end=se)
+            want = Canon(orc.run(s.text, samples=raw, kbegin=kb, kend=ke)).R
+            from paper_conf_sc_senvs23_b200 import report
+            lines = report.canonical(ctx, kb, ke, hist=hist, n_samples=len(raw), n_invalid=0, ranked=got)
+            assert Canon(lines).R == want, (world, g_)
+            if se > sb:
+                with pytest.raises(gs.GsError, match="does not cover"):
+                    ctx.rank_sites(hist[(sb + 1) * row:se * row], slot_begin=sb + 1, slot_end=se)
 
 
 def test_host_input_and_topk(gs):

@@ -24,9 +24,9 @@ ap.add_argument("--only", default="all")
 a = ap.parse_args()
 s, tr = bench.build_workload(a.config, a.order)
 words = DeviceTrace(tr).packed()
-ctx = g.Context(hist_mode=a.mode)
+ctx = g.Context(hist_mode=a.mode, hist_row=19)   # compact rows, as bench.py
 ctx.load_sass(s.text)
-hist = torch.empty(ctx.n_instr * 32, dtype=torch.int32, device="cuda")
+hist = torch.empty(ctx.n_instr * 19, dtype=torch.int32, device="cuda")
 ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
 ctx.detect()
 torch.cuda.synchronize()

@@ -239,19 +239,27 @@ def main():
         f"{n_local} samples, {n_sites} sites")
     stream = torch.cuda.current_stream()
     hist_events = []
+    phase_events = []     # per timed step: events at detect | attribute | merge | rank boundaries
 
     def step(record_hist=False):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)] if record_hist else None
+        if ev:
+            ev[0].record(stream)
         ctx.detect(kb, ke)
-        if record_hist:
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
+        if ev:
+            ev[1].record(stream)
         ninv.zero_()
         ctx.attribute_samples(words, hist, ninv)
-        if record_hist:
-            e1.record(stream)
-            hist_events.append((e0, e1))
+        if ev:
+            ev[2].record(stream)
+            hist_events.append((ev[1], ev[2]))
         part = gdist.reduce_scatter_hist(hist, row, gdist.slot_ranges(s.first_slot, s.n_instr, world))
+        if ev:
+            ev[3].record(stream)
         ctx.rank_sites(part, k=None, out=ranked_dev, slot_begin=s0, slot_end=s1)
+        if ev:
+            ev[4].record(stream)
+            phase_events.append(ev)
 
     for _ in range(args.warmup):
         step()
@@ -277,6 +285,8 @@ def main():
     clk = clocks.stop()
     ms = ev0.elapsed_time(ev1) / args.steps
     hist_ms = float(np.mean([e0.elapsed_time(e1) for e0, e1 in hist_events]))
+    phases = {name: float(np.mean([ev[i].elapsed_time(ev[i + 1]) for ev in phase_events]))
+              for i, name in enumerate(["detect", "attribute", "merge", "rank"])}
     t = torch.tensor([ms, hist_ms], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -363,6 +373,7 @@ def main():
                 "ms_per_step": e2e_s * 1e3},
         "cpu_baseline": cpu,
         "sites": n_sites,
+        "phases_ms": phases,
     }
     print(json.dumps(out), flush=True)
     if world > 1:

@@ -194,6 +194,8 @@ Opnd parse_operand(const std::string& raw) {
 struct Instr {
   int pc = 0;
   int line = -1;                  // source line from //## File ..., line N
+  std::string file;               // ... and its file (a source line is the pair (file, line), R33)
+  std::string bra_label;          // nvdisasm: BRA `(.L_x_N) target label, resolved per kernel
   std::string op;                 // base mnemonic
   std::vector<std::string> mods;  // modifiers after the first '.'
   std::vector<Opnd> ops;
@@ -212,6 +214,7 @@ struct Kernel {
   int param_base = 0x380;
   std::vector<Instr> ins;
   size_t first_slot = 0;
+  std::map<std::string, int> labels;  // nvdisasm ".L_x_N:" -> pc of the next instruction
 };
 
 bool op_in(const std::string& op, std::initializer_list<const char*> l) {
@@ -264,9 +267,22 @@ struct ParseError { std::string msg; };
 
 int arch_param_base(int sm) { return sm >= 100 ? 0x380 : (sm >= 90 ? 0x210 : 0x160); }
 
+// Accepts cuobjdump -sass text ("Function : name" headers, hex branch targets) and nvdisasm text
+// (".text.name:" labels, "//## File "f", line N" with -g, branch targets as `(.L_x_N) labels).
 std::vector<Kernel> parse_sass(const std::string& text) {
   std::vector<Kernel> ks;
   int cur_sm = 100, line_no = 0, src_line = -1;
+  std::string src_file;
+  std::vector<std::string> pending;  // labels waiting for their instruction
+  auto new_kernel = [&](const std::string& name) {
+    Kernel k;
+    k.name = name;
+    k.param_base = arch_param_base(cur_sm);
+    ks.push_back(k);
+    src_line = -1;
+    src_file.clear();
+    pending.clear();
+  };
   size_t p = 0;
   while (p < text.size()) {
     size_t e = text.find('\n', p);
@@ -285,16 +301,22 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     }
     size_t fn = t.find("Function :");
     if (fn != std::string::npos) {
-      Kernel k;
-      k.name = trim(t.substr(fn + 10));
-      k.param_base = arch_param_base(cur_sm);
-      ks.push_back(k);
-      src_line = -1;
+      new_kernel(trim(t.substr(fn + 10)));
+      continue;
+    }
+    if (t.size() > 7 && t.rfind(".text.", 0) == 0 && t.back() == ':') {  // nvdisasm function label
+      new_kernel(t.substr(6, t.size() - 7));
+      continue;
+    }
+    if (t.size() > 3 && t.rfind(".L", 0) == 0 && t.back() == ':') {  // nvdisasm branch label
+      pending.push_back(t.substr(0, t.size() - 1));
       continue;
     }
     if (t.rfind("//##", 0) == 0) {  // nvdisasm -g line info: //## File "f", line N
       size_t ln = t.find("line ");
       if (ln != std::string::npos) src_line = atoi(t.c_str() + ln + 5);
+      size_t q0 = t.find('"'), q1 = q0 == std::string::npos ? q0 : t.find('"', q0 + 1);
+      src_file = q1 == std::string::npos ? std::string() : t.substr(q0 + 1, q1 - q0 - 1);
       continue;
     }
     if (t.size() < 4 || t[0] != '/' || t[1] != '*') continue;
@@ -308,18 +330,16 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     size_t semi = body.find(';');
     if (semi == std::string::npos) continue;
     body = trim(body.substr(0, semi));
-    if (ks.empty()) {  // instruction without a Function header (e.g. a paper listing)
-      Kernel k;
-      k.name = "<anonymous>";
-      k.param_base = arch_param_base(cur_sm);
-      ks.push_back(k);
-    }
+    if (ks.empty()) new_kernel("<anonymous>");  // instructions without a header (e.g. a paper listing)
     Kernel& K = ks.back();
     Instr I;
     I.pc = (int)strtol(pcs.c_str(), nullptr, 16);
     I.line = src_line;
+    I.file = src_file;
     if ((size_t)I.pc != K.ins.size() * 16)
       throw ParseError{"line " + std::to_string(line_no) + ": pc not 16-strided"};
+    for (auto& lb : pending) K.labels[lb] = I.pc;
+    pending.clear();
     // guard predicate
     if (!body.empty() && body[0] == '@') {
       size_t sp = body.find_first_of(" \t");
@@ -350,10 +370,20 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     decode_effects(I);
     if (I.op == "BRA" && !raw.empty()) {
       long long v;
-      if (parse_int(raw.back(), &v)) I.bra_target = v;
+      std::string last = trim(raw.back());
+      if (parse_int(last, &v)) I.bra_target = v;
+      else if (last.size() > 4 && last.rfind("`(", 0) == 0 && last.back() == ')')
+        I.bra_label = last.substr(2, last.size() - 3);
     }
     K.ins.push_back(I);
   }
+  // nvdisasm label targets: a label names the pc of the instruction after it (R28)
+  for (auto& k : ks)
+    for (auto& I : k.ins)
+      if (!I.bra_label.empty()) {
+        auto it = k.labels.find(I.bra_label);
+        if (it != k.labels.end()) I.bra_target = it->second;
+      }
   size_t slot = 0;
   for (auto& k : ks) { k.first_slot = slot; slot += k.ins.size(); }
   return ks;
@@ -687,6 +717,9 @@ void detect_kernel(int kid, const Kernel& K, const Config& C, std::vector<Site>&
 
 // ---------------------------------------------------------------- O13-O15
 struct RawSample { uint32_t kernel, pc, reason; };
+// pre-aggregated PC-sampling record (CUPTI CUpti_PCSamplingPCData shape: one (pc, stall reason)
+// with its sample count, P:215-227 / SURVEY [probe 8]); `count` samples of that (kernel, pc, reason)
+struct CountRec { uint32_t kernel, pc, reason, count; };
 
 const int kRel[NRULES] = {
     // bit r set = reason r in REL(rule).  long_scoreboard = 6, lg_throttle = 5, tex_throttle = 16
@@ -702,7 +735,7 @@ const int kRel[NRULES] = {
 }  // namespace
 
 int main(int argc, char** argv) {
-  std::string sass_path, samples_path, out_path;
+  std::string sass_path, samples_path, counts_path, out_path, join = "pc";
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
@@ -712,6 +745,8 @@ int main(int argc, char** argv) {
     auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
     if (s == "--sass") sass_path = nxt();
     else if (s == "--samples") samples_path = nxt();
+    else if (s == "--counts") counts_path = nxt();  // CountRec records, added to the same histogram
+    else if (s == "--join") join = nxt();            // pc (default) | line
     else if (s == "--out") out_path = nxt();
     else if (s == "--D") C.D = atoi(nxt().c_str());
     else if (s == "--R") C.R = atoi(nxt().c_str());
@@ -726,6 +761,7 @@ int main(int argc, char** argv) {
     else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
     else { fprintf(stderr, "unknown arg %s\n", s.c_str()); return 2; }
   }
+  if (join != "pc" && join != "line") { fprintf(stderr, "unknown join %s\n", join.c_str()); return 2; }
   auto now = [] { return std::chrono::steady_clock::now(); };
   auto secs = [](auto a, auto b) { return std::chrono::duration<double>(b - a).count(); };
   FILE* f = fopen(sass_path.c_str(), "rb");
@@ -774,27 +810,42 @@ int main(int argc, char** argv) {
               s.attrs.empty() ? "" : " ", s.attrs.c_str());
     }
   }
-  if (hist && !samples_path.empty()) {
+  if (hist && (!samples_path.empty() || !counts_path.empty())) {
     // O13: H[slot][reason] += 1 for every valid sample.
     size_t P = 0;
     for (auto& k : ks) P += k.ins.size();
     std::vector<uint64_t> H(P * 32, 0);
-    FILE* sf = fopen(samples_path.c_str(), "rb");
-    if (!sf) { fprintf(stderr, "cannot open %s\n", samples_path.c_str()); return 2; }
     uint64_t N = 0, invalid = 0;
-    std::vector<RawSample> buf(1 << 16);
+    auto valid = [&](uint32_t kernel, uint32_t pc, uint32_t reason) {
+      return kernel < ks.size() && pc % 16 == 0 && pc / 16 < ks[kernel].ins.size() && reason < (uint32_t)C.R;
+    };
     auto th0 = now();
-    while (size_t got = fread(buf.data(), sizeof(RawSample), buf.size(), sf)) {
-      for (size_t q = 0; q < got; q++) {
-        const RawSample& s = buf[q];
-        N++;
-        bool ok = s.kernel < ks.size() && s.pc % 16 == 0 && s.pc / 16 < ks[s.kernel].ins.size() &&
-                  s.reason < (uint32_t)C.R;
-        if (!ok) { invalid++; continue; }
-        H[(ks[s.kernel].first_slot + s.pc / 16) * 32 + s.reason]++;
+    if (!samples_path.empty()) {
+      FILE* sf = fopen(samples_path.c_str(), "rb");
+      if (!sf) { fprintf(stderr, "cannot open %s\n", samples_path.c_str()); return 2; }
+      std::vector<RawSample> buf(1 << 16);
+      while (size_t got = fread(buf.data(), sizeof(RawSample), buf.size(), sf)) {
+        for (size_t q = 0; q < got; q++) {
+          const RawSample& s = buf[q];
+          N++;
+          if (!valid(s.kernel, s.pc, s.reason)) { invalid++; continue; }
+          H[(ks[s.kernel].first_slot + s.pc / 16) * 32 + s.reason]++;
+        }
       }
+      fclose(sf);
     }
-    fclose(sf);
+    if (!counts_path.empty()) {
+      // pre-aggregated records: H[slot][reason] += count (the same histogram as `count` samples)
+      FILE* cf = fopen(counts_path.c_str(), "rb");
+      if (!cf) { fprintf(stderr, "cannot open %s\n", counts_path.c_str()); return 2; }
+      CountRec r;
+      while (fread(&r, sizeof r, 1, cf) == 1) {
+        N += r.count;
+        if (!valid(r.kernel, r.pc, r.reason)) { invalid += r.count; continue; }
+        H[(ks[r.kernel].first_slot + r.pc / 16) * 32 + r.reason] += r.count;
+      }
+      fclose(cf);
+    }
     auto th1 = now();
     uint64_t mass = 0;
     for (size_t b = 0; b < H.size(); b++)
@@ -809,16 +860,36 @@ int main(int argc, char** argv) {
     for (size_t k = 0; k < ks.size(); k++)
       for (size_t i = 0; i < ks[k].ins.size(); i++)
         for (int r = 0; r < 32; r++) ktot[k] += H[(ks[k].first_slot + i) * 32 + r];
-    struct Ranked { const Site* s; uint64_t rel, tot; };
+    // The row a site is joined with (R18, R33): join=pc -> the site PC's row;
+    // join=line -> the sum of the rows of every instruction of the kernel on the same source line
+    // (file, line) as the site ("stall reasons ... at the line numbers identified"), or
+    // the site PC's row when the site has no line information.
+    auto site_row = [&](const Site& s) {
+      std::vector<uint64_t> row(32, 0);
+      const Kernel& K = ks[s.k];
+      const Instr& I = K.ins[s.idx];
+      if (join == "pc" || I.line < 0) {
+        for (int r = 0; r < 32; r++) row[r] = H[(K.first_slot + s.idx) * 32 + r];
+        return row;
+      }
+      for (size_t i = 0; i < K.ins.size(); i++) {
+        bool same = (int)i == s.idx;
+        if (join == "line" && I.line >= 0) same = K.ins[i].line == I.line && K.ins[i].file == I.file;
+        if (!same) continue;
+        for (int r = 0; r < 32; r++) row[r] += H[(K.first_slot + i) * 32 + r];
+      }
+      return row;
+    };
+    struct Ranked { const Site* s; uint64_t rel, tot; std::vector<uint64_t> row; };
     std::vector<Ranked> rk;
     for (auto& s : sites) {
-      size_t slot = ks[s.k].first_slot + (size_t)s.idx;
+      std::vector<uint64_t> row = site_row(s);
       uint64_t tot = 0, rel = 0;
       for (int r = 0; r < 32; r++) {
-        tot += H[slot * 32 + r];
-        if (kRel[s.rule] == -1 || (kRel[s.rule] >> r) & 1) rel += H[slot * 32 + r];
+        tot += row[r];
+        if (kRel[s.rule] == -1 || (kRel[s.rule] >> r) & 1) rel += row[r];
       }
-      rk.push_back({&s, rel, tot});
+      rk.push_back({&s, rel, tot, row});
     }
     // O15 rank: (rel desc, tot desc, kernel asc, idx asc, rule asc)
     std::sort(rk.begin(), rk.end(), [](const Ranked& a, const Ranked& b) {
@@ -833,9 +904,8 @@ int main(int argc, char** argv) {
     if (timing) fprintf(stderr, "TIME rank_s=%.6f sites=%zu\n", secs(th1, tr1), rk.size());
     for (size_t q = 0; q < lim && !quiet; q++) {
       const Site& s = *rk[q].s;
-      size_t slot = ks[s.k].first_slot + (size_t)s.idx;
-      std::string h;
-      for (int r = 0; r < C.R; r++) h += (r ? "," : "") + std::to_string(H[slot * 32 + r]);
+      std::string h;  // reported counts are 32-bit, saturating (R34)
+      for (int r = 0; r < C.R; r++) h += (r ? "," : "") + std::to_string(std::min<uint64_t>(rk[q].row[r], 0xffffffffull));
       fprintf(out, "R %zu %d %d %s rel=%llu tot=%llu ktot=%llu h=%s\n", q, s.k, s.idx, kRuleName[s.rule],
               (unsigned long long)rk[q].rel, (unsigned long long)rk[q].tot, (unsigned long long)ktot[s.k], h.c_str());
     }

@@ -17,3 +17,14 @@ for cap in 24 32 40 64; do
   cuobjdump -sass $T/spill.$cap.cubin > spill.r$cap.sm_100a.sass
 done
 rm -rf $T
+# Line-info pairs: ONE cubin per kernel (compiled with -lineinfo), disassembled twice — cuobjdump
+# -sass (hex branch targets, no lines) and nvdisasm -g -c (".text.f:" labels, `(.L_x_N) branch
+# labels, //## File "f", line N). Both texts must give the same detection (tests/test_oracle_pins.py).
+mkdir -p lineinfo
+T=$(mktemp -d)
+for k in sgemm_naive jacobi mixbench atomics spill; do
+  nvcc -arch=sm_100a -cubin -O3 -lineinfo -maxrregcount=32 -o $T/$k.cubin src/$k.cu
+  cuobjdump -sass $T/$k.cubin > lineinfo/$k.cuobjdump.sass
+  nvdisasm -g -c $T/$k.cubin > lineinfo/$k.nvdisasm.sass
+done
+rm -rf $T

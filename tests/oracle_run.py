@@ -21,8 +21,9 @@ def build_oracle(force: bool = False) -> str:
 
 
 def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, kbegin=0, kend=-1,
-        detect=True, hist=True, timing=False) -> str:
-    """sass: path or text/bytes. samples: [N,3] uint32 raw triples. Returns canonical text."""
+        detect=True, hist=True, timing=False, counts: np.ndarray | None = None, join: str = "pc") -> str:
+    """sass: path or text/bytes. samples: [N,3] uint32 raw triples. counts: [M,4] uint32
+    pre-aggregated (kernel, pc, reason, count) records. join: pc | line. Returns canonical text."""
     build_oracle()
     tmp = []
     try:
@@ -42,6 +43,14 @@ def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, k
             f.close()
             tmp.append(f.name)
             cmd += ["--samples", f.name]
+        if counts is not None:
+            f = tempfile.NamedTemporaryFile("wb", suffix=".bin", delete=False)
+            np.ascontiguousarray(counts, dtype=np.uint32).tofile(f)
+            f.close()
+            tmp.append(f.name)
+            cmd += ["--counts", f.name]
+        if join != "pc":
+            cmd += ["--join", join]
         if not detect:
             cmd.append("--no-detect")
         if not hist:

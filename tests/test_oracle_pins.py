@@ -282,3 +282,115 @@ def test_configs_generate_and_run():
         assert len(c.K) == {"C1": 1, "C2": 3}[cfg]
         assert sum(k["n"] for k in c.kstats()) == s.P
         assert c.sites("SPILL") if cfg == "C1" else c.sites("VEC")
+
+
+# --------------------------------------------------------------------------- nvdisasm text (O1)
+LINEINFO = ["sgemm_naive", "jacobi", "mixbench", "atomics", "spill"]
+
+
+def _strip_lines(lines):
+    import re
+    return [re.sub(r" line=\S+", "", x) for x in lines]
+
+
+@pytest.mark.parametrize("name", LINEINFO)
+def test_nvdisasm_and_cuobjdump_of_one_cubin_agree(name):
+    """One cubin, two disassemblers: nvdisasm -g (".text.f:" function labels, `(.L_x_N) branch
+    labels, //## line info) and cuobjdump -sass (hex branch targets) must give identical kernels
+    and sites (only the line= attribute differs). Pins the label resolution (loop marks, R28)."""
+    a = Canon(orc.run(golden(f"lineinfo/{name}.cuobjdump.sass")))
+    b = Canon(orc.run(golden(f"lineinfo/{name}.nvdisasm.sass")))
+    assert a.K == b.K and len(a.K) >= 1
+    assert _strip_lines(a.S) == _strip_lines(b.S)
+    assert all("line=-" in x for x in a.S)
+    assert all("line=-" not in x for x in b.S)
+    if name in ("sgemm_naive", "atomics", "spill"):
+        assert any(s["ld"] != "0" for s in b.sites())   # loops found through labels
+
+
+def test_nvdisasm_lines_are_the_source_lines():
+    """jacobi.cu: the five Told[...] loads sit on the source lines that read Told, the six
+    conversions on the lines with (float) casts (tests/golden/src/jacobi.cu)."""
+    src = open(golden("src/jacobi.cu")).read().splitlines()
+    told = {i + 1 for i, t in enumerate(src) if "Told[" in t}
+    casts = {i + 1 for i, t in enumerate(src) if "(float)" in t}
+    c = Canon(orc.run(golden("lineinfo/jacobi.nvdisasm.sass")))
+    assert {int(s["line"]) for s in c.sites("RO")} == told and len(told) == 5
+    conv = c.sites("CONV")
+    assert len(conv) == 6 and {int(s["line"]) for s in conv} <= casts
+
+
+def _nvdisasm_line_table(path):
+    """independent test-side parse: instruction index -> (file, line) of an nvdisasm -g listing"""
+    import re
+    out, cur = [], None
+    for t in open(path):
+        m = re.match(r'\s*//## File "([^"]*)", line (\d+)', t)
+        if m:
+            cur = (m.group(1), int(m.group(2)))
+            continue
+        if re.match(r"\s*/\*[0-9a-f]{4,}\*/\s", t):
+            out.append(cur)
+    return out
+
+
+def test_line_join_closed_form():
+    """join=line (R33): a site's row is the sum of the count-table rows of every
+    instruction on its source line; tot, rel and h follow from the table and an independent parse
+    of the //## line markers."""
+    from gen import samples as gs
+    path = golden("lineinfo/jacobi.nvdisasm.sass")
+    lines = _nvdisasm_line_table(path)
+    n = len(lines)
+    rng = np.random.default_rng(31)
+    tab = np.zeros((n, 32), np.int64)
+    tab[:, :19] = rng.integers(0, 50, (n, 19))
+    raw = gs.Trace(tab, [0], [n], order="shuffled", seed=31).raw()
+    pc = Canon(orc.run(path, samples=raw))
+    ln = Canon(orc.run(path, samples=raw, join="line"))
+    assert ln.H == pc.H and ln.S == pc.S
+    rel_sets = {"VEC": [6], "SPILL": [5, 6], "SHMEM": [6], "GATOM": [5], "RO": [6], "TEX": [6, 16],
+                "CONV": list(range(32))}
+    got = {}
+    for r in ln.R:
+        f = r.split()
+        kv = dict(x.split("=") for x in f[5:])
+        got[(int(f[3]), f[4])] = kv
+    assert len(got) == len(pc.R)
+    for s in ln.sites():
+        row = tab[[i for i in range(n) if lines[i] == lines[s["idx"]]]].sum(axis=0)
+        kv = got[(s["idx"], s["rule"])]
+        assert int(kv["tot"]) == int(row.sum())
+        assert int(kv["rel"]) == int(row[rel_sets[s["rule"]]].sum())
+        assert kv["h"] == ",".join(str(int(x)) for x in row[:19])
+    # a line holding several instructions really aggregates
+    assert any(int(got[(s["idx"], s["rule"])]["tot"]) > int(tab[s["idx"]].sum()) for s in ln.sites())
+    # without line information join=line is join=pc
+    plain = golden("lineinfo/jacobi.cuobjdump.sass")
+    assert Canon(orc.run(plain, samples=raw, join="line")).R == Canon(orc.run(plain, samples=raw)).R
+
+
+def test_count_records_equal_expanded_samples():
+    """Pre-aggregated (kernel, pc, reason, count) records (CUPTI PC-sampling shape, SURVEY §8f
+    row 3) give exactly the histogram, totals and ranking of the same samples one by one,
+    including invalid records (counted by their sample count)."""
+    path = golden("sgemm_naive.sm_100a.sass")
+    n = len(orc.sass_ops(path))
+    rng = np.random.default_rng(7)
+    m = 400
+    rec = np.zeros((m, 4), np.uint32)
+    rec[:, 0] = 0
+    rec[:, 1] = rng.integers(0, n, m) * 16
+    rec[:, 2] = rng.integers(0, 19, m)
+    rec[:, 3] = rng.integers(0, 40, m)
+    rec[:5, 1] += 4            # pc not 16-aligned -> invalid
+    rec[5:8, 2] = 25           # reason >= R -> invalid
+    rec[8:10, 0] = 3           # kernel out of range -> invalid
+    raw = np.repeat(rec[:, :3], rec[:, 3].astype(np.int64), axis=0)
+    a = Canon(orc.run(path, counts=rec))
+    b = Canon(orc.run(path, samples=raw))
+    assert a.H == b.H and a.N == b.N and a.R == b.R
+    assert int(a.N["invalid"]) == int(rec[:10, 3].sum())
+    # samples and records together add up
+    c = Canon(orc.run(path, samples=raw, counts=rec))
+    assert c.H == {k: 2 * v for k, v in b.H.items()}

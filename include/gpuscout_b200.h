@@ -52,10 +52,18 @@ typedef struct {
                                column r, the row padded to 32), or n_reasons -> compact rows holding only
                                the active reasons (4*R bytes per slot: less to zero, write and reduce
                                across GPUs). Any other value -> GS_E_INVAL.         */
-  uint32_t reserved;
+  uint32_t join_mode;       /* which histogram rows a site is joined with, GS_JOIN_*. default PC     */
 } gs_config;
 
 enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3 };
+
+/* Join granularity (R18, R33):
+ *   GS_JOIN_PC   the site PC's row ("attributed to the instruction detected");
+ *   GS_JOIN_LINE the sum of the rows of every instruction of the kernel on the site's source line
+ *                (file, line) from nvdisasm -g ("stall reasons ... at the line numbers identified",
+ *                P:325-327); a site without line information keeps its PC row.
+ * Ranked counts[] are the joined row, saturated to 2^32-1; rel and tot are exact. */
+enum { GS_JOIN_PC = 0, GS_JOIN_LINE = 1 };
 
 /* Rule ids (paper §4) — also the rank tie-break order. */
 enum { GS_VEC = 0, GS_SPILL = 1, GS_SHMEM = 2, GS_GATOM = 3, GS_RO = 4, GS_TEX = 5, GS_CONV = 6 };
@@ -100,7 +108,7 @@ const char *gs_last_error(const gs_ctx *ctx);
 /* Library build string (arch, version). */
 const char *gs_version(void);
 
-/* a-1: parse cuobjdump / nvdisasm SASS text (host memory, borrowed for the call; `len`
+/* a-1: parse cuobjdump -sass / nvdisasm [-g] SASS text (host memory, borrowed for the call; `len`
  * bytes, need not be NUL-terminated), pack one 16-byte record per instruction and upload them.
  * Replaces any previously loaded SASS and invalidates sites. Host-synchronous; the upload is
  * enqueued on the context stream. Parse errors -> GS_E_PARSE with the 1-based line number. */
@@ -145,8 +153,18 @@ gs_status gs_pack_samples(gs_ctx *ctx, const uint32_t *d_raw, uint64_t n, uint32
 gs_status gs_attribute_samples(gs_ctx *ctx, const uint32_t *samples, uint64_t n, int32_t *d_hist,
                                unsigned long long *d_n_invalid, int accumulate);
 
+/* a-9 for PRE-AGGREGATED PC-sampling data (CUPTI's CUpti_PCSamplingPCData gives, per PC, a sample
+ * count per stall reason): d_recs (device) holds n records of four
+ * uint32 {kernel, pc byte offset, reason, count}; H[slot*row + reason] += count for every valid
+ * record (validity as gs_pack_samples, R30), and *d_n_invalid (device u64) += count of every
+ * invalid one, so that sum(H) + n_invalid = sum(count). d_hist (device, n_instr*row int32) is
+ * zeroed first unless accumulate != 0; bins must stay below 2^31. Async. */
+gs_status gs_attribute_counts(gs_ctx *ctx, const uint32_t *d_recs, uint64_t n, int32_t *d_hist,
+                              unsigned long long *d_n_invalid, int accumulate);
+
 /* a-11, a-12 (R20): join the (already all-reduced) histogram onto the sites of the
- * last gs_detect and rank them by (rel desc, tot desc, kernel, idx, rule). Writes the first
+ * last gs_detect (rows per gs_config.join_mode) and rank them by (rel desc, tot desc, kernel, idx,
+ * rule). Writes the first
  * min(k, n_sites) rows to `out` (host or device; k = UINT64_MAX -> all) and the row count to
  * *n_out. Synchronises the stream. */
 gs_status gs_rank_sites(gs_ctx *ctx, const int32_t *d_hist, uint64_t k, gs_ranked_site *out,

@@ -17,6 +17,7 @@ LIB_PATH = os.path.join(HERE, "libgpuscout_b200.so")
 
 GS_OK, GS_E_INVAL, GS_E_PARSE, GS_E_RANGE, GS_E_CUDA, GS_E_NOMEM, GS_E_STATE = 0, -1, -2, -3, -4, -5, -6
 GS_HIST_AUTO, GS_HIST_GLOBAL, GS_HIST_PRIVATE, GS_HIST_WINDOW = 0, 1, 2, 3
+GS_JOIN_PC, GS_JOIN_LINE = 0, 1
 RULES = ["VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX", "CONV"]
 TERMS = ["NONE", "PARAM", "CONST", "ENTRY", "SREG", "MEMORY", "IMM", "TRUNC"]
 
@@ -35,7 +36,7 @@ class GsConfig(ctypes.Structure):
     _fields_ = [("trace_depth", ctypes.c_uint32), ("n_reasons", ctypes.c_uint32),
                 ("shmem_min_arith", ctypes.c_uint32), ("shmem_min_loads", ctypes.c_uint32),
                 ("hist_mode", ctypes.c_uint32), ("hist_counter_bits", ctypes.c_uint32),
-                ("hist_row", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("hist_row", ctypes.c_uint32), ("join_mode", ctypes.c_uint32)]
 
 
 class GsError(RuntimeError):
@@ -45,7 +46,7 @@ class GsError(RuntimeError):
 _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
-           "gs_attribute_samples", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
+           "gs_attribute_samples", "gs_attribute_counts", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
 
 
 def launch_count() -> int:
@@ -76,6 +77,7 @@ def load_library(path: str = LIB_PATH):
         "gs_kernel_stats_get": (I32, [P, P, SZ]),
         "gs_pack_samples": (I32, [P, P, U64, P, P]),
         "gs_attribute_samples": (I32, [P, P, U64, P, P, I32]),
+        "gs_attribute_counts": (I32, [P, P, U64, P, P, I32]),
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
         "gs_rank_sites_slice": (I32, [P, P, U64, U64, U64, P, ctypes.POINTER(U64)]),
         "gs_last_hist_mode": (I32, [P]),
@@ -107,7 +109,7 @@ class Context:
 
     def __init__(self, device: int | None = None, stream=None, trace_depth: int = 64, n_reasons: int = 19,
                  shmem_min_arith: int = 1, shmem_min_loads: int = 2, hist_mode: int = GS_HIST_AUTO,
-                 hist_counter_bits: int = 0, hist_row: int = 32):
+                 hist_counter_bits: int = 0, hist_row: int = 32, join_mode: int = GS_JOIN_PC):
         import torch
         if not torch.cuda.is_available():
             raise GsError("no CUDA device: the library has no CPU fallback")
@@ -118,7 +120,7 @@ class Context:
         self.torch_stream = stream
         handle = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
         cfg = GsConfig(trace_depth, n_reasons, shmem_min_arith, shmem_min_loads, hist_mode, hist_counter_bits,
-                       hist_row)
+                       hist_row, join_mode)
         self.n_reasons = n_reasons
         self.hist_row = hist_row or 32  # bins per histogram row: 32, or n_reasons (compact)
         self.trace_depth = trace_depth
@@ -226,6 +228,18 @@ class Context:
                                                 1 if accumulate else 0), "gs_attribute_samples")
         return hist, n_invalid
 
+    def attribute_counts(self, recs, hist=None, n_invalid=None, accumulate: bool = False):
+        """recs: device int32/uint32 tensor [M, 4] of pre-aggregated (kernel, pc, reason, count)."""
+        import torch
+        dev = torch.device("cuda", self.device)
+        if hist is None:
+            hist = torch.empty(self.n_instr * self.hist_row, dtype=torch.int32, device=dev)
+        if n_invalid is None:
+            n_invalid = torch.zeros(1, dtype=torch.int64, device=dev)
+        self._check(self.L.gs_attribute_counts(self.h, recs.data_ptr(), recs.shape[0], hist.data_ptr(),
+                                               n_invalid.data_ptr(), 1 if accumulate else 0), "gs_attribute_counts")
+        return hist, n_invalid
+
     def last_hist_mode(self) -> int:
         return self.L.gs_last_hist_mode(self.h)
 
@@ -265,6 +279,10 @@ def gs_pack_samples(ctx: Context, raw, words=None, n_invalid=None):
 
 def gs_attribute_samples(ctx: Context, samples, hist=None, n_invalid=None, accumulate: bool = False):
     return ctx.attribute_samples(samples, hist, n_invalid, accumulate)
+
+
+def gs_attribute_counts(ctx: Context, recs, hist=None, n_invalid=None, accumulate: bool = False):
+    return ctx.attribute_counts(recs, hist, n_invalid, accumulate)
 
 
 def gs_rank_sites(ctx: Context, hist, k: int | None = None, out=None):

@@ -33,6 +33,11 @@ void free_loaded(gs_ctx* c) {
   if (c->d_kd) cudaFree(c->d_kd);
   if (c->d_wd) cudaFree(c->d_wd);
   if (c->d_cbase) cudaFree(c->d_cbase);
+  if (c->d_lgrp) cudaFree(c->d_lgrp);
+  if (c->d_goff) cudaFree(c->d_goff);
+  if (c->d_gslot) cudaFree(c->d_gslot);
+  c->d_lgrp = c->d_goff = c->d_gslot = nullptr;
+  c->n_lgroups = 0;
   c->d_rec = nullptr;
   c->d_kd = nullptr;
   c->d_wd = nullptr;
@@ -72,7 +77,7 @@ gs_status gs_create(gs_ctx** out, int device, void* cuda_stream, const gs_config
   if (!c->cfg.shmem_min_loads) c->cfg.shmem_min_loads = 2;
   if (!c->cfg.hist_row) c->cfg.hist_row = 32;
   if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_WINDOW ||
-      (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) ||
+      (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) || c->cfg.join_mode > GS_JOIN_LINE ||
       (c->cfg.hist_counter_bits != 0 && c->cfg.hist_counter_bits != 16 && c->cfg.hist_counter_bits != 32)) {
     delete c;
     return GS_E_INVAL;
@@ -152,6 +157,29 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   }
   c->cbase_h.push_back((uint32_t)c->n_cand);
   c->n_win = (uint32_t)c->wd_h.size();
+  // source-line groups (R33): global id = kernel's base + kernel-local (file, line) key; CSR of slots
+  std::vector<uint32_t> lgrp, goff, gslot;
+  {
+    uint64_t G = 0;
+    for (auto& k : ks) G += k.n_lkeys;
+    if (G) {
+      lgrp.assign(P, ~0u);
+      goff.assign(G + 1, 0);
+      uint32_t gb = 0, sl = 0;
+      for (auto& k : ks) {
+        for (size_t i = 0; i < k.lkeys.size(); i++)
+          if (k.lkeys[i] >= 0) { lgrp[sl + i] = gb + (uint32_t)k.lkeys[i]; goff[lgrp[sl + i] + 1]++; }
+        gb += k.n_lkeys;
+        sl += (uint32_t)k.recs.size();
+      }
+      for (uint64_t g = 0; g < G; g++) goff[g + 1] += goff[g];
+      gslot.assign(goff[G], 0);
+      std::vector<uint32_t> fill(goff.begin(), goff.end() - 1);
+      for (uint32_t q = 0; q < P; q++)
+        if (lgrp[q] != ~0u) gslot[fill[lgrp[q]]++] = q;
+      c->n_lgroups = (uint32_t)G;
+    }
+  }
   if (c->n_cand > 0xffffffffull) return fail(c, GS_E_RANGE, "too many candidate instructions");
   GS_CUDA(c, cudaMalloc((void**)&c->d_rec, std::max<uint64_t>(P, 1) * sizeof(Rec)));
   GS_CUDA(c, cudaMalloc((void**)&c->d_kd, std::max<size_t>(ks.size(), 1) * sizeof(KDesc)));
@@ -164,6 +192,15 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     GS_CUDA(c, cudaMemcpyAsync(c->d_wd, c->wd_h.data(), c->wd_h.size() * sizeof(WDesc), cudaMemcpyHostToDevice,
                                c->stream));
   GS_CUDA(c, cudaMemcpyAsync(c->d_cbase, c->cbase_h.data(), c->cbase_h.size() * 4, cudaMemcpyHostToDevice, c->stream));
+  if (c->n_lgroups) {
+    GS_CUDA(c, cudaMalloc((void**)&c->d_lgrp, lgrp.size() * 4));
+    GS_CUDA(c, cudaMalloc((void**)&c->d_goff, goff.size() * 4));
+    GS_CUDA(c, cudaMalloc((void**)&c->d_gslot, std::max<size_t>(gslot.size(), 1) * 4));
+    GS_CUDA(c, cudaMemcpyAsync(c->d_lgrp, lgrp.data(), lgrp.size() * 4, cudaMemcpyHostToDevice, c->stream));
+    GS_CUDA(c, cudaMemcpyAsync(c->d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, c->stream));
+    if (!gslot.empty())
+      GS_CUDA(c, cudaMemcpyAsync(c->d_gslot, gslot.data(), gslot.size() * 4, cudaMemcpyHostToDevice, c->stream));
+  }
   gs_status s = detect_alloc(c);
   if (s != GS_OK) return s;
   // pageable source buffers: wait for the copies before they go out of scope
@@ -279,6 +316,17 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
   }
   GS_CUDA(c, cudaStreamSynchronize(c->stream));
   return GS_OK;
+}
+
+gs_status gs_attribute_counts(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_hist,
+                              unsigned long long* d_n_invalid, int accumulate) {
+  if (!c || (n && !d_recs) || !d_n_invalid) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_attribute_counts before gs_load_sass");
+  if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
+  if (n && !is_device_ptr(d_recs)) return fail(c, GS_E_INVAL, "count records must be device memory");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  return counts_run(c, d_recs, n, d_hist, d_n_invalid, accumulate);
 }
 
 gs_status gs_rank_sites_slice(gs_ctx* c, const int32_t* d_hist, uint64_t slot_begin, uint64_t slot_end, uint64_t k,

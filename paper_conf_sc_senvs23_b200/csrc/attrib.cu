@@ -86,6 +86,31 @@ __global__ void k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc
   count_invalid(bad, d_n_invalid);
 }
 
+// Pre-aggregated records {kernel, pc, reason, count} (CUPTI PC-sampling shape): one 128-bit load
+// per record, one L2 atomic per valid record (records are already one per (pc, reason), so there
+// is nothing to privatise); invalid records add their count to n_invalid.
+__global__ void k_counts(const uint4* __restrict__ rec, uint64_t n, const KDesc* __restrict__ kd, uint32_t nk,
+                         uint32_t nr, uint32_t row, int32_t* __restrict__ H, unsigned long long* d_n_invalid) {
+  unsigned long long bad = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4 r = __ldg(rec + i);  // x kernel, y pc, z reason, w count
+    bool ok = r.x < nk && (r.y & 15u) == 0 && r.z < nr;
+    uint32_t first = 0;
+    if (ok) {
+      const KDesc K = kd[r.x];
+      ok = (r.y >> 4) < K.n;
+      first = K.first;
+    }
+    if (ok) {
+      if (r.w) atomicAdd(H + (uint64_t)(first + (r.y >> 4)) * row + r.z, (int32_t)r.w);
+    } else {
+      bad += r.w;
+    }
+  }
+  for (int o = 16; o; o >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, o);
+  if ((threadIdx.x & 31) == 0 && bad) atomicAdd(d_n_invalid, bad);
+}
+
 // -------------------------------------------------------------------------------- GLOBAL
 __global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* __restrict__ s, uint64_t n,
                                                                 uint32_t pnr, Div dv, int32_t* __restrict__ H,
@@ -586,6 +611,23 @@ gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_
   if (!n) return GS_OK;
   k_pack<<<(unsigned)((n + 255) / 256), 256, 0, c->stream>>>(d_raw, n, c->d_kd, c->n_kernels, c->cfg.n_reasons,
                                                              d_words, d_n_invalid);
+  count_launch();
+  GS_CUDA(c, cudaGetLastError());
+  return GS_OK;
+}
+
+gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_hist, unsigned long long* d_n_invalid,
+                     int accumulate) {
+  cudaStream_t st = c->stream;
+  const uint32_t row = c->cfg.hist_row;
+  if (!accumulate && c->n_instr) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * row * 4, st));
+  if (!n) return GS_OK;
+  if (reinterpret_cast<uintptr_t>(d_recs) & 15u) return fail(c, GS_E_INVAL, "count records must be 16-byte aligned");
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+  const uint64_t blocks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 8, (n + 255) / 256));
+  k_counts<<<(unsigned)blocks, 256, 0, st>>>(reinterpret_cast<const uint4*>(d_recs), n, c->d_kd, c->n_kernels,
+                                             c->cfg.n_reasons, row, d_hist, d_n_invalid);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;

@@ -61,12 +61,16 @@ struct gs_ctx {
   std::vector<gs::WDesc> wd_h;
   std::vector<uint32_t> cbase_h;  // candidate base per window (n_win + 1)
   std::vector<int32_t> lines_h;
+  uint32_t n_lgroups = 0;             // source-line groups (kernel, file, line), 0 without line info
 
   // ---- device copies
   gs::Rec* d_rec = nullptr;
   gs::KDesc* d_kd = nullptr;
   gs::WDesc* d_wd = nullptr;
   uint32_t* d_cbase = nullptr;
+  uint32_t* d_lgrp = nullptr;   // per slot: its source-line group, ~0u if none (only when n_lgroups)
+  uint32_t* d_goff = nullptr;   // group -> first entry of d_gslot (n_lgroups + 1)
+  uint32_t* d_gslot = nullptr;  // slots ordered by group
 
   // ---- detection scratch
   uint32_t* d_tab = nullptr;  // n_win x 320 last-writer summaries -> carry-in tables
@@ -107,6 +111,8 @@ struct gs_ctx {
   size_t sort_tmp_bytes = 0;
   unsigned long long* d_ktot = nullptr;
   gs_ranked_site* d_ranked = nullptr;
+  uint32_t* d_jrow = nullptr;   // GS_JOIN_LINE: joined row per site (32 u32, saturated)
+  uint64_t jrow_cap = 0;
   uint64_t ranked_cap = 0;
   uint32_t* h_stage[2] = {nullptr, nullptr};  // pinned staging for host sample input
   uint32_t* d_stage[2] = {nullptr, nullptr};
@@ -146,6 +152,8 @@ gs_status detect_alloc(gs_ctx* c);  // after a load
 void detect_free(gs_ctx* c);
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
                            unsigned long long* d_n_invalid);
+gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_hist, unsigned long long* d_n_invalid,
+                     int accumulate);
 gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,
                    unsigned long long* d_n_invalid, int accumulate, bool zero_first);
 // d_hist holds the rows of slots [slot0, ...) (row width cfg.hist_row)

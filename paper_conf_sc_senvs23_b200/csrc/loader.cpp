@@ -1,17 +1,21 @@
 // loader.cpp — SASS text -> packed 16-byte records (§2.1).
 //
 // Product code (host side of gs_load_sass). Written independently of oracle/gs_oracle.cpp from the
-// readings in DESIGN.md §3 (R1, R2, R6, R7, R23-R28). Kernels are parsed in parallel: a first
-// sequential pass only finds "Function :" headers and arch lines; each kernel's lines are then
-// tokenised by a worker thread into records.
+// readings in DESIGN.md §3 (R1, R2, R6, R7, R23-R28, R33). Kernels are parsed in parallel: a first
+// sequential pass only finds kernel headers (cuobjdump "Function : f", nvdisasm ".text.f:") and
+// arch lines; each kernel's lines are then tokenised by a worker thread into records. nvdisasm
+// branch targets are labels (BRA `(.L_x_3)); a label names the pc of the next instruction, and
+// only backward targets matter (R13), so a label is resolved when its branch is reached.
 #include <algorithm>
 #include <atomic>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
 #include <string>
 #include <thread>
+#include <utility>
 #include <vector>
 
 #include "loader.h"
@@ -365,11 +369,20 @@ struct Segment {
   bool header;        // false for an anonymous leading kernel
 };
 
+// nvdisasm function label ".text.<name>:"
+inline bool is_fn_label(Sv t) { return t.n > 7 && starts(t, ".text.") && t[t.n - 1] == ':'; }
+// nvdisasm branch label ".L_x_N:"
+inline bool is_br_label(Sv t) { return t.n > 3 && starts(t, ".L") && t[t.n - 1] == ':'; }
+
 bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::string* err) {
   pk->name = seg.name;
   pk->param_base = (uint32_t)param_base_for(seg.sm);
   long lineno = seg.first_line;
   int32_t src_line = -1;
+  std::string src_file;
+  std::map<std::pair<std::string, int32_t>, int32_t> lkey;  // (file, line) -> kernel-local key
+  std::map<std::string, long long> labels;                  // branch label -> pc
+  std::vector<std::string> pending;
   size_t p = seg.begin;
   while (p < seg.end) {
     const char* nl = (const char*)memchr(text + p, '\n', seg.end - p);
@@ -379,9 +392,16 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     p = e + 1;
     lineno++;
     if (!t.n) continue;
-    if (starts(t, "//##")) {
+    if (starts(t, "//##")) {  // nvdisasm -g: //## File "f", line N
       size_t at;
       if (contains(t, "line ", &at)) src_line = atoi(std::string(t.p + at + 5, t.n - at - 5).c_str());
+      const char* q0 = (const char*)memchr(t.p, '"', t.n);
+      const char* q1 = q0 ? (const char*)memchr(q0 + 1, '"', t.n - (size_t)(q0 + 1 - t.p)) : nullptr;
+      src_file = q1 ? std::string(q0 + 1, (size_t)(q1 - q0 - 1)) : std::string();
+      continue;
+    }
+    if (is_br_label(t)) {
+      pending.emplace_back(t.p, t.n - 1);
       continue;
     }
     if (t.n < 4 || t[0] != '/' || t[1] != '*') continue;
@@ -402,15 +422,41 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
       *err = "line " + std::to_string(cur) + ": pc not 16-strided";
       return false;
     }
+    for (auto& lb : pending) labels[lb] = pc;
+    pending.clear();
+    Sv ins{body.p, semi};
+    std::string subst;  // `(.L_x_N) -> 0x<pc> when the label is already known (a backward target)
+    const char* bq = (const char*)memchr(ins.p, '`', ins.n);
+    if (bq && bq + 1 < ins.p + ins.n && bq[1] == '(') {
+      const char* rp = (const char*)memchr(bq, ')', (size_t)(ins.p + ins.n - bq));
+      if (rp) {
+        auto it = labels.find(std::string(bq + 2, (size_t)(rp - bq - 2)));
+        if (it != labels.end()) {
+          char hx[32];
+          snprintf(hx, sizeof hx, "0x%llx", it->second);
+          subst.assign(ins.p, (size_t)(bq - ins.p));
+          subst += hx;
+          subst.append(rp + 1, (size_t)(ins.p + ins.n - rp - 1));
+          ins = Sv{subst.data(), subst.size()};
+        }
+      }
+    }
     Rec r;
     std::string msg;
-    if (!pack_line(Sv{body.p, semi}, cur, pk->recs.size(), &r, &msg)) {
+    if (!pack_line(ins, cur, pk->recs.size(), &r, &msg)) {
       *err = "line " + std::to_string(cur) + ": " + msg;
       return false;
     }
     pk->recs.push_back(r);
     pk->lines.push_back(src_line);
+    int32_t key = -1;
+    if (src_line >= 0) {
+      auto ins_it = lkey.emplace(std::make_pair(src_file, src_line), (int32_t)lkey.size());
+      key = ins_it.first->second;
+    }
+    pk->lkeys.push_back(key);
   }
+  pk->n_lkeys = (uint32_t)lkey.size();
   return true;
 }
 
@@ -444,14 +490,14 @@ bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedK
         sm = atoi(std::string(t.p + at + 12, t.n - at - 12).c_str());
       } else if (contains(t, ".target") && contains(t, "sm_", &at)) {
         sm = atoi(std::string(t.p + at + 3, t.n - at - 3).c_str());
-      } else if (contains(t, "Function :", &at)) {
+      } else if (contains(t, "Function :", &at) || is_fn_label(t)) {
         if (!segs.empty()) segs.back().end = p;
         Segment s;
         s.begin = e + 1 > len ? len : e + 1;
         s.end = len;
         s.first_line = lineno + 1;
         s.sm = sm;
-        Sv nm = trim(Sv{t.p + at + 10, t.n - at - 10});
+        Sv nm = is_fn_label(t) ? Sv{t.p + 6, t.n - 7} : trim(Sv{t.p + at + 10, t.n - at - 10});
         s.name.assign(nm.p, nm.n);
         s.header = true;
         segs.push_back(s);

@@ -12,9 +12,11 @@ struct ParsedKernel {
   uint32_t param_base = 0x380;
   std::vector<Rec> recs;
   std::vector<int32_t> lines;  // source line per instruction, -1 if unknown
+  std::vector<int32_t> lkeys;  // source-line key per instruction: kernel-local id of (file, line), -1 if unknown
+  uint32_t n_lkeys = 0;
 };
 
-// Parses cuobjdump / nvdisasm text into per-kernel packed records using up to n_threads threads.
+// Parses cuobjdump -sass / nvdisasm [-g] text into per-kernel packed records using up to n_threads threads.
 // Returns false and sets *err ("line N: ...") on malformed input.
 bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedKernel>* out, std::string* err);
 

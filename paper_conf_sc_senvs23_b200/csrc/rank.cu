@@ -115,6 +115,42 @@ __global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int
   }
 }
 
+// GS_JOIN_LINE (R33): one warp per site, lane = reason; the site's row is the sum of
+// the rows of its source-line group (CSR goff/gslot), or its own PC row without line info.
+__global__ void k_join_line(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H,
+                            uint32_t slot0, uint32_t row, const KDesc* __restrict__ kd,
+                            const uint32_t* __restrict__ lgrp, const uint32_t* __restrict__ goff,
+                            const uint32_t* __restrict__ gslot, unsigned long long* __restrict__ rel_out,
+                            unsigned long long* __restrict__ tot_out, uint32_t* __restrict__ jrow,
+                            unsigned long long* __restrict__ mx) {
+  const uint64_t s = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (s >= ns) return;
+  const uint32_t lane = threadIdx.x & 31u;
+  const gs_site st = sites[s];
+  const uint32_t slot = kd[st.kernel].first + st.idx;
+  const uint32_t g = lgrp[slot];
+  unsigned long long v = 0;
+  if (g == ~0u) {
+    if (lane < row) v = (uint32_t)__ldg(H + (uint64_t)(slot - slot0) * row + lane);
+  } else {
+    for (uint32_t q = goff[g]; q < goff[g + 1]; q++)
+      if (lane < row) v += (uint32_t)__ldg(H + (uint64_t)(__ldg(gslot + q) - slot0) * row + lane);
+  }
+  const uint32_t m = kRelMask[st.rule];
+  unsigned long long tot = v, rel = ((m >> lane) & 1u) ? v : 0;
+  for (int o = 16; o; o >>= 1) {
+    tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    rel += __shfl_xor_sync(0xffffffffu, rel, o);
+  }
+  jrow[s * 32 + lane] = v > 0xffffffffull ? 0xffffffffu : (uint32_t)v;
+  if (lane == 0) {
+    rel_out[s] = rel;
+    tot_out[s] = tot;
+    atomicMax(mx, rel);
+    atomicMax(mx + 1, tot);
+  }
+}
+
 // key = ((maskR - rel) << bt) | (maskT - tot); vals = site index
 __global__ void k_keys_packed(const unsigned long long* __restrict__ rel, const unsigned long long* __restrict__ tot,
                               uint64_t ns, int bt, unsigned long long mask_r, unsigned long long mask_t,
@@ -136,21 +172,20 @@ __global__ void k_keys_field(const unsigned long long* __restrict__ val, const u
   if (!order) vals[i] = s;
 }
 
+// one warp per ranked row; counts from the PC row of H, or the joined row jrow (GS_JOIN_LINE)
 __global__ void k_emit(const uint32_t* __restrict__ order, uint64_t kk, const gs_site* __restrict__ sites,
-                       const int32_t* __restrict__ H, uint32_t slot0, uint32_t row, const KDesc* __restrict__ kd,
-                       const unsigned long long* __restrict__ ktot, gs_ranked_site* __restrict__ out) {
-  const uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);  // one warp per row
+                       const int32_t* __restrict__ H, uint32_t slot0, uint32_t row, const uint32_t* __restrict__ jrow,
+                       const unsigned long long* __restrict__ rel_a, const unsigned long long* __restrict__ tot_a,
+                       const KDesc* __restrict__ kd, const unsigned long long* __restrict__ ktot,
+                       gs_ranked_site* __restrict__ out) {
+  const uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
   if (q >= kk) return;
   const int lane = threadIdx.x & 31;
-  const gs_site st = sites[order[q]];
+  const uint32_t si = order[q];
+  const gs_site st = sites[si];
   const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx - slot0;
-  const uint32_t c = (uint32_t)lane < row ? (uint32_t)H[slot * row + lane] : 0u;
-  const uint32_t m = kRelMask[st.rule];
-  unsigned long long tot = c, rel = ((m >> lane) & 1u) ? c : 0;
-  for (int o = 16; o; o >>= 1) {
-    tot += __shfl_xor_sync(0xffffffffu, tot, o);
-    rel += __shfl_xor_sync(0xffffffffu, rel, o);
-  }
+  const uint32_t c = jrow ? jrow[(uint64_t)si * 32 + lane] : ((uint32_t)lane < row ? (uint32_t)H[slot * row + lane] : 0u);
+  const unsigned long long rel = rel_a[si], tot = tot_a[si];
   gs_ranked_site* r = out + q;
   r->counts[lane] = c;
   if (lane == 0) {
@@ -219,8 +254,15 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
     void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
     const unsigned grid = (unsigned)((ns + 255) / 256);
-    const bool vec = row == 32 && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0;
-    k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, vec, c->d_kd, d_rel, d_tot, d_max);
+    const bool line = c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups;
+    if (line) {
+      GS_CUDA(c, dev_grow(&c->d_jrow, &c->jrow_cap, ns * 32));
+      k_join_line<<<(unsigned)((ns + 7) / 8), 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, c->d_kd, c->d_lgrp,
+                                                            c->d_goff, c->d_gslot, d_rel, d_tot, c->d_jrow, d_max);
+    } else {
+      const bool vec = row == 32 && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0;
+      k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, vec, c->d_kd, d_rel, d_tot, d_max);
+    }
     count_launch();
     GS_CUDA(c, cudaGetLastError());
     unsigned long long mx[2];
@@ -259,7 +301,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
         GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
         dst = c->d_ranked;
       }
-      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row, c->d_kd,
+      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
+                                                        line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
                                                         c->d_ktot, dst);
       count_launch();
       GS_CUDA(c, cudaGetLastError());
@@ -282,6 +325,9 @@ void rank_free(gs_ctx* c) {
   if (c->d_sort_tmp) cudaFree(c->d_sort_tmp);
   if (c->d_ktot) cudaFree(c->d_ktot);
   if (c->d_ranked) cudaFree(c->d_ranked);
+  if (c->d_jrow) cudaFree(c->d_jrow);
+  c->d_jrow = nullptr;
+  c->jrow_cap = 0;
   c->d_sort_tmp = nullptr;
   c->d_ktot = nullptr;
   c->d_ranked = nullptr;

@@ -16,7 +16,9 @@ pytestmark = [pytest.mark.gpu, pytest.mark.usefixtures("oracle_bin")]
 FIXTURES = ["listing1.sass", "sgemm_naive.sm_100a.sass", "sgemm_naive.sm_70.sass", "jacobi.sm_100a.sass",
             "jacobi.sm_70.sass", "mixbench.sm_100a.sass", "mixbench.sm_70.sass", "atomics.sm_100a.sass",
             "atomics.sm_70.sass", "conv.sm_100a.sass", "spill.r24.sm_100a.sass", "spill.r32.sm_100a.sass",
-            "spill.r40.sm_100a.sass", "spill.r64.sm_100a.sass"]
+            "spill.r40.sm_100a.sass", "spill.r64.sm_100a.sass"] + \
+    [f"lineinfo/{k}.{d}.sass" for k in ("sgemm_naive", "jacobi", "mixbench", "atomics", "spill")
+     for d in ("cuobjdump", "nvdisasm")]
 
 
 @pytest.fixture(scope="module")
@@ -95,10 +97,10 @@ def test_trace_depth_edges(gs):
 
 
 # ------------------------------------------------------------------------------ full flow
-def _flow(gs, text, raw, hist_mode=0, host_input=False, k=None, n_reasons=19, hist_row=32):
+def _flow(gs, text, raw, hist_mode=0, host_input=False, k=None, n_reasons=19, hist_row=32, join_mode=0):
     import torch
     from paper_conf_sc_senvs23_b200 import report
-    ctx = _ctx(gs, hist_mode=hist_mode, n_reasons=n_reasons, hist_row=hist_row)
+    ctx = _ctx(gs, hist_mode=hist_mode, n_reasons=n_reasons, hist_row=hist_row, join_mode=join_mode)
     ctx.load_sass(text)
     ctx.detect()
     raw_t = torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda()
@@ -181,6 +183,71 @@ def test_rank_against_histogram_slice(gs, row):
             if se > sb:
                 with pytest.raises(gs.GsError, match="does not cover"):
                     ctx.rank_sites(hist[(sb + 1) * row:se * row], slot_begin=sb + 1, slot_end=se)
+
+
+@pytest.mark.parametrize("name", ["jacobi", "sgemm_naive", "mixbench", "spill"])
+@pytest.mark.parametrize("row", [32, 19])
+def test_line_join_parity(gs, name, row):
+    """GS_JOIN_LINE on nvdisasm -g text: each site joined with the sum of its source line's rows
+    (R33), against the oracle's --join line; on cuobjdump text (no lines) it is the PC
+    join."""
+    from gen import samples as gsm
+    for disasm in ("nvdisasm", "cuobjdump"):
+        text = _read(f"lineinfo/{name}.{disasm}.sass")
+        o_pc = Canon(orc.run(text))
+        n = sum(int(k["n"]) for k in o_pc.kstats())
+        first = [int(k["first"]) for k in o_pc.kstats()]
+        nk = [int(k["n"]) for k in o_pc.kstats()]
+        rng = np.random.default_rng(41)
+        tab = np.zeros((n, 32), np.int64)
+        tab[:, :19] = rng.integers(0, 30, (n, 19))
+        raw = gsm.Trace(tab, first, nk, order="shuffled", seed=41).raw()
+        g, _ = _flow(gs, text, raw, hist_row=row, join_mode=1)
+        o = Canon(orc.run(text, samples=raw, join="line"))
+        assert g.S == o.S and g.H == o.H and g.N == o.N
+        assert g.R == o.R, (name, disasm)
+
+
+def test_attribute_counts_parity(gs):
+    """gs_attribute_counts: pre-aggregated (kernel, pc, reason, count) records (CUPTI PC-sampling
+    shape) against the oracle's --counts, invalid records included; plus accumulate on top of
+    per-sample attribution."""
+    import torch
+    from paper_conf_sc_senvs23_b200 import report
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    rng = np.random.default_rng(43)
+    m = 50_000
+    rec = np.zeros((m, 4), np.uint32)
+    rec[:, 0] = rng.integers(0, len(s.n_instr), m)
+    rec[:, 1] = (rng.integers(0, 1 << 20, m) % s.n_instr[rec[:, 0]]) * 16
+    rec[:, 2] = rng.integers(0, 19, m)
+    rec[:, 3] = rng.integers(0, 1000, m)
+    rec[:7, 1] += 8
+    rec[7:11, 2] = 19
+    rec[11:13, 0] = len(s.n_instr)
+    rec[13:15, 1] = s.n_instr[rec[13:15, 0]] * 16
+    for row in (32, 19):
+        ctx = _ctx(gs, hist_row=row)
+        ctx.load_sass(s.text)
+        ctx.detect()
+        recs = torch.from_numpy(rec.view(np.int32).copy()).cuda()
+        hist, ninv = ctx.attribute_counts(recs)
+        ranked = ctx.rank_sites(hist)
+        torch.cuda.synchronize()
+        g = Canon(report.canonical(ctx, hist=hist, n_samples=int(rec[:, 3].sum()), n_invalid=int(ninv.item()),
+                                   ranked=ranked))
+        o = Canon(orc.run(s.text, counts=rec))
+        assert g.H == o.H and g.N == o.N and g.R == o.R
+        # samples + records accumulate into one histogram
+        raw = rec[15:2000]
+        raw = np.repeat(raw[:, :3], raw[:, 3].astype(np.int64), axis=0)
+        words, _ = ctx.pack_samples(torch.from_numpy(raw.view(np.int32).copy()).cuda())
+        hist2, _ = ctx.attribute_samples(words)
+        hist2, _ = ctx.attribute_counts(recs, hist=hist2, accumulate=True)
+        o2 = Canon(orc.run(s.text, samples=raw, counts=rec))
+        h2 = hist2.cpu().numpy().reshape(-1, row)
+        assert {(int(a), int(b)): int(h2[a, b]) for a, b in zip(*np.nonzero(h2))} == o2.H
 
 
 def test_host_input_and_topk(gs):

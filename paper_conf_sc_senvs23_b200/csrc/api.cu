@@ -99,6 +99,7 @@ void gs_destroy(gs_ctx* c) {
   free_loaded(c);
   attrib_free(c);
   rank_free(c);
+  if (c->h_pin) cudaFreeHost(c->h_pin);
   delete c;
 }
 

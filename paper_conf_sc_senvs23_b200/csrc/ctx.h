@@ -107,6 +107,7 @@ struct gs_ctx {
   unsigned long long* d_rank_keys[2] = {nullptr, nullptr};
   uint32_t* d_rank_vals[2] = {nullptr, nullptr};
   uint64_t rank_cap = 0;
+  int rank_bits_guess[2] = {-1, -1};  // bit widths of max(rel), max(tot) used by the last rank call
   void* d_sort_tmp = nullptr;
   size_t sort_tmp_bytes = 0;
   unsigned long long* d_ktot = nullptr;
@@ -114,6 +115,8 @@ struct gs_ctx {
   uint32_t* d_jrow = nullptr;   // GS_JOIN_LINE: joined row per site (32 u32, saturated)
   uint64_t jrow_cap = 0;
   uint64_t ranked_cap = 0;
+  void* h_pin = nullptr;  // pinned host scratch for small D2H results (async copies, no hidden sync)
+  size_t h_pin_bytes = 0;
   uint32_t* h_stage[2] = {nullptr, nullptr};  // pinned staging for host sample input
   uint32_t* d_stage[2] = {nullptr, nullptr};
   cudaEvent_t ev_stage[2] = {nullptr, nullptr};
@@ -133,6 +136,17 @@ gs_status cuda_fail(gs_ctx* c, cudaError_t e, const char* what);
     cudaError_t e_ = (call);                                \
     if (e_ != cudaSuccess) return gs::cuda_fail(ctx, e_, #call); \
   } while (0)
+
+// pinned host scratch of at least `bytes` (contents not preserved)
+inline cudaError_t pin_grow(gs_ctx* c, size_t bytes) {
+  if (c->h_pin && c->h_pin_bytes >= bytes) return cudaSuccess;
+  if (c->h_pin) cudaFreeHost(c->h_pin);
+  c->h_pin = nullptr;
+  c->h_pin_bytes = 0;
+  cudaError_t e = cudaHostAlloc(&c->h_pin, bytes < 4096 ? 4096 : bytes, cudaHostAllocDefault);
+  if (e == cudaSuccess) c->h_pin_bytes = bytes < 4096 ? 4096 : bytes;
+  return e;
+}
 
 template <typename T>
 cudaError_t dev_grow(T** p, uint64_t* cap, uint64_t need) {

@@ -417,7 +417,9 @@ __global__ void k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca,
 __global__ void k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
                         uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, const uint32_t* __restrict__ narith,
                         const uint32_t* __restrict__ site_off, gs_site* __restrict__ sites,
-                        uint32_t* __restrict__ chain) {
+                        uint32_t* __restrict__ chain, uint64_t site_cap, uint64_t chain_cap) {
+  // Launched before the host knows the totals: writes past the buffers' current capacities are
+  // skipped, and the host relaunches after growing them when a total exceeds its capacity.
   const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (c >= nc) return;
   const uint32_t f = ca.flags[c];
@@ -428,7 +430,7 @@ __global__ void k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ k
   const unsigned long long coff = ca.choff[c];
   // chain: re-chase and store kernel-local indices
   uint32_t n = 0;
-  if (ca.depth[c])
+  if (ca.depth[c] && coff + ca.depth[c] <= chain_cap)
     chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, [&](uint32_t j) { chain[coff + n++] = j; });
   uint32_t so = site_off[c];
   for (uint32_t rule = 0; rule < 7; rule++) {
@@ -467,7 +469,8 @@ __global__ void k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ k
       s.a0 = (int32_t)gt.nall[ca.grp[c]];
     }
     if (rule == GS_CONV) { s.depth = 0; s.term_kind = GS_T_NONE; s.term_value = 0; }
-    sites[so++] = s;
+    if (so < site_cap) sites[so] = s;
+    so++;
   }
 }
 
@@ -569,7 +572,11 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     GS_CUDA(c, cudaGetLastError());
   }
   unsigned long long* d_tot = c->cand.choff + nc;  // two totals after the offsets
-  unsigned long long tot[2] = {0, 0};
+  // pinned: [0, 16) the two totals, then the per-kernel counters (async D2H, one synchronisation)
+  GS_CUDA(c, pin_grow(c, 16 + (uint64_t)c->n_kernels * sizeof(gs_kernel_stats)));
+  unsigned long long* tot = static_cast<unsigned long long*>(c->h_pin);
+  gs_kernel_stats* kst_pin = reinterpret_cast<gs_kernel_stats*>(static_cast<char*>(c->h_pin) + 16);
+  tot[0] = tot[1] = 0;
   if (nc) {
     const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
     k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
@@ -587,22 +594,33 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     s = scan_u32(c, c->cand.nsite, c->cand.soff, nc, d_tot + 1);
     if (s != GS_OK) return s;
     GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
-    GS_CUDA(c, cudaStreamSynchronize(st));
   }
-  const uint64_t ns = tot[1], nch = tot[0];
-  if (nch > 0xffffffffull) return fail(c, GS_E_RANGE, "chain pool exceeds 2^32 entries");
-  GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
-  GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
-  if (nc && ns) {
+  // sites and chains into the buffers as they are (one host synchronisation per call); if a total
+  // turns out larger than its buffer, grow it and write again
+  auto write = [&]() -> gs_status {
+    if (!nc || (!c->sites_cap && !c->chain_cap)) return GS_OK;
     k_write<<<(uint32_t)((nc + 255) / 256), 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
-                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain); count_launch();
+                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain,
+                                                         c->sites_cap, c->chain_cap); count_launch();
     GS_CUDA(c, cudaGetLastError());
-  }
-  c->kstats_h.assign(c->n_kernels, gs_kernel_stats{});
+    return GS_OK;
+  };
+  gs_status ws = write();
+  if (ws != GS_OK) return ws;
   if (c->n_kernels)
-    GS_CUDA(c, cudaMemcpyAsync(c->kstats_h.data(), c->d_kstats, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats),
+    GS_CUDA(c, cudaMemcpyAsync(kst_pin, c->d_kstats, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats),
                                cudaMemcpyDeviceToHost, st));
   GS_CUDA(c, cudaStreamSynchronize(st));
+  c->kstats_h.assign(kst_pin, kst_pin + c->n_kernels);
+  const uint64_t ns = tot[1], nch = tot[0];
+  if (nch > 0xffffffffull) return fail(c, GS_E_RANGE, "chain pool exceeds 2^32 entries");
+  if (ns > c->sites_cap || nch > c->chain_cap) {
+    GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
+    GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
+    ws = write();
+    if (ws != GS_OK) return ws;
+    GS_CUDA(c, cudaStreamSynchronize(st));
+  }
   c->n_sites = ns;
   c->n_chain = nch;
   c->det_kb = kb; c->det_ke = ke; c->det_c0 = c0; c->det_c1 = c1;

@@ -265,49 +265,74 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     }
     count_launch();
     GS_CUDA(c, cudaGetLastError());
-    unsigned long long mx[2];
+    // The packed sort key needs the bit widths of max(rel) and max(tot). They are read back with
+    // one async copy; the sort itself is enqueued right away with the widths of the previous call
+    // (padded to whole 8-bit radix digits, which costs no extra pass) and redone with the exact
+    // widths only when this call's maxima do not fit them (one host synchronisation otherwise).
+    GS_CUDA(c, pin_grow(c, 16));
+    unsigned long long* mx = static_cast<unsigned long long*>(c->h_pin);
     GS_CUDA(c, cudaMemcpyAsync(mx, d_max, 16, cudaMemcpyDeviceToHost, st));
+    auto passes = [](int bits) { return (uint64_t)(bits + 7) / 8 + 2; };  // onesweep digits + hist + scan
+    const auto sort_emit = [&](int br, int bt) -> gs_status {
+      const uint32_t* order = v0;
+      size_t b1 = cub_bytes;
+      if (br + bt <= 64) {
+        k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
+        count_launch();
+        if (br + bt > 0) {
+          cub::DoubleBuffer<unsigned long long> dk(k0, k1);
+          cub::DoubleBuffer<uint32_t> dv(v0, v1);
+          GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, dk, dv, (int)ns, 0, br + bt, st));
+          count_launch(passes(br + bt));
+          order = dv.Current();
+        }
+      } else {
+        k_keys_field<<<grid, 256, 0, st>>>(d_tot, nullptr, ns, mask_of(bt), k0, v0);
+        count_launch();
+        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v0, v1, (int)ns, 0, bt, st));
+        count_launch(passes(bt));
+        k_keys_field<<<grid, 256, 0, st>>>(d_rel, v1, ns, mask_of(br), k0, nullptr);
+        count_launch();
+        b1 = cub_bytes;
+        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v1, v0, (int)ns, 0, br, st));
+        count_launch(passes(br));
+        order = v0;
+      }
+      GS_CUDA(c, cudaGetLastError());
+      if (kk) {
+        gs_ranked_site* dst = out;
+        if (out_is_host) {
+          GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
+          dst = c->d_ranked;
+        }
+        k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
+                                                          line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
+                                                          c->d_ktot, dst);
+        count_launch();
+        GS_CUDA(c, cudaGetLastError());
+        if (out_is_host)
+          GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));
+      }
+      return GS_OK;
+    };
+    const int gr = c->rank_bits_guess[0], gt = c->rank_bits_guess[1];
+    if (gr >= 0) {
+      gs_status s2 = sort_emit(gr, gt);
+      if (s2 != GS_OK) return s2;
+    }
     GS_CUDA(c, cudaStreamSynchronize(st));
     const int br = bits_of(mx[0]), bt = bits_of(mx[1]);
-    const uint32_t* order = v0;
-    size_t b1 = cub_bytes;
-    auto passes = [](int bits) { return (uint64_t)(bits + 7) / 8 + 2; };  // onesweep digits + hist + scan
-    if (br + bt <= 64) {
-      k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
-      count_launch();
-      if (br + bt > 0) {
-        cub::DoubleBuffer<unsigned long long> dk(k0, k1);
-        cub::DoubleBuffer<uint32_t> dv(v0, v1);
-        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, dk, dv, (int)ns, 0, br + bt, st));
-        count_launch(passes(br + bt));
-        order = dv.Current();
-      }
+    if (br + bt <= 64) {  // next call's widths: this call's, slack spread to fill the last digit
+      const int slack = ((br + bt + 7) / 8) * 8 - (br + bt);
+      c->rank_bits_guess[0] = std::min(64, br + slack / 2);
+      c->rank_bits_guess[1] = std::min(64, bt + slack - slack / 2);
+      if (c->rank_bits_guess[0] + c->rank_bits_guess[1] > 64) c->rank_bits_guess[0] = c->rank_bits_guess[1] = -1;
     } else {
-      k_keys_field<<<grid, 256, 0, st>>>(d_tot, nullptr, ns, mask_of(bt), k0, v0);
-      count_launch();
-      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v0, v1, (int)ns, 0, bt, st));
-      count_launch(passes(bt));
-      k_keys_field<<<grid, 256, 0, st>>>(d_rel, v1, ns, mask_of(br), k0, nullptr);
-      count_launch();
-      b1 = cub_bytes;
-      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v1, v0, (int)ns, 0, br, st));
-      count_launch(passes(br));
-      order = v0;
+      c->rank_bits_guess[0] = c->rank_bits_guess[1] = -1;
     }
-    GS_CUDA(c, cudaGetLastError());
-    if (kk) {
-      gs_ranked_site* dst = out;
-      if (out_is_host) {
-        GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
-        dst = c->d_ranked;
-      }
-      k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
-                                                        line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
-                                                        c->d_ktot, dst);
-      count_launch();
-      GS_CUDA(c, cudaGetLastError());
-      if (out_is_host)
-        GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));
+    if (gr < 0 || br > gr || bt > gt) {
+      gs_status s2 = sort_emit(br, bt);
+      if (s2 != GS_OK) return s2;
     }
   }
   GS_CUDA(c, cudaStreamSynchronize(st));

@@ -250,6 +250,50 @@ def test_attribute_counts_parity(gs):
         assert {(int(a), int(b)): int(h2[a, b]) for a, b in zip(*np.nonzero(h2))} == o2.H
 
 
+def test_rank_repeated_calls(gs):
+    """gs_rank_sites enqueues its sort with the key widths of the previous call and redoes it when
+    the new maxima do not fit: small -> large -> small histograms on one context, each against the
+    oracle."""
+    import torch
+    from paper_conf_sc_senvs23_b200 import report
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    ctx = _ctx(gs, hist_row=19)
+    ctx.load_sass(s.text)
+    ctx.detect()
+    for n, seed in ((20_000, 51), (3_000_000, 52), (50_000, 53), (50_000, 54)):
+        raw, _ = _samples(s, n, "shuffled", seed=seed, n_bad=0)
+        words, _ = ctx.pack_samples(torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda())
+        hist, _ = ctx.attribute_samples(words)
+        for k in (None, 7):
+            ranked = ctx.rank_sites(hist, k=k)
+            g = Canon(report.canonical(ctx, hist=hist, n_samples=len(raw), n_invalid=0, ranked=ranked))
+            o = Canon(orc.run(s.text, samples=raw, k=-1 if k is None else k))
+            assert g.R == o.R, (n, k)
+
+
+def test_detect_repeated_calls(gs):
+    """gs_detect writes sites into the buffers of the previous call and rewrites after growing them
+    when the totals do not fit: few -> many -> few sites on one context."""
+    from gen import sass as gsass
+    small = _read("listing1.sass")
+    big = gsass.config_sass("C2").text
+    ctx = _ctx(gs)
+    for text in (small, big, small, big):
+        ctx.load_sass(text)
+        ctx.detect()
+        from paper_conf_sc_senvs23_b200 import report
+        g = Canon(report.canonical(ctx))
+        o = Canon(orc.run(text))
+        assert g.S == o.S and g.K == o.K
+    # kernel ranges of growing size on one load
+    ctx.load_sass(big)
+    for kb, ke in ((0, 1), (0, 3), (1, 2), (0, 3)):
+        ctx.detect(kb, ke)
+        from paper_conf_sc_senvs23_b200 import report
+        assert Canon(report.canonical(ctx, kb, ke)).S == Canon(orc.run(big, kbegin=kb, kend=ke)).S
+
+
 def test_host_input_and_topk(gs):
     from gen import sass as gsass
     s = gsass.config_sass("C1")

@@ -255,6 +255,21 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
 template <bool P16>
 __device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t row, uint32_t nbins, int32_t* H, uint32_t t,
                       uint32_t nt) {
+  if (P16 && row == nr && ((ws * nr) & 1u) == 0 && (reinterpret_cast<uintptr_t>(H) & 7u) == 0) {
+    // compact rows: the two bins of word i are adjacent int32 of H (window-relative bins 2i, 2i+1
+    // at H[ws*R + 2i], 8-byte aligned), so one 64-bit L2 atomic adds both halves. Exact: bins stay
+    // below 2^31, so the low word never carries into the high one.
+    unsigned long long* H2 = reinterpret_cast<unsigned long long*>(H + (uint64_t)ws * nr);
+    for (uint32_t i = t; 2 * i < nbins; i += nt) {
+      const uint32_t v = tab[i];
+      if (v) {
+        tab[i] = 0;
+        if (2 * i + 1 < nbins) atomicAdd(H2 + i, (unsigned long long)(v & 0xffffu) | ((unsigned long long)(v >> 16) << 32));
+        else atomicAdd(H + (uint64_t)ws * nr + 2 * i, (int32_t)(v & 0xffffu));  // last, unpaired bin
+      }
+    }
+    return;
+  }
   const uint32_t per = P16 ? 2u : 1u;
   const uint32_t stride = per * nt, step_q = stride / nr, step_r = stride % nr;
   uint32_t q = (per * t) / nr, r = (per * t) % nr;
@@ -326,12 +341,18 @@ __device__ __forceinline__ uint32_t kernel_of(uint32_t slot, const KDesc* __rest
 }
 
 // the window for a slot: its whole kernel when that fits, else nslots slots centred on it inside
-// the kernel
-__device__ uint32_t window_for(uint32_t slot, const KDesc* __restrict__ kd, uint32_t nk, uint32_t nslots) {
+// the kernel; moved down one slot when its first bin ws*R is odd (the 64-bit pair flush wants an
+// even first bin; the extra slot in front is harmless, a slot lost at the end is deferred)
+__device__ uint32_t window_for(uint32_t slot, const KDesc* __restrict__ kd, uint32_t nk, uint32_t nslots, uint32_t nr) {
   const KDesc K = kd[kernel_of(slot, kd, nk)];
-  if (K.n <= nslots) return K.first;
-  uint32_t cws = slot > nslots / 2 ? slot - nslots / 2 : 0;
-  return min(max(cws, K.first), K.first + K.n - nslots);
+  uint32_t ws;
+  if (K.n <= nslots) {
+    ws = K.first;
+  } else {
+    const uint32_t cws = slot > nslots / 2 ? slot - nslots / 2 : 0;
+    ws = min(max(cws, K.first), K.first + K.n - nslots);
+  }
+  return ((ws * nr) & 1u) ? ws - 1 : ws;
 }
 
 // median slot of one valid-or-not probe per lane (~0u if no lane holds a valid word)
@@ -528,7 +549,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t med = probe_median(mine, slot);
         if (med == 0xffffffffu) return cur == kNoWindow ? 0u : cur;
         if (!outm && med - cur >= nslots / 8 && med - cur < nslots - nslots / 8) return cur;
-        return window_for(med, kd, nk, nslots);
+        return window_for(med, kd, nk, nslots, nr);
       };
       // two runs: valid probes all in k0 or k1 (k0 != k1), every k0 probe before every k1 probe
       const bool two_runs = okm && k0 != k1 && (m0 | m1) == okm && 31 - __clz(m0) < __ffs(m1) - 1;

@@ -12,6 +12,7 @@ ap.add_argument("--bits", type=int, default=0)
 ap.add_argument("--mode", type=int, default=0)
 ap.add_argument("--order", default="trace")
 ap.add_argument("--iters", type=int, default=10)
+ap.add_argument("--row", type=int, default=19, help="histogram row width (19 compact, as bench.py, or 32)")
 a = ap.parse_args()
 import torch  # noqa: E402
 
@@ -23,9 +24,9 @@ from gen.device import DeviceTrace  # noqa: E402
 
 s, tr = bench.build_workload("C4", a.order)
 words = DeviceTrace(tr).packed()
-ctx = binding.Context(hist_mode=a.mode, hist_counter_bits=a.bits)
+ctx = binding.Context(hist_mode=a.mode, hist_counter_bits=a.bits, hist_row=a.row)
 ctx.load_sass(s.text)
-hist = torch.empty(ctx.n_instr * 32, dtype=torch.int32, device="cuda")
+hist = torch.empty(ctx.n_instr * a.row, dtype=torch.int32, device="cuda")
 ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
 for _ in range(3):
     ctx.attribute_samples(words, hist, ninv)
@@ -38,5 +39,5 @@ e1.record()
 torch.cuda.synchronize()
 ms = e0.elapsed_time(e1) / a.iters
 print(f"lib={a.lib or 'default'} bits={a.bits} mode={a.mode} order={a.order}: {ms:.3f} ms, "
-      f"{tr.N / ms / 1e6:.1f} G samples/s, frac {(4 * tr.N + 128 * ctx.n_instr) / ms / 1e6 / 6555.8:.3f} "
+      f"{tr.N / ms / 1e6:.1f} G samples/s, frac {(4 * tr.N + 4 * a.row * ctx.n_instr) / ms / 1e6 / 6549.8:.3f} "
       f"n_invalid {int(ninv.item())}")

@@ -587,7 +587,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[k]);
     if (it.last) break;
+#if defined(GS_DIAG) && GS_DIAG == 10  // diagnostic: n_invalid counts items
+    if (ct == 0) atomicAdd(d_n_invalid, 1ull);
+#endif
     if (it.ws != ws) {  // window switch: every counter is done with the old window
+#if defined(GS_DIAG) && GS_DIAG == 9  // diagnostic: n_invalid counts window switches
+      if (ct == 0) atomicAdd(d_n_invalid, 1ull);
+#endif
       bar_counters();
       if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
       bar_counters();

@@ -62,6 +62,8 @@ struct Opnd {
   long long coff = 0;          // K_CREF: offset (immediate part)
   int base = kNoReg;           // K_MEM: first register term of the address
   long long off = 0;           // K_MEM: sum of immediate terms
+  bool wide = false;           // K_MEM: the base is a 64-bit pair (Rb.64)
+  bool pred_var = false;       // K_PRED: a real predicate (not PT / UPT)
 };
 
 std::string trim(const std::string& s) {
@@ -169,7 +171,9 @@ Opnd parse_operand(const std::string& raw) {
       p = c + 1;
     }
     Opnd inner;
-    parse_bracket(u.substr(last_open + 1, last_close - last_open - 1), &inner, true);
+    const std::string ib = u.substr(last_open + 1, last_close - last_open - 1);
+    parse_bracket(ib, &inner, true);
+    o.wide = ib.find(".64") != std::string::npos;
     o.base = inner.base;
     o.off = inner.off;
     for (int r : inner.regs) o.regs.push_back(r);
@@ -182,7 +186,11 @@ Opnd parse_operand(const std::string& raw) {
     if (p.size() >= 2 && p[0] == 'U' && p[1] == 'P') p = p.substr(2);
     else if (!p.empty() && p[0] == 'P') p = p.substr(1);
     else p = "#";
-    if (p == "T" || (p.size() == 1 && p[0] >= '0' && p[0] <= '7')) { o.kind = K_PRED; return o; }
+    if (p == "T" || (p.size() == 1 && p[0] >= '0' && p[0] <= '7')) {
+      o.kind = K_PRED;
+      o.pred_var = p != "T";
+      return o;
+    }
   }
   long long v;
   if (parse_int(t, &v)) { o.kind = K_IMM; return o; }
@@ -196,6 +204,7 @@ struct Instr {
   int line = -1;                  // source line from //## File ..., line N
   std::string file;               // ... and its file (a source line is the pair (file, line), R33)
   std::string bra_label;          // nvdisasm: BRA `(.L_x_N) target label, resolved per kernel
+  bool guarded = false;           // @Pn / @!Pn guard (not @PT)
   std::string op;                 // base mnemonic
   std::vector<std::string> mods;  // modifiers after the first '.'
   std::vector<Opnd> ops;
@@ -342,6 +351,7 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     pending.clear();
     // guard predicate
     if (!body.empty() && body[0] == '@') {
+      I.guarded = body.rfind("@PT", 0) != 0 && body.rfind("@UPT", 0) != 0;
       size_t sp = body.find_first_of(" \t");
       body = trim(body.substr(sp));
     }
@@ -715,6 +725,100 @@ void detect_kernel(int kid, const Kernel& K, const Config& C, std::vector<Site>&
   }
 }
 
+// ---------------------------------------------------------------- O16 register pressure
+// "GPUscout presents the number of additional registers needed by each SASS instruction"
+// (SURVEY §8f row 4). Live general-purpose registers per
+// instruction by backward dataflow over the kernel's control-flow graph (reading R36):
+//   live_in(i) = uses(i) ∪ (live_out(i) \ defs(i))   (a guarded instruction kills nothing)
+//   live_out(i) = ∪ live_in(s), s ∈ succ(i)           (BRA target; fall-through unless an
+//                                                      unguarded BRA / EXIT / RET)
+//   count(i) = |live_in(i) ∪ defs(i)|, R1 (the stack pointer) counted live after its definition.
+// Only R0..R254 (nvdisasm's "GPR #" column). additional(i) = count(i) - count(i-1).
+
+bool is_64type(const std::string& m) { return m == "F64" || m == "S64" || m == "U64"; }
+bool is_type(const std::string& m) {
+  return is_64type(m) || m == "F32" || m == "F16" || m == "BF16" || m == "S32" || m == "U32" || m == "S16" ||
+         m == "U16" || m == "S8" || m == "U8" || m == "TF32";
+}
+// register width of a store / atomic data operand (R36): .128 -> 4, .64 or a 64-bit type -> 2
+int data_width(const Instr& I) {
+  for (auto& m : I.mods) if (m == "128") return 4;
+  for (auto& m : I.mods) if (m == "64" || is_64type(m)) return 2;
+  return 1;
+}
+
+// GPR uses of instruction I, pair/quad registers expanded (R36)
+std::set<int> gpr_uses(const Instr& I) {
+  std::set<int> u;
+  int srcw = op_in(I.op, {"DADD", "DMUL", "DFMA", "DSETP", "DMNMX"}) ? 2 : 1;
+  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I", "F2FP", "I2FP", "F2IP"})) {
+    std::vector<std::string> types;
+    for (auto& m : I.mods) if (is_type(m)) types.push_back(m);
+    if (types.size() >= 2 && is_64type(types[1])) srcw = 2;  // second type = source type
+  }
+  const bool store_like = op_in(I.op, {"STG", "STS", "STL", "ST", "RED", "REDG", "ATOMG", "ATOM", "ATOMS"});
+  int srcidx = 0;  // index among the non-predicate operands after the destination
+  for (size_t k = 0; k < I.ops.size(); k++) {
+    if ((int)k == I.dst_pos) continue;
+    const Opnd& o = I.ops[k];
+    for (int r : o.regs) {
+      if (r >= 255) continue;  // RZ, uniform registers
+      int w = 1;
+      // a memory base is a 64-bit pair when written Rb.64 (sm_100) or when the access is .E
+      // ("extended", 64-bit addresses: sm_70's LDG.E [R8] reads R8:R9)
+      if (o.kind == K_MEM) w = (r == o.base && (o.wide || I.has_mod("E"))) ? 2 : 1;
+      else if (o.kind == K_CREF) w = 1;
+      else if (store_like && k > 0) w = data_width(I);
+      else if (I.op == "IMAD" && I.has_mod("WIDE") && srcidx == 2) w = 2;
+      else w = srcw;
+      for (int q = 0; q < w; q++) u.insert(r + q);
+    }
+    if ((int)k > I.dst_pos && o.kind != K_PRED) srcidx++;
+  }
+  return u;
+}
+
+std::vector<int> live_counts(const Kernel& K) {
+  const int n = (int)K.ins.size();
+  std::vector<std::set<int>> use(n), def(n);
+  std::vector<std::vector<int>> succ(n);
+  int r1def = -1;
+  for (int i = 0; i < n; i++) {
+    const Instr& I = K.ins[i];
+    use[i] = gpr_uses(I);
+    if (I.dst != kNoReg && I.dst < 255)
+      for (int q = 0; q < I.dst_w; q++) def[i].insert(I.dst + q);
+    if (r1def < 0 && def[i].count(1)) r1def = i;
+    bool cond = I.guarded;
+    if (I.op == "BRA")
+      for (size_t k = 0; k + 1 < I.ops.size(); k++) cond |= I.ops[k].kind == K_PRED && I.ops[k].pred_var;
+    const bool branch = I.op == "BRA" && I.bra_target >= 0 && I.bra_target / 16 < n;
+    if (branch) succ[i].push_back((int)(I.bra_target / 16));
+    const bool ends = (I.op == "EXIT" || I.op == "RET" || branch) && !cond;
+    if (!ends && i + 1 < n) succ[i].push_back(i + 1);
+  }
+  std::vector<std::set<int>> in(n);
+  for (bool changed = true; changed;) {  // round-robin to the fixed point
+    changed = false;
+    for (int i = n - 1; i >= 0; i--) {
+      std::set<int> out;
+      for (int s : succ[i]) out.insert(in[s].begin(), in[s].end());
+      std::set<int> li = use[i];
+      for (int r : out)
+        if (K.ins[i].guarded || !def[i].count(r)) li.insert(r);
+      if (li != in[i]) { in[i] = li; changed = true; }
+    }
+  }
+  std::vector<int> cnt(n);
+  for (int i = 0; i < n; i++) {
+    std::set<int> c = in[i];
+    c.insert(def[i].begin(), def[i].end());
+    if (r1def >= 0 && i > r1def) c.insert(1);
+    cnt[i] = (int)c.size();
+  }
+  return cnt;
+}
+
 // ---------------------------------------------------------------- O13-O15
 struct RawSample { uint32_t kernel, pc, reason; };
 // pre-aggregated PC-sampling record (CUPTI CUpti_PCSamplingPCData shape: one (pc, stall reason)
@@ -739,7 +843,7 @@ int main(int argc, char** argv) {
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
-  bool detect = true, hist = true, timing = false, quiet = false;
+  bool detect = true, hist = true, timing = false, quiet = false, liveness = false;
   for (int a = 1; a < argc; a++) {
     std::string s = argv[a];
     auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
@@ -756,6 +860,7 @@ int main(int argc, char** argv) {
     else if (s == "--kbegin") kbegin = atoi(nxt().c_str());
     else if (s == "--kend") kend = atoi(nxt().c_str());
     else if (s == "--no-detect") detect = false;
+    else if (s == "--liveness") liveness = true;   // L lines: live GPRs per instruction (O16)
     else if (s == "--no-hist") hist = false;
     else if (s == "--time") timing = true;
     else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
@@ -810,6 +915,12 @@ int main(int argc, char** argv) {
               s.attrs.empty() ? "" : " ", s.attrs.c_str());
     }
   }
+  if (liveness)
+    for (int k = kbegin; k < kend; k++) {
+      std::vector<int> cnt = live_counts(ks[k]);
+      for (size_t i = 0; i < cnt.size(); i++)
+        fprintf(out, "L %d %zu %d %d\n", k, i, cnt[i], cnt[i] - (i ? cnt[i - 1] : 0));
+    }
   if (hist && (!samples_path.empty() || !counts_path.empty())) {
     // O13: H[slot][reason] += 1 for every valid sample.
     size_t P = 0;

@@ -9,12 +9,14 @@ for arch in sm_100a sm_70; do
   for k in sgemm_naive jacobi mixbench atomics conv; do
     nvcc -arch=$arch -cubin -O3 -o $T/$k.$arch.cubin src/$k.cu
     cuobjdump -sass $T/$k.$arch.cubin > $k.$arch.sass
+    nvdisasm -lrm count -c $T/$k.$arch.cubin > $k.$arch.lrm.txt   # nvdisasm's register life ranges
   done
 done
 for cap in 24 32 40 64; do
   nvcc -arch=sm_100a -cubin -O3 -maxrregcount=$cap -Xptxas -v -o $T/spill.$cap.cubin src/spill.cu \
      2> spill.r$cap.ptxas.txt
   cuobjdump -sass $T/spill.$cap.cubin > spill.r$cap.sm_100a.sass
+  nvdisasm -lrm count -c $T/spill.$cap.cubin > spill.r$cap.sm_100a.lrm.txt
 done
 rm -rf $T
 # Line-info pairs: ONE cubin per kernel (compiled with -lineinfo), disassembled twice — cuobjdump
@@ -26,5 +28,7 @@ for k in sgemm_naive jacobi mixbench atomics spill; do
   nvcc -arch=sm_100a -cubin -O3 -lineinfo -maxrregcount=32 -o $T/$k.cubin src/$k.cu
   cuobjdump -sass $T/$k.cubin > lineinfo/$k.cuobjdump.sass
   nvdisasm -g -c $T/$k.cubin > lineinfo/$k.nvdisasm.sass
+  # nvdisasm's own register life ranges (GPR/PRED/UGPR counts per instruction): the pin of O16
+  nvdisasm -lrm count -c $T/$k.cubin > lineinfo/$k.lrm.txt
 done
 rm -rf $T

@@ -394,3 +394,48 @@ def test_count_records_equal_expanded_samples():
     # samples and records together add up
     c = Canon(orc.run(path, samples=raw, counts=rec))
     assert c.H == {k: 2 * v for k, v in b.H.items()}
+
+
+# --------------------------------------------------------------------------- O16 register pressure
+def _lrm_gpr(path):
+    """nvdisasm -lrm count listing -> per function the 'GPR #' column per instruction (test-side parse)"""
+    import re
+    out, cur = [], None
+    for t in open(path):
+        m = re.match(r"\s*\.text\.(\S+):", t)
+        if m:
+            cur = []
+            out.append(cur)
+            continue
+        m = re.match(r"\s*/\*[0-9a-f]{4,}\*/.*;\s*//\s*\|\s*(\d*)\s*\|", t)
+        if m and cur is not None:
+            cur.append(int(m.group(1) or 0))
+    return out
+
+
+LRM_FIXTURES = [(f"lineinfo/{k}.{d}.sass", f"lineinfo/{k}.lrm.txt") for k in LINEINFO
+                for d in ("nvdisasm", "cuobjdump")] + \
+    [(f"{k}.{a}.sass", f"{k}.{a}.lrm.txt") for k in ("sgemm_naive", "jacobi", "mixbench", "atomics", "conv")
+     for a in ("sm_100a", "sm_70")] + \
+    [(f"spill.r{c}.sm_100a.sass", f"spill.r{c}.sm_100a.lrm.txt") for c in (24, 32, 40, 64)]
+
+
+@pytest.mark.parametrize("sass,lrm", LRM_FIXTURES)
+def test_register_pressure_equals_nvdisasm_life_ranges(sass, lrm):
+    """O16 (P:541-554 "the number of additional registers needed by each SASS instruction"): the
+    live-GPR count of every instruction equals nvdisasm's own life-range analysis of the same cubin
+    (nvdisasm -lrm count, GPR column), from either disassembler's text; 'additional' is the
+    difference to the previous instruction."""
+    want = _lrm_gpr(golden(lrm))
+    for text in (golden(sass),):
+        got = {}
+        for line in orc.run(text, liveness=True).splitlines():
+            if line.startswith("L "):
+                _, k, i, c, a = line.split()
+                got.setdefault(int(k), []).append((int(c), int(a)))
+        assert len(got) == len(want)
+        for k, w in enumerate(want):
+            g = got[k][:len(w)]   # nvdisasm -lrm omits the trailing NOP padding
+            assert len(got[k]) >= len(w)
+            assert [c for c, _ in g] == w, (sass, k)
+            assert [a for _, a in g] == [w[0]] + [w[i] - w[i - 1] for i in range(1, len(w))]

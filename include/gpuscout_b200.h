@@ -178,6 +178,16 @@ gs_status gs_rank_sites(gs_ctx *ctx, const int32_t *d_hist, uint64_t k, gs_ranke
 gs_status gs_rank_sites_slice(gs_ctx *ctx, const int32_t *d_hist, uint64_t slot_begin, uint64_t slot_end,
                               uint64_t k, gs_ranked_site *out, uint64_t *n_out);
 
+/* Register pressure ("the number of additional registers needed by each SASS
+ * instruction"; also P:452): for every instruction of
+ * kernels [k_begin, k_end), the number of general-purpose registers (R0..R254) live at it,
+ * |live_in ∪ defs| by backward dataflow over the kernel's control-flow graph (R36; equal
+ * to nvdisasm's life-range "GPR #" column). d_live is a caller-owned DEVICE array indexed by global
+ * slot (n_instr entries); slots outside the range are left untouched. The additional registers of
+ * instruction i are d_live[i] - d_live[i-1] (the first instruction of a kernel: d_live[i]).
+ * Enqueued on the stream; synchronises once (basic-block count). */
+gs_status gs_register_pressure(gs_ctx *ctx, uint32_t k_begin, uint32_t k_end, uint16_t *d_live);
+
 /* Number of CUDA kernels this library has launched in the process so far (its own kernels plus
  * the CUB radix-sort kernels of gs_rank_sites). Lets a harness count launches in a timed region. */
 uint64_t gs_launch_count(void);

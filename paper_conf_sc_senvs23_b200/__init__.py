@@ -6,8 +6,8 @@ multi-GPU orchestration (dist.py).
 """
 from .binding import (GS_JOIN_LINE, GS_JOIN_PC, GS_HIST_AUTO, GS_HIST_GLOBAL, GS_HIST_PRIVATE, GS_HIST_WINDOW, RANKED_DTYPE, RULES,
                       SITE_DTYPE, Context, GsError, gs_attribute_counts, gs_attribute_samples, gs_detect, gs_load_sass,
-                      gs_pack_samples, gs_rank_sites, gs_rank_sites_slice, load_library)
+                      gs_pack_samples, gs_rank_sites, gs_rank_sites_slice, gs_register_pressure, load_library)
 
 __all__ = ["Context", "GsError", "load_library", "gs_load_sass", "gs_detect", "gs_pack_samples",
-           "gs_attribute_samples", "gs_attribute_counts", "gs_rank_sites", "gs_rank_sites_slice", "SITE_DTYPE", "RANKED_DTYPE", "RULES", "GS_HIST_AUTO",
+           "gs_attribute_samples", "gs_attribute_counts", "gs_rank_sites", "gs_rank_sites_slice", "gs_register_pressure", "SITE_DTYPE", "RANKED_DTYPE", "RULES", "GS_HIST_AUTO",
            "GS_HIST_GLOBAL", "GS_HIST_PRIVATE", "GS_HIST_WINDOW", "GS_JOIN_PC", "GS_JOIN_LINE"]

@@ -46,7 +46,7 @@ class GsError(RuntimeError):
 _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
-           "gs_attribute_samples", "gs_attribute_counts", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
+           "gs_attribute_samples", "gs_attribute_counts", "gs_register_pressure", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
 
 
 def launch_count() -> int:
@@ -78,6 +78,7 @@ def load_library(path: str = LIB_PATH):
         "gs_pack_samples": (I32, [P, P, U64, P, P]),
         "gs_attribute_samples": (I32, [P, P, U64, P, P, I32]),
         "gs_attribute_counts": (I32, [P, P, U64, P, P, I32]),
+        "gs_register_pressure": (I32, [P, U32, U32, P]),
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
         "gs_rank_sites_slice": (I32, [P, P, U64, U64, U64, P, ctypes.POINTER(U64)]),
         "gs_last_hist_mode": (I32, [P]),
@@ -240,6 +241,16 @@ class Context:
                                                n_invalid.data_ptr(), 1 if accumulate else 0), "gs_attribute_counts")
         return hist, n_invalid
 
+    def register_pressure(self, k_begin: int = 0, k_end: int | None = None, out=None):
+        """Live GPRs per instruction (int16 device tensor indexed by slot; kernels outside
+        [k_begin, k_end) untouched). Additional registers of slot i: out[i] - out[i-1]."""
+        import torch
+        k_end = self.n_kernels if k_end is None else k_end
+        if out is None:
+            out = torch.zeros(max(1, self.n_instr), dtype=torch.int16, device=torch.device("cuda", self.device))
+        self._check(self.L.gs_register_pressure(self.h, k_begin, k_end, out.data_ptr()), "gs_register_pressure")
+        return out
+
     def last_hist_mode(self) -> int:
         return self.L.gs_last_hist_mode(self.h)
 
@@ -283,6 +294,10 @@ def gs_attribute_samples(ctx: Context, samples, hist=None, n_invalid=None, accum
 
 def gs_attribute_counts(ctx: Context, recs, hist=None, n_invalid=None, accumulate: bool = False):
     return ctx.attribute_counts(recs, hist, n_invalid, accumulate)
+
+
+def gs_register_pressure(ctx: Context, k_begin: int = 0, k_end: int | None = None, out=None):
+    return ctx.register_pressure(k_begin, k_end, out)
 
 
 def gs_rank_sites(ctx: Context, hist, k: int | None = None, out=None):

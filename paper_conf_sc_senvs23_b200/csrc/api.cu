@@ -37,6 +37,7 @@ void free_loaded(gs_ctx* c) {
   if (c->d_goff) cudaFree(c->d_goff);
   if (c->d_gslot) cudaFree(c->d_gslot);
   c->d_lgrp = c->d_goff = c->d_gslot = nullptr;
+  liveness_free(c);
   c->n_lgroups = 0;
   c->d_rec = nullptr;
   c->d_kd = nullptr;
@@ -126,6 +127,9 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   c->lines_h.clear();
   c->lines_h.reserve(P);
   c->cbase_h.clear();
+  c->use_off_h.assign(1, 0);
+  c->use_reg_h.clear();
+  c->tgt_h.clear();
   c->n_cand = c->n_ldg = c->n_store = 0;
   std::vector<Rec> recs;
   recs.reserve(P);
@@ -153,6 +157,12 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     }
     slot += K.n;
     recs.insert(recs.end(), pk.recs.begin(), pk.recs.end());
+    {  // register-pressure inputs, offsets made global
+      const uint32_t base = (uint32_t)c->use_reg_h.size();
+      for (size_t i = 1; i < pk.use_off.size(); i++) c->use_off_h.push_back(base + pk.use_off[i]);
+      c->use_reg_h.insert(c->use_reg_h.end(), pk.use_reg.begin(), pk.use_reg.end());
+      c->tgt_h.insert(c->tgt_h.end(), pk.tgt.begin(), pk.tgt.end());
+    }
     c->lines_h.insert(c->lines_h.end(), pk.lines.begin(), pk.lines.end());
     c->names.push_back(std::move(pk.name));
   }
@@ -328,6 +338,17 @@ gs_status gs_attribute_counts(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int
   if (n && !is_device_ptr(d_recs)) return fail(c, GS_E_INVAL, "count records must be device memory");
   GS_CUDA(c, cudaSetDevice(c->device));
   return counts_run(c, d_recs, n, d_hist, d_n_invalid, accumulate);
+}
+
+gs_status gs_register_pressure(gs_ctx* c, uint32_t k_begin, uint32_t k_end, uint16_t* d_live) {
+  if (!c) return GS_E_INVAL;
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_register_pressure before gs_load_sass");
+  if (k_begin > k_end || k_end > c->n_kernels) return fail(c, GS_E_INVAL, "bad kernel range");
+  if (!d_live && k_end > k_begin) return fail(c, GS_E_INVAL, "null output");
+  if (d_live && !is_device_ptr(d_live)) return fail(c, GS_E_INVAL, "output must be device memory");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  return liveness_run(c, k_begin, k_end, d_live);
 }
 
 gs_status gs_rank_sites_slice(gs_ctx* c, const int32_t* d_hist, uint64_t slot_begin, uint64_t slot_end, uint64_t k,

@@ -62,6 +62,9 @@ struct gs_ctx {
   std::vector<uint32_t> cbase_h;  // candidate base per window (n_win + 1)
   std::vector<int32_t> lines_h;
   uint32_t n_lgroups = 0;             // source-line groups (kernel, file, line), 0 without line info
+  std::vector<uint32_t> use_off_h;     // register-pressure inputs (R36), uploaded on first use:
+  std::vector<uint8_t> use_reg_h;      //   GPR uses per slot (CSR, global offsets), branch targets
+  std::vector<int32_t> tgt_h;          //   (kernel-local index, -1 none)
 
   // ---- device copies
   gs::Rec* d_rec = nullptr;
@@ -71,6 +74,11 @@ struct gs_ctx {
   uint32_t* d_lgrp = nullptr;   // per slot: its source-line group, ~0u if none (only when n_lgroups)
   uint32_t* d_goff = nullptr;   // group -> first entry of d_gslot (n_lgroups + 1)
   uint32_t* d_gslot = nullptr;  // slots ordered by group
+  uint32_t* d_use_off = nullptr;  // register pressure inputs on the device (lazy)
+  uint8_t* d_use_reg = nullptr;
+  int32_t* d_tgt = nullptr;
+  void* d_lv = nullptr;           // liveness scratch
+  size_t lv_bytes = 0;
 
   // ---- detection scratch
   uint32_t* d_tab = nullptr;  // n_win x 320 last-writer summaries -> carry-in tables
@@ -174,6 +182,8 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
 gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k, gs_ranked_site* out,
                    bool out_is_host, uint64_t* n_out);
 void attrib_free(gs_ctx* c);
+gs_status liveness_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint16_t* d_live);
+void liveness_free(gs_ctx* c);
 void rank_free(gs_ctx* c);
 
 // device-wide exclusive scan of u32 counts into u32 or u64 offsets; total written to *d_total

@@ -109,6 +109,8 @@ struct Operand {
   int base = -1;             // T_MEM base register
   int regs[8];               // all registers inside (brackets too), in order
   int nregs = 0;
+  bool wide = false;         // T_MEM: base written Rb.64
+  bool predvar = false;      // T_PRED: a real predicate (not PT / UPT)
   void add(int r) { if (nregs < 8) regs[nregs++] = r; }
 };
 
@@ -163,7 +165,10 @@ Operand classify(Sv raw) {
       size_t c = i;
       while (c < u.n && u[c] != ']') c++;
       long long dummy = 0;
-      if (i == lb) scan_bracket(Sv{u.p + i + 1, c - i - 1}, &o, true, &o.imm);
+      if (i == lb) {
+        scan_bracket(Sv{u.p + i + 1, c - i - 1}, &o, true, &o.imm);
+        o.wide = contains(Sv{u.p + i + 1, c - i - 1}, ".64");
+      }
       else scan_bracket(Sv{u.p + i + 1, c - i - 1}, &o, false, &dummy);
       i = c + 1;
     }
@@ -171,7 +176,11 @@ Operand classify(Sv raw) {
   }
   int r = reg_id(u);
   if (r >= 0) { o.k = T_REG; o.reg = r; o.add(r); return o; }
-  if (is_pred(u)) { o.k = T_PRED; return o; }
+  if (is_pred(u)) {
+    o.k = T_PRED;
+    o.predvar = u[u.n - 1] != 'T';
+    return o;
+  }
   o.k = T_MISC;  // immediates, floats, SR_*, B0, PR, ...
   return o;
 }
@@ -206,10 +215,27 @@ struct Line {
   long lineno;
 };
 
+// Register-pressure inputs of one instruction (O16 / R36): GPR uses with operand widths expanded,
+// guard, exit, predicate operand of a branch, branch target (pc) or unresolved label.
+struct LiveOut {
+  std::vector<uint8_t>* uses = nullptr;
+  bool guarded = false, exit = false, brpred = false;
+  long long target = -1;
+  std::string label;
+};
+
+inline bool is64type(Sv m) { return m.eq("F64") || m.eq("S64") || m.eq("U64"); }
+inline bool istype(Sv m) {
+  static const char* k[] = {"F64", "S64", "U64", "F32", "F16", "BF16", "S32", "U32", "S16", "U16", "S8", "U8", "TF32"};
+  for (auto* x : k) if (m.eq(x)) return true;
+  return false;
+}
+
 // One instruction -> record. Returns false with msg on a malformed line.
-bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg) {
+bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, LiveOut* lo) {
   body = trim(body);
   if (body.n && body[0] == '@') {  // guard predicate
+    lo->guarded = !starts(body, "@PT") && !starts(body, "@UPT");
     size_t i = 0;
     while (i < body.n && !is_ws(body[i])) i++;
     body = trim(Sv{body.p + i, body.n - i});
@@ -353,6 +379,49 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg) {
       }
     }
   }
+  // register-pressure inputs (R36)
+  lo->exit = mn.eq("EXIT") || mn.eq("RET");
+  if (op == OP_BRA) {
+    for (int q = 0; q + 1 < no; q++) lo->brpred |= ops[q].k == T_PRED && ops[q].predvar;
+    long long t;
+    Sv lt = trim(raw_last);
+    if (no > 0 && to_int(lt, &t)) lo->target = t;
+    else if (lt.n > 4 && lt[0] == '`' && lt[1] == '(' && lt[lt.n - 1] == ')') lo->label.assign(lt.p + 2, lt.n - 3);
+  }
+  {
+    int srcw = (op == OP_DADD || op == OP_DMUL || op == OP_DFMA || op == OP_DMNMX || mn.eq("DSETP")) ? 2 : 1;
+    if (cls & C_CONV) {
+      int nt = 0;
+      for (int q = 0; q < nm; q++)
+        if (istype(mods[q]) && nt++ == 1 && is64type(mods[q])) srcw = 2;  // second type = source
+    }
+    const bool store_like = op == OP_STG || op == OP_STS || op == OP_STL || op == OP_ST || op == OP_RED ||
+                            op == OP_REDG || op == OP_ATOMG || op == OP_ATOM || op == OP_ATOMS;
+    int dataw = 1;
+    for (int q = 0; q < nm; q++) if (mods[q].eq("64") || is64type(mods[q])) dataw = 2;
+    for (int q = 0; q < nm; q++) if (mods[q].eq("128")) dataw = 4;
+    const bool ext = has("E"), wide_imad = op == OP_IMAD && has("WIDE");
+    int srcidx = 0;
+    for (int q = 0; q < no; q++) {
+      if (q == dpos) continue;
+      const Operand& o = ops[q];
+      for (int t = 0; t < o.nregs; t++) {
+        const int r = o.regs[t];
+        if (r < 0 || r >= 255) continue;  // RZ and uniform registers
+        int w;
+        if (o.k == T_MEM) w = (r == o.base && (o.wide || ext)) ? 2 : 1;
+        else if (o.k == T_CREF) w = 1;
+        else if (store_like && q > 0) w = dataw;
+        else if (wide_imad && srcidx == 2) w = 2;
+        else w = srcw;
+        for (int k2 = 0; k2 < w && r + k2 < 255; k2++) lo->uses->push_back((uint8_t)(r + k2));
+      }
+      if (q > dpos && o.k != T_PRED) srcidx++;
+    }
+  }
+  if (lo->guarded) flags |= F_PRED;
+  if (lo->exit) flags |= F_EXIT;
+  if (lo->brpred) flags |= F_BRPRED;
   if (cbank > 31) { *msg = "constant bank > 31"; return false; }
   *out = make_rec(op, flags, aw, dstw, pk, cbank, dst, ptr, s[0], s[1], s[2], s[3], imm);
   (void)lineno;
@@ -383,6 +452,8 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
   std::map<std::pair<std::string, int32_t>, int32_t> lkey;  // (file, line) -> kernel-local key
   std::map<std::string, long long> labels;                  // branch label -> pc
   std::vector<std::string> pending;
+  std::vector<std::pair<size_t, std::string>> fwd;          // branches to labels not seen yet
+  pk->use_off.assign(1, 0);
   size_t p = seg.begin;
   while (p < seg.end) {
     const char* nl = (const char*)memchr(text + p, '\n', seg.end - p);
@@ -443,10 +514,15 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     }
     Rec r;
     std::string msg;
-    if (!pack_line(ins, cur, pk->recs.size(), &r, &msg)) {
+    LiveOut lo;
+    lo.uses = &pk->use_reg;
+    if (!pack_line(ins, cur, pk->recs.size(), &r, &msg, &lo)) {
       *err = "line " + std::to_string(cur) + ": " + msg;
       return false;
     }
+    pk->use_off.push_back((uint32_t)pk->use_reg.size());
+    pk->tgt.push_back(lo.target >= 0 && lo.target % 16 == 0 ? (int32_t)(lo.target / 16) : -1);
+    if (lo.target < 0 && !lo.label.empty()) fwd.emplace_back(pk->recs.size(), lo.label);
     pk->recs.push_back(r);
     pk->lines.push_back(src_line);
     int32_t key = -1;
@@ -457,6 +533,11 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     pk->lkeys.push_back(key);
   }
   pk->n_lkeys = (uint32_t)lkey.size();
+  for (auto& pl : pending) labels[pl] = 16LL * (long long)pk->recs.size();  // labels after the last instruction
+  for (auto& f : fwd) {  // forward label targets (backward ones were substituted in place)
+    auto it = labels.find(f.second);
+    if (it != labels.end()) pk->tgt[f.first] = (int32_t)(it->second / 16);
+  }
   return true;
 }
 

@@ -14,6 +14,11 @@ struct ParsedKernel {
   std::vector<int32_t> lines;  // source line per instruction, -1 if unknown
   std::vector<int32_t> lkeys;  // source-line key per instruction: kernel-local id of (file, line), -1 if unknown
   uint32_t n_lkeys = 0;
+  // register-pressure inputs (R36): GPR uses per instruction (CSR, widths expanded) and branch
+  // targets (kernel-local instruction index, -1 if none / unresolved)
+  std::vector<uint32_t> use_off;  // n + 1
+  std::vector<uint8_t> use_reg;
+  std::vector<int32_t> tgt;
 };
 
 // Parses cuobjdump -sass / nvdisasm [-g] text into per-kernel packed records using up to n_threads threads.

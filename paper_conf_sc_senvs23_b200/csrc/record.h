@@ -83,7 +83,12 @@ GS_HD uint32_t op_class(uint32_t op) {
 }
 
 // flags
-enum : uint32_t { F_CONSTANT = 1, F_HASMEM = 2, F_BRA_OK = 4 };
+enum : uint32_t {
+  F_CONSTANT = 1, F_HASMEM = 2, F_BRA_OK = 4,
+  F_PRED = 8,     // guarded by a predicate other than PT (kills no register, R36)
+  F_EXIT = 16,    // EXIT / RET
+  F_BRPRED = 32,  // BRA with a predicate operand (conditional, e.g. BRA.U !UP0)
+};
 // access width codes
 enum : uint32_t { AW_NONE = 0, AW_8 = 1, AW_16 = 2, AW_32 = 3, AW_64 = 4, AW_128 = 5 };
 // pointer-operand kinds

@@ -331,3 +331,59 @@ def test_parse_error_reported(gs):
     ctx = _ctx(gs)
     with pytest.raises(gs.GsError, match="line 3"):
         ctx.load_sass("\t\tFunction : x\n        /*0000*/ NOP ;\n        /*0020*/ NOP ;\n")
+
+
+# ------------------------------------------------------------------------------ register pressure
+def _oracle_live(text, kb=0, ke=-1):
+    out = {}
+    for line in orc.run(text, liveness=True, kbegin=kb, kend=ke).splitlines():
+        if line.startswith("L "):
+            _, k, i, c, _a = line.split()
+            out[(int(k), int(i))] = int(c)
+    return out
+
+
+def _gpu_live(gs, text, kb=0, ke=None):
+    import torch
+    ctx = _ctx(gs)
+    ctx.load_sass(text)
+    first, n = ctx.kernel_table()
+    ke = ctx.n_kernels if ke is None else ke
+    live = ctx.register_pressure(kb, ke, out=torch.full((max(1, ctx.n_instr),), -1, dtype=torch.int16,
+                                                        device="cuda")).cpu().numpy()
+    got = {(k, i): int(live[first[k] + i]) for k in range(kb, ke) for i in range(int(n[k]))}
+    untouched = all(int(live[first[k] + i]) == -1 for k in range(ctx.n_kernels) if not kb <= k < ke
+                    for i in range(int(n[k])))
+    return got, untouched
+
+
+LIVE_TEXTS = ["lineinfo/sgemm_naive.nvdisasm.sass", "lineinfo/mixbench.nvdisasm.sass", "lineinfo/atomics.cuobjdump.sass",
+              "lineinfo/spill.nvdisasm.sass", "jacobi.sm_70.sass", "sgemm_naive.sm_70.sass", "conv.sm_100a.sass",
+              "spill.r24.sm_100a.sass", "listing1.sass"]
+
+
+@pytest.mark.parametrize("name", LIVE_TEXTS)
+def test_register_pressure_parity_fixtures(gs, name):
+    """gs_register_pressure against the oracle's O16 (itself pinned to nvdisasm's life ranges)."""
+    text = _read(name)
+    got, _ = _gpu_live(gs, text)
+    assert got == _oracle_live(text)
+
+
+def test_register_pressure_parity_generated(gs):
+    """Generated multi-kernel SASS (loops, spills, conversions) and random branchy streams; a
+    kernel range leaves the other kernels untouched."""
+    from gen import sass as gsass
+    for cfg, scale in (("C1", 1.0), ("C2", 1.0), ("C3", 0.002), ("C5", 0.01)):
+        s = gsass.config_sass(cfg, scale=scale) if cfg in ("C3", "C5") else gsass.config_sass(cfg)
+        got, _ = _gpu_live(gs, s.text)
+        assert got == _oracle_live(s.text), cfg
+    s = gsass.config_sass("C2")
+    got, untouched = _gpu_live(gs, s.text, 1, 2)
+    assert untouched and got == _oracle_live(s.text, 1, 2)
+    rng = random.Random(17)
+    for _ in range(40):
+        ks = [brute.random_stream(rng, rng.randint(1, 6)) for _ in range(rng.randint(1, 4))]
+        text = brute.render(ks)
+        got, _ = _gpu_live(gs, text)
+        assert got == _oracle_live(text)

@@ -36,14 +36,25 @@ namespace gs {
 namespace {
 
 constexpr int kThreadsGlobal = 512;
-constexpr int kThreads = 1024;
-constexpr uint32_t kTableWords = 56 * 1024 - 32;   // + 32 spare words (one per lane) = 224 KB
-constexpr uint32_t kMaxRanges = 3;
-#ifndef GS_TILE4
-#define GS_TILE4 16384
+#ifndef GS_HIST_THREADS
+#define GS_HIST_THREADS 1024
 #endif
-constexpr uint32_t kTile4 = GS_TILE4;              // uint4 per WINDOW tile (64K samples)
-constexpr int kVec = 4;                            // 128-bit loads in flight per thread
+#ifndef GS_KVEC
+#define GS_KVEC 8
+#endif
+constexpr int kThreads = GS_HIST_THREADS;
+#ifndef GS_TABLE_WORDS
+#define GS_TABLE_WORDS (56 * 1024 - 32)
+#endif
+constexpr uint32_t kTableWords = GS_TABLE_WORDS;   // + 32 spare words (one per lane) = 224 KB
+constexpr uint32_t kMaxRanges = 3;
+constexpr uint32_t kMinTableWords = 8192;          // smallest WINDOW table (32 KB)
+#ifndef GS_TILE4
+#define GS_TILE4 (4 * GS_KVEC * (GS_HIST_THREADS - 32))
+#endif
+constexpr uint32_t kTile4 = GS_TILE4;              // uint4 per WINDOW tile: 4 batches of the counters
+
+constexpr int kVec = GS_KVEC;                          // 128-bit loads in flight per thread
 constexpr uint32_t kNoWindow = 0xffffffffu;
 
 // x / d for x < 2^32, 1 <= d <= 32: floor(x * ceil(2^40 / d) / 2^40) (error < 2^37 / 2^40 < 1/d);
@@ -414,6 +425,80 @@ __device__ __forceinline__ void count_ring(const uint32_t* ring, uint32_t b, uin
   }
 }
 
+// ---------------------------------------------------------------------- WINDOW counting loop
+// The hot loop keeps only the stream position, the window and the table live: everything the rare
+// path needs (deferral ring, histogram, divisor) is read from shared memory / re-loaded inside the
+// out-of-line rare_w, so that ptxas can issue all kVec 128-bit loads of a batch before its first
+// atomic (with the rare state live, it delayed the last load behind the atomics, exposing the HBM
+// latency twice per batch).
+constexpr uint32_t kNct = kThreads - 32;  // counting threads of the WINDOW kernel
+
+// the rare part of one batch of nv uint4 at s4[i + u * kNct], re-read from L1/L2: outside the
+// window (deferred / invalid), or a 16-bit half that needs draining. Returns the invalid count.
+template <bool P16>
+__device__ __noinline__ uint32_t rare_w(const uint4* __restrict__ s4, uint64_t i, uint32_t nv, Win W, uint32_t* tab,
+                                        uint32_t flag, uint32_t am, const Spill* sS) {
+  const Spill S = *sS;
+  uint32_t bad = 0;
+  for (uint32_t u = 0; u < nv; u++) {
+    const uint4 v = __ldg(s4 + i + (uint64_t)u * kNct);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      const uint32_t off = w[q] - W.wb;
+      out_of_window<OUT_DEFER>(am, off >= W.lim, w[q], S, bad);
+      if (P16 && flag && off < W.lim && ((tab[off >> 1] >> ((off & 1u) << 4)) & 0x8000u))
+        drain16(tab, off >> 1, (off & 1u) << 4, w[q], S.dv, S.H);
+    }
+  }
+  return bad;
+}
+
+// per-sample fast path of one batch; returns the lane's flag (nonzero: rare work in this batch)
+template <bool P16, int N>
+__device__ __forceinline__ uint32_t hot_w(const uint32_t (&w)[N], Win W, uint32_t* tab, uint32_t spare) {
+  uint32_t flag = 0;
+#pragma unroll
+  for (int q = 0; q < N; q++) {
+    const uint32_t off = w[q] - W.wb;
+    const bool in = off < W.lim;
+    if (P16) {
+      const uint32_t inc = 1u << ((off & 1u) << 4);
+      flag |= atomicAdd(tab + (in ? off >> 1 : spare), inc) & (in ? inc << 15 : 0xffffffffu);
+    } else {
+      atomicAdd(tab + (in ? off : spare), 1u);
+      flag |= in ? 0u : 1u;
+    }
+  }
+  return flag;
+}
+
+template <bool P16>
+__device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, uint64_t i0, uint64_t i1, uint32_t ct,
+                                                 Win W, uint32_t* tab, uint32_t spare, const Spill* sS) {
+  uint32_t bad = 0;
+  uint64_t i = i0 + ct;
+  for (; i + (kVec - 1) * kNct < i1; i += kVec * kNct) {
+    uint32_t w[4 * kVec];
+#pragma unroll
+    for (int u = 0; u < kVec; u++) {
+      const uint4 v = __ldg(s4 + i + u * kNct);
+      w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
+    }
+    const uint32_t flag = hot_w<P16>(w, W, tab, spare);
+    const uint32_t am = __activemask();
+    if (__any_sync(am, flag)) bad += rare_w<P16>(s4, i, kVec, W, tab, flag, am, sS);
+  }
+  for (; i < i1; i += kNct) {
+    const uint4 v = __ldg(s4 + i);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+    const uint32_t flag = hot_w<P16>(w, W, tab, spare);
+    const uint32_t am = __activemask();
+    if (__any_sync(am, flag)) bad += rare_w<P16>(s4, i, 1, W, tab, flag, am, sS);
+  }
+  return bad;
+}
+
 // ---------------------------------------------------------------------- PRIVATE
 // fixed slot range per CTA (range = blockIdx % n_ranges); the CTA walks its sample chunk
 template <bool P16>
@@ -461,6 +546,23 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {  // 
       "r"(parity)
       : "memory");
 }
+// the producer's wait for a free item slot: back off between polls so that the spinning warp
+// does not take shared-memory cycles from the counters' atomics
+__device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity) {
+  uint32_t ok = 0;
+  for (;;) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    if (ok) return;
+#ifndef GS_BACKOFF_NS
+#define GS_BACKOFF_NS 500
+#endif
+    if (GS_BACKOFF_NS) __nanosleep(GS_BACKOFF_NS);
+  }
+}
 // the 31 counting warps only (warp 0 keeps producing)
 __device__ __forceinline__ void bar_counters() { asm volatile("bar.sync 1, %0;" ::"r"(kThreads - 32) : "memory"); }
 
@@ -491,15 +593,17 @@ template <bool P16>
 __global__ void __launch_bounds__(kThreads, 1)
     k_hist_window(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv,
                   const KDesc* __restrict__ kd, uint32_t nk, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
-                  unsigned long long* d_n_invalid, unsigned long long* rng, uint32_t* __restrict__ defer_ring) {
-  extern __shared__ uint32_t tab[];
+                  unsigned long long* d_n_invalid, unsigned long long* rng, uint32_t* __restrict__ defer_ring,
+                  uint32_t tw) {
+  extern __shared__ uint32_t tab[];  // tw counter words + 32 spare words
   __shared__ Item items[kItems];
   __shared__ __align__(8) uint64_t full[kItems], empty[kItems];
   __shared__ uint32_t sh_ndefer[2];
+  __shared__ Spill sh_S;  // the counters' rare-path state (written at window switches)
   const uint32_t pnr = P * nr;
-  const uint32_t nslots = (P16 ? 2 * kTableWords : kTableWords) / nr;
+  const uint32_t nslots = (P16 ? 2 * tw : tw) / nr;
   const uint32_t lane = threadIdx.x & 31u;
-  for (uint32_t i = threadIdx.x; i < kTableWords + 32; i += blockDim.x) tab[i] = i < kTableWords ? 0u : 1u;
+  for (uint32_t i = threadIdx.x; i < tw + 32; i += blockDim.x) tab[i] = i < tw ? 0u : 1u;
   if (threadIdx.x < kItems) {
     mbar_init(&full[threadIdx.x], 1);
     mbar_init(&empty[threadIdx.x], kThreads / 32 - 1);
@@ -520,7 +624,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const auto publish = [&](uint64_t a4, uint64_t b4, uint32_t ws, uint32_t last) {
       const uint32_t k = j % kItems;
       if (lane == 0) {
-        mbar_wait(&empty[k], ((j / kItems) & 1u) ^ 1u);
+        mbar_wait_backoff(&empty[k], ((j / kItems) & 1u) ^ 1u);
         items[k] = Item{a4, b4, ws, last};
         mbar_arrive(&full[k]);
       }
@@ -574,15 +678,23 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   // --------------------------------------------------------------------------- counters
   const uint32_t ct = threadIdx.x - 32, nct = kThreads - 32;
-  const uint32_t spare = kTableWords + lane;
+  const uint32_t spare = tw + lane;
   const uint4* s4 = reinterpret_cast<const uint4*>(s);
   uint32_t* const ring0 = defer_ring + (uint64_t)blockIdx.x * 2 * kDeferCap;
   uint32_t bad = 0, ws = kNoWindow, epoch = 0, dstart0 = 0, dstart1 = 0;
   Win W{0, 0};
   Spill S{pnr, dv, H, &sh_ndefer[0], ring0, 0};
+#if defined(GS_DIAG) && GS_DIAG == 11  // diagnostic: per-CTA timeline (printf)
+  long long d_t0 = clock64(), d_wait = 0, d_flush = 0, d_ring = 0, d_count = 0;
+  uint32_t d_sw = 0, d_items = 0;
+  uint64_t d_words = 0;
+#define GS_T(acc, ...) { const long long _a = clock64(); __VA_ARGS__; acc += clock64() - _a; }
+#else
+#define GS_T(acc, ...) { __VA_ARGS__; }
+#endif
   for (uint32_t j = 0;; j++) {
     const uint32_t k = j % kItems;
-    mbar_wait(&full[k], (j / kItems) & 1u);
+    GS_T(d_wait, mbar_wait(&full[k], (j / kItems) & 1u));
     const Item it = items[k];
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[k]);
@@ -594,15 +706,17 @@ __global__ void __launch_bounds__(kThreads, 1)
 #if defined(GS_DIAG) && GS_DIAG == 9  // diagnostic: n_invalid counts window switches
       if (ct == 0) atomicAdd(d_n_invalid, 1ull);
 #endif
-      bar_counters();
-      if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
-      bar_counters();
+      GS_T(d_flush, bar_counters(); if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
+           bar_counters());
+#if defined(GS_DIAG) && GS_DIAG == 11
+      d_sw++;
+#endif
       ws = it.ws;
       W = Win{ws * nr, min(nslots, P - min(P, ws)) * nr};
       if (ws != kNoWindow && j) {  // the ended epoch's deferred samples, against the new window
         const uint32_t h = epoch & 1u, dend = sh_ndefer[h], db = h ? dstart1 : dstart0;
         if (dend != db)  // positions past the capacity went to L2 when they were deferred
-          count_ring<P16>(ring0 + h * kDeferCap, db, min(dend - db, kDeferCap), W, tab, spare, one, S, bad, ct, nct);
+          GS_T(d_ring, count_ring<P16>(ring0 + h * kDeferCap, db, min(dend - db, kDeferCap), W, tab, spare, one, S, bad, ct, nct));
         if (h) dstart1 = dend;
         else dstart0 = dend;
         epoch++;
@@ -611,8 +725,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       S.cnt = &sh_ndefer[h];
       S.ring = ring0 + h * kDeferCap;
       S.base = h ? dstart1 : dstart0;
+      if (ct == 0) sh_S = S;
+      bar_counters();
     }
-    count_span<OUT_DEFER, P16>(s4, it.a4, it.b4, ct, nct, W, tab, spare, one, S, bad);
+    GS_T(d_count, bad += count_span_w<P16>(s4, it.a4, it.b4, ct, W, tab, spare, &sh_S));
+#if defined(GS_DIAG) && GS_DIAG == 11
+    d_items++;
+    d_words += 4 * (it.b4 - it.a4);
+#endif
   }
   bar_counters();
   {  // the last epoch's deferred samples: what is not in the current window goes to L2
@@ -627,8 +747,18 @@ __global__ void __launch_bounds__(kThreads, 1)
       else bad++;
     }
   count_invalid(bad, d_n_invalid);
+  long long d_f0 = clock64();
   bar_counters();
   if (ws != kNoWindow) flush<P16>(tab, ws, nr, dv.row, W.lim, H, ct, nct);
+#if defined(GS_DIAG) && GS_DIAG == 11
+  bar_counters();
+  if (ct == 0)
+    printf("DIAG11 cta %u sm_clk total %lld wait %lld flush %lld ring %lld count %lld final_flush %lld switches %u items %u words %llu\n",
+           blockIdx.x, clock64() - d_t0, d_wait, d_flush, d_ring, d_count, clock64() - d_f0, d_sw, d_items,
+           (unsigned long long)d_words);
+#else
+  (void)d_f0;
+#endif
 }
 
 }  // namespace
@@ -703,11 +833,20 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
-  const size_t smem = (size_t)(kTableWords + 32) * 4;
   const bool dyn = mode == GS_HIST_WINDOW;
+  // WINDOW: a table just large enough for the largest kernel (+1 slot for the even window base).
+  // The rest of the SM's 256 KB stays L1, which stages the counters' in-flight 128-bit loads: with
+  // a 224-KB table the L1 (~28 KB) capped the loads in flight and the pass ran 30% slower.
+  uint32_t tw = kTableWords;
+  if (dyn) {
+    const uint64_t need = bits == 16 ? ((uint64_t)(max_kn + 1) * nr + 1) / 2 : (uint64_t)(max_kn + 1) * nr;
+    tw = (uint32_t)std::min<uint64_t>(kTableWords, (std::max<uint64_t>(need, kMinTableWords) + 31) & ~31ull);
+  }
+  c->last_hist_table_words = tw;
+  const size_t smem = (size_t)(tw + 32) * 4;
   uint64_t chunks;
   if (dyn) {
-    chunks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms, n / (2ull * kTableWords) + 1));
+    chunks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms, n / (2ull * tw) + 1));
   } else {
     chunks = std::max<uint64_t>(1, (uint64_t)dev_sms / n_ranges);
     chunks = std::min<uint64_t>(chunks, std::max<uint64_t>(1, n / (2ull * kTableWords)));
@@ -730,7 +869,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     ls = prep(kern);
     if (ls == GS_OK)
       kern<<<(uint32_t)chunks, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, chunk, 1u, d_hist,
-                                                     d_n_invalid, c->d_tileq, c->d_defer);
+                                                     d_n_invalid, c->d_tileq, c->d_defer, tw);
   } else {
     const auto kern = bits == 16 ? k_hist_smem<true> : k_hist_smem<false>;
     ls = prep(kern);

@@ -108,6 +108,7 @@ struct gs_ctx {
 
   // ---- attribution / ranking scratch
   int last_hist_mode = 0, last_hist_bits = 0;
+  uint32_t last_hist_table_words = 0;  // WINDOW table size of the last histogram launch
   unsigned long long* d_tileq = nullptr;  // WINDOW histogram work-stealing queue
   uint64_t tileq_cap = 0;
   uint32_t* d_defer = nullptr;  // WINDOW histogram: per-CTA rings of deferred (out-of-window) samples

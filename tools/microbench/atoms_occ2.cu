@@ -1,3 +1,6 @@
+#ifndef NLOG
+#define NLOG 28
+#endif
 // Microbenchmark: shared-memory atomic counting rate on a C4-shaped stream (2^28 words, 1 GB >
 // L2): 80% of samples on a hot 10% of a 77824-bin window, 20% uniform. Compares
 //   A  1 CTA x 1024 thr / SM, 16-bit pairs (38912 words), returning atomics + flag vote, 16 samples/thread batch
@@ -93,12 +96,12 @@ __global__ void __launch_bounds__(1024, 1) k_h2(const uint4* __restrict__ s, uin
   }
   __syncthreads(); if(threadIdx.x==0) out[blockIdx.x]=t[5]+acc;
 }
-int main(){
-  const uint64_t n=1ull<<28; uint32_t *s,*o; CK(cudaMalloc(&s,n*4)); CK(cudaMalloc(&o,4096*4));
-  k_gen<<<1184,512>>>(s,n,77824); CK(cudaDeviceSynchronize());
+int main(){ setvbuf(stdout, NULL, _IONBF, 0); printf("start\n");
+  const uint64_t n=1ull<<NLOG; uint32_t *s,*o; CK(cudaMalloc(&s,n*4)); CK(cudaMalloc(&o,4096*4));
+  k_gen<<<1184,512>>>(s,n,77824); CK(cudaDeviceSynchronize()); printf("gen done\n");
   cudaEvent_t a,b; cudaEventCreate(&a); cudaEventCreate(&b);
   auto timeit=[&](const char* nm, auto f){ for(int w=0;w<2;w++) f(); CK(cudaGetLastError()); cudaEventRecord(a); for(int r=0;r<10;r++) f(); cudaEventRecord(b); cudaEventSynchronize(b);
-     float ms; cudaEventElapsedTime(&ms,a,b); ms/=10; printf("%-58s %8.3f ms %8.1f Gsamp/s  (x4 = %.3f ms for 2^30)\n",nm,ms,n/ms/1e6, 4*ms); return 0; };
+     float ms; cudaEventElapsedTime(&ms,a,b); ms/=10; printf("%-58s %8.3f ms %8.1f Gsamp/s  (x%d = %.3f ms for 2^30)\n",nm,ms,n/ms/1e6, (int)((1ull<<30)/n), ((1ull<<30)/n)*ms); return 0; };
   #define RUN(NM, BITS, RET, V, CPS) { auto k=k_h<BITS,RET,V>; size_t sm=(77824/(32/BITS)+32)*4; \
     CK(cudaFuncSetAttribute(k,cudaFuncAttributeMaxDynamicSharedMemorySize,(int)sm)); int occ=0; \
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ,k,1024,sm); cudaFuncAttributes fa; cudaFuncGetAttributes(&fa,k); \

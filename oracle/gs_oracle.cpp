@@ -850,7 +850,7 @@ int main(int argc, char** argv) {
     if (s == "--sass") sass_path = nxt();
     else if (s == "--samples") samples_path = nxt();
     else if (s == "--counts") counts_path = nxt();  // CountRec records, added to the same histogram
-    else if (s == "--join") join = nxt();            // pc (default) | line
+    else if (s == "--join") join = nxt();            // pc (default) | line | consumer
     else if (s == "--out") out_path = nxt();
     else if (s == "--D") C.D = atoi(nxt().c_str());
     else if (s == "--R") C.R = atoi(nxt().c_str());
@@ -866,7 +866,7 @@ int main(int argc, char** argv) {
     else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
     else { fprintf(stderr, "unknown arg %s\n", s.c_str()); return 2; }
   }
-  if (join != "pc" && join != "line") { fprintf(stderr, "unknown join %s\n", join.c_str()); return 2; }
+  if (join != "pc" && join != "line" && join != "consumer") { fprintf(stderr, "unknown join %s\n", join.c_str()); return 2; }
   auto now = [] { return std::chrono::steady_clock::now(); };
   auto secs = [](auto a, auto b) { return std::chrono::duration<double>(b - a).count(); };
   FILE* f = fopen(sass_path.c_str(), "rb");
@@ -975,10 +975,39 @@ int main(int argc, char** argv) {
     // join=line -> the sum of the rows of every instruction of the kernel on the same source line
     // (file, line) as the site ("stall reasons ... at the line numbers identified"), or
     // the site PC's row when the site has no line information.
+    // join=consumer (R37, [probe 9]: scoreboard stalls are sampled at the
+    // instruction waiting for the data, not at its producer): the site PC's row plus the rows of
+    // its direct consumers, the instructions j of the kernel that read a GPR (uses as in O16,
+    // pairs expanded) whose last writer before j (linear order, predicated writes count, as O3)
+    // is the site instruction. Each consumer counts once.
+    std::map<int, std::vector<std::vector<int>>> consumers;
+    auto consumers_of = [&](int k) -> const std::vector<std::vector<int>>& {
+      auto it = consumers.find(k);
+      if (it != consumers.end()) return it->second;
+      const Kernel& K = ks[k];
+      std::vector<std::vector<int>> cons(K.ins.size());
+      std::vector<int> lw(255, -1);  // last writer of R0..R254 so far
+      for (size_t j = 0; j < K.ins.size(); j++) {
+        const Instr& J = K.ins[j];
+        std::set<int> defs;
+        for (int r : gpr_uses(J))
+          if (lw[r] >= 0) defs.insert(lw[r]);
+        for (int d : defs) cons[d].push_back((int)j);
+        if (J.dst != kNoReg && J.dst < 255)
+          for (int w = 0; w < J.dst_w && J.dst + w < 255; w++) lw[J.dst + w] = (int)j;
+      }
+      return consumers.emplace(k, std::move(cons)).first->second;
+    };
     auto site_row = [&](const Site& s) {
       std::vector<uint64_t> row(32, 0);
       const Kernel& K = ks[s.k];
       const Instr& I = K.ins[s.idx];
+      if (join == "consumer") {
+        for (int r = 0; r < 32; r++) row[r] = H[(K.first_slot + s.idx) * 32 + r];
+        for (int j : consumers_of(s.k)[s.idx])
+          for (int r = 0; r < 32; r++) row[r] += H[(K.first_slot + j) * 32 + r];
+        return row;
+      }
       if (join == "pc" || I.line < 0) {
         for (int r = 0; r < 32; r++) row[r] = H[(K.first_slot + s.idx) * 32 + r];
         return row;

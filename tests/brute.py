@@ -254,3 +254,29 @@ def detect(kernels: list[list[Ins]], D=64, TA=1, TL=2):
                 ch = ",".join(map(str, chain)) if chain else "-"
                 slines.append(f"S {k} {i} {rule} line=- ld={ld} term={term} d={len(chain)} chain={ch}{attrs}")
     return klines, slines
+
+
+# ----------------------------------------------------------------------------- consumer join (R37)
+def gpr_uses(x: Ins) -> set:
+    """GPRs the instruction reads, register pairs expanded (O16 / R36 for this grammar): the
+    64-bit memory bases rendered ``[Rb.64]`` (LDG, STG, REDG) and the addend of IMAD.WIDE are
+    pairs; every other operand is one register."""
+    u = set()
+    for q, (k, v) in enumerate(x.srcs):
+        if k == "R" and v != 255:
+            u.add(v)
+            if fam(x) == "IMAD" and q == 2:
+                u.add(v + 1)
+    if x.base is not None:
+        u.add(x.base)
+        if fam(x) in ("LDG", "STG", "REDG"):
+            u.add(x.base + 1)
+    if x.data is not None:
+        u.add(x.data)
+    return u
+
+
+def consumers(ins, i):
+    """Instructions j > i reading a register whose last writer before j is i (brute force)."""
+    return [j for j in range(i + 1, len(ins))
+            if any(last_writer(ins, j, r) == i for r in gpr_uses(ins[j]))]

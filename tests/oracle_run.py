@@ -24,7 +24,7 @@ def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, k
         detect=True, hist=True, timing=False, counts: np.ndarray | None = None, join: str = "pc",
         liveness: bool = False) -> str:
     """sass: path or text/bytes. samples: [N,3] uint32 raw triples. counts: [M,4] uint32
-    pre-aggregated (kernel, pc, reason, count) records. join: pc | line. Returns canonical text."""
+    pre-aggregated (kernel, pc, reason, count) records. join: pc | line | consumer. Returns canonical text."""
     build_oracle()
     tmp = []
     try:

@@ -370,6 +370,87 @@ def test_line_join_closed_form():
     assert Canon(orc.run(plain, samples=raw, join="line")).R == Canon(orc.run(plain, samples=raw)).R
 
 
+def _ranked_rows(c):
+    got = {}
+    for r in c.R:
+        f = r.split()
+        kv = dict(x.split("=") for x in f[5:])
+        got[(int(f[2]), int(f[3]), f[4])] = kv
+    return got
+
+
+REL_SETS = {"VEC": [6], "SPILL": [5, 6], "SHMEM": [6], "GATOM": [5], "RO": [6], "TEX": [6, 16],
+            "CONV": list(range(32))}
+
+
+def test_consumer_join_brute_force():
+    """join=consumer (R37): a site's row is its PC row plus the rows of the
+    instructions that read a register it wrote (last writer = the site). Checked against an O(n^3)
+    brute force on random tiny streams (tests/brute.py: backward rescans, its own register-use
+    rules) with random count tables."""
+    from gen import samples as gs
+    rng = random.Random(37)
+    nrng = np.random.default_rng(37)
+    checked = 0
+    for _ in range(150):
+        ks = [brute.random_stream(rng, rng.randint(2, 7)) for _ in range(rng.randint(1, 2))]
+        n_instr = [len(k) for k in ks]
+        first = list(np.cumsum([0] + n_instr[:-1]))
+        tab = np.zeros((sum(n_instr), 32), np.int64)
+        tab[:, :19] = nrng.integers(0, 9, (sum(n_instr), 19))
+        if tab.sum() == 0:
+            continue
+        raw = gs.Trace(tab, first, n_instr, order="shuffled", seed=rng.randrange(1000)).raw()
+        text = brute.render(ks)
+        pc = Canon(orc.run(text, samples=raw))
+        cs = Canon(orc.run(text, samples=raw, join="consumer"))
+        assert cs.H == pc.H and cs.S == pc.S and cs.K == pc.K
+        got = _ranked_rows(cs)
+        assert len(got) == len(pc.R)
+        for s in cs.sites():
+            k, i = s["k"], s["idx"]
+            rows = [first[k] + i] + [first[k] + j for j in brute.consumers(ks[k], i)]
+            row = tab[rows].sum(axis=0)
+            kv = got[(k, i, s["rule"])]
+            assert int(kv["tot"]) == int(row.sum()), text
+            assert int(kv["rel"]) == int(row[REL_SETS[s["rule"]]].sum()), text
+            assert kv["h"] == ",".join(str(int(x)) for x in row[:19]), text
+            checked += 1
+    assert checked > 100
+
+
+def test_consumer_join_hand_example():
+    """A hand-checked stream: the load's two readers are its consumers; the reader after the
+    register is overwritten is not; a store has no consumers (its row alone)."""
+    from gen import samples as gs
+    ins = [
+        brute.Ins("LDC.64", dst=2, width=2, srcs=[("C", 0x380)]),
+        brute.Ins("LDG.E", dst=4, base=2, off=0),                        # 1: RO site
+        brute.Ins("FFMA", dst=5, srcs=[("R", 4), ("R", 4), ("R", 0)]),   # 2: consumer of 1 (once)
+        brute.Ins("I2F", dst=6, srcs=[("R", 4)]),                        # 3: consumer of 1; CONV site
+        brute.Ins("MOV", dst=4, srcs=[("I", 16)]),                       # 4: overwrites R4
+        brute.Ins("FFMA", dst=1, srcs=[("R", 4), ("R", 6), ("R", 5)]),   # 5: consumer of 4, 3, 2
+        brute.Ins("LDC.64", dst=8, width=2, srcs=[("C", 0x388)]),
+        brute.Ins("REDG.E.ADD.STRONG.GPU", base=8, off=0, data=1),       # 7: GATOM site, no dst
+    ]
+    assert brute.consumers(ins, 1) == [2, 3]
+    assert brute.consumers(ins, 3) == [5]
+    assert brute.consumers(ins, 7) == []
+    n = len(ins)
+    tab = np.zeros((n, 32), np.int64)
+    for i in range(n):
+        tab[i, 6] = 10 ** i          # long_scoreboard: one decimal digit per instruction
+        tab[i, 13] = 1
+    raw = gs.Trace(tab, [0], [n], order="shuffled", seed=5).raw()
+    c = Canon(orc.run(brute.render([ins]), samples=raw, join="consumer"))
+    assert {(s["idx"], s["rule"]) for s in c.sites()} == {(1, "RO"), (3, "CONV"), (7, "GATOM")}
+    got = _ranked_rows(c)
+    assert int(got[(0, 1, "RO")]["rel"]) == 10 + 100 + 1000
+    assert int(got[(0, 1, "RO")]["tot"]) == 10 + 100 + 1000 + 3
+    assert int(got[(0, 3, "CONV")]["tot"]) == 1000 + 100000 + 2
+    assert int(got[(0, 7, "GATOM")]["tot"]) == 10 ** 7 + 1
+
+
 def test_count_records_equal_expanded_samples():
     """Pre-aggregated (kernel, pc, reason, count) records (CUPTI PC-sampling shape, SURVEY §8f
     row 3) give exactly the histogram, totals and ranking of the same samples one by one,

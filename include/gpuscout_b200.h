@@ -62,8 +62,13 @@ enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW
  *   GS_JOIN_LINE the sum of the rows of every instruction of the kernel on the site's source line
  *                (file, line) from nvdisasm -g ("stall reasons ... at the line numbers identified",
  *                P:325-327); a site without line information keeps its PC row.
+ *   GS_JOIN_CONSUMER the site PC's row plus the rows of its direct consumers: every instruction j
+ *                of the kernel that reads a general-purpose register (pairs expanded) whose last
+ *                writer before j is the site instruction (R37; scoreboard stalls are
+ *                sampled at the instruction waiting for the data). gs_detect builds the consumer
+ *                groups when this mode is configured.
  * Ranked counts[] are the joined row, saturated to 2^32-1; rel and tot are exact. */
-enum { GS_JOIN_PC = 0, GS_JOIN_LINE = 1 };
+enum { GS_JOIN_PC = 0, GS_JOIN_LINE = 1, GS_JOIN_CONSUMER = 2 };
 
 /* Rule ids (paper §4) — also the rank tie-break order. */
 enum { GS_VEC = 0, GS_SPILL = 1, GS_SHMEM = 2, GS_GATOM = 3, GS_RO = 4, GS_TEX = 5, GS_CONV = 6 };

@@ -78,7 +78,7 @@ gs_status gs_create(gs_ctx** out, int device, void* cuda_stream, const gs_config
   if (!c->cfg.shmem_min_loads) c->cfg.shmem_min_loads = 2;
   if (!c->cfg.hist_row) c->cfg.hist_row = 32;
   if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_WINDOW ||
-      (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) || c->cfg.join_mode > GS_JOIN_LINE ||
+      (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) || c->cfg.join_mode > GS_JOIN_CONSUMER ||
       (c->cfg.hist_counter_bits != 0 && c->cfg.hist_counter_bits != 16 && c->cfg.hist_counter_bits != 32)) {
     delete c;
     return GS_E_INVAL;

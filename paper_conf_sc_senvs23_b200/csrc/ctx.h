@@ -121,7 +121,19 @@ struct gs_ctx {
   size_t sort_tmp_bytes = 0;
   unsigned long long* d_ktot = nullptr;
   gs_ranked_site* d_ranked = nullptr;
-  uint32_t* d_jrow = nullptr;   // GS_JOIN_LINE: joined row per site (32 u32, saturated)
+  uint32_t* d_jrow = nullptr;   // GS_JOIN_LINE / GS_JOIN_CONSUMER: joined row per site (32 u32, saturated)
+  // GS_JOIN_CONSUMER (R37), built by gs_detect: per GPR use its defining slot, and per slot the
+  // group {slot, its consumers} (CSR over global slots, valid for the detected kernels)
+  uint32_t* d_cdef = nullptr;   // per use (global use index): def slot or ~0u
+  uint64_t cdef_cap = 0;
+  uint32_t* d_ccnt = nullptr;   // per slot (+1): 1 + consumers
+  uint64_t ccnt_cap = 0;
+  uint32_t* d_cgoff = nullptr;  // per slot (+1): first entry of d_cgslot
+  uint64_t cgoff_cap = 0;
+  uint32_t* d_cgslot = nullptr; // the slot itself, then its consumers
+  uint64_t cgslot_cap = 0;
+  unsigned long long* d_ctot = nullptr;
+  bool cons_ready = false;      // the consumer groups belong to the current detection
   uint64_t jrow_cap = 0;
   uint64_t ranked_cap = 0;
   void* h_pin = nullptr;  // pinned host scratch for small D2H results (async copies, no hidden sync)
@@ -184,6 +196,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
                    bool out_is_host, uint64_t* n_out);
 void attrib_free(gs_ctx* c);
 gs_status liveness_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint16_t* d_live);
+// upload the packer's GPR use lists and branch targets (once per gs_load_sass)
+gs_status uses_upload(gs_ctx* c);
 void liveness_free(gs_ctx* c);
 void rank_free(gs_ctx* c);
 

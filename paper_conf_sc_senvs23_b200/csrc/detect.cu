@@ -279,6 +279,88 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
   }
 }
 
+// ------------------------------------------------------------------------------------------ C'
+// Consumer join (GS_JOIN_CONSUMER, reading R37; [probe 9]: scoreboard stalls are sampled at the
+// instruction that waits for the data). Per window (one warp), the same reaching-definition
+// machinery as k_resolve: for every GPR use q of instruction j (the packer's use lists, pairs
+// expanded as in R36) cdef[q] = RD(j, reg) (~0u for ENTRY or when j already reads another
+// register of the same definition), and ccnt[def] += 1.
+__global__ void __launch_bounds__(kWarps * 32) k_consumers(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+                                                           uint32_t w0, uint32_t nw, const uint32_t* __restrict__ tab,
+                                                           const uint32_t* __restrict__ use_off,
+                                                           const uint8_t* __restrict__ use_reg, uint32_t* cdef,
+                                                           uint32_t* ccnt) {
+  __shared__ uint32_t tabS[kWarps][256];  // GPR entries of the carried last-writer table
+  __shared__ uint32_t cm[kWarps][256];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t w = w0 + blockIdx.x * kWarps + warp;
+  if (w >= w0 + nw) return;
+  for (int r = lane; r < 256; r += 32) {
+    tabS[warp][r] = tab[(uint64_t)w * kNumRegs + r];
+    cm[warp][r] = 0;
+  }
+  __syncwarp();
+  const WDesc W = wd[w];
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t gt = ~((2u << lane) - 1u);
+  uint32_t* T = tabS[warp];
+  uint32_t* M = cm[warp];
+  for (uint32_t b = 0; b < W.len; b += 32) {
+    const uint32_t i = b + lane;
+    const bool valid = i < W.len;
+    const uint64_t g = (uint64_t)W.start + i;
+    const uint64_t gbase = (uint64_t)W.start + b;
+    const Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
+    const uint32_t dst = r_dst(r), dw = r_dstw(r);
+    const bool writes = valid && dw && dst < 255;  // GPR definitions only
+    if (writes)
+      for (uint32_t q = 0; q < dw && dst + q < 255; q++) atomicOr(&M[dst + q], 1u << lane);
+    __syncwarp();
+    if (valid) {
+      const uint32_t q0 = use_off[g], q1 = use_off[g + 1];
+      for (uint32_t q = q0; q < q1; q++) {
+        const uint32_t reg = use_reg[q];
+        const uint32_t m = M[reg] & lt;
+        const uint32_t v = m ? (uint32_t)((gbase + (31u - __clz(m)) + 1) << 1) : T[reg];
+        uint32_t d = v ? (v >> 1) - 1u : ~0u;
+        for (uint32_t p = q0; p < q && d != ~0u; p++)
+          if (cdef[p] == d) d = ~0u;  // j counts once per definition
+        cdef[q] = d;
+        if (d != ~0u) atomicAdd(ccnt + d, 1u);
+      }
+    }
+    __syncwarp();
+    if (writes) {
+      const uint32_t v = (uint32_t)((g + 1) << 1);
+      for (uint32_t q = 0; q < dw && dst + q < 255; q++)
+        if ((M[dst + q] & gt) == 0) T[dst + q] = v;
+    }
+    __syncwarp();
+    if (writes)
+      for (uint32_t q = 0; q < dw && dst + q < 255; q++) M[dst + q] = 0;
+    __syncwarp();
+  }
+}
+
+// slots [s0, s0 + n): 1 (the slot's own row) before the consumers are counted; ccnt[s0 + n] = 0
+__global__ void k_cons_init(uint32_t* ccnt, uint64_t s0, uint64_t n) {
+  const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (i <= n) ccnt[s0 + i] = i < n ? 1u : 0u;
+}
+
+// group of slot s = {s, its consumers}: gslot[goff[s]] = s, consumers after it (any order)
+__global__ void k_cons_fill(uint64_t s0, uint64_t n, const uint32_t* __restrict__ use_off,
+                            const uint32_t* __restrict__ cdef, const uint32_t* __restrict__ goff, uint32_t* ccnt,
+                            uint32_t* gslot) {
+  const uint64_t s = s0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (s >= s0 + n) return;
+  gslot[goff[s]] = (uint32_t)s;
+  for (uint32_t q = use_off[s], e = use_off[s + 1]; q < e; q++) {
+    const uint32_t d = cdef[q];
+    if (d != ~0u) gslot[goff[d] + atomicSub(ccnt + d, 1u) - 1u] = (uint32_t)s;
+  }
+}
+
 // ------------------------------------------------------------------------------------------ D
 struct TraceOut {
   uint32_t tk, tv, depth;
@@ -514,7 +596,46 @@ void detect_free(gs_ctx* c) {
   c->d_sites = nullptr; c->sites_cap = 0; c->n_sites = 0;
   c->d_chain = nullptr; c->chain_cap = 0; c->n_chain = 0;
   c->d_scan_tmp = nullptr; c->scan_tmp_bytes = 0;
+  void* cp[] = {c->d_cdef, c->d_ccnt, c->d_cgoff, c->d_cgslot, c->d_ctot};
+  for (void* p : cp)
+    if (p) cudaFree(p);
+  c->d_cdef = c->d_ccnt = c->d_cgoff = c->d_cgslot = nullptr;
+  c->d_ctot = nullptr;
+  c->cdef_cap = c->ccnt_cap = c->cgoff_cap = c->cgslot_cap = 0;
+  c->cons_ready = false;
   c->detected = false;
+}
+
+// GS_JOIN_CONSUMER: consumer groups of the slots of kernels [kb, ke) (R37)
+gs_status consumers_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint32_t w0, uint32_t nw) {
+  cudaStream_t st = c->stream;
+  c->cons_ready = false;
+  const uint64_t s0 = kb < c->n_kernels ? c->kd_h[kb].first : c->n_instr;
+  const uint64_t s1 = ke < c->n_kernels ? c->kd_h[ke].first : c->n_instr;
+  const uint64_t n = s1 - s0;
+  gs_status us = uses_upload(c);
+  if (us != GS_OK) return us;
+  const uint64_t nuse = c->use_off_h.empty() ? 0 : c->use_off_h.back();
+  GS_CUDA(c, dev_grow(&c->d_cdef, &c->cdef_cap, nuse ? nuse : 1));
+  GS_CUDA(c, dev_grow(&c->d_ccnt, &c->ccnt_cap, c->n_instr + 1));
+  GS_CUDA(c, dev_grow(&c->d_cgoff, &c->cgoff_cap, c->n_instr + 1));
+  GS_CUDA(c, dev_grow(&c->d_cgslot, &c->cgslot_cap, n + (c->use_off_h[s1] - c->use_off_h[s0]) + 1));
+  if (!c->d_ctot) GS_CUDA(c, cudaMalloc((void**)&c->d_ctot, 8));
+  k_cons_init<<<(unsigned)((n + 1 + 255) / 256), 256, 0, st>>>(c->d_ccnt, s0, n); count_launch();
+  if (nw) {
+    k_consumers<<<(nw + kWarps - 1) / kWarps, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_use_off,
+                                                                    c->d_use_reg, c->d_cdef, c->d_ccnt); count_launch();
+  }
+  GS_CUDA(c, cudaGetLastError());
+  us = scan_u32(c, c->d_ccnt + s0, c->d_cgoff + s0, n + 1, c->d_ctot);
+  if (us != GS_OK) return us;
+  if (n) {
+    k_cons_fill<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(s0, n, c->d_use_off, c->d_cdef, c->d_cgoff, c->d_ccnt,
+                                                            c->d_cgslot); count_launch();
+    GS_CUDA(c, cudaGetLastError());
+  }
+  c->cons_ready = true;
+  return GS_OK;
 }
 
 gs_status detect_alloc(gs_ctx* c) {
@@ -570,6 +691,11 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
                                            c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand); count_launch();
     GS_CUDA(c, cudaGetLastError());
+  }
+  c->cons_ready = false;
+  if (c->cfg.join_mode == GS_JOIN_CONSUMER) {
+    const gs_status cs = consumers_run(c, kb, ke, w0, nw);
+    if (cs != GS_OK) return cs;
   }
   unsigned long long* d_tot = c->cand.choff + nc;  // two totals after the offsets
   // pinned: [0, 16) the two totals, then the per-kernel counters (async D2H, one synchronisation)

@@ -196,6 +196,20 @@ T* carve(char*& p, uint64_t n) {
 
 }  // namespace
 
+gs_status uses_upload(gs_ctx* c) {
+  if (c->d_use_off) return GS_OK;  // first use: upload the packer's GPR use lists
+  cudaStream_t st = c->stream;
+  GS_CUDA(c, cudaMalloc((void**)&c->d_use_off, c->use_off_h.size() * 4));
+  GS_CUDA(c, cudaMalloc((void**)&c->d_use_reg, std::max<size_t>(c->use_reg_h.size(), 1)));
+  GS_CUDA(c, cudaMalloc((void**)&c->d_tgt, std::max<size_t>(c->tgt_h.size(), 1) * 4));
+  GS_CUDA(c, cudaMemcpyAsync(c->d_use_off, c->use_off_h.data(), c->use_off_h.size() * 4, cudaMemcpyHostToDevice, st));
+  if (!c->use_reg_h.empty())
+    GS_CUDA(c, cudaMemcpyAsync(c->d_use_reg, c->use_reg_h.data(), c->use_reg_h.size(), cudaMemcpyHostToDevice, st));
+  if (!c->tgt_h.empty())
+    GS_CUDA(c, cudaMemcpyAsync(c->d_tgt, c->tgt_h.data(), c->tgt_h.size() * 4, cudaMemcpyHostToDevice, st));
+  return GS_OK;
+}
+
 gs_status liveness_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint16_t* d_live) {
   cudaStream_t st = c->stream;
   if (ke <= kb) return GS_OK;
@@ -203,15 +217,9 @@ gs_status liveness_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint16_t* d_live) {
   const uint32_t s1 = ke < c->n_kernels ? c->kd_h[ke].first : (uint32_t)c->n_instr;
   const uint64_t n = s1 - s0, nk = ke - kb;
   if (!n) return GS_OK;
-  if (!c->d_use_off) {  // first use: upload the packer's register-pressure inputs
-    GS_CUDA(c, cudaMalloc((void**)&c->d_use_off, c->use_off_h.size() * 4));
-    GS_CUDA(c, cudaMalloc((void**)&c->d_use_reg, std::max<size_t>(c->use_reg_h.size(), 1)));
-    GS_CUDA(c, cudaMalloc((void**)&c->d_tgt, std::max<size_t>(c->tgt_h.size(), 1) * 4));
-    GS_CUDA(c, cudaMemcpyAsync(c->d_use_off, c->use_off_h.data(), c->use_off_h.size() * 4, cudaMemcpyHostToDevice, st));
-    if (!c->use_reg_h.empty())
-      GS_CUDA(c, cudaMemcpyAsync(c->d_use_reg, c->use_reg_h.data(), c->use_reg_h.size(), cudaMemcpyHostToDevice, st));
-    if (!c->tgt_h.empty())
-      GS_CUDA(c, cudaMemcpyAsync(c->d_tgt, c->tgt_h.data(), c->tgt_h.size() * 4, cudaMemcpyHostToDevice, st));
+  {
+    const gs_status us = uses_upload(c);
+    if (us != GS_OK) return us;
   }
   // scratch sized for the worst case (every instruction a block): leader, excl, block arrays
   const uint64_t need = 8 * ((n * 4 + 255) / 256 * 256) + 3 * ((n * kW * 4 + 255) / 256 * 256) +

@@ -117,6 +117,8 @@ __global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int
 
 // GS_JOIN_LINE (R33): one warp per site, lane = reason; the site's row is the sum of
 // the rows of its source-line group (CSR goff/gslot), or its own PC row without line info.
+// GS_JOIN_CONSUMER (R37): lgrp == nullptr, the group of a slot is the slot itself (its own row
+// and its consumers' rows).
 __global__ void k_join_line(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H,
                             uint32_t slot0, uint32_t row, const KDesc* __restrict__ kd,
                             const uint32_t* __restrict__ lgrp, const uint32_t* __restrict__ goff,
@@ -128,7 +130,7 @@ __global__ void k_join_line(const gs_site* __restrict__ sites, uint64_t ns, cons
   const uint32_t lane = threadIdx.x & 31u;
   const gs_site st = sites[s];
   const uint32_t slot = kd[st.kernel].first + st.idx;
-  const uint32_t g = lgrp[slot];
+  const uint32_t g = lgrp ? lgrp[slot] : slot;
   unsigned long long v = 0;
   if (g == ~0u) {
     if (lane < row) v = (uint32_t)__ldg(H + (uint64_t)(slot - slot0) * row + lane);
@@ -254,11 +256,14 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
     void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
     const unsigned grid = (unsigned)((ns + 255) / 256);
-    const bool line = c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups;
+    const bool cons = c->cfg.join_mode == GS_JOIN_CONSUMER;
+    if (cons && !c->cons_ready) return fail(c, GS_E_STATE, "consumer join: gs_detect ran in another join mode");
+    const bool line = (c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups) || cons;
     if (line) {
       GS_CUDA(c, dev_grow(&c->d_jrow, &c->jrow_cap, ns * 32));
-      k_join_line<<<(unsigned)((ns + 7) / 8), 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, c->d_kd, c->d_lgrp,
-                                                            c->d_goff, c->d_gslot, d_rel, d_tot, c->d_jrow, d_max);
+      k_join_line<<<(unsigned)((ns + 7) / 8), 256, 0, st>>>(
+          c->d_sites, ns, d_hist, slot0, row, c->d_kd, cons ? nullptr : c->d_lgrp, cons ? c->d_cgoff : c->d_goff,
+          cons ? c->d_cgslot : c->d_gslot, d_rel, d_tot, c->d_jrow, d_max);
     } else {
       const bool vec = row == 32 && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0;
       k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, vec, c->d_kd, d_rel, d_tot, d_max);

@@ -208,6 +208,69 @@ def test_line_join_parity(gs, name, row):
         assert g.R == o.R, (name, disasm)
 
 
+@pytest.mark.parametrize("name", ["listing1.sass", "sgemm_naive.sm_100a.sass", "jacobi.sm_70.sass",
+                                  "mixbench.sm_100a.sass", "spill.r24.sm_100a.sass", "conv.sm_100a.sass"])
+@pytest.mark.parametrize("row", [32, 19])
+def test_consumer_join_parity(gs, name, row):
+    """GS_JOIN_CONSUMER (R37): each site joined with its PC row plus the rows of its direct
+    consumers, against the oracle's --join consumer."""
+    from gen import samples as gsm
+    text = _read(name)
+    o_pc = Canon(orc.run(text))
+    first = [int(k["first"]) for k in o_pc.kstats()]
+    nk = [int(k["n"]) for k in o_pc.kstats()]
+    rng = np.random.default_rng(47)
+    tab = np.zeros((sum(nk), 32), np.int64)
+    tab[:, :19] = rng.integers(0, 30, (sum(nk), 19))
+    raw = gsm.Trace(tab, first, nk, order="shuffled", seed=47).raw()
+    g, _ = _flow(gs, text, raw, hist_row=row, join_mode=gs.GS_JOIN_CONSUMER)
+    o = Canon(orc.run(text, samples=raw, join="consumer"))
+    assert g.S == o.S and g.H == o.H and g.N == o.N
+    assert g.R == o.R, name
+
+
+def test_consumer_join_parity_streams_and_configs(gs):
+    """GS_JOIN_CONSUMER on random tiny streams (pairs, overwrites, several kernels) and on the C2
+    and scaled C4 configurations, including a detection shard ranked against its histogram slice."""
+    import torch
+    from gen import samples as gsm
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    rng = random.Random(53)
+    for _ in range(25):
+        ks = [brute.random_stream(rng, rng.randint(2, 7)) for _ in range(rng.randint(1, 3))]
+        nk = [len(k) for k in ks]
+        first = list(np.cumsum([0] + nk[:-1]))
+        tab = np.zeros((sum(nk), 32), np.int64)
+        tab[:, :19] = np.random.default_rng(rng.randrange(99)).integers(0, 5, (sum(nk), 19))
+        if not tab.any():
+            continue
+        raw = gsm.Trace(tab, first, nk, order="shuffled", seed=3).raw()
+        text = brute.render(ks)
+        g, _ = _flow(gs, text, raw, join_mode=gs.GS_JOIN_CONSUMER)
+        assert g.R == Canon(orc.run(text, samples=raw, join="consumer")).R, text
+    for cfg, scale in (("C2", 1), ("C4", 0.02)):
+        s = gsass.config_sass(cfg, scale=scale)
+        raw, _ = _samples(s, 200_000, "shuffled", seed=59)
+        g, _ = _flow(gs, s.text, raw, hist_row=19, join_mode=gs.GS_JOIN_CONSUMER)
+        o = Canon(orc.run(s.text, samples=raw, join="consumer"))
+        assert g.S == o.S and g.R == o.R, cfg
+    s = gsass.config_sass("C2")
+    raw, _ = _samples(s, 100_000, "shuffled", seed=61, n_bad=0)
+    ctx = _ctx(gs, hist_row=19, join_mode=gs.GS_JOIN_CONSUMER)
+    ctx.load_sass(s.text)
+    raw_t = torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda()
+    words, _ = ctx.pack_samples(raw_t)
+    hist, _ = ctx.attribute_samples(words)
+    for kb, ke in ((1, 2), (0, 3), (2, 3)):
+        ctx.detect(kb, ke)
+        sb, se = int(s.first_slot[kb]), int(s.first_slot[ke]) if ke < len(s.first_slot) else int(sum(s.n_instr))
+        got = ctx.rank_sites(hist[sb * 19:se * 19].clone(), slot_begin=sb, slot_end=se)
+        lines = report.canonical(ctx, kb, ke, hist=hist, n_samples=len(raw), n_invalid=0, ranked=got)
+        want = Canon(orc.run(s.text, samples=raw, kbegin=kb, kend=ke, join="consumer")).R
+        assert Canon(lines).R == want, (kb, ke)
+
+
 def test_attribute_counts_parity(gs):
     """gs_attribute_counts: pre-aggregated (kernel, pc, reason, count) records (CUPTI PC-sampling
     shape) against the oracle's --counts, invalid records included; plus accumulate on top of

@@ -485,36 +485,108 @@ __device__ uint32_t eval_rules(const Rec& ri, uint64_t c, const CandArrays& ca, 
   return f;
 }
 
-__global__ void k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca, GroupTable gt, RootSet rs,
-                        const uint32_t* __restrict__ narith, RuleCfg rc) {
-  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (c >= nc) return;
-  const Rec ri = ld_rec(rec, ca.idx[c]);
-  const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc);
-  ca.flags[c] = (uint8_t)f;
-  ca.nsite[c] = __popc(f);
-  ca.soff[c] = f ? ca.depth[c] : 0;  // chain length (scanned into choff)
+// Site and chain-pool compaction (a-7) without separate scan passes: k_rules leaves one packed
+// (chains << 32 | sites) sum per 256-candidate tile, one CTA scans the tile sums, and k_write
+// re-derives each candidate's offsets inside its tile with a block scan.
+constexpr int kCT = 256;  // candidates per tile (k_rules / k_write CTA)
+
+__device__ __forceinline__ unsigned long long warp_incl64(unsigned long long v) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long x = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += x;
+  }
+  return v;
+}
+// exclusive scan over the CTA of one value per thread (blockDim.x = NT); *total = the CTA's sum
+template <int NT>
+__device__ __forceinline__ unsigned long long block_excl64(unsigned long long v, unsigned long long* total) {
+  __shared__ unsigned long long wsum[NT / 32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const unsigned long long inc = warp_incl64(v);
+  if (lane == 31) wsum[warp] = inc;
+  __syncthreads();
+  if (warp == 0) {
+    unsigned long long x = lane < NT / 32 ? wsum[lane] : 0;
+    x = warp_incl64(x);
+    if (lane < NT / 32) wsum[lane] = x;
+  }
+  __syncthreads();
+  const unsigned long long before = warp ? wsum[warp - 1] : 0;
+  *total = wsum[NT / 32 - 1];
+  __syncthreads();
+  return before + inc - v;
+}
+// per candidate: sites (low 32 bits) and chain-pool entries (high 32 bits); a tile's sums fit
+__device__ __forceinline__ unsigned long long site_chain(uint32_t f, uint32_t depth) {
+  return ((unsigned long long)(f ? depth : 0u) << 32) | (unsigned long long)__popc(f);
 }
 
-__global__ void k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
-                        uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, const uint32_t* __restrict__ narith,
-                        const uint32_t* __restrict__ site_off, gs_site* __restrict__ sites,
-                        uint32_t* __restrict__ chain, uint64_t site_cap, uint64_t chain_cap) {
+__global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca, GroupTable gt,
+                                               RootSet rs, const uint32_t* __restrict__ narith, RuleCfg rc,
+                                               unsigned long long* __restrict__ tsum) {
+  const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
+  unsigned long long v = 0;
+  if (c < nc) {
+    const Rec ri = ld_rec(rec, ca.idx[c]);
+    const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc);
+    ca.flags[c] = (uint8_t)f;
+    v = site_chain(f, ca.depth[c]);
+  }
+  unsigned long long tot;
+  block_excl64<kCT>(v, &tot);
+  if (threadIdx.x == 0) tsum[blockIdx.x] = tot;
+}
+
+// one CTA: exclusive prefixes of the tile sums, sites and chains as separate u64 counters;
+// tot[0] = chain-pool entries, tot[1] = sites
+__global__ void __launch_bounds__(1024) k_tile_prefix(const unsigned long long* __restrict__ tsum, uint64_t nt,
+                                                      unsigned long long* __restrict__ pre_s,
+                                                      unsigned long long* __restrict__ pre_c,
+                                                      unsigned long long* __restrict__ tot) {
+  unsigned long long cs = 0, cc = 0;
+  for (uint64_t b = 0; b < nt; b += 1024) {
+    const uint64_t i = b + threadIdx.x;
+    const unsigned long long v = i < nt ? tsum[i] : 0;
+    unsigned long long ts, tc;
+    const unsigned long long es = block_excl64<1024>(v & 0xffffffffull, &ts);
+    const unsigned long long ec = block_excl64<1024>(v >> 32, &tc);
+    if (i < nt) {
+      pre_s[i] = cs + es;
+      pre_c[i] = cc + ec;
+    }
+    cs += ts;
+    cc += tc;
+  }
+  if (threadIdx.x == 0) {
+    tot[0] = cc;
+    tot[1] = cs;
+  }
+}
+
+__global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, const KDesc* __restrict__ kd,
+                                               const uint32_t* __restrict__ ptrrd, uint64_t nc, uint32_t D, CandArrays ca,
+                                               GroupTable gt, const uint32_t* __restrict__ narith,
+                                               const unsigned long long* __restrict__ pre_s,
+                                               const unsigned long long* __restrict__ pre_c, gs_site* __restrict__ sites,
+                                               uint32_t* __restrict__ chain, uint64_t site_cap, uint64_t chain_cap) {
   // Launched before the host knows the totals: writes past the buffers' current capacities are
   // skipped, and the host relaunches after growing them when a total exceeds its capacity.
-  const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (c >= nc) return;
-  const uint32_t f = ca.flags[c];
+  const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
+  const uint32_t f = c < nc ? ca.flags[c] : 0u;
+  unsigned long long tot;
+  const unsigned long long ex = block_excl64<kCT>(site_chain(f, c < nc ? ca.depth[c] : 0u), &tot);
   if (!f) return;
   const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
   const KDesc K = kd[kernel];
   const Rec ri = ld_rec(rec, g);
-  const unsigned long long coff = ca.choff[c];
+  const unsigned long long coff = pre_c[blockIdx.x] + (ex >> 32);
   // chain: re-chase and store kernel-local indices
   uint32_t n = 0;
   if (ca.depth[c] && coff + ca.depth[c] <= chain_cap)
     chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, [&](uint32_t j) { chain[coff + n++] = j; });
-  uint32_t so = site_off[c];
+  uint64_t so = pre_s[blockIdx.x] + (ex & 0xffffffffull);
   for (uint32_t rule = 0; rule < 7; rule++) {
     if (!((f >> rule) & 1u)) continue;
     gs_site s;
@@ -652,7 +724,7 @@ gs_status detect_alloc(gs_ctx* c) {
   A(c->cand.idx, NC * 4); A(c->cand.kernel, NC * 4); A(c->cand.base_rd, NC * 4); A(c->cand.data_rd, NC * 4);
   A(c->cand.tv, NC * 4); A(c->cand.grp, NC * 4); A(c->cand.nsite, NC * 4); A(c->cand.soff, NC * 4 + 4);
   A(c->cand.ld, NC); A(c->cand.tk, NC); A(c->cand.depth, NC); A(c->cand.flags, NC);
-  A(c->cand.choff, NC * 8 + 16);
+  A(c->cand.choff, 24 * ((NC + kCT - 1) / kCT) + 16);  // tile sums, prefixes, totals (k_rules / k_write)
   c->grp.cap = pow2_at_least(2 * c->n_ldg + 16);
   A(c->grp.key, (uint64_t)c->grp.cap * 8);
   A(c->grp.nload, (uint64_t)c->grp.cap * 4); A(c->grp.n32, (uint64_t)c->grp.cap * 4);
@@ -697,7 +769,13 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     const gs_status cs = consumers_run(c, kb, ke, w0, nw);
     if (cs != GS_OK) return cs;
   }
-  unsigned long long* d_tot = c->cand.choff + nc;  // two totals after the offsets
+  // tile sums, their exclusive prefixes (sites, chains) and the two totals, carved from cand.choff
+  // (3 x ceil(NC / 256) u64 + 2)
+  const uint64_t ntile = (nc + kCT - 1) / kCT;
+  unsigned long long* d_tsum = c->cand.choff;
+  unsigned long long* d_pre_s = d_tsum + ntile;
+  unsigned long long* d_pre_c = d_pre_s + ntile;
+  unsigned long long* d_tot = d_pre_c + ntile;
   // pinned: [0, 16) the two totals, then the per-kernel counters (async D2H, one synchronisation)
   GS_CUDA(c, pin_grow(c, 16 + (uint64_t)c->n_kernels * sizeof(gs_kernel_stats)));
   unsigned long long* tot = static_cast<unsigned long long*>(c->h_pin);
@@ -711,23 +789,20 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
                                    c->d_kstats); count_launch();
     GS_CUDA(c, cudaGetLastError());
-    k_rules<<<gridc, 256, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
-                                   RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}); count_launch();
+    k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
+                                             RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum);
+    count_launch();
+    k_tile_prefix<<<1, 1024, 0, st>>>(d_tsum, ntile, d_pre_s, d_pre_c, d_tot); count_launch();
     GS_CUDA(c, cudaGetLastError());
-    // chain offsets (u64) from chain lengths stored in soff, then site offsets in place of soff
-    gs_status s = scan_u32_to_u64(c, c->cand.soff, c->cand.choff, nc, d_tot);
-    if (s != GS_OK) return s;
-    s = scan_u32(c, c->cand.nsite, c->cand.soff, nc, d_tot + 1);
-    if (s != GS_OK) return s;
     GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
   }
   // sites and chains into the buffers as they are (one host synchronisation per call); if a total
   // turns out larger than its buffer, grow it and write again
   auto write = [&]() -> gs_status {
     if (!nc || (!c->sites_cap && !c->chain_cap)) return GS_OK;
-    k_write<<<(uint32_t)((nc + 255) / 256), 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
-                                                         c->d_narith, c->cand.soff, c->d_sites, c->d_chain,
-                                                         c->sites_cap, c->chain_cap); count_launch();
+    k_write<<<(uint32_t)((nc + kCT - 1) / kCT), kCT, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
+                                                             c->d_narith, d_pre_s, d_pre_c, c->d_sites, c->d_chain,
+                                                             c->sites_cap, c->chain_cap); count_launch();
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   };

@@ -72,44 +72,49 @@ __global__ void __launch_bounds__(kKtotThreads) k_ktot(const int32_t* __restrict
   }
 }
 
-__global__ void k_join(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H, uint32_t slot0,
-                       uint32_t row, bool vec, const KDesc* __restrict__ kd, unsigned long long* __restrict__ rel_out,
+// PC join (R18): one warp per 4 sites (8 lanes per site, 4 reasons per lane), rows read
+// coalesced; running maxima of rel and tot for the packed sort key.
+__global__ void __launch_bounds__(256) k_join(const gs_site* __restrict__ sites, uint64_t ns, const int32_t* __restrict__ H, uint32_t slot0,
+                       uint32_t row, const KDesc* __restrict__ kd, unsigned long long* __restrict__ rel_out,
                        unsigned long long* __restrict__ tot_out, unsigned long long* __restrict__ mx) {
-  const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const uint32_t lane = threadIdx.x & 31u, sub = lane & 7u;
+  const uint64_t s = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 3;
   unsigned long long tot = 0, rel = 0;
   if (s < ns) {
     const gs_site st = sites[s];
-    const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx - slot0;
+    const uint64_t slot = (uint64_t)__ldg(&kd[st.kernel].first) + st.idx - slot0;
     const uint32_t m = kRelMask[st.rule];
-    if (vec) {  // 32-wide, 16-byte aligned rows
-      const int4* r4 = reinterpret_cast<const int4*>(H + slot * 32);
+    const int32_t* r1 = H + slot * row;
 #pragma unroll
-      for (int q = 0; q < 8; q++) {
-        const int4 v = __ldg(r4 + q);
-        const uint32_t c[4] = {(uint32_t)v.x, (uint32_t)v.y, (uint32_t)v.z, (uint32_t)v.w};
-#pragma unroll
-        for (int t = 0; t < 4; t++) {
-          tot += c[t];
-          if ((m >> (4 * q + t)) & 1u) rel += c[t];
-        }
-      }
-    } else {
-      const int32_t* r1 = H + slot * row;
-      for (uint32_t t = 0; t < row; t++) {
+    for (uint32_t t = sub; t < 32; t += 8) {
+      if (t < row) {
         const uint32_t c = (uint32_t)__ldg(r1 + t);
         tot += c;
         if ((m >> t) & 1u) rel += c;
       }
     }
+  }
+#pragma unroll
+  for (int o = 4; o; o >>= 1) {  // within the 8 lanes of a site
+    tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    rel += __shfl_xor_sync(0xffffffffu, rel, o);
+  }
+  if (s < ns && sub == 0) {
     rel_out[s] = rel;
     tot_out[s] = tot;
   }
   unsigned long long mr = rel, mt = tot;
-  for (int o = 16; o; o >>= 1) {
+  for (int o = 16; o >= 8; o >>= 1) {
     mr = max(mr, __shfl_xor_sync(0xffffffffu, mr, o));
     mt = max(mt, __shfl_xor_sync(0xffffffffu, mt, o));
   }
-  if ((threadIdx.x & 31) == 0) {
+  // one pair of atomics per CTA: the maxima go to two addresses every CTA updates
+  __shared__ unsigned long long bm[2][8];
+  const uint32_t w = threadIdx.x >> 5;
+  if (lane == 0) { bm[0][w] = mr; bm[1][w] = mt; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (uint32_t v = 1; v < (blockDim.x >> 5); v++) { mr = max(mr, bm[0][v]); mt = max(mt, bm[1][v]); }
     atomicMax(mx, mr);
     atomicMax(mx + 1, mt);
   }
@@ -174,31 +179,44 @@ __global__ void k_keys_field(const unsigned long long* __restrict__ val, const u
   if (!order) vals[i] = s;
 }
 
-// one warp per ranked row; counts from the PC row of H, or the joined row jrow (GS_JOIN_LINE)
-__global__ void k_emit(const uint32_t* __restrict__ order, uint64_t kk, const gs_site* __restrict__ sites,
-                       const int32_t* __restrict__ H, uint32_t slot0, uint32_t row, const uint32_t* __restrict__ jrow,
-                       const unsigned long long* __restrict__ rel_a, const unsigned long long* __restrict__ tot_a,
-                       const KDesc* __restrict__ kd, const unsigned long long* __restrict__ ktot,
-                       gs_ranked_site* __restrict__ out) {
-  const uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
+// ranked rows, one thread per row (the order -> site -> kernel -> histogram-row chain of every
+// row in flight at once); counts from the PC row of H, or the joined row jrow
+__global__ void __launch_bounds__(256) k_emit(const uint32_t* __restrict__ order, uint64_t kk,
+                                              const gs_site* __restrict__ sites, const int32_t* __restrict__ H,
+                                              uint32_t slot0, uint32_t row, const uint32_t* __restrict__ jrow,
+                                              const unsigned long long* __restrict__ rel_a,
+                                              const unsigned long long* __restrict__ tot_a,
+                                              const KDesc* __restrict__ kd, const unsigned long long* __restrict__ ktot,
+                                              gs_ranked_site* __restrict__ out) {
+  const uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (q >= kk) return;
-  const int lane = threadIdx.x & 31;
-  const uint32_t si = order[q];
+  const uint32_t si = __ldg(order + q);
   const gs_site st = sites[si];
-  const uint64_t slot = (uint64_t)kd[st.kernel].first + st.idx - slot0;
-  const uint32_t c = jrow ? jrow[(uint64_t)si * 32 + lane] : ((uint32_t)lane < row ? (uint32_t)H[slot * row + lane] : 0u);
-  const unsigned long long rel = rel_a[si], tot = tot_a[si];
   gs_ranked_site* r = out + q;
-  r->counts[lane] = c;
-  if (lane == 0) {
-    r->kernel = st.kernel;
-    r->idx = st.idx;
-    r->rule = st.rule;
-    r->pad = 0;
-    r->rel = rel;
-    r->tot = tot;
-    r->ktot = ktot[st.kernel];
+  uint2* c2 = reinterpret_cast<uint2*>(r->counts);  // counts[] is 8-byte aligned
+  if (jrow) {
+    const uint4* j4 = reinterpret_cast<const uint4*>(jrow + (uint64_t)si * 32);
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      const uint4 v = __ldg(j4 + t);
+      c2[2 * t] = make_uint2(v.x, v.y);
+      c2[2 * t + 1] = make_uint2(v.z, v.w);
+    }
+  } else {
+    const int32_t* h = H + ((uint64_t)__ldg(&kd[st.kernel].first) + st.idx - slot0) * row;
+    uint32_t c[32];
+#pragma unroll
+    for (uint32_t t = 0; t < 32; t++) c[t] = t < row ? (uint32_t)__ldg(h + t) : 0u;
+#pragma unroll
+    for (int t = 0; t < 16; t++) c2[t] = make_uint2(c[2 * t], c[2 * t + 1]);
   }
+  r->kernel = st.kernel;
+  r->idx = st.idx;
+  r->rule = st.rule;
+  r->pad = 0;
+  r->rel = rel_a[si];
+  r->tot = tot_a[si];
+  r->ktot = ktot[st.kernel];
 }
 
 int bits_of(unsigned long long v) { return v ? 64 - __builtin_clzll(v) : 0; }
@@ -265,8 +283,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
           c->d_sites, ns, d_hist, slot0, row, c->d_kd, cons ? nullptr : c->d_lgrp, cons ? c->d_cgoff : c->d_goff,
           cons ? c->d_cgslot : c->d_gslot, d_rel, d_tot, c->d_jrow, d_max);
     } else {
-      const bool vec = row == 32 && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0;
-      k_join<<<grid, 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, vec, c->d_kd, d_rel, d_tot, d_max);
+      k_join<<<(unsigned)((ns * 8 + 255) / 256), 256, 0, st>>>(c->d_sites, ns, d_hist, slot0, row, c->d_kd, d_rel,
+                                                               d_tot, d_max);
     }
     count_launch();
     GS_CUDA(c, cudaGetLastError());
@@ -310,7 +328,7 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
           GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
           dst = c->d_ranked;
         }
-        k_emit<<<(unsigned)((kk + 7) / 8), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
+k_emit<<<(unsigned)((kk + 255) / 256), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
                                                           line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
                                                           c->d_ktot, dst);
         count_launch();

@@ -21,7 +21,11 @@ ap.add_argument("--order", default="trace")
 ap.add_argument("--mode", type=int, default=0)
 ap.add_argument("--steps", type=int, default=3)
 ap.add_argument("--only", default="all")
+ap.add_argument("--lib", default=None)
 a = ap.parse_args()
+if a.lib:
+    from paper_conf_sc_senvs23_b200 import binding
+    binding.load_library(a.lib)
 s, tr = bench.build_workload(a.config, a.order)
 words = DeviceTrace(tr).packed()
 ctx = g.Context(hist_mode=a.mode, hist_row=19)   # compact rows, as bench.py

@@ -316,27 +316,43 @@ __device__ __forceinline__ uint32_t n_tiles(uint64_t c, uint64_t chunk, uint64_t
   const uint64_t a4 = c * chunk / 4, e = (c + 1) * chunk < n ? (c + 1) * chunk : n, e4 = e / 4;
   return e4 > a4 ? (uint32_t)((e4 - a4 + kTile4 - 1) / kTile4) : 0u;
 }
+// Called by the whole producer warp (result broadcast). Own chunk: lane 0 takes the next tile from
+// the front. Stealing: the 32 lanes read the queue words of all chunks in parallel (a serial scan
+// by one lane took longer than the tiles it was meant to rebalance), pick the chunk with the most
+// tiles left and take its last tile with one CAS.
 __device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, uint32_t grid, uint64_t chunk,
                                         uint64_t n) {
-  const uint32_t mine = n_tiles(me, chunk, n);
-  for (;;) {  // own chunk, front to back
-    const unsigned long long o = *(volatile unsigned long long*)(rng + me);
-    const uint32_t head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
-    if (head + stolen >= mine) break;
-    if (atomicCAS(rng + me, o, o + (1ull << 32)) == o) return ((unsigned long long)me << 32) | head;
+  const uint32_t lane = threadIdx.x & 31u;
+  unsigned long long got = ~0ull;
+  if (lane == 0) {
+    const uint32_t mine = n_tiles(me, chunk, n);
+    for (;;) {  // own chunk, front to back
+      const unsigned long long o = *(volatile unsigned long long*)(rng + me);
+      const uint32_t head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
+      if (head + stolen >= mine) break;
+      if (atomicCAS(rng + me, o, o + (1ull << 32)) == o) { got = ((unsigned long long)me << 32) | head; break; }
+    }
   }
+  got = __shfl_sync(0xffffffffu, got, 0);
+  if (got != ~0ull) return got;
   for (;;) {  // steal from the back of the chunk with the most tiles left
     uint32_t best = grid, best_left = 0;
-    for (uint32_t v = 0; v < grid; v++) {
+    for (uint32_t v = lane; v < grid; v += 32) {
       const unsigned long long o = *(volatile unsigned long long*)(rng + v);
       const uint32_t nt = n_tiles(v, chunk, n), used = (uint32_t)(o >> 32) + (uint32_t)o;
       if (nt > used && nt - used > best_left) { best_left = nt - used; best = v; }
     }
-    if (best == grid) return ~0ull;
-    const unsigned long long o = *(volatile unsigned long long*)(rng + best);
-    const uint32_t nt = n_tiles(best, chunk, n), head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
-    if (head + stolen >= nt) continue;
-    if (atomicCAS(rng + best, o, o + 1ull) == o) return ((unsigned long long)best << 32) | (nt - 1 - stolen);
+    const uint32_t mx = __reduce_max_sync(0xffffffffu, best_left);
+    if (mx == 0) return ~0ull;
+    const uint32_t cand = __reduce_min_sync(0xffffffffu, best_left == mx ? best : 0xffffffffu);
+    if (lane == 0) {
+      const unsigned long long o = *(volatile unsigned long long*)(rng + cand);
+      const uint32_t nt = n_tiles(cand, chunk, n), head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
+      if (head + stolen < nt && atomicCAS(rng + cand, o, o + 1ull) == o)
+        got = ((unsigned long long)cand << 32) | (nt - 1 - stolen);
+    }
+    got = __shfl_sync(0xffffffffu, got, 0);
+    if (got != ~0ull) return got;
   }
 }
 
@@ -566,7 +582,10 @@ __device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity
 // the 31 counting warps only (warp 0 keeps producing)
 __device__ __forceinline__ void bar_counters() { asm volatile("bar.sync 1, %0;" ::"r"(kThreads - 32) : "memory"); }
 
-constexpr uint32_t kItems = 8;  // descriptor ring depth
+#ifndef GS_ITEMS
+#define GS_ITEMS 8
+#endif
+constexpr uint32_t kItems = GS_ITEMS;  // descriptor ring depth
 struct Item {
   uint64_t a4, b4;  // uint4 range of the stream
   uint32_t ws;      // window (first slot) for the range
@@ -632,9 +651,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       j++;
     };
     for (;;) {
-      unsigned long long tile = 0;
-      if (lane == 0) tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
-      tile = __shfl_sync(0xffffffffu, tile, 0);
+      const unsigned long long tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
       if (tile == ~0ull) break;
       uint64_t a4, b4;
       span(tile, a4, b4);

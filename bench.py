@@ -364,7 +364,7 @@ def main():
         "instrs_per_s": s.P / (ms_max * 1e-3),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "kernel": "gs_attribute_samples (histogram pass)",
-                     "hist_mode": ["auto", "global", "private", "window"][mode] if 0 <= mode < 4 else mode,
+                     "hist_mode": ["auto", "global", "private", "window", "partition"][mode] if 0 <= mode < 5 else mode,
                      "kernel_ms": hist_ms_max, "algorithmic_bytes": alg_bytes, "peak_source": peak_src},
         "clocks": clk,
         "gpu_launches": int(launches),

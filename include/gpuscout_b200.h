@@ -55,7 +55,7 @@ typedef struct {
   uint32_t join_mode;       /* which histogram rows a site is joined with, GS_JOIN_*. default PC     */
 } gs_config;
 
-enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3 };
+enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3, GS_HIST_PARTITION = 4 };
 
 /* Join granularity (R18, R33):
  *   GS_JOIN_PC   the site PC's row ("attributed to the instruction detected");

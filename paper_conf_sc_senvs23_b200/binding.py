@@ -16,7 +16,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libgpuscout_b200.so")
 
 GS_OK, GS_E_INVAL, GS_E_PARSE, GS_E_RANGE, GS_E_CUDA, GS_E_NOMEM, GS_E_STATE = 0, -1, -2, -3, -4, -5, -6
-GS_HIST_AUTO, GS_HIST_GLOBAL, GS_HIST_PRIVATE, GS_HIST_WINDOW = 0, 1, 2, 3
+GS_HIST_AUTO, GS_HIST_GLOBAL, GS_HIST_PRIVATE, GS_HIST_WINDOW, GS_HIST_PARTITION = 0, 1, 2, 3, 4
 GS_JOIN_PC, GS_JOIN_LINE, GS_JOIN_CONSUMER = 0, 1, 2
 RULES = ["VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX", "CONV"]
 TERMS = ["NONE", "PARAM", "CONST", "ENTRY", "SREG", "MEMORY", "IMM", "TRUNC"]

@@ -77,7 +77,7 @@ gs_status gs_create(gs_ctx** out, int device, void* cuda_stream, const gs_config
   if (!c->cfg.shmem_min_arith) c->cfg.shmem_min_arith = 1;
   if (!c->cfg.shmem_min_loads) c->cfg.shmem_min_loads = 2;
   if (!c->cfg.hist_row) c->cfg.hist_row = 32;
-  if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_WINDOW ||
+  if (c->cfg.trace_depth > 255 || c->cfg.n_reasons > 32 || c->cfg.hist_mode > GS_HIST_PARTITION ||
       (c->cfg.hist_row != 32 && c->cfg.hist_row != c->cfg.n_reasons) || c->cfg.join_mode > GS_JOIN_CONSUMER ||
       (c->cfg.hist_counter_bits != 0 && c->cfg.hist_counter_bits != 16 && c->cfg.hist_counter_bits != 32)) {
     delete c;

@@ -451,13 +451,13 @@ constexpr uint32_t kNct = kThreads - 32;  // counting threads of the WINDOW kern
 
 // the rare part of one batch of nv uint4 at s4[i + u * kNct], re-read from L1/L2: outside the
 // window (deferred / invalid), or a 16-bit half that needs draining. Returns the invalid count.
-template <bool P16>
+template <bool P16, uint32_t NCT>
 __device__ __noinline__ uint32_t rare_w(const uint4* __restrict__ s4, uint64_t i, uint32_t nv, Win W, uint32_t* tab,
                                         uint32_t flag, uint32_t am, const Spill* sS) {
   const Spill S = *sS;
   uint32_t bad = 0;
   for (uint32_t u = 0; u < nv; u++) {
-    const uint4 v = __ldg(s4 + i + (uint64_t)u * kNct);
+    const uint4 v = __ldg(s4 + i + (uint64_t)u * NCT);
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int q = 0; q < 4; q++) {
@@ -489,28 +489,28 @@ __device__ __forceinline__ uint32_t hot_w(const uint32_t (&w)[N], Win W, uint32_
   return flag;
 }
 
-template <bool P16>
+template <bool P16, uint32_t NCT = kNct>
 __device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, uint64_t i0, uint64_t i1, uint32_t ct,
                                                  Win W, uint32_t* tab, uint32_t spare, const Spill* sS) {
   uint32_t bad = 0;
   uint64_t i = i0 + ct;
-  for (; i + (kVec - 1) * kNct < i1; i += kVec * kNct) {
+  for (; i + (kVec - 1) * NCT < i1; i += kVec * NCT) {
     uint32_t w[4 * kVec];
 #pragma unroll
     for (int u = 0; u < kVec; u++) {
-      const uint4 v = __ldg(s4 + i + u * kNct);
+      const uint4 v = __ldg(s4 + i + u * NCT);
       w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
     }
     const uint32_t flag = hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16>(s4, i, kVec, W, tab, flag, am, sS);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, kVec, W, tab, flag, am, sS);
   }
-  for (; i < i1; i += kNct) {
+  for (; i < i1; i += NCT) {
     const uint4 v = __ldg(s4 + i);
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
     const uint32_t flag = hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16>(s4, i, 1, W, tab, flag, am, sS);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, 1, W, tab, flag, am, sS);
   }
   return bad;
 }
@@ -778,6 +778,275 @@ __global__ void __launch_bounds__(kThreads, 1)
 #endif
 }
 
+// ---------------------------------------------------------------------- PARTITION
+// For streams without locality (e.g. samples in random order): a WINDOW would see most samples
+// outside any window (L2 atomics, ~0.12 T samples/s). Instead the samples are first partitioned by
+// bucket = slot >> bshift (2^bshift slots, one shared-memory table), then every bucket is counted
+// with its own window, where every sample is inside:
+//   k_pcount   per CTA chunk: samples per bucket (shared counters), invalid words counted
+//   k_pscan    one CTA: bucket regions (4-word aligned starts) and each chunk's offset per bucket
+//   k_pscatter per CTA chunk, tiles of 8K samples: counting sort of the tile in shared memory by
+//              bucket, runs written to the bucket regions (coalesced within a run)
+//   k_pcount_hist  per CTA a contiguous share of the partitioned array, bucket by bucket
+constexpr int kPT = 1024;                  // threads of the partition kernels
+constexpr uint32_t kPMaxBuckets = 2048;
+constexpr uint32_t kPTile = kPT * 8;       // samples per scatter tile
+
+__device__ __forceinline__ uint32_t bucket_of(uint32_t w, Div dv, uint32_t bshift) { return divq(w, dv) >> bshift; }
+
+__global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
+                                                uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
+                                                uint32_t* __restrict__ cnt, unsigned long long* d_n_invalid) {
+  __shared__ uint32_t h[kPMaxBuckets];
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) h[b] = 0;
+  __syncthreads();
+  const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);  // chunk is a multiple of 4 words
+  const uint4* s4 = reinterpret_cast<const uint4*>(s);
+  uint32_t bad = 0;
+  uint64_t i = a / 4 + threadIdx.x;
+  const uint64_t e4 = e / 4;
+  for (; i + 3 * kPT < e4; i += 4 * kPT) {
+    uint4 v[4];
+#pragma unroll
+    for (int u = 0; u < 4; u++) v[u] = __ldg(s4 + i + u * kPT);
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t w[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        if (w[q] < pnr) atomicAdd(&h[bucket_of(w[q], dv, bshift)], 1u);
+        else bad++;
+      }
+    }
+  }
+  for (; i < e4; i += kPT) {
+    const uint4 v = __ldg(s4 + i);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      if (w[q] < pnr) atomicAdd(&h[bucket_of(w[q], dv, bshift)], 1u);
+      else bad++;
+    }
+  }
+  for (uint64_t j = e4 * 4 + threadIdx.x; j < e; j += kPT) {  // the stream's last < 4 words
+    if (s[j] < pnr) atomicAdd(&h[bucket_of(s[j], dv, bshift)], 1u);
+    else bad++;
+  }
+  count_invalid(bad, d_n_invalid);
+  __syncthreads();
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) cnt[(uint64_t)blockIdx.x * B + b] = h[b];
+}
+
+// bstart[b]: first word of bucket b's region (4-aligned), bstart[B] = end; off[c][b] = where chunk c
+// writes its bucket-b samples (in place of cnt)
+__global__ void __launch_bounds__(kPT) k_pscan(uint32_t* __restrict__ cnt, uint32_t nchunk, uint32_t B,
+                                               unsigned long long* __restrict__ bstart, uint32_t* __restrict__ out) {
+  __shared__ unsigned long long tot[kPMaxBuckets], pre[kPMaxBuckets];
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) {
+    unsigned long long t = 0;
+#pragma unroll 8
+    for (uint32_t c = 0; c < nchunk; c++) t += cnt[(uint64_t)c * B + b];
+    tot[b] = t;
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {  // warp scan of the 4-aligned region sizes, 64 buckets per lane at most
+    const uint32_t lane = threadIdx.x, per = (B + 31) / 32;
+    unsigned long long sum = 0;
+    for (uint32_t q = 0; q < per; q++) {
+      const uint32_t b = lane * per + q;
+      if (b < B) sum += (tot[b] + 3) & ~3ull;
+    }
+    unsigned long long inc = sum;
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    unsigned long long p = inc - sum;
+    for (uint32_t q = 0; q < per; q++) {
+      const uint32_t b = lane * per + q;
+      if (b < B) {
+        pre[b] = p;
+        bstart[b] = p;
+        p += (tot[b] + 3) & ~3ull;
+      }
+    }
+    if (lane == 31) bstart[B] = inc;
+  }
+  __syncthreads();
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) {
+    const unsigned long long e = pre[b] + tot[b], e4 = b + 1 < B ? pre[b + 1] : (e + 3) & ~3ull;
+    for (unsigned long long q = e; q < e4; q++) out[q] = 0xffffffffu;  // padding: invalid words
+    unsigned long long p = 0;
+    for (uint32_t c = 0; c < nchunk; c++) {
+      const uint32_t x = cnt[(uint64_t)c * B + b];
+      cnt[(uint64_t)c * B + b] = (uint32_t)p;  // offset within the bucket (< 2^32)
+      p += x;
+    }
+  }
+}
+
+// the 8 contiguous words of thread t in the tile at t0 (two 128-bit loads when the tile is whole)
+__device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t0, uint64_t e, uint32_t (&w)[8]) {
+  const uint64_t base = t0 + (uint64_t)threadIdx.x * 8;
+  if (base + 8 <= e) {
+    const uint4 v0 = __ldg(reinterpret_cast<const uint4*>(s + base));
+    const uint4 v1 = __ldg(reinterpret_cast<const uint4*>(s + base) + 1);
+    w[0] = v0.x; w[1] = v0.y; w[2] = v0.z; w[3] = v0.w; w[4] = v1.x; w[5] = v1.y; w[6] = v1.z; w[7] = v1.w;
+  } else {
+#pragma unroll
+    for (int q = 0; q < 8; q++) w[q] = base + q < e ? s[base + q] : 0xffffffffu;
+  }
+}
+
+__global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
+                                                  uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
+                                                  const uint32_t* __restrict__ off,
+                                                  const unsigned long long* __restrict__ bstart,
+                                                  uint32_t* __restrict__ out) {
+  __shared__ unsigned long long cur[kPMaxBuckets];
+  __shared__ uint32_t th[kPMaxBuckets], toff[kPMaxBuckets];
+  extern __shared__ uint32_t stage[];  // kPTile words (dynamic)
+  __shared__ uint32_t wsum[kPT / 32];
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) {
+    cur[b] = bstart[b] + off[(uint64_t)blockIdx.x * B + b];
+    th[b] = 0;
+  }
+  __syncthreads();
+  const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  uint32_t nw[8];
+  if (a < e) load8(s, a, e, nw);
+  for (uint64_t t0 = a; t0 < e; t0 += kPTile) {
+    uint32_t w[8], bk[8], r[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) w[q] = nw[q];
+    if (t0 + kPTile < e) load8(s, t0 + kPTile, e, nw);  // next tile in flight during this one
+#pragma unroll
+    for (int q = 0; q < 8; q++) bk[q] = w[q] < pnr ? bucket_of(w[q], dv, bshift) : 0xffffffffu;
+    // ranks within the tile's buckets: one shared atomic per run of equal buckets in the thread's
+    // 8 words, and one per warp when the whole warp holds a single bucket (trace order)
+    const uint32_t bk_lane0 = __shfl_sync(0xffffffffu, bk[0], 0);  // outside any condition (all lanes)
+    const bool uni = __all_sync(0xffffffffu, bk[0] == bk[7] && bk[0] == bk_lane0 && bk[0] != 0xffffffffu);
+    bool same = true;
+#pragma unroll
+    for (int q = 1; q < 8; q++) same &= bk[q] == bk[0];
+    if (uni && __all_sync(0xffffffffu, same)) {
+      uint32_t r0 = 0;
+      if (lane == 0) r0 = atomicAdd(&th[bk[0]], 256u);
+      r0 = __shfl_sync(0xffffffffu, r0, 0) + 8 * lane;
+#pragma unroll
+      for (int q = 0; q < 8; q++) r[q] = r0 + q;
+    } else {
+      uint32_t run = 1;
+#pragma unroll
+      for (int q = 7; q >= 0; q--) {  // run length from q to the end of its run
+        r[q] = (q < 7 && bk[q + 1] == bk[q]) ? run + 1 : 1;
+        run = r[q];
+      }
+#pragma unroll
+      for (int q = 0; q < 8; q++) {
+        if (bk[q] == 0xffffffffu) continue;
+        if (q == 0 || bk[q - 1] != bk[q]) r[q] = atomicAdd(&th[bk[q]], r[q]);
+        else r[q] = r[q - 1] + 1;
+      }
+    }
+    __syncthreads();
+    // exclusive scan of th over the buckets (two per thread for B <= 2048)
+    uint32_t x0 = 0, x1 = 0;
+    const uint32_t b0 = 2 * threadIdx.x, b1 = b0 + 1;
+    if (b0 < B) x0 = th[b0];
+    if (b1 < B) x1 = th[b1];
+    uint32_t v = x0 + x1, inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    if (lane == 31) wsum[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+      uint32_t y = wsum[lane], yi = y;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t z = __shfl_up_sync(0xffffffffu, yi, o);
+        if (lane >= o) yi += z;
+      }
+      wsum[lane] = yi - y;
+    }
+    __syncthreads();
+    const uint32_t ex = wsum[warp] + inc - v;
+    if (b0 < B) toff[b0] = ex;
+    if (b1 < B) toff[b1] = ex + x0;
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < 8; q++)
+      if (bk[q] != 0xffffffffu) stage[toff[bk[q]] + r[q]] = w[q];
+    __syncthreads();
+    // the tile's valid samples, bucket-sorted in stage[0, nv): runs to the bucket regions
+    const uint32_t nv = toff[B - 1] + th[B - 1];
+    for (uint32_t p = threadIdx.x; p < nv; p += kPT) {
+      const uint32_t x = stage[p];
+      const uint32_t b = bucket_of(x, dv, bshift);
+      out[cur[b] + (p - toff[b])] = x;
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < B; b += kPT) {
+      cur[b] += th[b];
+      th[b] = 0;
+    }
+    __syncthreads();
+  }
+}
+
+// per CTA: uint4 [c0, c1) of the partitioned array, bucket by bucket; every sample of bucket b is
+// inside its window [b << bshift, (b + 1) << bshift) (16-bit counters, drains only)
+template <bool P16>
+__global__ void __launch_bounds__(kPT, 1)
+    k_pcount_hist(const uint32_t* __restrict__ ps, const unsigned long long* __restrict__ bstart, uint32_t B,
+                  uint64_t chunk4, uint32_t P, uint32_t nr, Div dv, uint32_t bshift, int32_t* __restrict__ H,
+                  uint32_t tw) {
+  extern __shared__ uint32_t tab[];
+  __shared__ Spill sh_S;
+  for (uint32_t i = threadIdx.x; i < tw + 32; i += kPT) tab[i] = i < tw ? 0u : 1u;
+  if (threadIdx.x == 0) sh_S = Spill{P * nr, dv, H, nullptr, nullptr, 0};
+  __syncthreads();
+  const uint4* s4 = reinterpret_cast<const uint4*>(ps);
+  const uint64_t end4 = bstart[B] / 4;
+  const uint64_t c0 = blockIdx.x * chunk4, c1 = min(end4, c0 + chunk4);
+  if (c0 >= c1) return;
+  const uint32_t spare = tw + (threadIdx.x & 31u);
+  // first bucket touching c0: last b with bstart[b] / 4 <= c0
+  uint32_t lo = 0, hi = B;
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (bstart[mid] / 4 <= c0) lo = mid;
+    else hi = mid;
+  }
+  uint32_t ws = 0xffffffffu;
+  Win W{0, 0};
+  uint32_t bad = 0;
+  for (uint32_t b = lo; b < B; b++) {
+    const unsigned long long bs = bstart[b];
+    if (bs / 4 >= c1) break;
+    const unsigned long long we = bstart[b + 1];  // 4-aligned; the padding words hold ~0u (invalid)
+    const uint64_t a4 = c0 > bs / 4 ? c0 : (uint64_t)(bs / 4), e4 = c1 < we / 4 ? c1 : (uint64_t)(we / 4);
+    if (a4 >= e4) continue;
+    const uint32_t nws = b << bshift;
+    if (nws != ws) {
+      __syncthreads();
+      if (ws != 0xffffffffu) flush<P16>(tab, ws, nr, dv.row, W.lim, H, threadIdx.x, kPT);
+      __syncthreads();
+      ws = nws;
+      W = Win{ws * nr, min(1u << bshift, P - ws) * nr};
+    }
+    bad += count_span_w<P16, kPT>(s4, a4, e4, threadIdx.x, W, tab, spare, &sh_S);
+  }
+  (void)bad;  // the padding words (~0u) are counted as invalid here and ignored: invalid samples
+              // were counted by k_pcount
+  __syncthreads();
+  if (ws != 0xffffffffu) flush<P16>(tab, ws, nr, dv.row, W.lim, H, threadIdx.x, kPT);
+}
+
 }  // namespace
 
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
@@ -804,6 +1073,59 @@ gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_h
                                              c->cfg.n_reasons, row, d_hist, d_n_invalid);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
+  return GS_OK;
+}
+
+// GS_HIST_PARTITION (see the kernels): partition by bucket, then count each bucket in its window.
+// d_words is 16-byte aligned here (hist_run peeled the head); the histogram is already zeroed.
+gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,
+                        unsigned long long* d_n_invalid, int dev_sms) {
+  cudaStream_t st = c->stream;
+  const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
+  const Div dv = make_div(nr, c->cfg.hist_row);
+  // bucket = 2^bshift slots whose 16-bit counters fit the largest table
+  uint32_t bshift = 1;
+  while (bshift < 30 && ((((uint64_t)2 << bshift) * nr + 1) / 2) <= kTableWords) bshift++;
+  uint32_t B = (uint32_t)(((uint64_t)P + (1ull << bshift) - 1) >> bshift);
+  if (B > kPMaxBuckets) return fail(c, GS_E_RANGE, "GS_HIST_PARTITION: more than 2048 buckets");
+  const uint32_t tw = (uint32_t)(((((uint64_t)1 << bshift) * nr + 1) / 2 + 31) & ~31ull);
+  const uint64_t nchunk = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 2, (n + kPTile - 1) / kPTile));
+  uint64_t chunk = (n + nchunk - 1) / nchunk;
+  chunk = (chunk + kPTile - 1) / kPTile * kPTile;  // whole tiles (multiple of 4 words)
+  const uint64_t nch = (n + chunk - 1) / chunk;
+  // scratch: counts/offsets [nch][B] u32, bucket starts [B + 1] u64, partitioned copy (+ padding)
+  const uint64_t need = nch * B * 4 + 256 + (B + 1) * 8 + 256 + (n + 4ull * B + 4) * 4;
+  if (c->part_bytes < need) {
+    if (c->d_part) cudaFree(c->d_part);
+    c->d_part = nullptr;
+    c->part_bytes = 0;
+    GS_CUDA(c, cudaMalloc(&c->d_part, need));
+    c->part_bytes = need;
+  }
+  char* p = static_cast<char*>(c->d_part);
+  uint32_t* cnt = reinterpret_cast<uint32_t*>(p);
+  p += (nch * B * 4 + 255) / 256 * 256;
+  unsigned long long* bstart = reinterpret_cast<unsigned long long*>(p);
+  p += ((B + 1) * 8 + 255) / 256 * 256;
+  uint32_t* ps = reinterpret_cast<uint32_t*>(p);
+  k_pcount<<<(unsigned)nch, kPT, 0, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, d_n_invalid);
+  count_launch();
+  k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
+  count_launch();
+  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 4)));
+  k_pscatter<<<(unsigned)nch, kPT, kPTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
+  count_launch();
+  GS_CUDA(c, cudaGetLastError());
+  const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4
+  const uint64_t chunk4 = (total4 + dev_sms - 1) / dev_sms;
+  const size_t smem = (size_t)(tw + 32) * 4;
+  GS_CUDA(c, cudaFuncSetAttribute(k_pcount_hist<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  k_pcount_hist<true><<<(unsigned)dev_sms, kPT, smem, st>>>(ps, bstart, B, chunk4, P, nr, dv, bshift, d_hist, tw);
+  count_launch();
+  GS_CUDA(c, cudaGetLastError());
+  c->last_hist_mode = GS_HIST_PARTITION;
+  c->last_hist_bits = 16;
+  c->last_hist_table_words = tw;
   return GS_OK;
 }
 
@@ -850,6 +1172,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
+  if (mode == GS_HIST_PARTITION) return partition_run(c, d_words, n, d_hist, d_n_invalid, dev_sms);
   const bool dyn = mode == GS_HIST_WINDOW;
   // WINDOW: a table just large enough for the largest kernel (+1 slot for the even window base).
   // The rest of the SM's 256 KB stays L1, which stages the counters' in-flight 128-bit loads: with
@@ -901,6 +1224,9 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
 }
 
 void attrib_free(gs_ctx* c) {
+  if (c->d_part) cudaFree(c->d_part);
+  c->d_part = nullptr;
+  c->part_bytes = 0;
   if (c->d_tileq) cudaFree(c->d_tileq);
   c->d_tileq = nullptr;
   c->tileq_cap = 0;

@@ -109,6 +109,8 @@ struct gs_ctx {
   // ---- attribution / ranking scratch
   int last_hist_mode = 0, last_hist_bits = 0;
   uint32_t last_hist_table_words = 0;  // WINDOW table size of the last histogram launch
+  void* d_part = nullptr;              // PARTITION scratch: counts, bucket starts, partitioned copy
+  size_t part_bytes = 0;
   unsigned long long* d_tileq = nullptr;  // WINDOW histogram work-stealing queue
   uint64_t tileq_cap = 0;
   uint32_t* d_defer = nullptr;  // WINDOW histogram: per-CTA rings of deferred (out-of-window) samples

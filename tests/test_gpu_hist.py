@@ -8,7 +8,7 @@ import pytest
 
 pytestmark = pytest.mark.gpu
 
-MODES = [0, 1, 2, 3]   # AUTO, GLOBAL, PRIVATE, WINDOW
+MODES = [0, 1, 2, 3, 4]   # AUTO, GLOBAL, PRIVATE, WINDOW, PARTITION
 
 
 @pytest.fixture(scope="module")
@@ -53,7 +53,7 @@ def test_c4_full_size_closed_form(gs, order):
     s = gsass.config_sass("C4")
     tab = gsm.table_c4(s.cls, s.first_slot, s.n_instr, 1 << 30, key=0x6E5C0004)
     tr = gsm.Trace(tab, s.first_slot, s.n_instr, order=order, seed=1)
-    _check(gs, s, tr, [0, 3] if order == "trace" else [0, 1, 3])
+    _check(gs, s, tr, [0, 3, 4] if order == "trace" else [0, 1, 3, 4])
 
 
 def test_c5_skew_closed_form(gs):

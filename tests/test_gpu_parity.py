@@ -129,6 +129,7 @@ def _samples(s, n, order, seed, n_bad=100):
     ("C1", 16384, "trace", 0), ("C1", 16384, "shuffled", 1), ("C1", 16384, "shuffled", 2),
     ("C2", 400_000, "trace", 0), ("C2", 400_000, "shuffled", 1), ("C2", 400_000, "shuffled", 2),
     ("C1", 16384, "trace", 3), ("C2", 400_000, "trace", 3), ("C2", 400_000, "shuffled", 3),
+    ("C1", 16384, "shuffled", 4), ("C2", 400_000, "trace", 4), ("C2", 400_000, "shuffled", 4),
 ])
 def test_full_flow_parity(gs, cfg, n, order, mode):
     from gen import sass as gsass
@@ -142,7 +143,8 @@ def test_full_flow_parity(gs, cfg, n, order, mode):
 
 
 @pytest.mark.parametrize("cfg,n,order,mode", [("C1", 16384, "shuffled", 0), ("C2", 400_000, "trace", 0),
-                                              ("C2", 400_000, "shuffled", 1), ("C2", 400_000, "trace", 3)])
+                                              ("C2", 400_000, "shuffled", 1), ("C2", 400_000, "trace", 3),
+                                              ("C2", 400_000, "shuffled", 4)])
 def test_full_flow_parity_compact_rows(gs, cfg, n, order, mode):
     """gs_config.hist_row = R: histogram rows hold only the active reasons."""
     from gen import sass as gsass

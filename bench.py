@@ -192,7 +192,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--order", default="trace", choices=["trace", "shuffled"])
-    ap.add_argument("--hist-mode", type=int, default=0)
+    ap.add_argument("--hist-mode", type=int, default=-1,
+                    help="GS_HIST_* (default: AUTO for trace order, PARTITION for the unordered stream)")
     ap.add_argument("--hist-bits", type=int, default=0, choices=[0, 16, 32])
     ap.add_argument("--hist-row32", action="store_true", help="32-bin histogram rows instead of compact R-bin rows")
     ap.add_argument("--e2e-steps", type=int, default=5)
@@ -225,7 +226,8 @@ def main():
     n_local = b - a
     R = 19
     row = 32 if args.hist_row32 else R     # compact rows: 4*R B per slot to zero, write and reduce
-    ctx = g.Context(device=local, n_reasons=R, hist_mode=args.hist_mode, hist_counter_bits=args.hist_bits,
+    hist_mode = args.hist_mode if args.hist_mode >= 0 else (g.GS_HIST_PARTITION if args.order == "shuffled" else 0)
+    ctx = g.Context(device=local, n_reasons=R, hist_mode=hist_mode, hist_counter_bits=args.hist_bits,
                     hist_row=row)
     ctx.load_sass(s.text)
     P = ctx.n_instr

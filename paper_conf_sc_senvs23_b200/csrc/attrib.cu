@@ -898,22 +898,28 @@ __device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t
   }
 }
 
+// Four barriers per tile: ranks | scan (also resets the rank counters and advances the bucket
+// cursors by the previous tile's counts) | stage | write-out. The write-out reads each sample's
+// bucket from a shared byte/short array and its destination base dst[b] = cursor - tile offset.
 __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
                                                   uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
                                                   const uint32_t* __restrict__ off,
                                                   const unsigned long long* __restrict__ bstart,
                                                   uint32_t* __restrict__ out) {
-  __shared__ unsigned long long cur[kPMaxBuckets];
-  __shared__ uint32_t th[kPMaxBuckets], toff[kPMaxBuckets];
-  extern __shared__ uint32_t stage[];  // kPTile words (dynamic)
+  __shared__ unsigned long long dst[kPMaxBuckets];   // cursor of bucket b minus its tile offset
+  __shared__ uint32_t th[kPMaxBuckets], tcnt[kPMaxBuckets];
+  extern __shared__ uint32_t stage[];  // kPTile words, then kPTile u16 bucket ids (dynamic)
+  uint16_t* sbk = reinterpret_cast<uint16_t*>(stage + kPTile);
   __shared__ uint32_t wsum[kPT / 32];
-  for (uint32_t b = threadIdx.x; b < B; b += kPT) {
-    cur[b] = bstart[b] + off[(uint64_t)blockIdx.x * B + b];
-    th[b] = 0;
-  }
+  __shared__ uint32_t nv_sh;
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  const uint32_t b0 = 2 * threadIdx.x, b1 = b0 + 1;  // the two buckets this thread scans
+  unsigned long long cur0 = 0, cur1 = 0;              // their cursors (registers)
+  if (b0 < B) cur0 = bstart[b0] + off[(uint64_t)blockIdx.x * B + b0];
+  if (b1 < B) cur1 = bstart[b1] + off[(uint64_t)blockIdx.x * B + b1];
+  for (uint32_t b = threadIdx.x; b < B; b += kPT) th[b] = 0;
   __syncthreads();
   const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);
-  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   uint32_t nw[8];
   if (a < e) load8(s, a, e, nw);
   for (uint64_t t0 = a; t0 < e; t0 += kPTile) {
@@ -923,8 +929,8 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
     if (t0 + kPTile < e) load8(s, t0 + kPTile, e, nw);  // next tile in flight during this one
 #pragma unroll
     for (int q = 0; q < 8; q++) bk[q] = w[q] < pnr ? bucket_of(w[q], dv, bshift) : 0xffffffffu;
-    // ranks within the tile's buckets: one shared atomic per run of equal buckets in the thread's
-    // 8 words, and one per warp when the whole warp holds a single bucket (trace order)
+    // ranks within the tile's buckets: one shared atomic per sample, and one per warp when the
+    // whole warp holds a single bucket (trace order)
     const uint32_t bk_lane0 = __shfl_sync(0xffffffffu, bk[0], 0);  // outside any condition (all lanes)
     const bool uni = __all_sync(0xffffffffu, bk[0] == bk[7] && bk[0] == bk_lane0 && bk[0] != 0xffffffffu);
     bool same = true;
@@ -936,65 +942,67 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
       r0 = __shfl_sync(0xffffffffu, r0, 0) + 8 * lane;
 #pragma unroll
       for (int q = 0; q < 8; q++) r[q] = r0 + q;
-    } else {
-      uint32_t run = 1;
+    } else if (__all_sync(0xffffffffu, bk[0] != 0xffffffffu && bk[1] != 0xffffffffu && bk[2] != 0xffffffffu &&
+                                          bk[3] != 0xffffffffu && bk[4] != 0xffffffffu && bk[5] != 0xffffffffu &&
+                                          bk[6] != 0xffffffffu && bk[7] != 0xffffffffu)) {
 #pragma unroll
-      for (int q = 7; q >= 0; q--) {  // run length from q to the end of its run
-        r[q] = (q < 7 && bk[q + 1] == bk[q]) ? run + 1 : 1;
-        run = r[q];
-      }
+      for (int q = 0; q < 8; q++) r[q] = atomicAdd(&th[bk[q]], 1u);  // branch-free: all valid
+    } else {  // one shared atomic per valid sample
 #pragma unroll
-      for (int q = 0; q < 8; q++) {
-        if (bk[q] == 0xffffffffu) continue;
-        if (q == 0 || bk[q - 1] != bk[q]) r[q] = atomicAdd(&th[bk[q]], r[q]);
-        else r[q] = r[q - 1] + 1;
-      }
+      for (int q = 0; q < 8; q++) r[q] = bk[q] != 0xffffffffu ? atomicAdd(&th[bk[q]], 1u) : 0u;
     }
-    __syncthreads();
-    // exclusive scan of th over the buckets (two per thread for B <= 2048)
+    uint32_t vmask = 0;
+#pragma unroll
+    for (int q = 0; q < 8; q++) vmask |= bk[q] != 0xffffffffu ? 1u << q : 0u;
+    const bool allv = __all_sync(0xffffffffu, vmask == 0xffu);
+    __syncthreads();  // A: ranks done (and the previous tile's write-out)
     uint32_t x0 = 0, x1 = 0;
-    const uint32_t b0 = 2 * threadIdx.x, b1 = b0 + 1;
-    if (b0 < B) x0 = th[b0];
-    if (b1 < B) x1 = th[b1];
-    uint32_t v = x0 + x1, inc = v;
+    if (b0 < B) { x0 = th[b0]; th[b0] = 0; }
+    if (b1 < B) { x1 = th[b1]; th[b1] = 0; }
+    const uint32_t v = x0 + x1;
+    uint32_t inc = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
       if (lane >= o) inc += y;
     }
     if (lane == 31) wsum[warp] = inc;
-    __syncthreads();
+    __syncthreads();  // B
     if (warp == 0) {
-      uint32_t y = wsum[lane], yi = y;
+      const uint32_t y = wsum[lane];
+      uint32_t yi = y;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t z = __shfl_up_sync(0xffffffffu, yi, o);
         if (lane >= o) yi += z;
       }
       wsum[lane] = yi - y;
+      if (lane == 31) nv_sh = yi;
     }
-    __syncthreads();
-    const uint32_t ex = wsum[warp] + inc - v;
-    if (b0 < B) toff[b0] = ex;
-    if (b1 < B) toff[b1] = ex + x0;
-    __syncthreads();
+    __syncthreads();  // C
+    const uint32_t ex = wsum[warp] + inc - v;  // tile offset of bucket b0
+    if (b0 < B) { tcnt[b0] = ex; dst[b0] = cur0 - ex; cur0 += x0; }
+    if (b1 < B) { tcnt[b1] = ex + x0; dst[b1] = cur1 - (ex + x0); cur1 += x1; }
+    __syncthreads();  // D: offsets ready
+    if (allv) {
 #pragma unroll
-    for (int q = 0; q < 8; q++)
-      if (bk[q] != 0xffffffffu) stage[toff[bk[q]] + r[q]] = w[q];
-    __syncthreads();
-    // the tile's valid samples, bucket-sorted in stage[0, nv): runs to the bucket regions
-    const uint32_t nv = toff[B - 1] + th[B - 1];
-    for (uint32_t p = threadIdx.x; p < nv; p += kPT) {
-      const uint32_t x = stage[p];
-      const uint32_t b = bucket_of(x, dv, bshift);
-      out[cur[b] + (p - toff[b])] = x;
+      for (int q = 0; q < 8; q++) {
+        const uint32_t p = tcnt[bk[q]] + r[q];
+        stage[p] = w[q];
+        sbk[p] = (uint16_t)bk[q];
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < 8; q++)
+        if (bk[q] != 0xffffffffu) {
+          const uint32_t p = tcnt[bk[q]] + r[q];
+          stage[p] = w[q];
+          sbk[p] = (uint16_t)bk[q];
+        }
     }
-    __syncthreads();
-    for (uint32_t b = threadIdx.x; b < B; b += kPT) {
-      cur[b] += th[b];
-      th[b] = 0;
-    }
-    __syncthreads();
+    __syncthreads();  // E: staged
+    const uint32_t nv = nv_sh;
+    for (uint32_t p = threadIdx.x; p < nv; p += kPT) out[dst[sbk[p]] + p] = stage[p];
   }
 }
 
@@ -1112,8 +1120,8 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
-  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 4)));
-  k_pscatter<<<(unsigned)nch, kPT, kPTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
+  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 6)));
+  k_pscatter<<<(unsigned)nch, kPT, kPTile * 6, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4

@@ -448,6 +448,9 @@ __device__ __forceinline__ void count_ring(const uint32_t* ring, uint32_t b, uin
 // atomic (with the rare state live, it delayed the last load behind the atomics, exposing the HBM
 // latency twice per batch).
 constexpr uint32_t kNct = kThreads - 32;  // counting threads of the WINDOW kernel
+// 16-bit exactness: after a half reaches 0x8000 every counting thread adds at most one batch
+// (4 * kVec samples) before it drains it, so the half stays below 0x10000
+static_assert(kNct * 4 * kVec < 0x8000, "16-bit counters: too many increments in flight");
 
 // the rare part of one batch of nv uint4 at s4[i + u * kNct], re-read from L1/L2: outside the
 // window (deferred / invalid), or a 16-bit half that needs draining. Returns the invalid count.
@@ -1047,7 +1050,8 @@ __global__ void __launch_bounds__(kPT, 1)
       ws = nws;
       W = Win{ws * nr, min(1u << bshift, P - ws) * nr};
     }
-    bad += count_span_w<P16, kPT>(s4, a4, e4, threadIdx.x, W, tab, spare, &sh_S);
+    // warps 1..31 count (kNct threads: the 16-bit exactness bound below), warp 0 only flushes
+    if (threadIdx.x >= 32) bad += count_span_w<P16, kNct>(s4, a4, e4, threadIdx.x - 32, W, tab, spare, &sh_S);
   }
   (void)bad;  // the padding words (~0u) are counted as invalid here and ignored: invalid samples
               // were counted by k_pcount

@@ -1099,7 +1099,7 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   uint32_t bshift = 1;
   while (bshift < 30 && ((((uint64_t)2 << bshift) * nr + 1) / 2) <= kTableWords) bshift++;
   uint32_t B = (uint32_t)(((uint64_t)P + (1ull << bshift) - 1) >> bshift);
-  if (B > kPMaxBuckets) return fail(c, GS_E_RANGE, "GS_HIST_PARTITION: more than 2048 buckets");
+  if (B > kPMaxBuckets) return GS_E_RANGE;  // caller falls back to WINDOW (modules > 2048 tables)
   const uint32_t tw = (uint32_t)(((((uint64_t)1 << bshift) * nr + 1) / 2 + 31) & ~31ull);
   const uint64_t nchunk = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 2, (n + kPTile - 1) / kPTile));
   uint64_t chunk = (n + nchunk - 1) / nchunk;
@@ -1184,7 +1184,14 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   }
-  if (mode == GS_HIST_PARTITION) return partition_run(c, d_words, n, d_hist, d_n_invalid, dev_sms);
+  if (mode == GS_HIST_PARTITION) {
+    const gs_status ps = partition_run(c, d_words, n, d_hist, d_n_invalid, dev_sms);
+    if (ps != GS_E_RANGE) return ps;
+    mode = GS_HIST_WINDOW;  // more than 2048 bucket tables: the windowed strategy instead
+    bits = max_kn > nslots32 ? 16 : 32;
+    c->last_hist_mode = (int)mode;
+    c->last_hist_bits = (int)bits;
+  }
   const bool dyn = mode == GS_HIST_WINDOW;
   // WINDOW: a table just large enough for the largest kernel (+1 slot for the even window base).
   // The rest of the SM's 256 KB stays L1, which stages the counters' in-flight 128-bit loads: with

@@ -109,3 +109,29 @@ def test_unaligned_views_and_invalid_words(gs, offset):
         hist2, _ = ctx.attribute_samples(view, hist=hist.clone(), accumulate=True)
         assert torch.equal(hist2, 2 * want)
         ctx.close()
+
+
+@pytest.mark.parametrize("n", [1, 3, 5, 4097, 100_003])
+@pytest.mark.parametrize("nr", [19, 8])
+def test_small_and_ragged_streams_all_modes(gs, n, nr):
+    """Tiny and ragged sample counts (no whole 128-bit vector, partial tiles) with 8 or 19 active
+    reasons: every strategy equals the bincount of the words (closed form), invalid words counted."""
+    import torch
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    rng = np.random.default_rng(n + nr)
+    w = rng.integers(0, s.P * nr, n).astype(np.int64)
+    w[::7] = s.P * nr + 5                      # invalid words
+    bad = int((w >= s.P * nr).sum())
+    want_c = np.bincount(w[w < s.P * nr], minlength=s.P * nr).astype(np.int32)
+    words = torch.from_numpy(w.astype(np.int32)).cuda()
+    for mode in MODES:
+        for row in (32, nr):
+            ctx = gs.Context(hist_mode=mode, n_reasons=nr, hist_row=row)
+            ctx.load_sass(s.text)
+            hist, ninv = ctx.attribute_samples(words)
+            torch.cuda.synchronize()
+            got = hist.view(-1, row)[:, :nr].reshape(-1).cpu().numpy()
+            assert int(ninv.item()) == bad, (mode, row)
+            assert np.array_equal(got, want_c), (mode, row, n)
+            ctx.close()

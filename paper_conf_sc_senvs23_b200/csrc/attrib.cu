@@ -902,8 +902,8 @@ __device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t
 }
 
 // Four barriers per tile: ranks | scan (also resets the rank counters and advances the bucket
-// cursors by the previous tile's counts) | stage | write-out. The write-out reads each sample's
-// bucket from a shared byte/short array and its destination base dst[b] = cursor - tile offset.
+// cursors by the previous tile's counts) | stage | write-out. The write-out recomputes each
+// sample's bucket and reads its destination base dst[b] = cursor - tile offset.
 __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
                                                   uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
                                                   const uint32_t* __restrict__ off,
@@ -911,8 +911,7 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
                                                   uint32_t* __restrict__ out) {
   __shared__ unsigned long long dst[kPMaxBuckets];   // cursor of bucket b minus its tile offset
   __shared__ uint32_t th[kPMaxBuckets], tcnt[kPMaxBuckets];
-  extern __shared__ uint32_t stage[];  // kPTile words, then kPTile u16 bucket ids (dynamic)
-  uint16_t* sbk = reinterpret_cast<uint16_t*>(stage + kPTile);
+  extern __shared__ uint32_t stage[];  // kPTile words (dynamic)
   __shared__ uint32_t wsum[kPT / 32];
   __shared__ uint32_t nv_sh;
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
@@ -989,23 +988,18 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
     __syncthreads();  // D: offsets ready
     if (allv) {
 #pragma unroll
-      for (int q = 0; q < 8; q++) {
-        const uint32_t p = tcnt[bk[q]] + r[q];
-        stage[p] = w[q];
-        sbk[p] = (uint16_t)bk[q];
-      }
+      for (int q = 0; q < 8; q++) stage[tcnt[bk[q]] + r[q]] = w[q];
     } else {
 #pragma unroll
       for (int q = 0; q < 8; q++)
-        if (bk[q] != 0xffffffffu) {
-          const uint32_t p = tcnt[bk[q]] + r[q];
-          stage[p] = w[q];
-          sbk[p] = (uint16_t)bk[q];
-        }
+        if (bk[q] != 0xffffffffu) stage[tcnt[bk[q]] + r[q]] = w[q];
     }
     __syncthreads();  // E: staged
     const uint32_t nv = nv_sh;
-    for (uint32_t p = threadIdx.x; p < nv; p += kPT) out[dst[sbk[p]] + p] = stage[p];
+    for (uint32_t p = threadIdx.x; p < nv; p += kPT) {  // the bucket is recomputed (ALU, not smem)
+      const uint32_t x = stage[p];
+      out[dst[bucket_of(x, dv, bshift)] + p] = x;
+    }
   }
 }
 
@@ -1124,8 +1118,8 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
-  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 6)));
-  k_pscatter<<<(unsigned)nch, kPT, kPTile * 6, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
+  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 4)));
+  k_pscatter<<<(unsigned)nch, kPT, kPTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4

@@ -302,23 +302,31 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
   if (c->n_instr >= (1ull << 27)) return fail(c, GS_E_RANGE, "packed samples address at most 2^27 slots");
   GS_CUDA(c, cudaSetDevice(c->device));
   if (!n || is_device_ptr(samples)) return hist_run(c, samples, n, d_hist, d_n_invalid, accumulate, true);
-  // host input: stream chunks through two device staging buffers; the H2D copy of chunk i+1
-  // (copy engine) overlaps the histogram of chunk i
+  // host input: chunks through two device staging buffers; the H2D copy of chunk i+1 runs on a
+  // copy stream (copy engine) while the histogram of chunk i runs on the context's stream
   const size_t chunk = size_t(16) << 20;  // words
   if (c->stage_words < chunk) {
     attrib_free(c);
     for (int b = 0; b < 2; b++) {
       GS_CUDA(c, cudaMalloc((void**)&c->d_stage[b], chunk * 4));
       GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_stage[b], cudaEventDisableTiming));
+      GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_copied[b], cudaEventDisableTiming));
     }
+    GS_CUDA(c, cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
     c->stage_words = chunk;
   }
   if (!accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * c->cfg.hist_row * 4, c->stream));
+  // the copy stream starts after everything already enqueued on the context's stream
+  GS_CUDA(c, cudaEventRecord(c->ev_stage[0], c->stream));
+  GS_CUDA(c, cudaEventRecord(c->ev_stage[1], c->stream));
   uint64_t done = 0;
   int b = 0;
   while (done < n) {
     const uint64_t m = std::min<uint64_t>(chunk, n - done);
-    GS_CUDA(c, cudaMemcpyAsync(c->d_stage[b], samples + done, m * 4, cudaMemcpyHostToDevice, c->stream));
+    GS_CUDA(c, cudaStreamWaitEvent(c->copy_stream, c->ev_stage[b], 0));  // buffer b free again
+    GS_CUDA(c, cudaMemcpyAsync(c->d_stage[b], samples + done, m * 4, cudaMemcpyHostToDevice, c->copy_stream));
+    GS_CUDA(c, cudaEventRecord(c->ev_copied[b], c->copy_stream));
+    GS_CUDA(c, cudaStreamWaitEvent(c->stream, c->ev_copied[b], 0));
     gs_status s = hist_run(c, c->d_stage[b], m, d_hist, d_n_invalid, 1, false);
     if (s != GS_OK) return s;
     GS_CUDA(c, cudaEventRecord(c->ev_stage[b], c->stream));

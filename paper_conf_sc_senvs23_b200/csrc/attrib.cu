@@ -1250,10 +1250,14 @@ void attrib_free(gs_ctx* c) {
     if (c->h_stage[b]) cudaFreeHost(c->h_stage[b]);
     if (c->d_stage[b]) cudaFree(c->d_stage[b]);
     if (c->ev_stage[b]) cudaEventDestroy(c->ev_stage[b]);
+    if (c->ev_copied[b]) cudaEventDestroy(c->ev_copied[b]);
     c->h_stage[b] = nullptr;
     c->d_stage[b] = nullptr;
     c->ev_stage[b] = nullptr;
+    c->ev_copied[b] = nullptr;
   }
+  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
+  c->copy_stream = nullptr;
   c->stage_words = 0;
 }
 

@@ -142,7 +142,9 @@ struct gs_ctx {
   size_t h_pin_bytes = 0;
   uint32_t* h_stage[2] = {nullptr, nullptr};  // pinned staging for host sample input
   uint32_t* d_stage[2] = {nullptr, nullptr};
-  cudaEvent_t ev_stage[2] = {nullptr, nullptr};
+  cudaEvent_t ev_stage[2] = {nullptr, nullptr};   // histogram of staging buffer b done (ctx stream)
+  cudaEvent_t ev_copied[2] = {nullptr, nullptr};  // H2D into staging buffer b done (copy stream)
+  cudaStream_t copy_stream = nullptr;             // host input: H2D copies overlap the histogram
   size_t stage_words = 0;
 };
 

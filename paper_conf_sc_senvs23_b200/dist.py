@@ -55,13 +55,16 @@ def reduce_scatter_hist(hist, row: int, ranges, group=None):
     rows of slots ranges[g] = [s, e); returns that slice (a view of `hist`). One collective: NCCL's
     reduce_scatter (uneven parts run as grouped ncclReduce calls); on other backends one reduce per
     part. Single process: the slice of the whole histogram."""
+    import torch
     import torch.distributed as dist
     parts = [hist[s * row:e * row] for s, e in ranges]
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
         return parts[0] if len(parts) == 1 else hist
     me = dist.get_rank(group)
     if dist.get_backend(group) == "nccl":
-        dist.reduce_scatter(parts[me], parts, op=dist.ReduceOp.SUM, group=group)
+        out = torch.empty_like(parts[me])  # a separate output: no aliasing of an input part
+        dist.reduce_scatter(out, parts, op=dist.ReduceOp.SUM, group=group)
+        return out
     else:
         works = [dist.reduce(p, dst=g, op=dist.ReduceOp.SUM, group=group, async_op=True)
                  for g, p in enumerate(parts) if p.numel()]

@@ -243,6 +243,7 @@ def main():
     hist_events = []
     phase_events = []     # per timed step: events at detect | attribute | merge | rank boundaries
 
+    last_part = [None]   # this rank's summed histogram rows of the last step
     def step(record_hist=False):
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)] if record_hist else None
         if ev:
@@ -256,6 +257,7 @@ def main():
             ev[2].record(stream)
             hist_events.append((ev[1], ev[2]))
         part = gdist.reduce_scatter_hist(hist, row, gdist.slot_ranges(s.first_slot, s.n_instr, world))
+        last_part[0] = part
         if ev:
             ev[3].record(stream)
         ctx.rank_sites(part, k=None, out=ranked_dev, slot_begin=s0, slot_end=s1)
@@ -297,7 +299,7 @@ def main():
 
     # correctness guard on the bench configuration (closed form: mass and invalid count; with a
     # reduce-scatter each rank holds the summed rows of its own slot range)
-    mass = torch.tensor([int(hist[s0 * row:s1 * row].to(torch.int64).sum().item())], dtype=torch.int64, device="cuda")
+    mass = torch.tensor([int(last_part[0].to(torch.int64).sum().item())], dtype=torch.int64, device="cuda")
     if world > 1:
         dist.all_reduce(mass)
     assert int(mass.item()) == tr.N and int(ninv.item()) == 0, (int(mass.item()), tr.N, int(ninv.item()))

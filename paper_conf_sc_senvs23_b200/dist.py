@@ -52,7 +52,8 @@ def slot_ranges(first_slot, n_instr, world: int) -> list[tuple[int, int]]:
 
 def reduce_scatter_hist(hist, row: int, ranges, group=None):
     """Sum the per-rank histograms (rows of `row` bins, one per slot) and leave on rank g the summed
-    rows of slots ranges[g] = [s, e); returns that slice (a view of `hist`). One collective: NCCL's
+    rows of slots ranges[g] = [s, e); returns that slice (NCCL: a new tensor; otherwise a view of
+    `hist`). One collective: NCCL's
     reduce_scatter (uneven parts run as grouped ncclReduce calls); on other backends one reduce per
     part. Single process: the slice of the whole histogram."""
     import torch

@@ -210,9 +210,16 @@ def main():
 
     import torch
     import torch.distributed as dist
+    # GS_BENCH_DEVICE / GS_BENCH_BACKEND: functional checks of the multi-rank flow on one GPU
+    # (all ranks on one device over gloo); the default is one GPU per rank over NCCL
+    local = int(os.environ.get("GS_BENCH_DEVICE", local))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("GS_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     import paper_conf_sc_senvs23_b200 as g
     from paper_conf_sc_senvs23_b200 import binding, build as gbuild, dist as gdist
     from gen.device import DeviceTrace
@@ -312,6 +319,8 @@ def main():
     tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}_{args.order}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        if traffic and world > 1:   # captured on the whole stream: this rank's launch holds n_local samples
+            traffic = traffic * n_local / tr.N
 
     # e2e: same step through the C ABI with HOST buffers (pinned), copies inside the timed region
     host_words = torch.empty(n_local, dtype=torch.int32, pin_memory=True)

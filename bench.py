@@ -224,6 +224,7 @@ def main():
     from paper_conf_sc_senvs23_b200 import binding, build as gbuild, dist as gdist
     from gen.device import DeviceTrace
     gbuild.build()
+    torch.cuda.set_stream(torch.cuda.Stream())   # a non-default stream: the library may replay CUDA graphs on it
 
     t_setup = time.perf_counter()
     s, tr = build_workload(args.config, args.order)

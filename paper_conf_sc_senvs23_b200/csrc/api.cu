@@ -16,6 +16,8 @@ namespace gs {
 
 static std::atomic<uint64_t> g_launches{0};
 void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+void count_launch_undo(uint64_t n) { g_launches.fetch_sub(n, std::memory_order_relaxed); }
+uint64_t launch_count_now() { return g_launches.load(std::memory_order_relaxed); }
 
 gs_status fail(gs_ctx* c, gs_status s, const std::string& msg) {
   if (c) c->err = msg;

@@ -119,6 +119,9 @@ struct gs_ctx {
   uint32_t* d_rank_vals[2] = {nullptr, nullptr};
   uint64_t rank_cap = 0;
   int rank_bits_guess[2] = {-1, -1};  // bit widths of max(rel), max(tot) used by the last rank call
+  cudaGraphExec_t rank_exec = nullptr;  // the rank sequence as a CUDA graph, replayed while its key repeats
+  std::vector<uintptr_t> rank_key;
+  uint64_t rank_graph_launches = 0;
   void* d_sort_tmp = nullptr;
   size_t sort_tmp_bytes = 0;
   unsigned long long* d_ktot = nullptr;
@@ -152,6 +155,8 @@ namespace gs {
 
 // process-wide launch counter (gs_launch_count)
 void count_launch(uint64_t n = 1);
+void count_launch_undo(uint64_t n);
+uint64_t launch_count_now();
 
 // error helpers (set ctx->err, return status)
 gs_status fail(gs_ctx* c, gs_status s, const std::string& msg);

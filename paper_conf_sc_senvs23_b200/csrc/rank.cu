@@ -229,18 +229,15 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
   cudaStream_t st = c->stream;
   const uint64_t ns = c->n_sites;
   const uint64_t kk = std::min<uint64_t>(k, ns);
-  if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8));
-  unsigned long long* d_max = c->d_ktot + std::max<uint32_t>(c->n_kernels, 1);
-  GS_CUDA(c, cudaMemsetAsync(c->d_ktot, 0, ((uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2) * 8, st));
   const uint32_t row = c->cfg.hist_row;
-  if (c->det_ke > c->det_kb) {  // kernel totals of the detected kernels only
-    uint32_t max_n = 1;
-    for (uint32_t k = c->det_kb; k < c->det_ke; k++) max_n = std::max(max_n, c->kd_h[k].n);
-    dim3 grid(c->det_ke - c->det_kb, (max_n + kKtotSlotsPerCta - 1) / kKtotSlotsPerCta);
-    k_ktot<<<grid, kKtotThreads, 0, st>>>(d_hist, slot0, row, c->d_kd, c->det_kb, c->det_ke, c->d_ktot);
-    count_launch();
-    GS_CUDA(c, cudaGetLastError());
-  }
+  const uint64_t nkt = (uint64_t)std::max<uint32_t>(c->n_kernels, 1) + 2;
+  const bool cons = c->cfg.join_mode == GS_JOIN_CONSUMER;
+  if (cons && !c->cons_ready) return fail(c, GS_E_STATE, "consumer join: gs_detect ran in another join mode");
+  const bool line = (c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups) || cons;
+  // ---- every allocation first (the enqueue below may be captured into a CUDA graph)
+  if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, nkt * 8));
+  unsigned long long* d_max = c->d_ktot + (nkt - 2);
+  size_t cub_bytes = 0;
   if (ns) {
     if (c->rank_cap < ns) {
       for (int b = 0; b < 2; b++) {
@@ -256,12 +253,8 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
       }
       c->rank_cap = ns;
     }
-    unsigned long long* k0 = c->d_rank_keys[0];
-    unsigned long long* k1 = c->d_rank_keys[1];
-    uint32_t* v0 = c->d_rank_vals[0];
-    uint32_t* v1 = c->d_rank_vals[1];
-    size_t cub_bytes = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, k0, k1, v0, v1, (int)ns, 0, 64, st);
+    cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, c->d_rank_keys[0], c->d_rank_keys[1], c->d_rank_vals[0],
+                                    c->d_rank_vals[1], (int)ns, 0, 64, st);
     const size_t arr = ((ns * 8 + 255) / 256) * 256;  // rel and tot arrays live in the temp block
     if (c->sort_tmp_bytes < cub_bytes + 2 * arr) {
       if (c->d_sort_tmp) cudaFree(c->d_sort_tmp);
@@ -270,15 +263,74 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
       GS_CUDA(c, cudaMalloc(&c->d_sort_tmp, cub_bytes + 2 * arr));
       c->sort_tmp_bytes = cub_bytes + 2 * arr;
     }
-    unsigned long long* d_rel = reinterpret_cast<unsigned long long*>(c->d_sort_tmp);
-    unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
-    void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
-    const unsigned grid = (unsigned)((ns + 255) / 256);
-    const bool cons = c->cfg.join_mode == GS_JOIN_CONSUMER;
-    if (cons && !c->cons_ready) return fail(c, GS_E_STATE, "consumer join: gs_detect ran in another join mode");
-    const bool line = (c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups) || cons;
+    if (line) GS_CUDA(c, dev_grow(&c->d_jrow, &c->jrow_cap, ns * 32));
+    if (kk && out_is_host) GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
+  }
+  GS_CUDA(c, pin_grow(c, 16));
+  unsigned long long* mx = static_cast<unsigned long long*>(c->h_pin);
+  unsigned long long* k0 = c->d_rank_keys[0];
+  unsigned long long* k1 = c->d_rank_keys[1];
+  uint32_t* v0 = c->d_rank_vals[0];
+  uint32_t* v1 = c->d_rank_vals[1];
+  const size_t arr = ((ns * 8 + 255) / 256) * 256;
+  unsigned long long* d_rel = reinterpret_cast<unsigned long long*>(c->d_sort_tmp);
+  unsigned long long* d_tot = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_sort_tmp) + arr);
+  void* cub_tmp = static_cast<char*>(c->d_sort_tmp) + 2 * arr;
+  const unsigned grid = (unsigned)((ns + 255) / 256);
+  auto passes = [](int bits) { return (uint64_t)(bits + 7) / 8 + 2; };  // onesweep digits + hist + scan
+  // sort by the packed key and emit the first kk rows
+  const auto sort_emit = [&](int br, int bt) -> gs_status {
+    const uint32_t* order = v0;
+    size_t b1 = cub_bytes;
+    if (br + bt <= 64) {
+      k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
+      count_launch();
+      if (br + bt > 0) {
+        cub::DoubleBuffer<unsigned long long> dk(k0, k1);
+        cub::DoubleBuffer<uint32_t> dv(v0, v1);
+        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, dk, dv, (int)ns, 0, br + bt, st));
+        count_launch(passes(br + bt));
+        order = dv.Current();
+      }
+    } else {
+      k_keys_field<<<grid, 256, 0, st>>>(d_tot, nullptr, ns, mask_of(bt), k0, v0);
+      count_launch();
+      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v0, v1, (int)ns, 0, bt, st));
+      count_launch(passes(bt));
+      k_keys_field<<<grid, 256, 0, st>>>(d_rel, v1, ns, mask_of(br), k0, nullptr);
+      count_launch();
+      b1 = cub_bytes;
+      GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v1, v0, (int)ns, 0, br, st));
+      count_launch(passes(br));
+      order = v0;
+    }
+    GS_CUDA(c, cudaGetLastError());
+    if (kk) {
+      gs_ranked_site* dst = out_is_host ? c->d_ranked : out;
+      k_emit<<<(unsigned)((kk + 255) / 256), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
+                                                          line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
+                                                          c->d_ktot, dst);
+      count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      if (out_is_host)
+        GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));
+    }
+    return GS_OK;
+  };
+  const int gr = c->rank_bits_guess[0], gt = c->rank_bits_guess[1];
+  // kernel totals, join, maxima read-back, and (with the previous call's key widths) sort + emit
+  const auto enqueue_main = [&]() -> gs_status {
+    GS_CUDA(c, cudaMemsetAsync(c->d_ktot, 0, nkt * 8, st));
+    if (c->det_ke > c->det_kb) {  // kernel totals of the detected kernels only
+      uint32_t max_n = 1;
+      for (uint32_t q = c->det_kb; q < c->det_ke; q++) max_n = std::max(max_n, c->kd_h[q].n);
+      dim3 g2(c->det_ke - c->det_kb, (max_n + kKtotSlotsPerCta - 1) / kKtotSlotsPerCta);
+      k_ktot<<<g2, kKtotThreads, 0, st>>>(d_hist, slot0, row, c->d_kd, c->det_kb, c->det_ke, c->d_ktot);
+      count_launch();
+      GS_CUDA(c, cudaGetLastError());
+    }
+    if (!ns) return GS_OK;
     if (line) {
-      GS_CUDA(c, dev_grow(&c->d_jrow, &c->jrow_cap, ns * 32));
       k_join_line<<<(unsigned)((ns + 7) / 8), 256, 0, st>>>(
           c->d_sites, ns, d_hist, slot0, row, c->d_kd, cons ? nullptr : c->d_lgrp, cons ? c->d_cgoff : c->d_goff,
           cons ? c->d_cgslot : c->d_gslot, d_rel, d_tot, c->d_jrow, d_max);
@@ -292,57 +344,59 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     // one async copy; the sort itself is enqueued right away with the widths of the previous call
     // (padded to whole 8-bit radix digits, which costs no extra pass) and redone with the exact
     // widths only when this call's maxima do not fit them (one host synchronisation otherwise).
-    GS_CUDA(c, pin_grow(c, 16));
-    unsigned long long* mx = static_cast<unsigned long long*>(c->h_pin);
     GS_CUDA(c, cudaMemcpyAsync(mx, d_max, 16, cudaMemcpyDeviceToHost, st));
-    auto passes = [](int bits) { return (uint64_t)(bits + 7) / 8 + 2; };  // onesweep digits + hist + scan
-    const auto sort_emit = [&](int br, int bt) -> gs_status {
-      const uint32_t* order = v0;
-      size_t b1 = cub_bytes;
-      if (br + bt <= 64) {
-        k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
-        count_launch();
-        if (br + bt > 0) {
-          cub::DoubleBuffer<unsigned long long> dk(k0, k1);
-          cub::DoubleBuffer<uint32_t> dv(v0, v1);
-          GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, dk, dv, (int)ns, 0, br + bt, st));
-          count_launch(passes(br + bt));
-          order = dv.Current();
-        }
-      } else {
-        k_keys_field<<<grid, 256, 0, st>>>(d_tot, nullptr, ns, mask_of(bt), k0, v0);
-        count_launch();
-        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v0, v1, (int)ns, 0, bt, st));
-        count_launch(passes(bt));
-        k_keys_field<<<grid, 256, 0, st>>>(d_rel, v1, ns, mask_of(br), k0, nullptr);
-        count_launch();
-        b1 = cub_bytes;
-        GS_CUDA(c, cub::DeviceRadixSort::SortPairs(cub_tmp, b1, k0, k1, v1, v0, (int)ns, 0, br, st));
-        count_launch(passes(br));
-        order = v0;
+    if (gr >= 0) return sort_emit(gr, gt);
+    return GS_OK;
+  };
+  // The whole sequence is replayed as one CUDA graph while its parameters repeat (e.g. one rank
+  // call per step): a dozen launches of small kernels become one graph launch.
+  const uintptr_t key[] = {(uintptr_t)ns, (uintptr_t)kk, (uintptr_t)d_hist, slot0, row, (uintptr_t)out,
+                           out_is_host, (uintptr_t)(int64_t)gr, (uintptr_t)(int64_t)gt, line, cons, c->det_kb,
+                           c->det_ke, (uintptr_t)c->d_sites, (uintptr_t)c->d_sort_tmp, (uintptr_t)k0, (uintptr_t)v0,
+                           (uintptr_t)c->d_jrow, (uintptr_t)c->d_ranked, (uintptr_t)mx, (uintptr_t)c->d_ktot,
+                           (uintptr_t)c->d_kd, (uintptr_t)c->d_cgoff, (uintptr_t)c->d_cgslot, (uintptr_t)c->d_goff,
+                           (uintptr_t)c->d_gslot, (uintptr_t)c->d_lgrp, (uintptr_t)c->n_kernels};
+  constexpr size_t nkey = sizeof(key) / sizeof(key[0]);
+  static const bool no_graph = getenv("GS_NO_GRAPH") != nullptr;
+  bool host_ok = true;  // a captured D2H copy needs page-locked (or device) destination memory
+  if (kk && out_is_host) {
+    cudaPointerAttributes pa;
+    host_ok = cudaPointerGetAttributes(&pa, out) == cudaSuccess && pa.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+  }
+  // (the legacy / per-thread default streams cannot be captured: plain launches there)
+  const bool capturable = st != nullptr && st != cudaStreamLegacy && st != cudaStreamPerThread;
+  const bool use_graph = !no_graph && gr >= 0 && ns && host_ok && capturable;
+  if (use_graph) {
+    bool hit = c->rank_exec && c->rank_key.size() == nkey;
+    for (size_t q = 0; hit && q < nkey; q++) hit = c->rank_key[q] == key[q];
+    if (!hit) {
+      if (c->rank_exec) cudaGraphExecDestroy(c->rank_exec);
+      c->rank_exec = nullptr;
+      const uint64_t l0 = launch_count_now();
+      GS_CUDA(c, cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+      const gs_status s1 = enqueue_main();
+      cudaGraph_t g = nullptr;
+      const cudaError_t e = cudaStreamEndCapture(st, &g);
+      if (s1 != GS_OK) {
+        if (g) cudaGraphDestroy(g);
+        return s1;
       }
-      GS_CUDA(c, cudaGetLastError());
-      if (kk) {
-        gs_ranked_site* dst = out;
-        if (out_is_host) {
-          GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
-          dst = c->d_ranked;
-        }
-k_emit<<<(unsigned)((kk + 255) / 256), 256, 0, st>>>(order, kk, c->d_sites, d_hist, slot0, row,
-                                                          line ? c->d_jrow : nullptr, d_rel, d_tot, c->d_kd,
-                                                          c->d_ktot, dst);
-        count_launch();
-        GS_CUDA(c, cudaGetLastError());
-        if (out_is_host)
-          GS_CUDA(c, cudaMemcpyAsync(out, dst, kk * sizeof(gs_ranked_site), cudaMemcpyDeviceToHost, st));
-      }
-      return GS_OK;
-    };
-    const int gr = c->rank_bits_guess[0], gt = c->rank_bits_guess[1];
-    if (gr >= 0) {
-      gs_status s2 = sort_emit(gr, gt);
-      if (s2 != GS_OK) return s2;
+      GS_CUDA(c, e);
+      const cudaError_t ei = cudaGraphInstantiate(&c->rank_exec, g, 0);
+      cudaGraphDestroy(g);
+      GS_CUDA(c, ei);
+      c->rank_key.assign(key, key + nkey);
+      c->rank_graph_launches = launch_count_now() - l0;
+      count_launch_undo(c->rank_graph_launches);  // counted again when the graph runs
     }
+    GS_CUDA(c, cudaGraphLaunch(c->rank_exec, st));
+    count_launch(c->rank_graph_launches);
+  } else {
+    const gs_status s1 = enqueue_main();
+    if (s1 != GS_OK) return s1;
+  }
+  if (ns) {
     GS_CUDA(c, cudaStreamSynchronize(st));
     const int br = bits_of(mx[0]), bt = bits_of(mx[1]);
     if (br + bt <= 64) {  // next call's widths: this call's, slack spread to fill the last digit
@@ -364,6 +418,9 @@ k_emit<<<(unsigned)((kk + 255) / 256), 256, 0, st>>>(order, kk, c->d_sites, d_hi
 }
 
 void rank_free(gs_ctx* c) {
+  if (c->rank_exec) cudaGraphExecDestroy(c->rank_exec);
+  c->rank_exec = nullptr;
+  c->rank_key.clear();
   for (int b = 0; b < 2; b++) {
     if (c->d_rank_keys[b]) cudaFree(c->d_rank_keys[b]);
     if (c->d_rank_vals[b]) cudaFree(c->d_rank_vals[b]);

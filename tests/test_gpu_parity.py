@@ -452,3 +452,43 @@ def test_register_pressure_parity_generated(gs):
         text = brute.render(ks)
         got, _ = _gpu_live(gs, text)
         assert got == _oracle_live(text)
+
+
+def test_rank_graph_replay(gs):
+    """gs_rank_sites on a non-default stream replays its captured CUDA graph while the parameters
+    repeat: repeated calls, new histogram contents in the same buffer (larger maxima: the key widths
+    grow and the sort is redone) and a host output all equal a plain run on the default stream."""
+    import torch
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    s = gsass.config_sass("C2")
+    raw_a, _ = _samples(s, 50_000, "shuffled", seed=71, n_bad=0)
+    raw_b, _ = _samples(s, 2_000_000, "shuffled", seed=73, n_bad=0)
+    st = torch.cuda.Stream()
+
+    def canon(ctx, hist, n, rows):
+        return Canon(report.canonical(ctx, hist=hist, n_samples=n, n_invalid=0, ranked=rows)).R
+
+    with torch.cuda.stream(st):
+        ctx = _ctx(gs, hist_row=19)
+        ctx.load_sass(s.text)
+        ctx.detect()
+        hist = torch.empty(ctx.n_instr * 19, dtype=torch.int32, device="cuda")
+        ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ns = ctx.sites_device()[2]
+        dev_rows = torch.empty(ns * gs.RANKED_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+        got = []
+        for q, raw in enumerate((raw_a, raw_a, raw_a, raw_b, raw_b, raw_a)):
+            w, _ = ctx.pack_samples(torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda())
+            ctx.attribute_samples(w, hist, ninv)
+            if q % 2:   # device output: the captured graph path
+                n = ctx.rank_sites(hist, out=dev_rows)
+                rows = dev_rows.cpu().numpy().view(gs.RANKED_DTYPE)[:n]
+            else:       # host (pageable) output: plain launches
+                rows = ctx.rank_sites(hist)
+            got.append(canon(ctx, hist, len(raw), rows))
+        st.synchronize()
+    want_a = Canon(orc.run(s.text, samples=raw_a)).R
+    want_b = Canon(orc.run(s.text, samples=raw_b)).R
+    assert got[0] == got[1] == got[2] == got[5] == want_a
+    assert got[3] == got[4] == want_b

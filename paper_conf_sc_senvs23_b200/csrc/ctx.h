@@ -119,6 +119,9 @@ struct gs_ctx {
   uint32_t* d_rank_vals[2] = {nullptr, nullptr};
   uint64_t rank_cap = 0;
   int rank_bits_guess[2] = {-1, -1};  // bit widths of max(rel), max(tot) used by the last rank call
+  cudaGraphExec_t det_exec = nullptr;   // the detection sequence as a CUDA graph (see detect_run)
+  std::vector<uintptr_t> det_key;
+  uint64_t det_graph_launches = 0;
   cudaGraphExec_t rank_exec = nullptr;  // the rank sequence as a CUDA graph, replayed while its key repeats
   std::vector<uintptr_t> rank_key;
   uint64_t rank_graph_launches = 0;

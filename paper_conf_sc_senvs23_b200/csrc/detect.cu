@@ -675,6 +675,9 @@ void detect_free(gs_ctx* c) {
   c->d_ctot = nullptr;
   c->cdef_cap = c->ccnt_cap = c->cgoff_cap = c->cgslot_cap = 0;
   c->cons_ready = false;
+  if (c->det_exec) cudaGraphExecDestroy(c->det_exec);
+  c->det_exec = nullptr;
+  c->det_key.clear();
   c->detected = false;
 }
 
@@ -749,26 +752,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   const uint64_t c0 = c->cbase_h[w0], c1 = c->cbase_h[w1], nc = c1 - c0;
   const uint32_t D = c->cfg.trace_depth;
   c->detected = false;
-  GS_CUDA(c, cudaMemsetAsync(c->d_kstats, 0, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats), st));
-  if (nw) {
-    GS_CUDA(c, cudaMemsetAsync(c->d_wsum + w0, 0, (uint64_t)nw * 4, st));
-    GS_CUDA(c, cudaMemsetAsync(c->d_wev + w0, 0, (uint64_t)nw * 4, st));
-    const uint32_t grid = (nw + kWarps - 1) / kWarps;
-    k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
-                                           c->d_wev, c->d_narith, c->d_kstats); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    // candidate arrays are indexed relative to c0
-    k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
-                                           c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-  }
-  c->cons_ready = false;
-  if (c->cfg.join_mode == GS_JOIN_CONSUMER) {
-    const gs_status cs = consumers_run(c, kb, ke, w0, nw);
-    if (cs != GS_OK) return cs;
-  }
+  const bool cons = c->cfg.join_mode == GS_JOIN_CONSUMER;
   // tile sums, their exclusive prefixes (sites, chains) and the two totals, carved from cand.choff
   // (3 x ceil(NC / 256) u64 + 2)
   const uint64_t ntile = (nc + kCT - 1) / kCT;
@@ -781,21 +765,6 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   unsigned long long* tot = static_cast<unsigned long long*>(c->h_pin);
   gs_kernel_stats* kst_pin = reinterpret_cast<gs_kernel_stats*>(static_cast<char*>(c->h_pin) + 16);
   tot[0] = tot[1] = 0;
-  if (nc) {
-    const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
-    k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    const uint32_t gridc = (uint32_t)((nc + 255) / 256);
-    k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
-                                   c->d_kstats); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
-                                             RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum);
-    count_launch();
-    k_tile_prefix<<<1, 1024, 0, st>>>(d_tsum, ntile, d_pre_s, d_pre_c, d_tot); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
-  }
   // sites and chains into the buffers as they are (one host synchronisation per call); if a total
   // turns out larger than its buffer, grow it and write again
   auto write = [&]() -> gs_status {
@@ -806,11 +775,87 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     GS_CUDA(c, cudaGetLastError());
     return GS_OK;
   };
-  gs_status ws = write();
-  if (ws != GS_OK) return ws;
-  if (c->n_kernels)
-    GS_CUDA(c, cudaMemcpyAsync(kst_pin, c->d_kstats, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats),
-                               cudaMemcpyDeviceToHost, st));
+  // everything up to the speculative write and the read-backs (no allocation in here)
+  const auto enqueue = [&]() -> gs_status {
+    GS_CUDA(c, cudaMemsetAsync(c->d_kstats, 0, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats), st));
+    if (nw) {
+      GS_CUDA(c, cudaMemsetAsync(c->d_wsum + w0, 0, (uint64_t)nw * 4, st));
+      GS_CUDA(c, cudaMemsetAsync(c->d_wev + w0, 0, (uint64_t)nw * 4, st));
+      const uint32_t grid = (nw + kWarps - 1) / kWarps;
+      k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
+                                             c->d_wev, c->d_narith, c->d_kstats); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      // candidate arrays are indexed relative to c0
+      k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
+                                             c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+    }
+    if (cons) {
+      const gs_status cs = consumers_run(c, kb, ke, w0, nw);
+      if (cs != GS_OK) return cs;
+    }
+    if (nc) {
+      const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
+      k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      const uint32_t gridc = (uint32_t)((nc + 255) / 256);
+      k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
+                                         c->d_kstats); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
+                                               RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum);
+      count_launch();
+      k_tile_prefix<<<1, 1024, 0, st>>>(d_tsum, ntile, d_pre_s, d_pre_c, d_tot); count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
+    }
+    gs_status ws = write();
+    if (ws != GS_OK) return ws;
+    if (c->n_kernels)
+      GS_CUDA(c, cudaMemcpyAsync(kst_pin, c->d_kstats, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats),
+                                 cudaMemcpyDeviceToHost, st));
+    return GS_OK;
+  };
+  c->cons_ready = false;
+  // Replayed as one CUDA graph while (kernel range, buffers, capacities) repeat; not with the
+  // consumer join (it allocates), nor on the default streams (not capturable).
+  const uintptr_t key[] = {kb, ke, (uintptr_t)nc, D, (uintptr_t)c->sites_cap, (uintptr_t)c->chain_cap,
+                           (uintptr_t)c->d_sites, (uintptr_t)c->d_chain, (uintptr_t)c->h_pin,
+                           c->cfg.shmem_min_arith, c->cfg.shmem_min_loads, (uintptr_t)c->n_kernels};
+  constexpr size_t nkey = sizeof(key) / sizeof(key[0]);
+  static const bool no_graph = getenv("GS_NO_GRAPH") != nullptr;
+  const bool capturable = st != nullptr && st != cudaStreamLegacy && st != cudaStreamPerThread;
+  if (!no_graph && !cons && capturable) {
+    bool hit = c->det_exec && c->det_key.size() == nkey;
+    for (size_t q = 0; hit && q < nkey; q++) hit = c->det_key[q] == key[q];
+    if (!hit) {
+      if (c->det_exec) cudaGraphExecDestroy(c->det_exec);
+      c->det_exec = nullptr;
+      const uint64_t l0 = launch_count_now();
+      GS_CUDA(c, cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+      const gs_status s1 = enqueue();
+      cudaGraph_t g = nullptr;
+      const cudaError_t e = cudaStreamEndCapture(st, &g);
+      if (s1 != GS_OK) {
+        if (g) cudaGraphDestroy(g);
+        return s1;
+      }
+      GS_CUDA(c, e);
+      const cudaError_t ei = cudaGraphInstantiate(&c->det_exec, g, 0);
+      cudaGraphDestroy(g);
+      GS_CUDA(c, ei);
+      c->det_key.assign(key, key + nkey);
+      c->det_graph_launches = launch_count_now() - l0;
+      count_launch_undo(c->det_graph_launches);
+    }
+    GS_CUDA(c, cudaGraphLaunch(c->det_exec, st));
+    count_launch(c->det_graph_launches);
+  } else {
+    const gs_status s1 = enqueue();
+    if (s1 != GS_OK) return s1;
+  }
   GS_CUDA(c, cudaStreamSynchronize(st));
   c->kstats_h.assign(kst_pin, kst_pin + c->n_kernels);
   const uint64_t ns = tot[1], nch = tot[0];
@@ -818,7 +863,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   if (ns > c->sites_cap || nch > c->chain_cap) {
     GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
     GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
-    ws = write();
+    const gs_status ws = write();
     if (ws != GS_OK) return ws;
     GS_CUDA(c, cudaStreamSynchronize(st));
   }

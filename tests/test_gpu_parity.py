@@ -492,3 +492,21 @@ def test_rank_graph_replay(gs):
     want_b = Canon(orc.run(s.text, samples=raw_b)).R
     assert got[0] == got[1] == got[2] == got[5] == want_a
     assert got[3] == got[4] == want_b
+
+
+def test_detect_graph_replay(gs):
+    """gs_detect on a non-default stream (captured CUDA graph, replayed while the kernel range and
+    buffers repeat): repeated and alternating kernel ranges equal the oracle's K/S lines."""
+    import torch
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    s = gsass.config_sass("C4", scale=0.03)   # 7 kernels
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        ctx = _ctx(gs)
+        ctx.load_sass(s.text)
+        for kb, ke in [(0, 7), (0, 7), (2, 5), (2, 5), (0, 7), (5, 7)]:
+            ctx.detect(kb, ke)
+            g = Canon(report.canonical(ctx, kb, ke))
+            o = Canon(orc.run(s.text, kbegin=kb, kend=ke))
+            assert g.K == o.K and g.S == o.S, (kb, ke)

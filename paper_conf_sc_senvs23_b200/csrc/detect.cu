@@ -186,9 +186,16 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
   if (w >= w0 + nw) return;
-  for (int r = lane; r < kNumRegs; r += 32) {
-    tabS[warp][r] = tab[(uint64_t)w * kNumRegs + r];
-    cm[warp][r] = 0;
+  {  // the window's carried table: all ten loads of a lane in flight before the first store
+    static_assert(kNumRegs % 32 == 0, "registers per lane");
+    uint32_t tv[kNumRegs / 32];
+#pragma unroll
+    for (int u = 0; u < kNumRegs / 32; u++) tv[u] = __ldg(tab + (uint64_t)w * kNumRegs + lane + 32 * u);
+#pragma unroll
+    for (int u = 0; u < kNumRegs / 32; u++) {
+      tabS[warp][lane + 32 * u] = tv[u];
+      cm[warp][lane + 32 * u] = 0;
+    }
   }
   __syncwarp();
   const WDesc W = wd[w];
@@ -295,9 +302,15 @@ __global__ void __launch_bounds__(kWarps * 32) k_consumers(const Rec* __restrict
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
   if (w >= w0 + nw) return;
-  for (int r = lane; r < 256; r += 32) {
-    tabS[warp][r] = tab[(uint64_t)w * kNumRegs + r];
-    cm[warp][r] = 0;
+  {
+    uint32_t tv[8];
+#pragma unroll
+    for (int u = 0; u < 8; u++) tv[u] = __ldg(tab + (uint64_t)w * kNumRegs + lane + 32 * u);
+#pragma unroll
+    for (int u = 0; u < 8; u++) {
+      tabS[warp][lane + 32 * u] = tv[u];
+      cm[warp][lane + 32 * u] = 0;
+    }
   }
   __syncwarp();
   const WDesc W = wd[w];

@@ -14,6 +14,7 @@ ap.add_argument("--order", default="trace")
 ap.add_argument("--iters", type=int, default=10)
 ap.add_argument("--row", type=int, default=19, help="histogram row width (19 compact, as bench.py, or 32)")
 ap.add_argument("--synthetic", action="store_true", help="2^30 words on kernel 0 only: 80%% on a hot 10%% of its bins, 20%% uniform (the atoms_occ2 stream)")
+ap.add_argument("--accumulate", action="store_true", help="no histogram zeroing (timing only)")
 ap.add_argument("--check", action="store_true", help="compare the histogram with the count table")
 a = ap.parse_args()
 import torch  # noqa: E402
@@ -49,7 +50,7 @@ torch.cuda.synchronize()
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 e0.record()
 for _ in range(a.iters):
-    ctx.attribute_samples(words, hist, ninv)
+    ctx.attribute_samples(words, hist, ninv, accumulate=a.accumulate)
 e1.record()
 torch.cuda.synchronize()
 ms = e0.elapsed_time(e1) / a.iters

@@ -843,7 +843,7 @@ int main(int argc, char** argv) {
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
-  bool detect = true, hist = true, timing = false, quiet = false, liveness = false;
+  bool detect = true, hist = true, timing = false, quiet = false, liveness = false, no_hlines = false;
   for (int a = 1; a < argc; a++) {
     std::string s = argv[a];
     auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
@@ -864,6 +864,7 @@ int main(int argc, char** argv) {
     else if (s == "--no-hist") hist = false;
     else if (s == "--time") timing = true;
     else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
+    else if (s == "--no-hlines") no_hlines = true;  // full-size runs: every line but the H lines
     else { fprintf(stderr, "unknown arg %s\n", s.c_str()); return 2; }
   }
   if (join != "pc" && join != "line" && join != "consumer") { fprintf(stderr, "unknown join %s\n", join.c_str()); return 2; }
@@ -961,7 +962,7 @@ int main(int argc, char** argv) {
     uint64_t mass = 0;
     for (size_t b = 0; b < H.size(); b++)
       if (H[b]) {
-        if (!quiet) fprintf(out, "H %zu %zu %llu\n", b / 32, b % 32, (unsigned long long)H[b]);
+        if (!quiet && !no_hlines) fprintf(out, "H %zu %zu %llu\n", b / 32, b % 32, (unsigned long long)H[b]);
         mass += H[b];
       }
     fprintf(out, "N total=%llu valid=%llu invalid=%llu\n", (unsigned long long)N, (unsigned long long)mass,

@@ -22,7 +22,7 @@ def build_oracle(force: bool = False) -> str:
 
 def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, kbegin=0, kend=-1,
         detect=True, hist=True, timing=False, counts: np.ndarray | None = None, join: str = "pc",
-        liveness: bool = False) -> str:
+        liveness: bool = False, hlines: bool = True) -> str:
     """sass: path or text/bytes. samples: [N,3] uint32 raw triples. counts: [M,4] uint32
     pre-aggregated (kernel, pc, reason, count) records. join: pc | line | consumer. Returns canonical text."""
     build_oracle()
@@ -54,6 +54,8 @@ def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, k
             cmd += ["--join", join]
         if liveness:
             cmd.append("--liveness")
+        if not hlines:
+            cmd.append("--no-hlines")
         if not detect:
             cmd.append("--no-detect")
         if not hist:

@@ -510,3 +510,34 @@ def test_detect_graph_replay(gs):
             g = Canon(report.canonical(ctx, kb, ke))
             o = Canon(orc.run(s.text, kbegin=kb, kend=ke))
             assert g.K == o.K and g.S == o.S, (kb, ke)
+
+
+def test_c4_full_size_flow_parity(gs):
+    """The bench configuration itself (C4: 2^30 samples in trace order over 1,048,576 PCs, compact
+    rows, WINDOW): detection, attribution and ranking on the GPU against the oracle fed the same
+    histogram as pre-aggregated (kernel, pc, reason, count) records; every K, S and R line."""
+    import torch
+    import bench
+    from gen.device import DeviceTrace
+    from paper_conf_sc_senvs23_b200 import report
+    s, tr = bench.build_workload("C4", "trace")
+    tab = tr.table
+    words = DeviceTrace(tr).packed()
+    ctx = _ctx(gs, hist_row=19)
+    ctx.load_sass(s.text)
+    ctx.detect()
+    hist, ninv = ctx.attribute_samples(words)
+    del words
+    rows = ctx.rank_sites(hist)
+    torch.cuda.synchronize()
+    assert int(ninv.item()) == 0
+    g = Canon(report.canonical(ctx))
+    g_r = [f"R {q} {int(r['kernel'])} {int(r['idx'])} {gs.RULES[r['rule']]} rel={int(r['rel'])} "
+           f"tot={int(r['tot'])} ktot={int(r['ktot'])} h={','.join(str(int(x)) for x in r['counts'][:19])}"
+           for q, r in enumerate(rows)]
+    slot, reason = np.nonzero(tab)
+    k = np.searchsorted(s.first_slot, slot, side="right") - 1
+    counts = np.stack([k, (slot - s.first_slot[k]) * 16, reason, tab[slot, reason]], axis=1).astype(np.uint32)
+    o = Canon(orc.run(s.text, counts=counts, hlines=False))
+    assert g.K == o.K and g.S == o.S
+    assert len(g_r) == len(o.R) and g_r == o.R

@@ -512,18 +512,20 @@ def test_detect_graph_replay(gs):
             assert g.K == o.K and g.S == o.S, (kb, ke)
 
 
-def test_c4_full_size_flow_parity(gs):
-    """The bench configuration itself (C4: 2^30 samples in trace order over 1,048,576 PCs, compact
-    rows, WINDOW): detection, attribution and ranking on the GPU against the oracle fed the same
-    histogram as pre-aggregated (kernel, pc, reason, count) records; every K, S and R line."""
+@pytest.mark.parametrize("order,mode", [("trace", 0), ("shuffled", 4)])
+def test_c4_full_size_flow_parity(gs, order, mode):
+    """The bench configuration itself (C4: 2^30 samples over 1,048,576 PCs, compact rows; trace
+    order with AUTO = WINDOW, shuffled with PARTITION): detection, attribution and ranking on the GPU
+    against the oracle fed the same histogram as pre-aggregated (kernel, pc, reason, count) records;
+    every K, S and R line."""
     import torch
     import bench
     from gen.device import DeviceTrace
     from paper_conf_sc_senvs23_b200 import report
-    s, tr = bench.build_workload("C4", "trace")
+    s, tr = bench.build_workload("C4", order)
     tab = tr.table
     words = DeviceTrace(tr).packed()
-    ctx = _ctx(gs, hist_row=19)
+    ctx = _ctx(gs, hist_row=19, hist_mode=mode)
     ctx.load_sass(s.text)
     ctx.detect()
     hist, ninv = ctx.attribute_samples(words)

@@ -543,3 +543,14 @@ def test_c4_full_size_flow_parity(gs, order, mode):
     o = Canon(orc.run(s.text, counts=counts, hlines=False))
     assert g.K == o.K and g.S == o.S
     assert len(g_r) == len(o.R) and g_r == o.R
+
+
+def test_c3_full_size_detect_parity(gs):
+    """configs[2] at full size (C3: 10,000 kernels, 50M SASS instructions, the paper's dry run):
+    every K and S line (3.76M sites) equals the oracle's."""
+    from gen import sass as gsass
+    s = gsass.config_sass("C3")
+    g, _ = _detect_lines(gs, s.text)
+    o = Canon(orc.run(s.text, hist=False))
+    assert g.K == o.K
+    assert len(g.S) == len(o.S) and g.S == o.S

@@ -904,7 +904,8 @@ __device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t
 // Four barriers per tile: ranks | scan (also resets the rank counters and advances the bucket
 // cursors by the previous tile's counts) | stage | write-out. The write-out recomputes each
 // sample's bucket and reads its destination base dst[b] = cursor - tile offset.
-__global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
+template <int NT>
+__global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
                                                   uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
                                                   const uint32_t* __restrict__ off,
                                                   const unsigned long long* __restrict__ bstart,
@@ -912,23 +913,24 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
   __shared__ unsigned long long dst[kPMaxBuckets];   // cursor of bucket b minus its tile offset
   __shared__ uint32_t th[kPMaxBuckets], tcnt[kPMaxBuckets];
   extern __shared__ uint32_t stage[];  // kPTile words (dynamic)
-  __shared__ uint32_t wsum[kPT / 32];
+  constexpr uint32_t kTile = NT * 8, BPT = kPMaxBuckets / NT;  // samples per tile, buckets per thread
+  __shared__ uint32_t wsum[NT / 32];
   __shared__ uint32_t nv_sh;
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-  const uint32_t b0 = 2 * threadIdx.x, b1 = b0 + 1;  // the two buckets this thread scans
-  unsigned long long cur0 = 0, cur1 = 0;              // their cursors (registers)
-  if (b0 < B) cur0 = bstart[b0] + off[(uint64_t)blockIdx.x * B + b0];
-  if (b1 < B) cur1 = bstart[b1] + off[(uint64_t)blockIdx.x * B + b1];
-  for (uint32_t b = threadIdx.x; b < B; b += kPT) th[b] = 0;
+  const uint32_t bb = BPT * threadIdx.x;  // the buckets this thread scans: [bb, bb + BPT)
+  unsigned long long cur[BPT];            // their cursors (registers)
+#pragma unroll
+  for (uint32_t j = 0; j < BPT; j++) cur[j] = bb + j < B ? bstart[bb + j] + off[(uint64_t)blockIdx.x * B + bb + j] : 0;
+  for (uint32_t b = threadIdx.x; b < B; b += NT) th[b] = 0;
   __syncthreads();
   const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);
   uint32_t nw[8];
   if (a < e) load8(s, a, e, nw);
-  for (uint64_t t0 = a; t0 < e; t0 += kPTile) {
+  for (uint64_t t0 = a; t0 < e; t0 += kTile) {
     uint32_t w[8], bk[8], r[8];
 #pragma unroll
     for (int q = 0; q < 8; q++) w[q] = nw[q];
-    if (t0 + kPTile < e) load8(s, t0 + kPTile, e, nw);  // next tile in flight during this one
+    if (t0 + kTile < e) load8(s, t0 + kTile, e, nw);  // next tile in flight during this one
 #pragma unroll
     for (int q = 0; q < 8; q++) bk[q] = w[q] < pnr ? bucket_of(w[q], dv, bshift) : 0xffffffffu;
     // ranks within the tile's buckets: one shared atomic per sample, and one per warp when the
@@ -958,10 +960,13 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
     for (int q = 0; q < 8; q++) vmask |= bk[q] != 0xffffffffu ? 1u << q : 0u;
     const bool allv = __all_sync(0xffffffffu, vmask == 0xffu);
     __syncthreads();  // A: ranks done (and the previous tile's write-out)
-    uint32_t x0 = 0, x1 = 0;
-    if (b0 < B) { x0 = th[b0]; th[b0] = 0; }
-    if (b1 < B) { x1 = th[b1]; th[b1] = 0; }
-    const uint32_t v = x0 + x1;
+    uint32_t x[BPT], v = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < BPT; j++) {
+      x[j] = 0;
+      if (bb + j < B) { x[j] = th[bb + j]; th[bb + j] = 0; }
+      v += x[j];
+    }
     uint32_t inc = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -971,20 +976,23 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
     if (lane == 31) wsum[warp] = inc;
     __syncthreads();  // B
     if (warp == 0) {
-      const uint32_t y = wsum[lane];
+      const uint32_t y = lane < NT / 32 ? wsum[lane] : 0u;
       uint32_t yi = y;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t z = __shfl_up_sync(0xffffffffu, yi, o);
         if (lane >= o) yi += z;
       }
-      wsum[lane] = yi - y;
+      if (lane < NT / 32) wsum[lane] = yi - y;
       if (lane == 31) nv_sh = yi;
     }
     __syncthreads();  // C
-    const uint32_t ex = wsum[warp] + inc - v;  // tile offset of bucket b0
-    if (b0 < B) { tcnt[b0] = ex; dst[b0] = cur0 - ex; cur0 += x0; }
-    if (b1 < B) { tcnt[b1] = ex + x0; dst[b1] = cur1 - (ex + x0); cur1 += x1; }
+    uint32_t ex = wsum[warp] + inc - v;  // tile offset of bucket bb
+#pragma unroll
+    for (uint32_t j = 0; j < BPT; j++) {
+      if (bb + j < B) { tcnt[bb + j] = ex; dst[bb + j] = cur[j] - ex; cur[j] += x[j]; }
+      ex += x[j];
+    }
     __syncthreads();  // D: offsets ready
     if (allv) {
 #pragma unroll
@@ -996,7 +1004,7 @@ __global__ void __launch_bounds__(kPT) k_pscatter(const uint32_t* __restrict__ s
     }
     __syncthreads();  // E: staged
     const uint32_t nv = nv_sh;
-    for (uint32_t p = threadIdx.x; p < nv; p += kPT) {  // the bucket is recomputed (ALU, not smem)
+    for (uint32_t p = threadIdx.x; p < nv; p += NT) {  // the bucket is recomputed (ALU, not smem)
       const uint32_t x = stage[p];
       out[dst[bucket_of(x, dv, bshift)] + p] = x;
     }
@@ -1095,9 +1103,15 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   uint32_t B = (uint32_t)(((uint64_t)P + (1ull << bshift) - 1) >> bshift);
   if (B > kPMaxBuckets) return GS_E_RANGE;  // caller falls back to WINDOW (modules > 2048 tables)
   const uint32_t tw = (uint32_t)(((((uint64_t)1 << bshift) * nr + 1) / 2 + 31) & ~31ull);
-  const uint64_t nchunk = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 2, (n + kPTile - 1) / kPTile));
+#ifndef GS_PST
+#define GS_PST 1024
+#endif
+  constexpr int kPST = GS_PST;                  // scatter threads per CTA
+  constexpr uint32_t kSTile = kPST * 8;        // samples per scatter tile
+  const uint64_t nchunk = std::max<uint64_t>(
+      1, std::min<uint64_t>((uint64_t)dev_sms * (2048 / kPST), (n + kSTile - 1) / kSTile));
   uint64_t chunk = (n + nchunk - 1) / nchunk;
-  chunk = (chunk + kPTile - 1) / kPTile * kPTile;  // whole tiles (multiple of 4 words)
+  chunk = (chunk + kPTile - 1) / kPTile * kPTile;  // whole tiles of either kernel (multiple of 4 words)
   const uint64_t nch = (n + chunk - 1) / chunk;
   // scratch: counts/offsets [nch][B] u32, bucket starts [B + 1] u64, partitioned copy (+ padding)
   const uint64_t need = nch * B * 4 + 256 + (B + 1) * 8 + 256 + (n + 4ull * B + 4) * 4;
@@ -1118,8 +1132,8 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
-  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kPTile * 4)));
-  k_pscatter<<<(unsigned)nch, kPT, kPTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
+  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter<kPST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSTile * 4)));
+  k_pscatter<kPST><<<(unsigned)nch, kPST, kSTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4

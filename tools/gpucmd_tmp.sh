@@ -1,5 +1,6 @@
-python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-for o in shuffled trace; do
-timeout -s KILL 100 python tools/time_hist.py --iters 10 --check --order $o --mode 4 2>&1 | tail -2
-for v in pst512 pst256; do timeout -s KILL 100 python tools/time_hist.py --iters 10 --check --order $o --mode 4 --lib tools/libgs_$v.so 2>&1 | tail -2; done
-done
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1; tail -1 gpurun_out/smoke.log
+timeout -s KILL 1200 python -m pytest tests -m gpu -q > gpurun_out/gpu_tests.log 2>&1; tail -1 gpurun_out/gpu_tests.log
+timeout -s KILL 300 python bench.py > gpurun_out/bench_final.json 2> gpurun_out/bench_final.err; tail -1 gpurun_out/bench_final.json | cut -c1-200
+timeout -s KILL 300 python bench.py --order shuffled --no-cpu-baseline > gpurun_out/bench_final_shuffled.json 2>/dev/null
+timeout -s KILL 300 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_final_reference.json 2>/dev/null
+echo done

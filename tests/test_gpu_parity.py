@@ -505,7 +505,7 @@ def test_detect_graph_replay(gs):
     with torch.cuda.stream(st):
         ctx = _ctx(gs)
         ctx.load_sass(s.text)
-        for kb, ke in [(0, 7), (0, 7), (2, 5), (2, 5), (0, 7), (5, 7)]:
+        for kb, ke in [(0, 7), (0, 7), (2, 5), (2, 5), (0, 7), (5, 7), (5, 5), (5, 5), (6, 7)]:
             ctx.detect(kb, ke)
             g = Canon(report.canonical(ctx, kb, ke))
             o = Canon(orc.run(s.text, kbegin=kb, kend=ke))

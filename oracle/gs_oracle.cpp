@@ -24,7 +24,9 @@
 //   O12 CONV  datatype conversions                               P:746-761 §4.7
 //   O13 per-PC x stall-reason histogram of PC samples            P:215-227 §2.2
 //   O14 join of the histogram onto flagged sites
+//       join=pc (default), line ([R33]), consumer ([R37], SURVEY [probe 9])
 //   O15 ranking (total order on integers)                        [R20]
+//   O16 register pressure: live GPRs per instruction (--liveness) P:541-554, P:452 [R36]
 //
 // Output: the canonical result text on stdout or --out.
 #include <algorithm>

@@ -26,7 +26,7 @@
 //   O14 join of the histogram onto flagged sites
 //       join=pc (default), line ([R33]), consumer ([R37], SURVEY [probe 9])
 //   O15 ranking (total order on integers)                        [R20]
-//   O16 register pressure: live GPRs per instruction (--liveness) P:541-554, P:452 [R36]
+//   O16 register pressure: live GPRs per instruction (--liveness) P:541-554, P:452 [R36, R38]
 //
 // Output: the canonical result text on stdout or --out.
 #include <algorithm>
@@ -206,11 +206,14 @@ struct Instr {
   int line = -1;                  // source line from //## File ..., line N
   std::string file;               // ... and its file (a source line is the pair (file, line), R33)
   std::string bra_label;          // nvdisasm: BRA `(.L_x_N) target label, resolved per kernel
+  std::vector<std::string> brx_labels;  // nvdisasm: BRX ... (*"BRANCH_TARGETS .L_a,.L_b"*) (R38i)
+  std::vector<long long> brx_targets;   // ... resolved to pcs
   bool guarded = false;           // @Pn / @!Pn guard (not @PT)
   std::string op;                 // base mnemonic
   std::vector<std::string> mods;  // modifiers after the first '.'
   std::vector<Opnd> ops;
   int dst = kNoReg, dst_w = 0, dst_pos = -1;
+  int dst2 = kNoReg, dst2_pos = -1;  // second destination quad of a .256 load (R38a)
   std::vector<int> srcs;          // register sources (no RZ/URZ), O2
   int mem = -1;                   // index of the memory operand in ops
   long long bra_target = -1;      // BRA immediate target pc
@@ -223,6 +226,7 @@ struct Instr {
 struct Kernel {
   std::string name;
   int param_base = 0x380;
+  int regcount = -1;                  // REG:N of a cuobjdump -res-usage block, if the dump has one (R38k)
   std::vector<Instr> ins;
   size_t first_slot = 0;
   std::map<std::string, int> labels;  // nvdisasm ".L_x_N:" -> pc of the next instruction
@@ -233,40 +237,117 @@ bool op_in(const std::string& op, std::initializer_list<const char*> l) {
   return false;
 }
 
-// O2 destination width table (DESIGN.md §3 table W).
+// ---- register widths (R24, revised for sm_100a by R38; pinned to nvdisasm -lrm narrow) ----
+bool is_64type(const std::string& m) { return m == "F64" || m == "S64" || m == "U64"; }
+bool is_int_type(const std::string& m) {
+  return m == "S64" || m == "U64" || m == "S32" || m == "U32" || m == "S16" || m == "U16" || m == "S8" || m == "U8";
+}
+bool is_float_type(const std::string& m) {
+  return m == "F64" || m == "F32" || m == "F16" || m == "BF16" || m == "TF32" || m == "E4M3" || m == "E5M2";
+}
+bool is_type(const std::string& m) { return is_int_type(m) || is_float_type(m); }
+
+// R38e conversions: which type modifier names the destination and which the source.
+//   F2F, I2I: first type = destination, second = source (F2F.F32.F64);
+//   I2F, I2FP: the float type is the destination, the integer type the source (I2F.U64.RP: u64 -> f32);
+//   F2I, F2IP: the integer type is the destination, the float type the source (F2I.F64.TRUNC: f64 -> s32).
+// Returns the register widths {dst, src} (2 for a 64-bit type, else 1).
+std::pair<int, int> conv_widths(const Instr& I) {
+  std::vector<std::string> t;
+  for (auto& m : I.mods) if (is_type(m)) t.push_back(m);
+  std::string d, s;
+  if (op_in(I.op, {"F2F", "I2I"})) {
+    if (t.size() >= 1) d = t[0];
+    if (t.size() >= 2) s = t[1];
+  } else if (op_in(I.op, {"I2F", "I2FP"})) {
+    for (auto& m : t) (is_float_type(m) ? d : s) = m;
+  } else if (op_in(I.op, {"F2I", "F2IP"})) {
+    for (auto& m : t) (is_int_type(m) ? d : s) = m;
+  } else if (I.op == "F2FP") {
+    if (t.size() >= 1) d = t[0];
+    if (t.size() >= 2) s = t[1];
+  }
+  return {is_64type(d) ? 2 : 1, is_64type(s) ? 2 : 1};
+}
+
+// R38c warp-level MMA fragments: HMMA.<m><n><k>.<acc>[.<in>] on an m16n8kK tile holds, per thread,
+// A = 16*K*b/1024 and B = 8*K*b/1024 registers (b = input element bits: F16/BF16 16 (default), TF32
+// 32, E4M3/E5M2 8) and C = D = 4 registers for an F32 accumulator, 2 for F16.
+struct MmaRegs { int a = 1, b = 1, acc = 1; };
+MmaRegs mma_regs(const Instr& I) {
+  MmaRegs r;
+  int K = 8, bits = 16;
+  std::string acc;
+  for (size_t q = 0; q < I.mods.size(); q++) {
+    const std::string& m = I.mods[q];
+    if (q == 0 && m.size() >= 4 && isdigit((unsigned char)m[0])) K = atoi(m.c_str() + 3);  // "16816" -> 16, "1688" -> 8
+    else if (acc.empty() && is_float_type(m)) acc = m;
+    else if (m == "TF32") bits = 32;
+    else if (m == "E4M3" || m == "E5M2") bits = 8;
+  }
+  r.a = std::max(1, 16 * K * bits / 1024);
+  r.b = std::max(1, 8 * K * bits / 1024);
+  r.acc = acc == "F16" ? 2 : 4;
+  return r;
+}
+
+// R38d tensor-memory loads/stores (tcgen05.ld/st): LDTM[.<shape>].x<N>; registers per thread per
+// repetition: 32dp32bit (no shape modifier) 1, 16dp32bit 1, 16dp64bit 1, 16dp128bit 2, 16dp256bit 4.
+int tmem_regs(const Instr& I) {
+  int per = 1, x = 1;
+  for (auto& m : I.mods) {
+    if (m == "16dp128bit") per = 2;
+    else if (m == "16dp256bit") per = 4;
+    else if (m.size() > 1 && m[0] == 'x' && isdigit((unsigned char)m[1])) x = atoi(m.c_str() + 1);
+  }
+  return per * x;
+}
+
+// O2 destination width table (DESIGN.md §3 table W: R24 as revised by R38).
 int dst_width(const Instr& I) {
+  for (auto& m : I.mods) if (m == "256") return 4;      // R38a: each of the two destination quads
   for (auto& m : I.mods) if (m == "128") return 4;
-  if (I.op == "HMMA") return I.has_mod("F32") ? 4 : 2;
+  if (I.op == "HMMA") return mma_regs(I).acc;             // R38c
   if (I.op == "LDSM") {
     if (I.has_mod("4")) return 4;
     if (I.has_mod("2")) return 2;
     return 1;
   }
+  if (I.op == "LDTM") return tmem_regs(I);                // R38d
   for (auto& m : I.mods) if (m == "64" || m == "WIDE") return 2;
+  if (I.op == "CS2R") return I.has_mod("32") ? 1 : 2;     // R38b: CS2R writes a pair unless .32
+  if (I.op == "LEPC") return 2;                           // R38b: a 64-bit program counter
   if (op_in(I.op, {"DADD", "DMUL", "DFMA", "DMNMX"})) return 2;
-  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I"})) {
-    for (auto& m : I.mods) {  // the first type modifier is the destination type
-      if (m == "F64" || m == "S64" || m == "U64") return 2;
-      if (m == "F32" || m == "F16" || m == "BF16" || m == "S32" || m == "U32" || m == "S16" ||
-          m == "U16" || m == "S8" || m == "U8" || m == "TF32" || m == "E4M3" || m == "E5M2")
-        return 1;
-    }
-  }
+  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I", "I2FP", "F2IP", "F2FP"})) return conv_widths(I).first;  // R38e
   return 1;
+}
+
+// R38f opcodes whose register operands are all sources (a first register operand is not a
+// destination): WARPSYNC Rmask, BRX/JMX Rtarget, RET Rreturn, CALL Rtarget, NANOSLEEP Rns, BAR ... Rn.
+bool no_register_dst(const std::string& op) {
+  return op_in(op, {"WARPSYNC", "BRX", "BRXU", "JMX", "JMXU", "RET", "CALL", "NANOSLEEP", "BAR", "YIELD", "BPT"});
 }
 
 // O2: decode dst and sources.
 void decode_effects(Instr& I) {
   int d = -1;
-  if (!I.ops.empty() && I.ops[0].kind == K_REG) d = 0;
+  if (no_register_dst(I.op)) d = -1;
+  else if (!I.ops.empty() && I.ops[0].kind == K_REG) d = 0;
   else if (I.ops.size() >= 2 && I.ops[0].kind == K_PRED && I.ops[1].kind == K_REG && I.op != "FCHK")
     d = 1;  // SHFL PT, R0 ... ; ATOMG PT, R2 ... ; LOP3.LUT P0, R5 ...
+  int last_dst = d;
   if (d >= 0) {
     I.dst_pos = d;
     I.dst = I.ops[d].reg;
     I.dst_w = dst_width(I);
+    // R38a: a 256-bit load (LDG.E.ENL2.256 Ra, Rb, [..]) writes two register quads Ra and Rb
+    if (I.has_mod("256") && (size_t)d + 1 < I.ops.size() && I.ops[d + 1].kind == K_REG) {
+      I.dst2_pos = d + 1;
+      I.dst2 = I.ops[d + 1].reg;
+      last_dst = d + 1;
+    }
   }
-  for (size_t k = (size_t)(d + 1); k < I.ops.size(); k++)
+  for (size_t k = (size_t)(last_dst + 1); k < I.ops.size(); k++)
     for (int r : I.ops[k].regs)
       if (!is_zero_reg(r)) I.srcs.push_back(r);
   for (size_t k = 0; k < I.ops.size(); k++)
@@ -285,10 +366,14 @@ std::vector<Kernel> parse_sass(const std::string& text) {
   int cur_sm = 100, line_no = 0, src_line = -1;
   std::string src_file;
   std::vector<std::string> pending;  // labels waiting for their instruction
+  std::map<std::string, int> res_regs;  // cuobjdump -res-usage: function name -> REG:N (R38k)
+  std::string res_fn;
   auto new_kernel = [&](const std::string& name) {
     Kernel k;
     k.name = name;
     k.param_base = arch_param_base(cur_sm);
+    auto rr = res_regs.find(name);
+    if (rr != res_regs.end()) k.regcount = rr->second;
     ks.push_back(k);
     src_line = -1;
     src_file.clear();
@@ -308,6 +393,16 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     size_t tg = t.find(".target");
     if (tg != std::string::npos && t.find("sm_") != std::string::npos) {
       cur_sm = atoi(t.c_str() + t.find("sm_") + 3);
+      continue;
+    }
+    // cuobjdump -res-usage block: " Function <name>:" then "  REG:N STACK:..." (R38k)
+    if (t.rfind("Function ", 0) == 0 && t.size() > 10 && t.back() == ':' && t.find("Function :") == std::string::npos) {
+      res_fn = t.substr(9, t.size() - 10);
+      continue;
+    }
+    if (!res_fn.empty() && t.rfind("REG:", 0) == 0) {
+      res_regs[res_fn] = atoi(t.c_str() + 4);
+      res_fn.clear();
       continue;
     }
     size_t fn = t.find("Function :");
@@ -341,6 +436,26 @@ std::vector<Kernel> parse_sass(const std::string& text) {
     size_t semi = body.find(';');
     if (semi == std::string::npos) continue;
     body = trim(body.substr(0, semi));
+    // nvdisasm annotates indirect branches with their targets: (*"BRANCH_TARGETS .L_a,.L_b"*) (R38i)
+    std::vector<std::string> brx_labels;
+    size_t ann = body.find("(*\"");
+    if (ann != std::string::npos) {
+      std::string a = body.substr(ann);
+      body = trim(body.substr(0, ann));
+      size_t bt = a.find("BRANCH_TARGETS ");
+      if (bt != std::string::npos) {
+        std::string list = a.substr(bt + 15);
+        list = list.substr(0, list.find('"'));
+        size_t s = 0;
+        while (s <= list.size()) {
+          size_t e = list.find(',', s);
+          if (e == std::string::npos) e = list.size();
+          std::string lb = trim(list.substr(s, e - s));
+          if (!lb.empty()) brx_labels.push_back(lb);
+          s = e + 1;
+        }
+      }
+    }
     if (ks.empty()) new_kernel("<anonymous>");  // instructions without a header (e.g. a paper listing)
     Kernel& K = ks.back();
     Instr I;
@@ -367,7 +482,8 @@ std::vector<Kernel> parse_sass(const std::string& text) {
       I.mods.push_back(opc.substr(d0 + 1, d1 == std::string::npos ? std::string::npos : d1 - d0 - 1));
       d0 = d1;
     }
-    // split operands at top-level commas
+    // split operands at top-level commas; an operand list without a comma between two operands
+    // ("RET.REL.NODEC R2 0x0", "BRX R4 -0x43d0") is split at top-level blanks as well (R38i)
     std::vector<std::string> raw;
     int depth = 0;
     std::string cur;
@@ -375,6 +491,8 @@ std::vector<Kernel> parse_sass(const std::string& text) {
       if (ch == '[' || ch == '{') depth++;
       if (ch == ']' || ch == '}') depth--;
       if (ch == ',' && depth == 0) { raw.push_back(cur); cur.clear(); }
+      else if ((ch == ' ' || ch == '\t') && depth == 0 && !trim(cur).empty()) { raw.push_back(cur); cur.clear(); }
+      else if ((ch == ' ' || ch == '\t') && depth == 0) continue;
       else cur += ch;
     }
     if (!trim(cur).empty()) raw.push_back(cur);
@@ -387,15 +505,21 @@ std::vector<Kernel> parse_sass(const std::string& text) {
       else if (last.size() > 4 && last.rfind("`(", 0) == 0 && last.back() == ')')
         I.bra_label = last.substr(2, last.size() - 3);
     }
+    I.brx_labels = brx_labels;
     K.ins.push_back(I);
   }
   // nvdisasm label targets: a label names the pc of the instruction after it (R28)
   for (auto& k : ks)
-    for (auto& I : k.ins)
+    for (auto& I : k.ins) {
       if (!I.bra_label.empty()) {
         auto it = k.labels.find(I.bra_label);
         if (it != k.labels.end()) I.bra_target = it->second;
       }
+      for (auto& lb : I.brx_labels) {
+        auto it = k.labels.find(lb);
+        if (it != k.labels.end()) I.brx_targets.push_back(it->second);
+      }
+    }
   size_t slot = 0;
   for (auto& k : ks) { k.first_slot = slot; slot += k.ins.size(); }
   return ks;
@@ -430,6 +554,7 @@ int access_bits(const Instr& I) {
     if (m == "U16" || m == "S16") return 16;
     if (m == "64") return 64;
     if (m == "128") return 128;
+    if (m == "256") return 256;  // sm_100a LDG.E.ENL2.256: two register quads (R38a)
   }
   return 32;
 }
@@ -464,11 +589,12 @@ class KernelAnalysis {
     for (size_t i = 0; i < K.ins.size(); i++) {
       for (auto& q : rd_at[i]) q.second = lw[q.first];
       const Instr& I = K.ins[i];
-      if (I.dst != kNoReg && !is_zero_reg(I.dst))
-        for (int w = 0; w < I.dst_w; w++) {
-          int r = I.dst + w;
-          if ((is_ur(I.dst) && r <= 318) || (!is_ur(I.dst) && r <= 254)) lw[r] = (int)i;
-        }
+      for (int dreg : {I.dst, I.dst2})
+        if (dreg != kNoReg && !is_zero_reg(dreg))
+          for (int w = 0; w < I.dst_w; w++) {
+            int r = dreg + w;
+            if ((is_ur(dreg) && r <= 318) || (!is_ur(dreg) && r <= 254)) lw[r] = (int)i;
+          }
     }
   }
   int rd(int i, int r) const {
@@ -671,7 +797,7 @@ void detect_kernel(int kid, const Kernel& K, const Config& C, std::vector<Site>&
     if (is_conv(I.op)) st.conv++;
     if (I.op == "LDG" && I.mem >= 0) {
       int bits = access_bits(I);
-      if (bits == 64 || bits == 128) st.vec_already++;  // "already vectorised"
+      if (bits >= 64) st.vec_already++;  // "already vectorised" (64/128/256-bit)
       const Group& g = groups[key_of(i)];
       // O6 VEC: 32-bit LDG whose group has >= 2 distinct immediate offsets.
       if (bits == 32 && g.off32.size() >= 2) {
@@ -737,87 +863,145 @@ void detect_kernel(int kid, const Kernel& K, const Config& C, std::vector<Site>&
 //   count(i) = |live_in(i) ∪ defs(i)|, R1 (the stack pointer) counted live after its definition.
 // Only R0..R254 (nvdisasm's "GPR #" column). additional(i) = count(i) - count(i-1).
 
-bool is_64type(const std::string& m) { return m == "F64" || m == "S64" || m == "U64"; }
-bool is_type(const std::string& m) {
-  return is_64type(m) || m == "F32" || m == "F16" || m == "BF16" || m == "S32" || m == "U32" || m == "S16" ||
-         m == "U16" || m == "S8" || m == "U8" || m == "TF32";
-}
-// register width of a store / atomic data operand (R36): .128 -> 4, .64 or a 64-bit type -> 2
+// register width of a store / atomic data operand (R36, R38a/d): .256 -> 4 per data operand (two
+// quads), .128 -> 4, STSM .4/.2 -> 4/2, STTM as LDTM, .64 or a 64-bit type -> 2
 int data_width(const Instr& I) {
-  for (auto& m : I.mods) if (m == "128") return 4;
+  for (auto& m : I.mods) if (m == "256" || m == "128") return 4;
+  if (I.op == "STSM") return I.has_mod("4") ? 4 : (I.has_mod("2") ? 2 : 1);
+  if (I.op == "STTM") return tmem_regs(I);
   for (auto& m : I.mods) if (m == "64" || is_64type(m)) return 2;
   return 1;
 }
 
-// GPR uses of instruction I, pair/quad registers expanded (R36)
+// GPR uses of instruction I, pair/quad registers expanded (R36, R38)
 std::set<int> gpr_uses(const Instr& I) {
   std::set<int> u;
   int srcw = op_in(I.op, {"DADD", "DMUL", "DFMA", "DSETP", "DMNMX"}) ? 2 : 1;
-  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I", "F2FP", "I2FP", "F2IP"})) {
-    std::vector<std::string> types;
-    for (auto& m : I.mods) if (is_type(m)) types.push_back(m);
-    if (types.size() >= 2 && is_64type(types[1])) srcw = 2;  // second type = source type
-  }
-  const bool store_like = op_in(I.op, {"STG", "STS", "STL", "ST", "RED", "REDG", "ATOMG", "ATOM", "ATOMS"});
-  int srcidx = 0;  // index among the non-predicate operands after the destination
+  if (op_in(I.op, {"F2F", "I2F", "F2I", "I2I", "F2FP", "I2FP", "F2IP"})) srcw = conv_widths(I).second;  // R38e
+  const bool store_like =
+      op_in(I.op, {"STG", "STS", "STL", "ST", "RED", "REDG", "ATOMG", "ATOM", "ATOMS", "STSM", "STTM", "STAS"});
+  const bool mma = I.op == "HMMA";
+  const MmaRegs mr = mma ? mma_regs(I) : MmaRegs();
+  // IMAD.HI adds a 64-bit addend: hi32(a * b + c:c+1) (R38h)
+  const bool hi_add = I.op == "IMAD" && I.has_mod("HI");
+  // an indirect branch / call / return reads a 64-bit target address (R38g)
+  const bool target_pair = op_in(I.op, {"BRX", "BRXU", "JMX", "JMXU", "RET", "CALL"});
+  const int last_dst = I.dst2_pos >= 0 ? I.dst2_pos : I.dst_pos;
+  int last_mem = -1;  // .E ("extended" 64-bit global address) names the last memory operand (R38j)
+  for (size_t k = 0; k < I.ops.size(); k++)
+    if (I.ops[k].kind == K_MEM) last_mem = (int)k;
+  int srcidx = 0;  // index among the non-predicate operands after the destination(s)
   for (size_t k = 0; k < I.ops.size(); k++) {
-    if ((int)k == I.dst_pos) continue;
+    if ((int)k == I.dst_pos || (int)k == I.dst2_pos) continue;
     const Opnd& o = I.ops[k];
     for (int r : o.regs) {
       if (r >= 255) continue;  // RZ, uniform registers
       int w = 1;
       // a memory base is a 64-bit pair when written Rb.64 (sm_100) or when the access is .E
       // ("extended", 64-bit addresses: sm_70's LDG.E [R8] reads R8:R9)
-      if (o.kind == K_MEM) w = (r == o.base && (o.wide || I.has_mod("E"))) ? 2 : 1;
+      if (o.kind == K_MEM) w = (r == o.base && (o.wide || (I.has_mod("E") && (int)k == last_mem))) ? 2 : 1;
       else if (o.kind == K_CREF) w = 1;
+      else if (target_pair) w = 2;
       else if (store_like && k > 0) w = data_width(I);
+      else if (mma) w = srcidx == 0 ? mr.a : (srcidx == 1 ? mr.b : mr.acc);
       else if (I.op == "IMAD" && I.has_mod("WIDE") && srcidx == 2) w = 2;
+      else if (hi_add && srcidx == 2) w = 2;
       else w = srcw;
-      for (int q = 0; q < w; q++) u.insert(r + q);
+      for (int q = 0; q < w && r + q < 255; q++) u.insert(r + q);
     }
-    if ((int)k > I.dst_pos && o.kind != K_PRED) srcidx++;
+    if ((int)k > last_dst && o.kind != K_PRED) srcidx++;
   }
+  if (I.op == "CALL") { u.insert(0); u.insert(1); }  // R38g: the call reads R0 and the stack pointer R1
   return u;
 }
 
-std::vector<int> live_counts(const Kernel& K) {
+// R38g: registers a CALL may overwrite (the ABI's caller-saved GPRs, as nvdisasm's life ranges show
+// them on sm_100a): R0, R3..R15 and R32+8j..R35+8j (j = 0..8), limited to the kernel's registers.
+bool call_clobbered(int r) { return r == 0 || (r >= 3 && r <= 15) || (r >= 32 && r <= 99 && (r - 32) % 8 < 4); }
+
+// GPR definitions of instruction I: the destination(s) and the registers their width covers (O2,
+// R24, R38); a CALL defines its clobbered registers below `nregs` (the kernel's register count).
+std::set<int> gpr_defs(const Instr& I, int nregs = 255) {
+  std::set<int> d;
+  for (int dreg : {I.dst, I.dst2})
+    if (dreg != kNoReg && dreg < 255)
+      for (int q = 0; q < I.dst_w && dreg + q < 255; q++) d.insert(dreg + q);
+  if (I.op == "CALL")
+    for (int r = 0; r < nregs && r < 255; r++)
+      if (call_clobbered(r)) d.insert(r);
+  return d;
+}
+
+// The kernel's register count (R38k): REG:N of the dump's cuobjdump -res-usage block when it has
+// one, else one past the highest GPR any instruction reads or writes (widths expanded).
+int kernel_nregs(const Kernel& K) {
+  if (K.regcount > 0) return K.regcount;
+  int m = 0;
+  for (auto& I : K.ins) {
+    for (int r : gpr_uses(I)) m = std::max(m, r + 1);
+    for (int r : gpr_defs(I, 0)) m = std::max(m, r + 1);
+  }
+  return m;
+}
+
+std::vector<std::set<int>> live_sets(const Kernel& K) {
   const int n = (int)K.ins.size();
   std::vector<std::set<int>> use(n), def(n);
   std::vector<std::vector<int>> succ(n);
   int r1def = -1;
+  const int nregs = kernel_nregs(K);
   for (int i = 0; i < n; i++) {
     const Instr& I = K.ins[i];
     use[i] = gpr_uses(I);
-    if (I.dst != kNoReg && I.dst < 255)
-      for (int q = 0; q < I.dst_w; q++) def[i].insert(I.dst + q);
+    def[i] = gpr_defs(I, nregs);
     if (r1def < 0 && def[i].count(1)) r1def = i;
     bool cond = I.guarded;
+    // a branch with a predicate or register condition before its target (BRA.U !UP0, 0x..;
+    // BRA.DIV UR4, 0x..) may fall through (R38i)
     if (I.op == "BRA")
-      for (size_t k = 0; k + 1 < I.ops.size(); k++) cond |= I.ops[k].kind == K_PRED && I.ops[k].pred_var;
+      for (size_t k = 0; k + 1 < I.ops.size(); k++)
+        cond |= (I.ops[k].kind == K_PRED && I.ops[k].pred_var) || I.ops[k].kind == K_REG;
     const bool branch = I.op == "BRA" && I.bra_target >= 0 && I.bra_target / 16 < n;
     if (branch) succ[i].push_back((int)(I.bra_target / 16));
-    const bool ends = (I.op == "EXIT" || I.op == "RET" || branch) && !cond;
+    // an indirect branch continues at each of its listed targets (nvdisasm BRANCH_TARGETS, R38i)
+    const bool brx = op_in(I.op, {"BRX", "BRXU", "JMX", "JMXU"});
+    if (brx)
+      for (long long t : I.brx_targets)
+        if (t / 16 < n) succ[i].push_back((int)(t / 16));
+    const bool ends = (I.op == "EXIT" || I.op == "RET" || branch || brx) && !cond;
     if (!ends && i + 1 < n) succ[i].push_back(i + 1);
   }
+  // R38g: a RET hands the callee-saved registers (those a CALL does not clobber, below the kernel's
+  // register count; R1 is counted separately) back to the caller: they are live out of it
+  std::set<int> callee_saved;
+  for (int r = 0; r < nregs && r < 255; r++)
+    if (r != 1 && !call_clobbered(r)) callee_saved.insert(r);
   std::vector<std::set<int>> in(n);
   for (bool changed = true; changed;) {  // round-robin to the fixed point
     changed = false;
     for (int i = n - 1; i >= 0; i--) {
       std::set<int> out;
       for (int s : succ[i]) out.insert(in[s].begin(), in[s].end());
+      if (K.ins[i].op == "RET") out.insert(callee_saved.begin(), callee_saved.end());
       std::set<int> li = use[i];
       for (int r : out)
         if (K.ins[i].guarded || !def[i].count(r)) li.insert(r);
       if (li != in[i]) { in[i] = li; changed = true; }
     }
   }
-  std::vector<int> cnt(n);
+  std::vector<std::set<int>> live(n);
   for (int i = 0; i < n; i++) {
-    std::set<int> c = in[i];
-    c.insert(def[i].begin(), def[i].end());
-    if (r1def >= 0 && i > r1def) c.insert(1);
-    cnt[i] = (int)c.size();
+    live[i] = in[i];
+    live[i].insert(def[i].begin(), def[i].end());
+    if (r1def >= 0 && i > r1def) live[i].insert(1);
   }
+  return live;
+}
+
+// count(i) = |live_in(i) ∪ defs(i)| (+ R1 after its definition)
+std::vector<int> live_counts(const Kernel& K) {
+  std::vector<int> cnt;
+  for (auto& s : live_sets(K)) cnt.push_back((int)s.size());
   return cnt;
 }
 
@@ -845,7 +1029,8 @@ int main(int argc, char** argv) {
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
-  bool detect = true, hist = true, timing = false, quiet = false, liveness = false, no_hlines = false;
+  bool detect = true, hist = true, timing = false, quiet = false, liveness = false, no_hlines = false,
+       regsets = false;
   for (int a = 1; a < argc; a++) {
     std::string s = argv[a];
     auto nxt = [&]() { return std::string(a + 1 < argc ? argv[++a] : ""); };
@@ -863,6 +1048,7 @@ int main(int argc, char** argv) {
     else if (s == "--kend") kend = atoi(nxt().c_str());
     else if (s == "--no-detect") detect = false;
     else if (s == "--liveness") liveness = true;   // L lines: live GPRs per instruction (O16)
+    else if (s == "--regsets") regsets = true;     // G lines: GPR defs and uses per instruction (O16 inputs)
     else if (s == "--no-hist") hist = false;
     else if (s == "--time") timing = true;
     else if (s == "--quiet") quiet = true;  // timing runs: compute everything, print only K/N lines
@@ -923,6 +1109,19 @@ int main(int argc, char** argv) {
       std::vector<int> cnt = live_counts(ks[k]);
       for (size_t i = 0; i < cnt.size(); i++)
         fprintf(out, "L %d %zu %d %d\n", k, i, cnt[i], cnt[i] - (i ? cnt[i - 1] : 0));
+    }
+  if (regsets)  // the def / use / live sets of O16, one G line per instruction (test pins)
+    for (int k = kbegin; k < kend; k++) {
+      const int nregs = kernel_nregs(ks[k]);
+      const std::vector<std::set<int>> live = live_sets(ks[k]);
+      auto join = [](const std::set<int>& s) {
+        std::string r;
+        for (int x : s) r += (r.empty() ? "" : ",") + std::to_string(x);
+        return r.empty() ? std::string("-") : r;
+      };
+      for (size_t i = 0; i < ks[k].ins.size(); i++)
+        fprintf(out, "G %d %zu def=%s use=%s live=%s\n", k, i, join(gpr_defs(ks[k].ins[i], nregs)).c_str(),
+                join(gpr_uses(ks[k].ins[i])).c_str(), join(live[i]).c_str());
     }
   if (hist && (!samples_path.empty() || !counts_path.empty())) {
     // O13: H[slot][reason] += 1 for every valid sample.

@@ -32,3 +32,16 @@ for k in sgemm_naive jacobi mixbench atomics spill; do
   nvdisasm -lrm count -c $T/$k.cubin > lineinfo/$k.lrm.txt
 done
 rm -rf $T
+# sm_100a-native register forms (R38): wmma (HMMA / LDSM / CS2R pairs), 256-bit vector
+# loads and stores (LDG/STG.E.ENL2.256, two register quads), tcgen05 tensor memory (LDTM / STTM,
+# guardrail CALL / RET subroutines). The SASS text carries the -res-usage block (REG:N, R38k);
+# nvdisasm -lrm count gives the pinned live counts, -lrm narrow the per-register def/use/live table.
+mkdir -p b200
+T=$(mktemp -d)
+for k in wmma v8 tmem; do
+  nvcc -arch=sm_100a -cubin -O3 -o $T/$k.cubin src/$k.cu
+  cuobjdump -sass -res-usage $T/$k.cubin > b200/$k.sm_100a.sass
+  nvdisasm -lrm count -c $T/$k.cubin > b200/$k.sm_100a.lrm.txt
+  nvdisasm -lrm narrow -c $T/$k.cubin > b200/$k.sm_100a.narrow.txt
+done
+rm -rf $T

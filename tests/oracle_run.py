@@ -22,7 +22,7 @@ def build_oracle(force: bool = False) -> str:
 
 def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, kbegin=0, kend=-1,
         detect=True, hist=True, timing=False, counts: np.ndarray | None = None, join: str = "pc",
-        liveness: bool = False, hlines: bool = True) -> str:
+        liveness: bool = False, hlines: bool = True, regsets: bool = False) -> str:
     """sass: path or text/bytes. samples: [N,3] uint32 raw triples. counts: [M,4] uint32
     pre-aggregated (kernel, pc, reason, count) records. join: pc | line | consumer. Returns canonical text."""
     build_oracle()
@@ -54,6 +54,8 @@ def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, k
             cmd += ["--join", join]
         if liveness:
             cmd.append("--liveness")
+        if regsets:
+            cmd.append("--regsets")
         if not hlines:
             cmd.append("--no-hlines")
         if not detect:
@@ -117,6 +119,29 @@ class Canon:
 
 def golden(name: str) -> str:
     return os.path.join(GOLDEN, name)
+
+
+def golden_text(name: str) -> str:
+    """A fixture's text; `.xz` fixtures (the frozen torch SASS) are decompressed."""
+    import lzma
+    path = golden(name)
+    if path.endswith(".xz"):
+        with lzma.open(path, "rt") as f:
+            return f.read()
+    with open(path) as f:
+        return f.read()
+
+
+def regsets(text: str, **kw) -> dict:
+    """(kernel, idx) -> (defs, uses, live) of the oracle's O16 register model (G lines)."""
+    def ints(v):
+        return set() if v == "-" else set(map(int, v.split(",")))
+    out = {}
+    for line in run(text, regsets=True, hist=False, **kw).splitlines():
+        if line.startswith("G "):
+            f = line.split()
+            out[(int(f[1]), int(f[2]))] = (ints(f[3][4:]), ints(f[4][4:]), ints(f[5][5:]))
+    return out
 
 
 def sass_ops(path: str) -> dict:

@@ -498,7 +498,8 @@ LRM_FIXTURES = [(f"lineinfo/{k}.{d}.sass", f"lineinfo/{k}.lrm.txt") for k in LIN
                 for d in ("nvdisasm", "cuobjdump")] + \
     [(f"{k}.{a}.sass", f"{k}.{a}.lrm.txt") for k in ("sgemm_naive", "jacobi", "mixbench", "atomics", "conv")
      for a in ("sm_100a", "sm_70")] + \
-    [(f"spill.r{c}.sm_100a.sass", f"spill.r{c}.sm_100a.lrm.txt") for c in (24, 32, 40, 64)]
+    [(f"spill.r{c}.sm_100a.sass", f"spill.r{c}.sm_100a.lrm.txt") for c in (24, 32, 40, 64)] + \
+    [(f"b200/{k}.sm_100a.sass", f"b200/{k}.sm_100a.lrm.txt") for k in ("wmma", "v8", "tmem")]
 
 
 @pytest.mark.parametrize("sass,lrm", LRM_FIXTURES)
@@ -520,3 +521,75 @@ def test_register_pressure_equals_nvdisasm_life_ranges(sass, lrm):
             assert len(got[k]) >= len(w)
             assert [c for c, _ in g] == w, (sass, k)
             assert [a for _, a in g] == [w[0]] + [w[i] - w[i - 1] for i in range(1, len(w))]
+
+
+# --------------------------------------------------------------------------- O16 on sm_100a forms (R38)
+# nvdisasm -lrm narrow prints, per instruction, which GPRs it assigns, reads and keeps live. The
+# oracle's register model must give the same three sets on every instruction: this pins the
+# operand widths of the B200-native forms (R38): LDG/STG.E.ENL2.256 (two register quads), HMMA
+# fragments, LDSM/STSM, LDTM/STTM (tcgen05), CS2R/LEPC pairs, IMAD.HI's 64-bit addend, conversion
+# type roles, the call ABI (clobbers, callee-saved registers live at RET) and REG:N from -res-usage.
+B200_NARROW = [(f"b200/{k}.sm_100a.sass", f"b200/{k}.sm_100a.narrow.txt") for k in ("wmma", "v8", "tmem")] + [
+    ("torch/k1779_tcgen05_gemm.sass.xz", "torch/k1779_tcgen05_gemm.narrow.txt.xz"),
+    ("torch/cubin1810.sass.xz", "torch/cubin1810.narrow.txt.xz"),
+]
+
+
+def _narrow(name):
+    import lrm_table
+    return lrm_table.parse(orc.golden_text(name).splitlines(keepends=True))
+
+
+@pytest.mark.parametrize("sass,narrow", B200_NARROW)
+def test_register_sets_equal_nvdisasm_table(sass, narrow):
+    """Per instruction: oracle defs == nvdisasm '^'/'x' columns, uses == 'v'/'x', live == every
+    marked column (the set whose size is the count of O16)."""
+    want = _narrow(narrow)
+    got = orc.regsets(orc.golden_text(sass))
+    n = 0
+    for k, fn in enumerate(want):
+        for i, (txt, cnt, d, u, live) in enumerate(fn):
+            gd, gu, gl = got[(k, i)]
+            assert (gd, gu, gl) == (d, u, live), (sass, k, i, txt)
+            assert len(gl) == cnt
+            n += 1
+    assert n == sum(len(f) for f in want) and n > 0
+
+
+def test_real_torch_cubin_live_counts_equal_nvdisasm():
+    """A real sm_100 cubin of the torch wheel (ELF 1810 of libtorch_cuda.so: 200 kernels, 38,585
+    instructions, tests/golden/torch/make_torch_fixtures.sh): every L line equals nvdisasm -lrm count."""
+    import tempfile
+    with tempfile.NamedTemporaryFile("w", suffix=".txt", delete=False) as f:
+        f.write(orc.golden_text("torch/cubin1810.lrm.txt.xz"))
+    want = _lrm_gpr(f.name)
+    got = {}
+    for line in orc.run(orc.golden_text("torch/cubin1810.sass.xz"), liveness=True, hist=False).splitlines():
+        if line.startswith("L "):
+            _, k, i, c, a = line.split()
+            got.setdefault(int(k), []).append(int(c))
+    assert len(want) == len(got) == 200
+    assert sum(len(w) for w in want) == 38585
+    for k, w in enumerate(want):
+        assert got[k][:len(w)] == w, k
+
+
+def test_256bit_loads_are_already_vectorised():
+    """a load that already moves a vector (LDG.E.64 in the paper's DP mixbench) is
+    "already vectorised" and is not flagged. sm_100a's LDG.E.ENL2.256 fills two register quads
+    (R38a): it counts as already vectorised, is never a VEC site, and its second quad is a
+    destination (its last writer for later readers), not a source."""
+    text = orc.golden_text("b200/v8.sm_100a.sass")
+    c = Canon(orc.run(text))
+    ops = orc.sass_ops(golden("b200/v8.sm_100a.sass"))
+    ldg256 = [i for i, o in ops.items() if o.startswith("LDG") and o.endswith(".256")]
+    assert len(ldg256) == 1
+    assert c.kstats()[0]["vec_already"] == 1
+    assert ldg256[0] not in {s["idx"] for s in c.sites("VEC")}
+    # the two 32-bit loads off the second base form the only VEC group (offsets 0 and +4)
+    vec = c.sites("VEC")
+    assert len(vec) == 2 and {(s["min"], s["max"], s["n"], s["contig"]) for s in vec} == {("0", "4", "2", "1")}
+    g = orc.regsets(text)
+    i = ldg256[0]
+    assert g[(0, i)][0] == set(range(4, 12))  # LDG.E.ENL2.256 R4, R8, [R6.64]: R4..R11 written
+    assert g[(0, i)][1] == {6, 7}             # ... and only the address pair read

@@ -5,7 +5,7 @@
  *     each flagged memory instruction carrying a bounded backward def-use trace;
  *   - warp-stall attribution: PC samples with stall reasons aggregated per PC and
  *     attributed "to the instruction detected by the SASS Analysis engine".
- * Readings of the paper where it is silent are numbered R1..R31 in DESIGN.md §3.
+ * Readings of the paper where it is silent are numbered R1..R38 in DESIGN.md §3.
  *
  * Conventions (all entry points):
  *   - Every call returns a gs_status; no exception or abort crosses the ABI. On error the message
@@ -110,8 +110,10 @@ typedef struct {
 /* One ranked site (host or device output of gs_rank_sites). 168 bytes. */
 typedef struct {
   uint32_t kernel, idx, rule, pad;
-  uint64_t rel, tot, ktot; /* REL-reason samples, all samples at the site PC, kernel total */
-  uint32_t counts[32];     /* histogram row of the site PC                                           */
+  uint64_t rel, tot, ktot; /* REL-reason samples and all samples of the joined row, kernel total */
+  uint32_t counts[32];     /* the joined histogram row: the site PC row (GS_JOIN_PC), the sum over its  */
+                           /* source line (GS_JOIN_LINE) or over it and its consumers (GS_JOIN_CONSUMER);
+                              32-bit, saturating (R34)                                               */
 } gs_ranked_site;
 
 /* Create a context on `device` that enqueues on `cuda_stream` (a cudaStream_t; NULL = legacy

@@ -31,6 +31,7 @@ namespace {
 
 void free_loaded(gs_ctx* c) {
   detect_free(c);
+  rank_reset_graph(c);
   if (c->d_rec) cudaFree(c->d_rec);
   if (c->d_kd) cudaFree(c->d_kd);
   if (c->d_wd) cudaFree(c->d_wd);
@@ -132,6 +133,8 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   c->use_off_h.assign(1, 0);
   c->use_reg_h.clear();
   c->tgt_h.clear();
+  c->xoff_h.assign(1, 0);
+  c->xtgt_h.clear();
   c->n_cand = c->n_ldg = c->n_store = 0;
   std::vector<Rec> recs;
   recs.reserve(P);
@@ -141,7 +144,7 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     KDesc& K = c->kd_h[k];
     K.first = slot;
     K.n = (uint32_t)pk.recs.size();
-    K.param_base = pk.param_base;
+    K.param_base = pk.param_base | (std::min<uint32_t>(pk.nregs, 255u) << 16);
     K.win0 = (uint32_t)c->wd_h.size();
     for (uint32_t s = 0; s < K.n; s += kWin) {
       WDesc W{(uint32_t)k, slot + s, std::min(kWin, K.n - s), 0};
@@ -163,7 +166,11 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
       const uint32_t base = (uint32_t)c->use_reg_h.size();
       for (size_t i = 1; i < pk.use_off.size(); i++) c->use_off_h.push_back(base + pk.use_off[i]);
       c->use_reg_h.insert(c->use_reg_h.end(), pk.use_reg.begin(), pk.use_reg.end());
-      c->tgt_h.insert(c->tgt_h.end(), pk.tgt.begin(), pk.tgt.end());
+      const int32_t x0 = (int32_t)c->xoff_h.size() - 1;  // indirect-branch lists: global list ids
+      for (int32_t t : pk.tgt) c->tgt_h.push_back(t <= -2 ? t - x0 : t);
+      const uint32_t xbase = (uint32_t)c->xtgt_h.size();
+      for (size_t x = 1; x < pk.xtgt_off.size(); x++) c->xoff_h.push_back(xbase + pk.xtgt_off[x]);
+      c->xtgt_h.insert(c->xtgt_h.end(), pk.xtgt.begin(), pk.xtgt.end());
     }
     c->lines_h.insert(c->lines_h.end(), pk.lines.begin(), pk.lines.end());
     c->names.push_back(std::move(pk.name));

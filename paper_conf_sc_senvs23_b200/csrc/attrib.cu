@@ -236,8 +236,9 @@ template <int OUT, int N>
 __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t* tab, uint32_t spare, uint32_t one,
                                         const Spill& S, uint32_t& bad) {
   // Per sample: off, in, word, half increment, one returning shared atomic, one mask test. A lane
-  // outside the window adds to its spare word (never flushed; kept nonzero) and its mask is all
-  // ones, so the same test flags "outside the window" and "half already >= 0x8000". One vote per
+  // outside the window adds 2 to its spare word (never flushed; initialised to 1, so it stays odd
+  // and can never wrap to 0) and its mask is all ones, so the same test flags "outside the window"
+  // and "half already >= 0x8000". One vote per
   // batch; the rare path re-reads the words to find the halves to drain. Every thread that sees
   // a half >= 0x8000 checks it before its next batch, so a half overshoots 0x8000 by at most
   // (threads x batch) < 0x8000 increments before it is drained.
@@ -247,7 +248,7 @@ __device__ __forceinline__ void count16(const uint32_t (&w)[N], Win W, uint32_t*
     const uint32_t off = w[q] - W.wb;
     const bool in = off < W.lim;
     const uint32_t inc = one << ((off & 1u) << 4);
-    flag |= atomicAdd(tab + (in ? off >> 1 : spare), inc) & (in ? inc << 15 : 0xffffffffu);
+    flag |= atomicAdd(tab + (in ? off >> 1 : spare), in ? inc : 2u) & (in ? inc << 15 : 0xffffffffu);
   }
   const uint32_t am = __activemask();
   if (__any_sync(am, flag)) {
@@ -482,8 +483,8 @@ __device__ __forceinline__ uint32_t hot_w(const uint32_t (&w)[N], Win W, uint32_
     const uint32_t off = w[q] - W.wb;
     const bool in = off < W.lim;
     if (P16) {
-      const uint32_t inc = 1u << ((off & 1u) << 4);
-      flag |= atomicAdd(tab + (in ? off >> 1 : spare), inc) & (in ? inc << 15 : 0xffffffffu);
+      const uint32_t inc = 1u << ((off & 1u) << 4);  // spare word: +2 keeps it odd (nonzero)
+      flag |= atomicAdd(tab + (in ? off >> 1 : spare), in ? inc : 2u) & (in ? inc << 15 : 0xffffffffu);
     } else {
       atomicAdd(tab + (in ? off : spare), 1u);
       flag |= in ? 0u : 1u;
@@ -519,7 +520,13 @@ __device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, u
 }
 
 // ---------------------------------------------------------------------- PRIVATE
-// fixed slot range per CTA (range = blockIdx % n_ranges); the CTA walks its sample chunk
+// fixed slot range per CTA (range = blockIdx % n_ranges); the CTA walks its sample chunk.
+// 16-bit exactness (count16): the increment that takes a half from 0x7FFF to 0x8000 is not flagged,
+// every later one is, and a thread drains at the end of its batch. In the worst case every one of
+// the kThreads threads adds a whole batch (4 * kVec samples) to the half after it reached 0x8000
+// and before any drain, so the half peaks at 0x7FFF + kThreads * 4 * kVec: at most 0xFFFF, never a
+// carry into the neighbouring bin, iff kThreads * 4 * kVec <= 0x8000.
+static_assert(kThreads * 4 * kVec <= 0x8000, "PRIVATE 16-bit counters: a half could carry into its neighbour");
 template <bool P16>
 __global__ void __launch_bounds__(kThreads, 1)
     k_hist_smem(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv, uint32_t n_ranges,

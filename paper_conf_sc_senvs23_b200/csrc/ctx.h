@@ -64,7 +64,9 @@ struct gs_ctx {
   uint32_t n_lgroups = 0;             // source-line groups (kernel, file, line), 0 without line info
   std::vector<uint32_t> use_off_h;     // register-pressure inputs (R36), uploaded on first use:
   std::vector<uint8_t> use_reg_h;      //   GPR uses per slot (CSR, global offsets), branch targets
-  std::vector<int32_t> tgt_h;          //   (kernel-local index, -1 none)
+  std::vector<int32_t> tgt_h;          //   (kernel-local index, -1 none, -2 - x indirect-branch list x)
+  std::vector<uint32_t> xoff_h;        // indirect-branch successor lists (R38i, CSR over x)
+  std::vector<int32_t> xtgt_h;
 
   // ---- device copies
   gs::Rec* d_rec = nullptr;
@@ -77,6 +79,8 @@ struct gs_ctx {
   uint32_t* d_use_off = nullptr;  // register pressure inputs on the device (lazy)
   uint8_t* d_use_reg = nullptr;
   int32_t* d_tgt = nullptr;
+  uint32_t* d_xoff = nullptr;
+  int32_t* d_xtgt = nullptr;
   void* d_lv = nullptr;           // liveness scratch
   size_t lv_bytes = 0;
 
@@ -128,6 +132,7 @@ struct gs_ctx {
   void* d_sort_tmp = nullptr;
   size_t sort_tmp_bytes = 0;
   unsigned long long* d_ktot = nullptr;
+  uint64_t ktot_cap = 0;
   gs_ranked_site* d_ranked = nullptr;
   uint32_t* d_jrow = nullptr;   // GS_JOIN_LINE / GS_JOIN_CONSUMER: joined row per site (32 u32, saturated)
   // GS_JOIN_CONSUMER (R37), built by gs_detect: per GPR use its defining slot, and per slot the
@@ -212,6 +217,7 @@ gs_status liveness_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint16_t* d_live);
 gs_status uses_upload(gs_ctx* c);
 void liveness_free(gs_ctx* c);
 void rank_free(gs_ctx* c);
+void rank_reset_graph(gs_ctx* c);
 
 // device-wide exclusive scan of u32 counts into u32 or u64 offsets; total written to *d_total
 gs_status scan_u32(gs_ctx* c, const uint32_t* in, uint32_t* out, uint64_t n, unsigned long long* d_total);

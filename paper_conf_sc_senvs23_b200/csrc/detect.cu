@@ -99,11 +99,13 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
     const bool valid = i < W.len;
     const uint64_t g = (uint64_t)W.start + i;
     const Rec r = rr[u];
-    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r);
+    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), dst2 = r_dst2(r);
     if (valid && dw && reg_live(dst)) {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
       const uint32_t cap = reg_cap(dst);
       for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicMax(&last[warp][dst + q], v);
+      if (reg_live(dst2))  // second quad of a 256-bit load (R38a)
+        for (uint32_t q = 0; q < dw && dst2 + q <= reg_cap(dst2); q++) atomicMax(&last[warp][dst2 + q], v);
     }
     if (valid && op == OP_LDG) narith[g] = 0;
     if (valid && op == OP_BRA && (r_flags(r) & F_BRA_OK)) {
@@ -122,7 +124,8 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
       n_gatom += (cls & C_GATOM) ? 1 : 0;
       n_satom += (cls & C_SATOM) ? 1 : 0;
       n_conv += (cls & C_CONV) ? 1 : 0;
-      n_vec += (op == OP_LDG && (r_flags(r) & F_HASMEM) && (r_aw(r) == AW_64 || r_aw(r) == AW_128)) ? 1 : 0;
+      n_vec += (op == OP_LDG && (r_flags(r) & F_HASMEM) && (r_aw(r) == AW_64 || r_aw(r) == AW_128 || r_aw(r) == AW_256))
+                   ? 1 : 0;  // "already vectorised" (R38a)
     }
     }
   }
@@ -216,9 +219,13 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
     rnext = i + 32 < W.len ? ld_rec(rec, g + 32) : Rec{0, 0, 0, 0};
     const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
     const bool writes = valid && dw && reg_live(dst);
-    const uint32_t cap = reg_cap(dst);
+    const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
+    const bool writes2 = reg_live(dst2);
+    const uint32_t cap = reg_cap(dst), cap2 = reg_cap(dst2);
     if (writes)
       for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicOr(&M[dst + q], 1u << lane);
+    if (writes2)
+      for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++) atomicOr(&M[dst2 + q], 1u << lane);
     const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
     __syncwarp();
     // RD value: ((def + 1) << 1) | def_is_global_load, or 0 for ENTRY
@@ -278,10 +285,15 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
       for (uint32_t q = 0; q < dw && dst + q <= cap; q++)
         if ((M[dst + q] & gt) == 0) T[dst + q] = v;
+      if (writes2)
+        for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++)
+          if ((M[dst2 + q] & gt) == 0) T[dst2 + q] = v;
     }
     __syncwarp();
     if (writes)
       for (uint32_t q = 0; q < dw && dst + q <= cap; q++) M[dst + q] = 0;
+    if (writes2)
+      for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++) M[dst2 + q] = 0;
     __syncwarp();
   }
 }
@@ -326,8 +338,12 @@ __global__ void __launch_bounds__(kWarps * 32) k_consumers(const Rec* __restrict
     const Rec r = valid ? ld_rec(rec, g) : Rec{0, 0, 0, 0};
     const uint32_t dst = r_dst(r), dw = r_dstw(r);
     const bool writes = valid && dw && dst < 255;  // GPR definitions only
+    const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
+    const bool writes2 = dst2 < 255;
     if (writes)
       for (uint32_t q = 0; q < dw && dst + q < 255; q++) atomicOr(&M[dst + q], 1u << lane);
+    if (writes2)
+      for (uint32_t q = 0; q < dw && dst2 + q < 255; q++) atomicOr(&M[dst2 + q], 1u << lane);
     __syncwarp();
     if (valid) {
       const uint32_t q0 = use_off[g], q1 = use_off[g + 1];
@@ -347,10 +363,15 @@ __global__ void __launch_bounds__(kWarps * 32) k_consumers(const Rec* __restrict
       const uint32_t v = (uint32_t)((g + 1) << 1);
       for (uint32_t q = 0; q < dw && dst + q < 255; q++)
         if ((M[dst + q] & gt) == 0) T[dst + q] = v;
+      if (writes2)
+        for (uint32_t q = 0; q < dw && dst2 + q < 255; q++)
+          if ((M[dst2 + q] & gt) == 0) T[dst2 + q] = v;
     }
     __syncwarp();
     if (writes)
       for (uint32_t q = 0; q < dw && dst + q < 255; q++) M[dst + q] = 0;
+    if (writes2)
+      for (uint32_t q = 0; q < dw && dst2 + q < 255; q++) M[dst2 + q] = 0;
     __syncwarp();
   }
 }
@@ -397,7 +418,7 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restric
     if (cj & C_CONSTLOAD) {
       const int32_t off = r_imm(rj) + 4 * (int32_t)(r - r_dst(rj));
       const uint32_t bank = r_cbank(rj);
-      if (bank == 0 && off >= (int32_t)K.param_base) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
       else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
       break;
     }
@@ -407,7 +428,7 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restric
     if (pk == PK_CONST) {
       const int32_t off = r_imm(rj);
       const uint32_t bank = r_cbank(rj);
-      if (bank == 0 && off >= (int32_t)K.param_base) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
       else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
       break;
     }

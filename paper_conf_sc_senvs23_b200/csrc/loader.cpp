@@ -200,7 +200,7 @@ const OpName kOps[] = {
     {"IADD3", OP_IADD3}, {"VIADD", OP_VIADD}, {"IMAD", OP_IMAD}, {"IMUL", OP_IMUL},
     {"IMNMX", OP_IMNMX}, {"VIMNMX", OP_VIMNMX}, {"IABS", OP_IABS}, {"LEA", OP_LEA},
     {"ULEA", OP_ULEA}, {"UIADD3", OP_UIADD3}, {"UIMAD", OP_UIMAD}, {"HMMA", OP_HMMA},
-    {"DMNMX", OP_DMNMX}, {"FCHK", OP_FCHK},
+    {"DMNMX", OP_DMNMX}, {"FCHK", OP_FCHK}, {"CALL", OP_CALL}, {"RET", OP_RET}, {"BRX", OP_BRX},
 };
 
 uint8_t op_lookup(Sv m) {
@@ -215,20 +215,61 @@ struct Line {
   long lineno;
 };
 
-// Register-pressure inputs of one instruction (O16 / R36): GPR uses with operand widths expanded,
-// guard, exit, predicate operand of a branch, branch target (pc) or unresolved label.
+// Register-pressure inputs of one instruction (O16 / R36, R38): GPR uses with operand widths
+// expanded, guard, exit, predicate/register condition of a branch, branch target (pc) or unresolved
+// label, indirect-branch target labels, highest GPR touched.
 struct LiveOut {
   std::vector<uint8_t>* uses = nullptr;
   bool guarded = false, exit = false, brpred = false;
   long long target = -1;
   std::string label;
+  std::vector<std::string> brx;  // nvdisasm BRANCH_TARGETS of a BRX (R38i)
+  int maxreg = -1;
 };
 
 inline bool is64type(Sv m) { return m.eq("F64") || m.eq("S64") || m.eq("U64"); }
-inline bool istype(Sv m) {
-  static const char* k[] = {"F64", "S64", "U64", "F32", "F16", "BF16", "S32", "U32", "S16", "U16", "S8", "U8", "TF32"};
+inline bool isinttype(Sv m) {
+  static const char* k[] = {"S64", "U64", "S32", "U32", "S16", "U16", "S8", "U8"};
   for (auto* x : k) if (m.eq(x)) return true;
   return false;
+}
+inline bool isfloattype(Sv m) {
+  static const char* k[] = {"F64", "F32", "F16", "BF16", "TF32", "E4M3", "E5M2"};
+  for (auto* x : k) if (m.eq(x)) return true;
+  return false;
+}
+
+// R38e: register widths {destination, source} of a conversion from the roles of its type modifiers
+void conv_roles(Sv mn, const Sv* mods, int nm, uint32_t* dw, uint32_t* sw) {
+  Sv t[8];
+  int nt = 0;
+  for (int q = 0; q < nm && nt < 8; q++)
+    if (isinttype(mods[q]) || isfloattype(mods[q])) t[nt++] = mods[q];
+  Sv d{}, src{};
+  if (mn.eq("F2F") || mn.eq("I2I") || mn.eq("F2FP")) {
+    if (nt >= 1) d = t[0];
+    if (nt >= 2) src = t[1];
+  } else if (mn.eq("I2F") || mn.eq("I2FP")) {
+    for (int q = 0; q < nt; q++) (isfloattype(t[q]) ? d : src) = t[q];
+  } else if (mn.eq("F2I") || mn.eq("F2IP")) {
+    for (int q = 0; q < nt; q++) (isinttype(t[q]) ? d : src) = t[q];
+  }
+  *dw = d.n && is64type(d) ? 2 : 1;
+  *sw = src.n && is64type(src) ? 2 : 1;
+}
+
+// R38d: registers per thread of a tensor-memory access LDTM/STTM[.<shape>].x<N>
+uint32_t tmem_width(const Sv* mods, int nm) {
+  uint32_t per = 1, x = 1;
+  for (int q = 0; q < nm; q++) {
+    if (mods[q].eq("16dp128bit")) per = 2;
+    else if (mods[q].eq("16dp256bit")) per = 4;
+    else if (mods[q].n > 1 && mods[q][0] == 'x' && mods[q][1] >= '0' && mods[q][1] <= '9') {
+      x = 0;
+      for (size_t k = 1; k < mods[q].n && mods[q][k] >= '0' && mods[q][k] <= '9'; k++) x = x * 10 + (mods[q][k] - '0');
+    }
+  }
+  return per * x;
 }
 
 // One instruction -> record. Returns false with msg on a malformed line.
@@ -264,14 +305,18 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, L
   Sv raw_last;
   int no = 0;
   {
+    // operands are separated by top-level commas, or by blanks where SASS writes no comma
+    // ("RET.REL.NODEC R2 0x0", "BRX R4 -0x43d0", R38i)
     int depth = 0;
     size_t s = 0;
     for (size_t q = 0; q <= rest.n; q++) {
       char c = q < rest.n ? rest[q] : ',';
       if (c == '[' || c == '{') depth++;
       else if (c == ']' || c == '}') depth--;
-      if ((c == ',' && depth == 0) || q == rest.n) {
+      const bool blank = (c == ' ' || c == '\t') && depth == 0;
+      if ((c == ',' && depth == 0) || q == rest.n || blank) {
         Sv tok{rest.p + s, q - s};
+        if (blank && !trim(tok).n) { s = q + 1; continue; }
         if (q < rest.n || trim(tok).n) {
           if (no >= 16) { *msg = "too many operands"; return false; }
           ops[no++] = classify(tok);
@@ -281,32 +326,60 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, L
       }
     }
   }
-  // destination (R23)
-  int dpos = -1;
-  if (no >= 1 && ops[0].k == T_REG) dpos = 0;
+  // HMMA fragment widths (R38c): m16 n8 kK tile, input element bits b -> A = 16Kb/1024, B = 8Kb/1024
+  // registers, accumulator 4 (F32) or 2 (F16)
+  uint32_t mma_a = 1, mma_b = 1, mma_acc = 1;
+  if (op == OP_HMMA) {
+    uint32_t K = 8, bits = 16;
+    bool acc_seen = false, acc16 = false;
+    for (int q = 0; q < nm; q++) {
+      if (q == 0 && mods[q].n >= 4 && mods[q][0] >= '0' && mods[q][0] <= '9') {
+        K = 0;
+        for (size_t k = 3; k < mods[q].n; k++) K = K * 10 + (uint32_t)(mods[q][k] - '0');
+      } else if (!acc_seen && isfloattype(mods[q])) {
+        acc_seen = true;
+        acc16 = mods[q].eq("F16");
+      } else if (mods[q].eq("TF32")) bits = 32;
+      else if (mods[q].eq("E4M3") || mods[q].eq("E5M2")) bits = 8;
+    }
+    mma_a = std::max(1u, 16 * K * bits / 1024);
+    mma_b = std::max(1u, 8 * K * bits / 1024);
+    mma_acc = acc16 ? 2 : 4;
+  }
+  uint32_t cdw = 1, csw = 1;
+  const bool conv = op == OP_F2F || op == OP_I2F || op == OP_F2I || op == OP_I2I || op == OP_I2FP ||
+                    op == OP_F2IP || op == OP_F2FP;
+  if (conv) conv_roles(mn, mods, nm, &cdw, &csw);
+  // destination (R23); opcodes whose register operands are all read have none (R38f)
+  const bool no_dst = mn.eq("WARPSYNC") || mn.eq("BRX") || mn.eq("BRXU") || mn.eq("JMX") || mn.eq("JMXU") ||
+                      mn.eq("RET") || mn.eq("CALL") || mn.eq("NANOSLEEP") || mn.eq("BAR") || mn.eq("YIELD") ||
+                      mn.eq("BPT");
+  int dpos = -1, dpos2 = -1;
+  if (no_dst) dpos = -1;
+  else if (no >= 1 && ops[0].k == T_REG) dpos = 0;
   else if (no >= 2 && ops[0].k == T_PRED && ops[1].k == T_REG && op != OP_FCHK) dpos = 1;
-  uint32_t dst = kRegNone, dstw = 0;
+  uint32_t dst = kRegNone, dstw = 0, dst2 = kRegNone;
   if (dpos >= 0) {
     dst = (uint32_t)ops[dpos].reg;
-    // width table W (R24)
-    if (has("128")) dstw = 4;
-    else if (op == OP_HMMA) dstw = has("F32") ? 4 : 2;
+    // width table W (R24 as revised by R38)
+    if (has("256")) dstw = 4;  // R38a: each of the two destination quads
+    else if (has("128")) dstw = 4;
+    else if (op == OP_HMMA) dstw = mma_acc;
     else if (mn.eq("LDSM")) dstw = has("4") ? 4 : (has("2") ? 2 : 1);
+    else if (op == OP_LDTM) dstw = tmem_width(mods, nm);
     else if (has("64") || has("WIDE")) dstw = 2;
+    else if (op == OP_CS2R) dstw = has("32") ? 1 : 2;  // R38b
+    else if (mn.eq("LEPC")) dstw = 2;
     else if (op == OP_DADD || op == OP_DMUL || op == OP_DFMA || op == OP_DMNMX) dstw = 2;
-    else if (op == OP_F2F || op == OP_I2F || op == OP_F2I || op == OP_I2I) {
-      dstw = 1;
-      static const char* k64[] = {"F64", "S64", "U64"};
-      static const char* k32[] = {"F32", "F16", "BF16", "S32", "U32", "S16", "U16", "S8", "U8", "TF32", "E4M3", "E5M2"};
-      for (int q = 0; q < nm; q++) {
-        bool hit64 = false, hit32 = false;
-        for (auto* x : k64) hit64 |= mods[q].eq(x);
-        for (auto* x : k32) hit32 |= mods[q].eq(x);
-        if (hit64) { dstw = 2; break; }
-        if (hit32) break;
-      }
-    } else dstw = 1;
+    else if (conv) dstw = cdw;
+    else dstw = 1;
+    if (dstw > 255) { *msg = "destination wider than 255 registers"; return false; }
+    if (has("256") && dpos + 1 < no && ops[dpos + 1].k == T_REG) {  // R38a: LDG.E.ENL2.256 Ra, Rb
+      dpos2 = dpos + 1;
+      dst2 = (uint32_t)ops[dpos2].reg;
+    }
   }
+  const int last_dst = dpos2 >= 0 ? dpos2 : dpos;
   // memory operand
   int mem = -1;
   for (int q = 0; q < no; q++) if (ops[q].k == T_MEM) { mem = q; break; }
@@ -328,11 +401,16 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, L
       if (mods[q].eq("U16") || mods[q].eq("S16")) { aw = AW_16; break; }
       if (mods[q].eq("64")) { aw = AW_64; break; }
       if (mods[q].eq("128")) { aw = AW_128; break; }
+      if (mods[q].eq("256")) { aw = AW_256; break; }
     }
+  }
+  if (dst2 != kRegNone) {  // the second quad travels in s2 (record.h)
+    s[2] = dst2;
+    flags |= F_DST2;
   }
   if (cls & C_ARITH) {  // register sources after dst (R25), at most 4
     int ns = 0;
-    for (int q = dpos + 1; q < no; q++)
+    for (int q = last_dst + 1; q < no; q++)
       for (int t = 0; t < ops[q].nregs; t++) {
         int r = ops[q].regs[t];
         if (!reg_live((uint32_t)r)) continue;
@@ -379,45 +457,60 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, L
       }
     }
   }
-  // register-pressure inputs (R36)
+  // register-pressure inputs (R36, R38)
   lo->exit = mn.eq("EXIT") || mn.eq("RET");
-  if (op == OP_BRA) {
-    for (int q = 0; q + 1 < no; q++) lo->brpred |= ops[q].k == T_PRED && ops[q].predvar;
+  if (op == OP_BRA) {  // a predicate or register condition before the target may fall through (R38i)
+    for (int q = 0; q + 1 < no; q++) lo->brpred |= (ops[q].k == T_PRED && ops[q].predvar) || ops[q].k == T_REG;
     long long t;
     Sv lt = trim(raw_last);
     if (no > 0 && to_int(lt, &t)) lo->target = t;
     else if (lt.n > 4 && lt[0] == '`' && lt[1] == '(' && lt[lt.n - 1] == ')') lo->label.assign(lt.p + 2, lt.n - 3);
   }
   {
-    int srcw = (op == OP_DADD || op == OP_DMUL || op == OP_DFMA || op == OP_DMNMX || mn.eq("DSETP")) ? 2 : 1;
-    if (cls & C_CONV) {
-      int nt = 0;
-      for (int q = 0; q < nm; q++)
-        if (istype(mods[q]) && nt++ == 1 && is64type(mods[q])) srcw = 2;  // second type = source
-    }
+    const size_t use0 = lo->uses->size();
+    uint32_t srcw = (op == OP_DADD || op == OP_DMUL || op == OP_DFMA || op == OP_DMNMX || mn.eq("DSETP")) ? 2 : 1;
+    if (conv) srcw = csw;  // R38e
     const bool store_like = op == OP_STG || op == OP_STS || op == OP_STL || op == OP_ST || op == OP_RED ||
-                            op == OP_REDG || op == OP_ATOMG || op == OP_ATOM || op == OP_ATOMS;
-    int dataw = 1;
+                            op == OP_REDG || op == OP_ATOMG || op == OP_ATOM || op == OP_ATOMS || mn.eq("STSM") ||
+                            mn.eq("STTM") || mn.eq("STAS");
+    uint32_t dataw = 1;  // data operand width of a store (R36, R38a/d)
     for (int q = 0; q < nm; q++) if (mods[q].eq("64") || is64type(mods[q])) dataw = 2;
-    for (int q = 0; q < nm; q++) if (mods[q].eq("128")) dataw = 4;
+    if (mn.eq("STSM")) dataw = has("4") ? 4 : (has("2") ? 2 : 1);
+    if (mn.eq("STTM")) dataw = tmem_width(mods, nm);
+    for (int q = 0; q < nm; q++) if (mods[q].eq("128") || mods[q].eq("256")) dataw = 4;
     const bool ext = has("E"), wide_imad = op == OP_IMAD && has("WIDE");
+    const bool hi_add = op == OP_IMAD && has("HI");  // R38h: 64-bit addend
+    const bool target_pair = op == OP_BRX || op == OP_RET || op == OP_CALL || mn.eq("BRXU") || mn.eq("JMX") ||
+                             mn.eq("JMXU");  // R38g: 64-bit target address
+    int last_mem = -1;  // R38j: .E names the last memory operand
+    for (int q = 0; q < no; q++) if (ops[q].k == T_MEM) last_mem = q;
     int srcidx = 0;
     for (int q = 0; q < no; q++) {
-      if (q == dpos) continue;
+      if (q == dpos || q == dpos2) continue;
       const Operand& o = ops[q];
       for (int t = 0; t < o.nregs; t++) {
         const int r = o.regs[t];
         if (r < 0 || r >= 255) continue;  // RZ and uniform registers
-        int w;
-        if (o.k == T_MEM) w = (r == o.base && (o.wide || ext)) ? 2 : 1;
+        uint32_t w;
+        if (o.k == T_MEM) w = (r == o.base && (o.wide || (ext && q == last_mem))) ? 2 : 1;
         else if (o.k == T_CREF) w = 1;
+        else if (target_pair) w = 2;
         else if (store_like && q > 0) w = dataw;
-        else if (wide_imad && srcidx == 2) w = 2;
+        else if (op == OP_HMMA) w = srcidx == 0 ? mma_a : (srcidx == 1 ? mma_b : mma_acc);
+        else if ((wide_imad || hi_add) && srcidx == 2) w = 2;
         else w = srcw;
-        for (int k2 = 0; k2 < w && r + k2 < 255; k2++) lo->uses->push_back((uint8_t)(r + k2));
+        for (uint32_t k2 = 0; k2 < w && r + (int)k2 < 255; k2++) lo->uses->push_back((uint8_t)(r + k2));
       }
-      if (q > dpos && o.k != T_PRED) srcidx++;
+      if (q > last_dst && o.k != T_PRED) srcidx++;
     }
+    if (op == OP_CALL) {  // R38g: a call reads R0 and the stack pointer R1
+      lo->uses->push_back(0);
+      lo->uses->push_back(1);
+    }
+    // highest GPR touched (the kernel's register count when the dump has no REG:N, R38k)
+    for (size_t q = use0; q < lo->uses->size(); q++) lo->maxreg = std::max(lo->maxreg, (int)(*lo->uses)[q]);
+    for (uint32_t d : {dst, dst2})
+      if (d < 255) lo->maxreg = std::max(lo->maxreg, (int)std::min<uint32_t>(d + dstw - 1, 254));
   }
   if (lo->guarded) flags |= F_PRED;
   if (lo->exit) flags |= F_EXIT;
@@ -436,6 +529,7 @@ struct Segment {
   int sm;
   std::string name;
   bool header;        // false for an anonymous leading kernel
+  int regcount;       // REG:N of a cuobjdump -res-usage block for this function, -1 if none (R38k)
 };
 
 // nvdisasm function label ".text.<name>:"
@@ -453,6 +547,9 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
   std::map<std::string, long long> labels;                  // branch label -> pc
   std::vector<std::string> pending;
   std::vector<std::pair<size_t, std::string>> fwd;          // branches to labels not seen yet
+  std::vector<std::vector<std::string>> brx_labels;         // BRANCH_TARGETS of each BRX (R38i)
+  std::vector<size_t> brx_at;
+  int maxreg = -1;
   pk->use_off.assign(1, 0);
   size_t p = seg.begin;
   while (p < seg.end) {
@@ -496,6 +593,27 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     for (auto& lb : pending) labels[lb] = pc;
     pending.clear();
     Sv ins{body.p, semi};
+    // nvdisasm annotates an indirect branch with its targets: (*"BRANCH_TARGETS .L_a,.L_b"*) (R38i)
+    std::vector<std::string> targets;
+    for (size_t q = 0; q + 2 < ins.n; q++)
+      if (ins[q] == '(' && ins[q + 1] == '*' && ins[q + 2] == '"') {
+        Sv a{ins.p + q, ins.n - q};
+        size_t bt;
+        if (contains(a, "BRANCH_TARGETS ", &bt)) {
+          size_t e = bt + 15;
+          while (e < a.n && a[e] != '"') e++;
+          Sv list{a.p + bt + 15, e - bt - 15};
+          size_t s0 = 0;
+          for (size_t k = 0; k <= list.n; k++)
+            if (k == list.n || list[k] == ',') {
+              Sv lb = trim(Sv{list.p + s0, k - s0});
+              if (lb.n) targets.emplace_back(lb.p, lb.n);
+              s0 = k + 1;
+            }
+        }
+        ins = trim(Sv{ins.p, q});
+        break;
+      }
     std::string subst;  // `(.L_x_N) -> 0x<pc> when the label is already known (a backward target)
     const char* bq = (const char*)memchr(ins.p, '`', ins.n);
     if (bq && bq + 1 < ins.p + ins.n && bq[1] == '(') {
@@ -523,6 +641,12 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     pk->use_off.push_back((uint32_t)pk->use_reg.size());
     pk->tgt.push_back(lo.target >= 0 && lo.target % 16 == 0 ? (int32_t)(lo.target / 16) : -1);
     if (lo.target < 0 && !lo.label.empty()) fwd.emplace_back(pk->recs.size(), lo.label);
+    if (r_op(r) == OP_BRX && !targets.empty()) {  // multi-target entry, resolved at the end
+      pk->tgt.back() = -2 - (int32_t)brx_at.size();
+      brx_at.push_back(pk->recs.size());
+      brx_labels.push_back(std::move(targets));
+    }
+    maxreg = std::max(maxreg, lo.maxreg);
     pk->recs.push_back(r);
     pk->lines.push_back(src_line);
     int32_t key = -1;
@@ -538,6 +662,17 @@ bool parse_segment(const char* text, const Segment& seg, ParsedKernel* pk, std::
     auto it = labels.find(f.second);
     if (it != labels.end()) pk->tgt[f.first] = (int32_t)(it->second / 16);
   }
+  // indirect-branch successor lists (R38i): kernel-local instruction indices, CSR
+  pk->xtgt_off.assign(1, 0);
+  for (size_t b = 0; b < brx_at.size(); b++) {
+    for (auto& lb : brx_labels[b]) {
+      auto it = labels.find(lb);
+      if (it != labels.end() && it->second / 16 < (long long)pk->recs.size()) pk->xtgt.push_back((int32_t)(it->second / 16));
+    }
+    pk->xtgt_off.push_back((uint32_t)pk->xtgt.size());
+  }
+  // the kernel's register count (R38k): the dump's REG:N, else one past the highest GPR touched
+  pk->nregs = seg.regcount > 0 ? (uint32_t)seg.regcount : (uint32_t)(maxreg + 1);
   return true;
 }
 
@@ -558,6 +693,8 @@ bool is_instr_line(Sv t) {
 bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedKernel>* out, std::string* err) {
   // pass 1: segments
   std::vector<Segment> segs;
+  std::map<std::string, int> res_regs;  // cuobjdump -res-usage: " Function <name>:" / "  REG:N ..." (R38k)
+  std::string res_fn;
   int sm = 100;
   long lineno = 1;
   size_t p = 0;
@@ -567,7 +704,12 @@ bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedK
     Sv t = trim(Sv{text + p, e - p});
     size_t at;
     if (t.n) {
-      if (contains(t, "code for sm_", &at)) {
+      if (starts(t, "Function ") && t[t.n - 1] == ':' && !contains(t, "Function :")) {
+        res_fn.assign(t.p + 9, t.n - 10);
+      } else if (!res_fn.empty() && starts(t, "REG:")) {
+        res_regs[res_fn] = atoi(std::string(t.p + 4, std::min<size_t>(t.n - 4, 12)).c_str());
+        res_fn.clear();
+      } else if (contains(t, "code for sm_", &at)) {
         sm = atoi(std::string(t.p + at + 12, t.n - at - 12).c_str());
       } else if (contains(t, ".target") && contains(t, "sm_", &at)) {
         sm = atoi(std::string(t.p + at + 3, t.n - at - 3).c_str());
@@ -581,6 +723,8 @@ bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedK
         Sv nm = is_fn_label(t) ? Sv{t.p + 6, t.n - 7} : trim(Sv{t.p + at + 10, t.n - at - 10});
         s.name.assign(nm.p, nm.n);
         s.header = true;
+        auto rr = res_regs.find(s.name);
+        s.regcount = rr == res_regs.end() ? -1 : rr->second;
         segs.push_back(s);
       } else if (segs.empty() && !starts(t, "//##") && is_instr_line(t)) {
         Segment s;  // instructions before any Function header: one anonymous kernel
@@ -590,6 +734,7 @@ bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedK
         s.sm = sm;
         s.name = "<anonymous>";
         s.header = false;
+        s.regcount = -1;
         segs.push_back(s);
       }
     }

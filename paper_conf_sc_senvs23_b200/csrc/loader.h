@@ -18,7 +18,10 @@ struct ParsedKernel {
   // targets (kernel-local instruction index, -1 if none / unresolved)
   std::vector<uint32_t> use_off;  // n + 1
   std::vector<uint8_t> use_reg;
-  std::vector<int32_t> tgt;
+  std::vector<int32_t> tgt;       // -2 - x: indirect branch x with the successor list below (R38i)
+  std::vector<uint32_t> xtgt_off; // indirect-branch successor lists (CSR over x; kernel-local indices)
+  std::vector<int32_t> xtgt;
+  uint32_t nregs = 0;             // the kernel's GPR count (R38k): REG:N of -res-usage, else max touched + 1
 };
 
 // Parses cuobjdump -sass / nvdisasm [-g] text into per-kernel packed records using up to n_threads threads.

@@ -235,7 +235,9 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
   if (cons && !c->cons_ready) return fail(c, GS_E_STATE, "consumer join: gs_detect ran in another join mode");
   const bool line = (c->cfg.join_mode == GS_JOIN_LINE && c->n_lgroups) || cons;
   // ---- every allocation first (the enqueue below may be captured into a CUDA graph)
-  if (!c->d_ktot) GS_CUDA(c, cudaMalloc((void**)&c->d_ktot, nkt * 8));
+  if (ns > 0x7fffffffull) return fail(c, GS_E_RANGE, "more than 2^31-1 sites (the site sort takes int counts)");
+  // kernel totals + the two maxima: grown with the kernel count (a later gs_load_sass may load more)
+  GS_CUDA(c, dev_grow(&c->d_ktot, &c->ktot_cap, nkt));
   unsigned long long* d_max = c->d_ktot + (nkt - 2);
   size_t cub_bytes = 0;
   if (ns) {
@@ -417,6 +419,14 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
   return GS_OK;
 }
 
+// a new module invalidates the captured rank sequence (its k_ktot grid follows the kernel sizes)
+void rank_reset_graph(gs_ctx* c) {
+  if (c->rank_exec) cudaGraphExecDestroy(c->rank_exec);
+  c->rank_exec = nullptr;
+  c->rank_key.clear();
+  c->rank_bits_guess[0] = c->rank_bits_guess[1] = -1;
+}
+
 void rank_free(gs_ctx* c) {
   if (c->rank_exec) cudaGraphExecDestroy(c->rank_exec);
   c->rank_exec = nullptr;
@@ -435,6 +445,7 @@ void rank_free(gs_ctx* c) {
   c->jrow_cap = 0;
   c->d_sort_tmp = nullptr;
   c->d_ktot = nullptr;
+  c->ktot_cap = 0;
   c->d_ranked = nullptr;
   c->rank_cap = 0;
   c->sort_tmp_bytes = 0;

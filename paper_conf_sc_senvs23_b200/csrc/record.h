@@ -4,13 +4,14 @@
 // One record per instruction ("the instruction and the destination (+source) register numbers",
 // P:211-213), laid out so a warp loads 32 consecutive records with one coalesced uint4 per lane.
 //
-//   w0: op[0:8) | flags[8:16) | aw[16:19) | dstw[19:22) | pk[22:24) | cbank[24:29)
-//   w1: dst[0:9) | ptr[9:18) | s0[18:27)
+//   w0: op[0:8) | flags[8:16) | aw[16:19) | pk[19:21) | cbank[21:26) | dstw[26:32) (low 6 bits)
+//   w1: dst[0:9) | ptr[9:18) | s0[18:27) | dstw[27:29) (high 2 bits: widths up to 255, LDTM.x128)
 //   w2: s1[0:9)  | s2[9:18)  | s3[18:27)
 //   w3: imm (int32): memory offset / branch target (kernel-local index) / constant-bank offset
 //
 // Register ids (9 bits): GPR Rn -> n (RZ = 255), URn -> 256 + n (URZ = 319), none = 511.
-// Memory instructions: s0 = address base register, s1 = stored/data register.
+// Memory instructions: s0 = address base register, s1 = stored/data register; a 256-bit load
+// (LDG.E.ENL2.256 Ra, Rb, [..], R38a) carries its second destination quad Rb in s2 (F_DST2).
 // ARITH instructions (R12): s0..s3 = register sources (RZ/URZ dropped, at most 4).
 // pk = pointer-operand kind of the def-use trace step (R7): REG -> ptr register,
 // CONST -> c[cbank][imm], IMM -> the trace ends at an immediate.
@@ -40,6 +41,7 @@ enum Op : uint8_t {
   OP_FADD, OP_FMUL, OP_FFMA, OP_FMNMX, OP_DADD, OP_DMUL, OP_DFMA, OP_HADD2, OP_HMUL2, OP_HFMA2,
   OP_MUFU, OP_IADD3, OP_VIADD, OP_IMAD, OP_IMUL, OP_IMNMX, OP_VIMNMX, OP_IABS,
   OP_IMAD_MOV, OP_LEA, OP_ULEA, OP_UIADD3, OP_UIMAD, OP_HMMA, OP_DMNMX, OP_FCHK,
+  OP_CALL, OP_RET, OP_BRX,  // R38g/i: the call ABI and indirect branches (register pressure)
   OP_COUNT
 };
 
@@ -87,12 +89,16 @@ enum : uint32_t {
   F_CONSTANT = 1, F_HASMEM = 2, F_BRA_OK = 4,
   F_PRED = 8,     // guarded by a predicate other than PT (kills no register, R36)
   F_EXIT = 16,    // EXIT / RET
-  F_BRPRED = 32,  // BRA with a predicate operand (conditional, e.g. BRA.U !UP0)
+  F_BRPRED = 32,  // BRA with a predicate or register condition (BRA.U !UP0, BRA.DIV UR4; R38i)
+  F_DST2 = 64,    // second destination quad in s2 (256-bit load, R38a)
 };
 // access width codes
-enum : uint32_t { AW_NONE = 0, AW_8 = 1, AW_16 = 2, AW_32 = 3, AW_64 = 4, AW_128 = 5 };
+enum : uint32_t { AW_NONE = 0, AW_8 = 1, AW_16 = 2, AW_32 = 3, AW_64 = 4, AW_128 = 5, AW_256 = 6 };
 // pointer-operand kinds
 enum : uint32_t { PK_IMM = 0, PK_REG = 1, PK_CONST = 2 };
+// call ABI (R38g): registers a CALL may overwrite; the others (except R1) are callee-saved and live
+// out of a RET
+GS_HD bool call_clobbered(uint32_t r) { return r == 0 || (r >= 3 && r <= 15) || (r >= 32 && r <= 99 && (r - 32) % 8 < 4); }
 
 struct Rec {
   uint32_t w0, w1, w2;
@@ -103,9 +109,9 @@ static_assert(sizeof(Rec) == 16, "record is 16 bytes");
 GS_HD uint32_t r_op(const Rec& r) { return r.w0 & 0xffu; }
 GS_HD uint32_t r_flags(const Rec& r) { return (r.w0 >> 8) & 0xffu; }
 GS_HD uint32_t r_aw(const Rec& r) { return (r.w0 >> 16) & 7u; }
-GS_HD uint32_t r_dstw(const Rec& r) { return (r.w0 >> 19) & 7u; }
-GS_HD uint32_t r_pk(const Rec& r) { return (r.w0 >> 22) & 3u; }
-GS_HD uint32_t r_cbank(const Rec& r) { return (r.w0 >> 24) & 31u; }
+GS_HD uint32_t r_pk(const Rec& r) { return (r.w0 >> 19) & 3u; }
+GS_HD uint32_t r_cbank(const Rec& r) { return (r.w0 >> 21) & 31u; }
+GS_HD uint32_t r_dstw(const Rec& r) { return (r.w0 >> 26) | (((r.w1 >> 27) & 3u) << 6); }
 GS_HD uint32_t r_dst(const Rec& r) { return r.w1 & 511u; }
 GS_HD uint32_t r_ptr(const Rec& r) { return (r.w1 >> 9) & 511u; }
 GS_HD uint32_t r_s0(const Rec& r) { return (r.w1 >> 18) & 511u; }
@@ -113,13 +119,15 @@ GS_HD uint32_t r_s1(const Rec& r) { return r.w2 & 511u; }
 GS_HD uint32_t r_s2(const Rec& r) { return (r.w2 >> 9) & 511u; }
 GS_HD uint32_t r_s3(const Rec& r) { return (r.w2 >> 18) & 511u; }
 GS_HD int32_t r_imm(const Rec& r) { return r.w3; }
+// second destination quad of a 256-bit load (R38a), kRegNone otherwise
+GS_HD uint32_t r_dst2(const Rec& r) { return (r_flags(r) & F_DST2) ? r_s2(r) : (uint32_t)kRegNone; }
 
 GS_HD Rec make_rec(uint32_t op, uint32_t flags, uint32_t aw, uint32_t dstw, uint32_t pk, uint32_t cbank,
                    uint32_t dst, uint32_t ptr, uint32_t s0, uint32_t s1, uint32_t s2, uint32_t s3, int32_t imm) {
   Rec r;
-  r.w0 = (op & 0xffu) | ((flags & 0xffu) << 8) | ((aw & 7u) << 16) | ((dstw & 7u) << 19) | ((pk & 3u) << 22) |
-         ((cbank & 31u) << 24);
-  r.w1 = (dst & 511u) | ((ptr & 511u) << 9) | ((s0 & 511u) << 18);
+  r.w0 = (op & 0xffu) | ((flags & 0xffu) << 8) | ((aw & 7u) << 16) | ((pk & 3u) << 19) | ((cbank & 31u) << 21) |
+         ((dstw & 63u) << 26);
+  r.w1 = (dst & 511u) | ((ptr & 511u) << 9) | ((s0 & 511u) << 18) | (((dstw >> 6) & 3u) << 27);
   r.w2 = (s1 & 511u) | ((s2 & 511u) << 9) | ((s3 & 511u) << 18);
   r.w3 = imm;
   return r;
@@ -129,9 +137,11 @@ GS_HD Rec make_rec(uint32_t op, uint32_t flags, uint32_t aw, uint32_t dstw, uint
 struct KDesc {
   uint32_t first;       // global slot of instruction 0
   uint32_t n;           // instructions
-  uint32_t param_base;  // R1
+  uint32_t param_base;  // R1 (bits 0..15); the kernel's GPR count (R38k) in bits 16..31
   uint32_t win0;        // first window id
 };
+GS_HD uint32_t kd_param_base(const KDesc& k) { return k.param_base & 0xffffu; }
+GS_HD uint32_t kd_nregs(const KDesc& k) { return k.param_base >> 16; }
 
 // per-window descriptor (device): windows never cross kernels
 struct WDesc {

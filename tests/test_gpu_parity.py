@@ -18,7 +18,9 @@ FIXTURES = ["listing1.sass", "sgemm_naive.sm_100a.sass", "sgemm_naive.sm_70.sass
             "atomics.sm_70.sass", "conv.sm_100a.sass", "spill.r24.sm_100a.sass", "spill.r32.sm_100a.sass",
             "spill.r40.sm_100a.sass", "spill.r64.sm_100a.sass"] + \
     [f"lineinfo/{k}.{d}.sass" for k in ("sgemm_naive", "jacobi", "mixbench", "atomics", "spill")
-     for d in ("cuobjdump", "nvdisasm")]
+     for d in ("cuobjdump", "nvdisasm")] + \
+    ["b200/wmma.sm_100a.sass", "b200/v8.sm_100a.sass", "b200/tmem.sm_100a.sass", "b200/abi_brx.nvdisasm.sass",
+     "torch/k1779_tcgen05_gemm.sass.xz"]
 
 
 @pytest.fixture(scope="module")
@@ -44,6 +46,8 @@ def _detect_lines(gs, text, D=64, kb=0, ke=None, **kw):
 
 
 def _read(name):
+    if name.endswith(".xz"):
+        return orc.golden_text(name).encode()
     return open(golden(name), "rb").read()
 
 
@@ -424,7 +428,11 @@ def _gpu_live(gs, text, kb=0, ke=None):
 
 LIVE_TEXTS = ["lineinfo/sgemm_naive.nvdisasm.sass", "lineinfo/mixbench.nvdisasm.sass", "lineinfo/atomics.cuobjdump.sass",
               "lineinfo/spill.nvdisasm.sass", "jacobi.sm_70.sass", "sgemm_naive.sm_70.sass", "conv.sm_100a.sass",
-              "spill.r24.sm_100a.sass", "listing1.sass"]
+              "spill.r24.sm_100a.sass", "listing1.sass",
+              # sm_100a register forms (R38): HMMA/LDSM/CS2R, 256-bit quads, tcgen05 LDTM/STTM with the
+              # call ABI, BRX target lists, a CUTLASS tcgen05 GEMM kernel
+              "b200/wmma.sm_100a.sass", "b200/v8.sm_100a.sass", "b200/tmem.sm_100a.sass",
+              "b200/abi_brx.nvdisasm.sass", "torch/k1779_tcgen05_gemm.sass.xz"]
 
 
 @pytest.mark.parametrize("name", LIVE_TEXTS)
@@ -554,3 +562,47 @@ def test_c3_full_size_detect_parity(gs):
     o = Canon(orc.run(s.text, hist=False))
     assert g.K == o.K
     assert len(g.S) == len(o.S) and g.S == o.S
+
+
+def test_real_torch_cubin_parity(gs):
+    """A whole real sm_100 cubin of the torch wheel (ELF 1810 of libtorch_cuda.so, 200 kernels,
+    38,585 instructions; tests/golden/torch): the GPU's K/S lines and live-register counts equal the
+    oracle's, whose L lines equal nvdisasm -lrm count on every instruction (test_oracle_pins)."""
+    text = _read("torch/cubin1810.sass.xz")
+    g, _ = _detect_lines(gs, text)
+    o = Canon(orc.run(text, hist=False))
+    assert len(g.K) == 200 and g.K == o.K
+    assert g.S == o.S
+    got, _ = _gpu_live(gs, text)
+    assert got == _oracle_live(text)
+
+
+def test_reload_then_rank_graph(gs):
+    """one context, modules of 3 -> many -> 3 -> 1 kernels, each detected and ranked
+    through the captured rank graph (device output on a non-default stream): the kernel-total buffer
+    grows with the kernel count and a reload never replays a stale graph."""
+    import torch
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    mods = [gsass.config_sass("C2"), gsass.config_sass("C3", scale=0.004), gsass.config_sass("C2"),
+            gsass.config_sass("C1")]
+    assert len(mods[1].n_instr) > 30
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        ctx = _ctx(gs, hist_row=19)
+        for q, s in enumerate(mods):
+            raw, _ = _samples(s, 200_000, "shuffled", seed=91 + q, n_bad=0)
+            ctx.load_sass(s.text)
+            ctx.detect()
+            hist = torch.empty(ctx.n_instr * 19, dtype=torch.int32, device="cuda")
+            ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
+            w, _ = ctx.pack_samples(torch.from_numpy(raw.view(np.int32).reshape(-1, 3).copy()).cuda())
+            ctx.attribute_samples(w, hist, ninv)
+            ns = ctx.sites_device()[2]
+            dev_rows = torch.empty(max(ns, 1) * gs.RANKED_DTYPE.itemsize, dtype=torch.uint8, device="cuda")
+            for _ in range(2):  # capture, then replay
+                n = ctx.rank_sites(hist, out=dev_rows)
+                rows = dev_rows.cpu().numpy().view(gs.RANKED_DTYPE)[:n]
+                got = Canon(report.canonical(ctx, hist=hist, n_samples=len(raw), n_invalid=0, ranked=rows)).R
+                assert got == Canon(orc.run(s.text, samples=raw)).R, q
+        st.synchronize()

@@ -153,3 +153,125 @@ def sass_ops(path: str) -> dict:
         if m:
             ops[int(m.group(1), 16) // 16] = m.group(3)
     return ops
+
+
+# ------------------------------------------------------------------------------ sharded oracle
+def split_kernels(text: bytes) -> list[bytes]:
+    """cuobjdump text -> one text per kernel ("Function :" sections). The preamble (-res-usage
+    block, first arch line) goes with every section, and each later section also gets the last
+    "code for sm_NN" line before it. Test-side text slicing only: each section is parsed by the
+    oracle itself."""
+    def line_starts(needle):
+        out, p = [], text.find(needle)
+        while p >= 0:
+            out.append(text.rfind(b"\n", 0, p) + 1)
+            p = text.find(needle, p + len(needle))
+        return out
+    marks = line_starts(b"Function : ")
+    if not marks:
+        return [text]
+    arches = line_starts(b"code for sm_")
+    cuts = marks + [len(text)]
+    pre = text[:marks[0]]
+    out = [text[:cuts[1]]]
+    a = 0
+    for i in range(1, len(marks)):
+        while a + 1 < len(arches) and arches[a + 1] < marks[i]:
+            a += 1
+        arch = b""
+        if arches and arches[a] < marks[i]:
+            e = text.find(b"\n", arches[a])
+            arch = text[arches[a]:e + 1]
+        out.append(pre + arch + text[cuts[i]:cuts[i + 1]])
+    return out
+
+
+def run_sharded(sass: bytes, raw: np.ndarray | None, n_instr, shards: int, D=64, R=19, timing=False,
+                tmpdir: str | None = None):
+    """The all-cores oracle baseline (SURVEY §8d "the same oracle functions over kernel / sample
+    shards, merged by integer sums"): the module is cut into `shards` contiguous kernel ranges
+    balanced by instruction count, each with the samples of its kernels, and each range is a
+    complete, independent oracle run (histogram bins, kernel totals and sites are per kernel).
+    Runs the processes in parallel and merges their canonical outputs: kernel and slot numbers
+    shifted, N lines summed, R lines re-sorted by the total order (R20). The merged text equals the
+    single-process output (tests/test_oracle_pins.py). Returns (text, seconds of the parallel part
+    incl. the merge) when timing."""
+    import time
+    n_instr = np.asarray(n_instr, dtype=np.int64)
+    K = len(n_instr)
+    shards = max(1, min(shards, K))
+    csum = np.concatenate([[0], np.cumsum(n_instr)])
+    bounds = [0] + [int(np.searchsorted(csum, csum[-1] * p / shards)) for p in range(1, shards)] + [K]
+    bounds = sorted(set(min(max(b, 0), K) for b in bounds))
+    secs = split_kernels(sass) if not (tmpdir and os.path.exists(os.path.join(tmpdir, "shard0.sass"))) else [b""] * K
+    assert len(secs) == K, (len(secs), K)
+    build_oracle()
+    td = tmpdir or tempfile.mkdtemp()
+    jobs = []
+    for p in range(len(bounds) - 1):
+        kb, ke = bounds[p], bounds[p + 1]
+        if kb == ke:
+            continue
+        sp = os.path.join(td, f"shard{p}.sass")
+        reuse = tmpdir is not None and os.path.exists(sp)  # a caller's tmpdir keeps the inputs of repeated steps
+        if not reuse:
+            with open(sp, "wb") as f:
+                f.write(b"".join(secs[kb:ke]))
+        cmd = [ORACLE, "--sass", sp, "--D", str(D), "--R", str(R), "--no-hlines"]
+        if raw is not None and reuse:
+            cmd += ["--samples", os.path.join(td, f"shard{p}.bin")]
+        elif raw is not None:
+            kk = raw[:, 0].astype(np.int64)
+            sel = (kk >= kb) & (kk < ke) if p else ((kk < ke) | (kk >= K))  # invalid kernels: shard 0
+            part = raw[sel].copy()
+            ok = part[:, 0] < K
+            part[ok, 0] -= kb
+            rp = os.path.join(td, f"shard{p}.bin")
+            np.ascontiguousarray(part, dtype=np.uint32).tofile(rp)
+            cmd += ["--samples", rp]
+        jobs.append((kb, int(csum[kb]), cmd))
+    t0 = time.perf_counter()
+    procs = [subprocess.Popen(c, stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True) for _, _, c in jobs]
+    outs = [p.communicate() for p in procs]
+    for p, (o, e) in zip(procs, outs):
+        if p.returncode != 0:
+            raise RuntimeError(f"oracle shard failed: {e}")
+    head, klines, slines, rrows = None, [], [], []
+    tot = {"total": 0, "valid": 0, "invalid": 0}
+    have_n = False
+    for (kb, sb, _), (o, _) in zip(jobs, outs):
+        for line in o.splitlines():
+            f = line.split()
+            if line.startswith("#") or line.startswith("CFG"):
+                head = head or []
+                if line not in head:
+                    head.append(line)
+            elif f[0] == "K":
+                f[1] = str(int(f[1]) + kb)
+                f[3] = str(int(f[3]) + sb)
+                klines.append(" ".join(f))
+            elif f[0] == "S":
+                f[1] = str(int(f[1]) + kb)
+                slines.append(" ".join(f))
+            elif f[0] == "N":
+                have_n = True
+                for kv in f[1:]:
+                    a, b = kv.split("=")
+                    tot[a] += int(b)
+            elif f[0] == "R":
+                k = int(f[2]) + kb
+                rel = int(f[5].split("=")[1])
+                totv = int(f[6].split("=")[1])
+                rrows.append((-rel, -totv, k, int(f[3]), ["VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX",
+                                                           "CONV"].index(f[4]), f[4:]))
+    rrows.sort(key=lambda r: r[:5])
+    lines = head + klines + slines
+    if have_n:
+        lines.append(f"N total={tot['total']} valid={tot['valid']} invalid={tot['invalid']}")
+    lines += [f"R {q} {r[2]} {r[3]} " + " ".join(r[5]) for q, r in enumerate(rrows)]
+    secs_par = time.perf_counter() - t0
+    if tmpdir is None:
+        import shutil
+        shutil.rmtree(td, ignore_errors=True)
+    text = "\n".join(lines) + "\n"
+    return (text, secs_par) if timing else text

@@ -593,3 +593,25 @@ def test_256bit_loads_are_already_vectorised():
     i = ldg256[0]
     assert g[(0, i)][0] == set(range(4, 12))  # LDG.E.ENL2.256 R4, R8, [R6.64]: R4..R11 written
     assert g[(0, i)][1] == {6, 7}             # ... and only the address pair read
+
+
+# --------------------------------------------------------------------------- all-cores oracle baseline
+@pytest.mark.parametrize("name,shards", [("C2", 3), ("C2", 2), ("atomics.sm_70.sass", 2), ("b200/tmem.sm_100a.sass", 1)])
+def test_sharded_oracle_equals_single_process(name, shards):
+    """The all-cores oracle baseline runs independent kernel ranges in parallel and
+    merges by integer sums and the total order R20: its canonical text equals the single-process
+    oracle's (sm_70 param bases and -res-usage REG:N survive the split)."""
+    from gen import samples as gsm
+    from gen import sass as gsass
+    if name == "C2":
+        s = gsass.config_sass("C2")
+        text, n_instr = s.text, s.n_instr
+        tab = gsm.table_class_weighted(s.cls, 300_000, key=3)
+        raw = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=3).raw()
+        raw = gsm.interleave(raw, gsm.invalid_raw(len(n_instr), n_instr, 100, key=3), key=4)
+    else:
+        text = open(golden(name), "rb").read()
+        n_instr = [k["n"] for k in Canon(orc.run(text)).kstats()]
+        raw = None
+    want = orc.run(text, samples=raw, hlines=False) if raw is not None else orc.run(text, hist=False)
+    assert orc.run_sharded(text, raw, n_instr, shards) == want

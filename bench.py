@@ -199,6 +199,116 @@ def reference_arm(args, world, rank):
     }), flush=True)
 
 
+# ----------------------------------------------------------------------------------- extra lines
+def _time_events(fn, steps, warmup, stream):
+    """mean ms of fn() over `steps` calls, CUDA events on `stream`, after `warmup` calls"""
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / steps
+
+
+def extra_detect_c3(g, peak, steps, warmup):
+    """configs[2] (C3: 10,000 kernels, ~50M SASS instructions; the paper's dry run):
+    gs_load_sass host parse+pack+upload (wall) and gs_detect (CUDA events). Algorithmic bytes
+    (SURVEY §8d): 16 B read per instruction + 16 B per site + 4 B per chain step written."""
+    import torch
+    from gen import sass as gsass
+    s3 = gsass.config_sass("C3")
+    ctx = g.Context(n_reasons=19)
+    t0 = time.perf_counter()
+    ctx.load_sass(s3.text)
+    torch.cuda.synchronize()
+    parse_s = time.perf_counter() - t0
+    n_sites = ctx.detect()
+    _, _, ns, nc = ctx.sites_device()
+    ms = _time_events(ctx.detect, steps, warmup, torch.cuda.current_stream())
+    alg = 16.0 * ctx.n_instr + 16.0 * ns + 4.0 * nc
+    ach = alg / (ms * 1e-3) / 1e9
+    return {"workload": "C3", "kernels": ctx.n_kernels, "sass_instrs": ctx.n_instr, "sites": int(n_sites),
+            "chain_steps": int(nc), "detect_ms": ms, "instrs_per_s": ctx.n_instr / (ms * 1e-3),
+            "host_parse_pack_upload_s": parse_s, "text_bytes": len(s3.text),
+            "roofline": {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                         "algorithmic_bytes": alg}}
+
+
+def extra_c5(g, peak, steps, warmup):
+    """configs[4] (C5: 200M samples, 90% on 10 PCs, a 1M-PC module with 63/64/65-step chains):
+    the attribution pass in both orders (trace: AUTO, shuffled: PARTITION, as the main line)."""
+    import torch
+    from gen import samples as gsm
+    from gen import sass as gsass
+    from gen.device import DeviceTrace
+    s5 = gsass.config_sass("C5")
+    hot = [int(f) + 40 for f in s5.first_slot[:10]]
+    tab = gsm.table_c5(s5.cls, hot, 200_000_000, key=0x6E5C0005)
+    out = {"workload": "C5", "samples": int(tab.sum()), "sass_instrs": int(sum(s5.n_instr))}
+    R = 19
+    for order, mode in (("trace", 0), ("shuffled", g.GS_HIST_PARTITION)):
+        tr = gsm.Trace(tab, s5.first_slot, s5.n_instr, order=order, seed=2)
+        words = DeviceTrace(tr, torch.cuda.current_device()).packed()
+        ctx = g.Context(n_reasons=R, hist_mode=mode, hist_row=R)
+        ctx.load_sass(s5.text)
+        hist = torch.empty(ctx.n_instr * R, dtype=torch.int32, device="cuda")
+        ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ms = _time_events(lambda: ctx.attribute_samples(words, hist, ninv), steps, warmup,
+                          torch.cuda.current_stream())
+        assert int(hist.to(torch.int64).sum().item()) == tr.N
+        alg = 4.0 * tr.N + 4.0 * R * ctx.n_instr
+        ach = alg / (ms * 1e-3) / 1e9
+        out[order] = {"attribute_ms": ms, "samples_per_s": tr.N / (ms * 1e-3), "hist_mode": ctx.last_hist_mode(),
+                      "roofline": {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                                   "algorithmic_bytes": alg}}
+        del words, hist
+    return out
+
+
+def extra_pack_hist(g, ctx, words, hist, ninv, s, peak, steps, warmup):
+    """N1 + N2 (SURVEY §8d timing protocol): raw 12-byte (kernel, pc offset, reason) records of the
+    same trace through gs_pack_samples, then the histogram. The raw records are built on the device
+    from the packed words (input preparation, not timed)."""
+    import torch
+    R = 19
+    n = words.shape[0]
+    first = torch.from_numpy(np.asarray(s.first_slot, dtype=np.int64)).cuda()
+    raw = torch.empty((n, 3), dtype=torch.int32, device="cuda")
+    chunk = 1 << 26
+    for a in range(0, n, chunk):
+        w = words[a:a + chunk].to(torch.int64)
+        slot, reason = w // R, w % R
+        k = torch.searchsorted(first, slot, right=True) - 1
+        raw[a:a + chunk, 0] = k.to(torch.int32)
+        raw[a:a + chunk, 1] = ((slot - first[k]) * 16).to(torch.int32)
+        raw[a:a + chunk, 2] = reason.to(torch.int32)
+        del w, slot, reason, k
+    packed = torch.empty(n, dtype=torch.int32, device="cuda")
+    pinv = torch.zeros(1, dtype=torch.int64, device="cuda")
+    st = torch.cuda.current_stream()
+    pack_ms = _time_events(lambda: ctx.pack_samples(raw, packed, pinv), steps, warmup, st)
+    assert torch.equal(packed, words)
+
+    def both():
+        ctx.pack_samples(raw, packed, pinv)
+        ctx.attribute_samples(packed, hist, ninv)
+    both_ms = _time_events(both, steps, warmup, st)
+    del raw, packed
+    alg_pack = 16.0 * n            # 12 B read + 4 B written per record
+    alg_both = alg_pack + 4.0 * n + 4.0 * R * ctx.n_instr
+    return {"samples": n, "pack_ms": pack_ms, "pack_plus_hist_ms": both_ms,
+            "samples_per_s": n / (both_ms * 1e-3),
+            "pack_roofline": {"achieved": alg_pack / (pack_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                              "frac": alg_pack / (pack_ms * 1e-3) / 1e9 / peak},
+            "roofline": {"achieved": alg_both / (both_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                         "frac": alg_both / (both_ms * 1e-3) / 1e9 / peak, "algorithmic_bytes": alg_both}}
+
+
 def workload_config(args, s, tr, world):
     return {"workload": args.config, "kernels": len(s.n_instr), "sass_instrs": s.P, "samples": tr.N,
             "order": args.order, "reasons": 19, "trace_depth": 64, "parallelism": f"dp{world}",
@@ -223,6 +333,7 @@ def main():
     ap.add_argument("--cpu-samples", type=int, default=1 << 24,
                     help="samples in the oracle's bounded sample (with the full SASS) per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip the C3 detection / C5 / pack+hist lines")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -347,6 +458,15 @@ def main():
         if traffic and world > 1:   # captured on the whole stream: this rank's launch holds n_local samples
             traffic = traffic * n_local / tr.N
 
+    # extra lines (N = 1): N1 + N2 on this trace, configs[2] detection, configs[4] attribution
+    extras = {}
+    if world == 1 and not args.no_extras:
+        try:
+            extras["pack_hist"] = extra_pack_hist(g, ctx, words, hist, ninv, s, read_peaks()[0], 10, 3)
+        except Exception as e:  # noqa: BLE001
+            extras["pack_hist"] = {"failed": str(e)}
+        torch.cuda.empty_cache()
+
     # e2e: same step through the C ABI with HOST buffers (pinned), copies inside the timed region
     host_words = torch.empty(n_local, dtype=torch.int32, pin_memory=True)
     host_words.copy_(words)
@@ -373,6 +493,16 @@ def main():
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_s = float(te[0])
+
+    if world == 1 and not args.no_extras:
+        del host_words
+        torch.cuda.empty_cache()
+        for name, fn in (("detect_C3", extra_detect_c3), ("C5", extra_c5)):
+            try:
+                extras[name] = fn(g, read_peaks()[0], 10, 3)
+            except Exception as e:  # noqa: BLE001
+                extras[name] = {"failed": str(e)}
+            torch.cuda.empty_cache()
 
     if rank != 0:
         dist.destroy_process_group()
@@ -403,6 +533,7 @@ def main():
         "cpu_baseline": cpu,
         "sites": n_sites,
         "phases_ms": phases,
+        "extra": extras,
     }
     print(json.dumps(out), flush=True)
     if world > 1:

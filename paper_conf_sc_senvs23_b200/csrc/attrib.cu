@@ -78,22 +78,42 @@ __device__ __forceinline__ void count_invalid(uint32_t n_bad, unsigned long long
   if ((threadIdx.x & 31) == 0 && n_bad) atomicAdd(d_n_invalid, (unsigned long long)n_bad);
 }
 
-__global__ void k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc* __restrict__ kd, uint32_t nk,
-                       uint32_t nr, uint32_t* __restrict__ words, unsigned long long* d_n_invalid) {
-  const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  uint32_t bad = 0;
-  if (i < n) {
-    const uint32_t k = raw[3 * i], pc = raw[3 * i + 1], reason = raw[3 * i + 2];
-    bool ok = k < nk && (pc & 15u) == 0 && reason < nr;
-    uint32_t w = 0xffffffffu;
-    if (ok) {
-      const KDesc K = kd[k];
-      ok = (pc >> 4) < K.n;
-      if (ok) w = (K.first + (pc >> 4)) * nr + reason;
-    }
-    words[i] = w;
-    bad = ok ? 0 : 1;
+// one raw record (kernel, pc offset, reason) -> packed word (~0u if invalid, R30)
+__device__ __forceinline__ uint32_t pack1(uint32_t k, uint32_t pc, uint32_t reason, const KDesc* __restrict__ kd,
+                                          uint32_t nk, uint32_t nr, uint32_t& bad) {
+  bool ok = k < nk && (pc & 15u) == 0 && reason < nr;
+  uint32_t w = 0xffffffffu;
+  if (ok) {
+    const KDesc K = kd[k];
+    ok = (pc >> 4) < K.n;
+    if (ok) w = (K.first + (pc >> 4)) * nr + reason;
   }
+  bad += ok ? 0u : 1u;
+  return w;
+}
+
+// N1: four records (48 B = three 128-bit loads) -> one 128-bit store per thread, grid-stride over
+// the 16-byte-aligned body; the < 4 trailing records and an unaligned input take the scalar loop
+__global__ void __launch_bounds__(256) k_pack(const uint32_t* __restrict__ raw, uint64_t n, const KDesc* __restrict__ kd,
+                                              uint32_t nk, uint32_t nr, uint32_t* __restrict__ words,
+                                              unsigned long long* d_n_invalid) {
+  uint32_t bad = 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const bool vec = ((reinterpret_cast<uintptr_t>(raw) | reinterpret_cast<uintptr_t>(words)) & 15u) == 0;
+  const uint64_t n4 = vec ? n / 4 : 0;
+  const uint4* r4 = reinterpret_cast<const uint4*>(raw);
+  uint4* w4 = reinterpret_cast<uint4*>(words);
+  for (uint64_t i = t0; i < n4; i += stride) {
+    const uint4 a = __ldcs(r4 + 3 * i), b = __ldcs(r4 + 3 * i + 1), c = __ldcs(r4 + 3 * i + 2);
+    uint4 o;
+    o.x = pack1(a.x, a.y, a.z, kd, nk, nr, bad);
+    o.y = pack1(a.w, b.x, b.y, kd, nk, nr, bad);
+    o.z = pack1(b.z, b.w, c.x, kd, nk, nr, bad);
+    o.w = pack1(c.y, c.z, c.w, kd, nk, nr, bad);
+    __stcs(w4 + i, o);
+  }
+  for (uint64_t i = 4 * n4 + t0; i < n; i += stride) words[i] = pack1(raw[3 * i], raw[3 * i + 1], raw[3 * i + 2], kd, nk, nr, bad);
   count_invalid(bad, d_n_invalid);
 }
 
@@ -1073,8 +1093,11 @@ __global__ void __launch_bounds__(kPT, 1)
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
                            unsigned long long* d_n_invalid) {
   if (!n) return GS_OK;
-  k_pack<<<(unsigned)((n + 255) / 256), 256, 0, c->stream>>>(d_raw, n, c->d_kd, c->n_kernels, c->cfg.n_reasons,
-                                                             d_words, d_n_invalid);
+  const uint64_t want = (n + 4 * 256 - 1) / (4 * 256);   // a thread per 4 records, at most 32 CTAs per SM
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+  const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)dev_sms * 8));
+  k_pack<<<grid, 256, 0, c->stream>>>(d_raw, n, c->d_kd, c->n_kernels, c->cfg.n_reasons, d_words, d_n_invalid);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;

@@ -64,7 +64,12 @@ def reduce_scatter_hist(hist, row: int, ranges, group=None):
     me = dist.get_rank(group)
     if dist.get_backend(group) == "nccl":
         out = torch.empty_like(parts[me])  # a separate output: no aliasing of an input part
-        dist.reduce_scatter(out, parts, op=dist.ReduceOp.SUM, group=group)
+        if len({p.numel() for p in parts}) == 1 and hist.is_contiguous() and hist.numel() == out.numel() * len(parts):
+            # equal slot ranges (e.g. C4: 256 equal kernels): the parts are hist itself, in rank
+            # order, so the tensor form reads it in place (the list form copies the inputs first)
+            dist.reduce_scatter_tensor(out, hist, op=dist.ReduceOp.SUM, group=group)
+        else:
+            dist.reduce_scatter(out, parts, op=dist.ReduceOp.SUM, group=group)
         return out
     if hist.is_cuda:  # gloo with device tensors (functional checks on one GPU): one all_reduce
         dist.all_reduce(hist, op=dist.ReduceOp.SUM, group=group)

@@ -178,6 +178,26 @@ gs_status gs_attribute_samples(gs_ctx *ctx, const uint32_t *samples, uint64_t n,
 gs_status gs_attribute_counts(gs_ctx *ctx, const uint32_t *d_recs, uint64_t n, int32_t *d_hist,
                               unsigned long long *d_n_invalid, int accumulate);
 
+/* CUPTI PC-sampling ingest (§2.2; R39).
+ * gs_cupti_stall_reasons: the stall-reason table of cuptiPCSamplingGetStallReasons — n CUPTI
+ * indices and their names ("smsp__pcsamp_warps_issue_stalled_<reason>[_not_issued]", host strings,
+ * borrowed for the call). A name maps to one of the 19 ncu reasons (R17); "_not_issued" counters are
+ * a subset of the same samples and are skipped; other names are unknown (invalid). Kept until the
+ * next call. */
+gs_status gs_cupti_stall_reasons(gs_ctx *ctx, size_t n, const uint32_t *index, const char *const *names);
+/* gs_attribute_cupti: pc_data = CUpti_PCSamplingPCData[n_pcs] (cupti_pcsampling.h, 64-byte records,
+ * HOST memory as CUPTI returns it: functionName and stallReason are host pointers). Every
+ * (record, stall reason) adds its samples to H[slot*row + reason] with kernel = the loaded kernel
+ * named functionName, slot = first_slot + pcOffset/16; records of another cubin (cubin_crc != 0 and
+ * record crc different), an unknown function or reason, or an invalid pc (R30) add their samples to
+ * *d_n_invalid (device u64); skipped (_not_issued) samples are counted into *n_skipped (host, may be
+ * NULL); *n_records (host, may be NULL) = the flattened (record, reason) entries. d_hist as
+ * gs_attribute_counts (zeroed unless accumulate). The flattening runs on host threads into pinned
+ * memory; returns when the staging copy is done (the scatter-add is async). */
+gs_status gs_attribute_cupti(gs_ctx *ctx, const void *pc_data, size_t n_pcs, uint64_t cubin_crc, int32_t *d_hist,
+                             unsigned long long *d_n_invalid, int accumulate, unsigned long long *n_skipped,
+                             unsigned long long *n_records);
+
 /* a-11, a-12 (R20): join the (already all-reduced) histogram onto the sites of the
  * last gs_detect (rows per gs_config.join_mode) and rank them by (rel desc, tot desc, kernel, idx,
  * rule). Writes the first

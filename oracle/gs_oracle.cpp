@@ -23,6 +23,7 @@
 //   O11 TEX   texture candidates                                 P:717-744 §4.6
 //   O12 CONV  datatype conversions                               P:746-761 §4.7
 //   O13 per-PC x stall-reason histogram of PC samples            P:215-227 §2.2
+//       (raw samples, pre-aggregated count records [R35], CUPTI PC-sampling records [R39])
 //   O14 join of the histogram onto flagged sites
 //       join=pc (default), line ([R33]), consumer ([R37], SURVEY [probe 9])
 //   O15 ranking (total order on integers)                        [R20]
@@ -1011,6 +1012,13 @@ struct RawSample { uint32_t kernel, pc, reason; };
 // with its sample count, P:215-227 / SURVEY [probe 8]); `count` samples of that (kernel, pc, reason)
 struct CountRec { uint32_t kernel, pc, reason, count; };
 
+// The 19 ncu / CUPTI stall reasons in id order (R17, SURVEY [probe 9]); a CUPTI name is
+// "smsp__pcsamp_warps_issue_stalled_<reason>[_not_issued]" (R39).
+const char* kReasonName[19] = {"barrier", "branch_resolving", "dispatch_stall", "drain", "imc_miss",
+                               "lg_throttle", "long_scoreboard", "math_pipe_throttle", "membar",
+                               "mio_throttle", "misc", "no_instructions", "not_selected", "selected",
+                               "short_scoreboard", "sleeping", "tex_throttle", "wait", "warpgroup_arrive"};
+
 const int kRel[NRULES] = {
     // bit r set = reason r in REL(rule).  long_scoreboard = 6, lg_throttle = 5, tex_throttle = 16
     1 << 6,                 // VEC
@@ -1025,7 +1033,8 @@ const int kRel[NRULES] = {
 }  // namespace
 
 int main(int argc, char** argv) {
-  std::string sass_path, samples_path, counts_path, out_path, join = "pc";
+  std::string sass_path, samples_path, counts_path, cupti_path, out_path, join = "pc";
+  unsigned long long cupti_crc = 0;
   Config C;
   long long K_top = -1;
   int kbegin = 0, kend = -1;
@@ -1037,6 +1046,8 @@ int main(int argc, char** argv) {
     if (s == "--sass") sass_path = nxt();
     else if (s == "--samples") samples_path = nxt();
     else if (s == "--counts") counts_path = nxt();  // CountRec records, added to the same histogram
+    else if (s == "--cupti") cupti_path = nxt();    // CUPTI PC-sampling records (text form, R39)
+    else if (s == "--cupti-crc") cupti_crc = strtoull(nxt().c_str(), nullptr, 0);  // 0: any module
     else if (s == "--join") join = nxt();            // pc (default) | line | consumer
     else if (s == "--out") out_path = nxt();
     else if (s == "--D") C.D = atoi(nxt().c_str());
@@ -1123,7 +1134,7 @@ int main(int argc, char** argv) {
         fprintf(out, "G %d %zu def=%s use=%s live=%s\n", k, i, join(gpr_defs(ks[k].ins[i], nregs)).c_str(),
                 join(gpr_uses(ks[k].ins[i])).c_str(), join(live[i]).c_str());
     }
-  if (hist && (!samples_path.empty() || !counts_path.empty())) {
+  if (hist && (!samples_path.empty() || !counts_path.empty() || !cupti_path.empty())) {
     // O13: H[slot][reason] += 1 for every valid sample.
     size_t P = 0;
     for (auto& k : ks) P += k.ins.size();
@@ -1159,6 +1170,53 @@ int main(int argc, char** argv) {
       }
       fclose(cf);
     }
+    uint64_t skipped = 0;
+    if (!cupti_path.empty()) {
+      // CUPTI PC sampling (§2.2; SURVEY [probe 8]; R39): one record per (function, pc
+      // offset) with per-stall-reason sample counts; the stall-reason table maps CUPTI's indices to
+      // names. Text form (tests write it from the same records the library reads):
+      //   T <index> <name>                                        stall-reason table entry
+      //   P <cubinCrc> <functionName> <pcOffset> <index>:<samples> ...   one CUpti_PCSamplingPCData
+      // kernel = the kernel of the dump with that name; reason = the name's position in kReasonName
+      // after the prefix; "_not_issued" counters are a subset of the same samples: skipped; a
+      // foreign cubin (crc filter), unknown function or reason, or an invalid pc: invalid (R30).
+      FILE* pf = fopen(cupti_path.c_str(), "rb");
+      if (!pf) { fprintf(stderr, "cannot open %s\n", cupti_path.c_str()); return 2; }
+      std::map<unsigned long long, std::string> table;
+      std::map<std::string, int> kid;
+      for (size_t k = 0; k < ks.size(); k++) kid.emplace(ks[k].name, (int)k);
+      const std::string prefix = "smsp__pcsamp_warps_issue_stalled_", ni = "_not_issued";
+      char lb[1 << 16];
+      while (fgets(lb, sizeof lb, pf)) {
+        std::vector<std::string> f;
+        for (char* t = strtok(lb, " \t\r\n"); t; t = strtok(nullptr, " \t\r\n")) f.push_back(t);
+        if (f.size() == 3 && f[0] == "T") { table[strtoull(f[1].c_str(), nullptr, 0)] = f[2]; continue; }
+        if (f.size() < 4 || f[0] != "P") continue;
+        const unsigned long long crc = strtoull(f[1].c_str(), nullptr, 0);
+        const unsigned long long pc = strtoull(f[3].c_str(), nullptr, 0);
+        auto ki = kid.find(f[2]);
+        for (size_t q = 4; q < f.size(); q++) {
+          const size_t c = f[q].find(':');
+          const unsigned long long idx = strtoull(f[q].substr(0, c).c_str(), nullptr, 0);
+          const unsigned long long cnt = strtoull(f[q].substr(c + 1).c_str(), nullptr, 0);
+          std::string name = table.count(idx) ? table[idx] : std::string();
+          if (name.size() > ni.size() && name.compare(name.size() - ni.size(), ni.size(), ni) == 0) {
+            skipped += cnt;
+            continue;
+          }
+          N += cnt;
+          int reason = -1;
+          if (name.compare(0, prefix.size(), prefix) == 0)
+            for (int r = 0; r < 19; r++)
+              if (name.substr(prefix.size()) == kReasonName[r]) reason = r;
+          const bool ok = (cupti_crc == 0 || crc == cupti_crc) && ki != kid.end() && reason >= 0 &&
+                          pc <= 0xffffffffull && valid((uint32_t)ki->second, (uint32_t)pc, (uint32_t)reason);
+          if (!ok) { invalid += cnt; continue; }
+          H[(ks[ki->second].first_slot + pc / 16) * 32 + reason] += cnt;
+        }
+      }
+      fclose(pf);
+    }
     auto th1 = now();
     uint64_t mass = 0;
     for (size_t b = 0; b < H.size(); b++)
@@ -1168,6 +1226,7 @@ int main(int argc, char** argv) {
       }
     fprintf(out, "N total=%llu valid=%llu invalid=%llu\n", (unsigned long long)N, (unsigned long long)mass,
             (unsigned long long)invalid);
+    if (!cupti_path.empty()) fprintf(out, "C skipped=%llu\n", (unsigned long long)skipped);  // _not_issued (R39)
     // O14 join: counts at the site's PC, site total, kernel total, REL sum.
     std::vector<uint64_t> ktot(ks.size(), 0);
     for (size_t k = 0; k < ks.size(); k++)

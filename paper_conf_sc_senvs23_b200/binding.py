@@ -46,7 +46,8 @@ class GsError(RuntimeError):
 _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
-           "gs_attribute_samples", "gs_attribute_counts", "gs_register_pressure", "gs_rank_sites", "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
+           "gs_attribute_samples", "gs_attribute_counts", "gs_cupti_stall_reasons", "gs_attribute_cupti", "gs_register_pressure", "gs_rank_sites",
+           "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
 
 
 def launch_count() -> int:
@@ -78,6 +79,9 @@ def load_library(path: str = LIB_PATH):
         "gs_pack_samples": (I32, [P, P, U64, P, P]),
         "gs_attribute_samples": (I32, [P, P, U64, P, P, I32]),
         "gs_attribute_counts": (I32, [P, P, U64, P, P, I32]),
+        "gs_cupti_stall_reasons": (I32, [P, SZ, P, P]),
+        "gs_attribute_cupti": (I32, [P, P, SZ, U64, P, P, I32, ctypes.POINTER(ctypes.c_ulonglong),
+                                     ctypes.POINTER(ctypes.c_ulonglong)]),
         "gs_register_pressure": (I32, [P, U32, U32, P]),
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
         "gs_rank_sites_slice": (I32, [P, P, U64, U64, U64, P, ctypes.POINTER(U64)]),
@@ -240,6 +244,27 @@ class Context:
         self._check(self.L.gs_attribute_counts(self.h, recs.data_ptr(), recs.shape[0], hist.data_ptr(),
                                                n_invalid.data_ptr(), 1 if accumulate else 0), "gs_attribute_counts")
         return hist, n_invalid
+
+    def cupti_stall_reasons(self, n: int, index_ptr: int, names_ptr: int):
+        """the stall-reason table of cuptiPCSamplingGetStallReasons: n CUPTI indices (uint32 array
+        address) and their names (char* array address)"""
+        self._check(self.L.gs_cupti_stall_reasons(self.h, n, index_ptr, names_ptr), "gs_cupti_stall_reasons")
+
+    def attribute_cupti(self, pc_data_ptr: int, n_pcs: int, cubin_crc: int = 0, hist=None, n_invalid=None,
+                        accumulate: bool = False):
+        """CUpti_PCSamplingPCData[n_pcs] at host address pc_data_ptr -> histogram. Returns
+        (hist, n_invalid device tensor, skipped samples, flattened entries)."""
+        import torch
+        dev = torch.device("cuda", self.device)
+        if hist is None:
+            hist = torch.empty(self.n_instr * self.hist_row, dtype=torch.int32, device=dev)
+        if n_invalid is None:
+            n_invalid = torch.zeros(1, dtype=torch.int64, device=dev)
+        sk, nr = ctypes.c_ulonglong(), ctypes.c_ulonglong()
+        self._check(self.L.gs_attribute_cupti(self.h, pc_data_ptr, n_pcs, cubin_crc, hist.data_ptr(), n_invalid.data_ptr(),
+                                              1 if accumulate else 0, ctypes.byref(sk), ctypes.byref(nr)),
+                    "gs_attribute_cupti")
+        return hist, n_invalid, sk.value, nr.value
 
     def register_pressure(self, k_begin: int = 0, k_end: int | None = None, out=None):
         """Live GPRs per instruction (int16 device tensor indexed by slot; kernels outside

@@ -16,7 +16,7 @@ LIB = os.path.join(HERE, "libgpuscout_b200.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CUDA_SRCS = ["api.cu", "detect.cu", "scan.cu", "attrib.cu", "rank.cu", "liveness.cu"]
-CXX_SRCS = ["loader.cpp"]
+CXX_SRCS = ["loader.cpp", "cupti.cpp"]
 HEADERS = ["ctx.h", "record.h", "loader.h"]
 
 

@@ -32,6 +32,7 @@ namespace {
 void free_loaded(gs_ctx* c) {
   detect_free(c);
   rank_reset_graph(c);
+  c->kernel_index.clear();
   if (c->d_rec) cudaFree(c->d_rec);
   if (c->d_kd) cudaFree(c->d_kd);
   if (c->d_wd) cudaFree(c->d_wd);
@@ -103,6 +104,7 @@ void gs_destroy(gs_ctx* c) {
   free_loaded(c);
   attrib_free(c);
   rank_free(c);
+  cupti_free(c);
   if (c->h_pin) cudaFreeHost(c->h_pin);
   delete c;
 }
@@ -355,6 +357,24 @@ gs_status gs_attribute_counts(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int
   if (n && !is_device_ptr(d_recs)) return fail(c, GS_E_INVAL, "count records must be device memory");
   GS_CUDA(c, cudaSetDevice(c->device));
   return counts_run(c, d_recs, n, d_hist, d_n_invalid, accumulate);
+}
+
+gs_status gs_cupti_stall_reasons(gs_ctx* c, size_t n, const uint32_t* index, const char* const* names) {
+  if (!c || (n && (!index || !names))) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  return cupti_reasons(c, n, index, names);
+}
+
+gs_status gs_attribute_cupti(gs_ctx* c, const void* pc_data, size_t n_pcs, uint64_t cubin_crc, int32_t* d_hist,
+                             unsigned long long* d_n_invalid, int accumulate, unsigned long long* n_skipped,
+                             unsigned long long* n_records) {
+  if (!c || (n_pcs && !pc_data) || !d_n_invalid) return fail(c, GS_E_INVAL, "null argument");
+  c->err.clear();
+  if (!c->loaded) return fail(c, GS_E_STATE, "gs_attribute_cupti before gs_load_sass");
+  if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
+  if (n_pcs && is_device_ptr(pc_data)) return fail(c, GS_E_INVAL, "CUPTI records must be host memory");
+  GS_CUDA(c, cudaSetDevice(c->device));
+  return cupti_run(c, pc_data, n_pcs, cubin_crc, d_hist, d_n_invalid, accumulate, n_skipped, n_records);
 }
 
 gs_status gs_register_pressure(gs_ctx* c, uint32_t k_begin, uint32_t k_end, uint16_t* d_live) {

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "../../include/gpuscout_b200.h"
@@ -131,6 +132,13 @@ struct gs_ctx {
   uint64_t rank_graph_launches = 0;
   void* d_sort_tmp = nullptr;
   size_t sort_tmp_bytes = 0;
+  // CUPTI ingest (cupti.cpp, R39): stall-reason index -> reason id (-2 skipped, -1 unknown), kernel
+  // name -> index of the loaded module, pinned staging + device copy of the flattened records
+  std::unordered_map<uint32_t, int> cupti_reason;
+  std::unordered_map<std::string, uint32_t> kernel_index;
+  void* h_cupti = nullptr;
+  void* d_cupti = nullptr;
+  uint64_t cupti_cap = 0;
   unsigned long long* d_ktot = nullptr;
   uint64_t ktot_cap = 0;
   gs_ranked_site* d_ranked = nullptr;
@@ -218,6 +226,12 @@ gs_status uses_upload(gs_ctx* c);
 void liveness_free(gs_ctx* c);
 void rank_free(gs_ctx* c);
 void rank_reset_graph(gs_ctx* c);
+gs_status cupti_reasons(gs_ctx* c, size_t n, const uint32_t* index, const char* const* names);
+gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int32_t* d_hist,
+                    unsigned long long* d_n_invalid, int accumulate, unsigned long long* n_skipped,
+                    unsigned long long* n_records);
+cudaError_t cupti_grow(gs_ctx* c, uint64_t n);
+void cupti_free(gs_ctx* c);
 
 // device-wide exclusive scan of u32 counts into u32 or u64 offsets; total written to *d_total
 gs_status scan_u32(gs_ctx* c, const uint32_t* in, uint32_t* out, uint64_t n, unsigned long long* d_total);

@@ -22,7 +22,8 @@ def build_oracle(force: bool = False) -> str:
 
 def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, kbegin=0, kend=-1,
         detect=True, hist=True, timing=False, counts: np.ndarray | None = None, join: str = "pc",
-        liveness: bool = False, hlines: bool = True, regsets: bool = False) -> str:
+        liveness: bool = False, hlines: bool = True, regsets: bool = False, cupti: str | None = None,
+        cupti_crc: int = 0) -> str:
     """sass: path or text/bytes. samples: [N,3] uint32 raw triples. counts: [M,4] uint32
     pre-aggregated (kernel, pc, reason, count) records. join: pc | line | consumer. Returns canonical text."""
     build_oracle()
@@ -50,6 +51,12 @@ def run(sass, samples: np.ndarray | None = None, D=64, R=19, TA=1, TL=2, k=-1, k
             f.close()
             tmp.append(f.name)
             cmd += ["--counts", f.name]
+        if cupti is not None:   # CUPTI PC-sampling records in their text form (gen/cupti.py)
+            f = tempfile.NamedTemporaryFile("w", suffix=".cupti", delete=False)
+            f.write(cupti)
+            f.close()
+            tmp.append(f.name)
+            cmd += ["--cupti", f.name, "--cupti-crc", str(cupti_crc)]
         if join != "pc":
             cmd += ["--join", join]
         if liveness:

@@ -606,3 +606,34 @@ def test_reload_then_rank_graph(gs):
                 got = Canon(report.canonical(ctx, hist=hist, n_samples=len(raw), n_invalid=0, ranked=rows)).R
                 assert got == Canon(orc.run(s.text, samples=raw)).R, q
         st.synchronize()
+
+
+@pytest.mark.parametrize("cfg,crc_filter,row", [("C2", True, 32), ("C2", False, 19), ("C1", True, 19)])
+def test_cupti_ingest_parity(gs, cfg, crc_filter, row):
+    """gs_cupti_stall_reasons + gs_attribute_cupti on CUPTI-shaped host
+    records (CUpti_PCSamplingPCData with host name / stall-reason pointers): histogram, invalid
+    and skipped weights, and the ranking equal the oracle reading the same records."""
+    import torch
+    from gen import cupti
+    from gen import samples as gsm
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    s = gsass.config_sass(cfg)
+    tab = gsm.table_class_weighted(s.cls, 300_000, key=13)
+    names = [ln.split(b"Function : ")[1].split()[0].decode() for ln in s.text.split(b"\n") if b"Function : " in ln]
+    buf = cupti.Buffer(tab, names, s.first_slot, s.n_instr, key=13)
+    crc = buf.crc if crc_filter else 0
+    ctx = _ctx(gs, hist_row=row)
+    ctx.load_sass(s.text)
+    ctx.detect()
+    ctx.cupti_stall_reasons(*buf.table_ptrs())
+    hist, ninv, skipped, nrec = ctx.attribute_cupti(buf.ptr(), buf.n, crc)
+    rows = ctx.rank_sites(hist)
+    torch.cuda.synchronize()
+    n_inv = int(ninv.item())
+    total = int(tab.sum()) + n_inv + (sum(w for _, _, w in buf.foreign_crc_bins) if not crc_filter else 0)
+    g = Canon(report.canonical(ctx, hist=hist, n_samples=total, n_invalid=n_inv, ranked=rows))
+    o = Canon(orc.run(s.text, cupti=buf.text, cupti_crc=crc))
+    assert g.H == o.H and g.N == o.N and g.R == o.R and g.S == o.S
+    assert f"C skipped={skipped}" in o.text and skipped == buf.skipped
+    assert nrec == sum(int(buf.pcdata[i].stallReasonCount) for i in range(buf.n))

@@ -615,3 +615,33 @@ def test_sharded_oracle_equals_single_process(name, shards):
         raw = None
     want = orc.run(text, samples=raw, hlines=False) if raw is not None else orc.run(text, hist=False)
     assert orc.run_sharded(text, raw, n_instr, shards) == want
+
+
+# --------------------------------------------------------------------------- CUPTI records (R39)
+def _module_names(text: bytes):
+    return [ln.split(b"Function : ")[1].split()[0].decode() for ln in text.split(b"\n") if b"Function : " in ln]
+
+
+def test_cupti_records_equal_count_table():
+    """CUPTI PC-sampling records (CUpti_PCSamplingPCData: per PC, samples per CUPTI stall-reason
+    index; SURVEY [probe 8]) built from an exact count table: the oracle's histogram is
+    the table; _not_issued counters (a subset of the same samples) are skipped; a foreign cubin,
+    an unknown function, an unknown reason and a misaligned pc are invalid (R39)."""
+    from gen import cupti
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    tab = gsm.table_class_weighted(s.cls, 200_000, key=9)
+    buf = cupti.Buffer(tab, _module_names(s.text), s.first_slot, s.n_instr, key=9)
+    c = Canon(orc.run(s.text, cupti=buf.text, cupti_crc=buf.crc, detect=False))
+    nz = np.nonzero(tab)
+    assert {(int(a), int(b)): int(tab[a, b]) for a, b in zip(*nz)} == c.H
+    assert c.N == {"total": str(int(tab.sum()) + buf.invalid_crc), "valid": str(int(tab.sum())),
+                   "invalid": str(buf.invalid_crc)}
+    assert f"C skipped={buf.skipped}" in c.text
+    # any cubin (crc 0): the foreign-cubin records of known functions count too
+    c0 = Canon(orc.run(s.text, cupti=buf.text, cupti_crc=0, detect=False))
+    want = {(int(a), int(b)): int(tab[a, b]) for a, b in zip(*nz)}
+    for slot, r, w in buf.foreign_crc_bins:
+        want[(slot, r)] = want.get((slot, r), 0) + w
+    assert c0.H == want and c0.N["invalid"] == str(buf.invalid_any)

@@ -309,6 +309,38 @@ def extra_pack_hist(g, ctx, words, hist, ninv, s, peak, steps, warmup):
                          "frac": alg_both / (both_ms * 1e-3) / 1e9 / peak, "algorithmic_bytes": alg_both}}
 
 
+def extra_cupti(g, s, peak, steps, warmup):
+    """CUPTI ingest: the C4 count table as CUpti_PCSamplingPCData host records (one
+    per PC, all-samples + not-issued counters per reason) through gs_attribute_cupti: host flattening
+    into pinned memory, one H2D copy, the weighted device scatter-add. Wall clock per call (the host
+    part dominates), records/s and the samples they represent per second."""
+    import torch
+    from gen import cupti
+    from gen import samples as gsm
+    tab = gsm.table_c4(s.cls, s.first_slot, s.n_instr, 1 << 30, key=0x6E5C0004)
+    names = [ln.split(b"Function : ")[1].split()[0].decode() for ln in s.text.split(b"\n") if b"Function : " in ln]
+    buf = cupti.FastBuffer(tab, names, s.first_slot)
+    R = 19
+    ctx = g.Context(n_reasons=R, hist_row=R)
+    ctx.load_sass(s.text)
+    ctx.cupti_stall_reasons(*buf.table_ptrs())
+    hist = torch.empty(ctx.n_instr * R, dtype=torch.int32, device="cuda")
+    ninv = torch.zeros(1, dtype=torch.int64, device="cuda")
+    ts = []
+    for i in range(warmup + steps):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        _, _, sk, nrec = ctx.attribute_cupti(buf.ptr(), buf.n, buf.crc, hist, ninv)
+        torch.cuda.synchronize()
+        if i >= warmup:
+            ts.append(time.perf_counter() - t0)
+    assert int(hist.to(torch.int64).sum().item()) == buf.samples and sk == buf.skipped and int(ninv.item()) == 0
+    sec = float(np.median(ts))
+    return {"records": buf.n, "entries": int(nrec), "samples": buf.samples, "ms_per_call": sec * 1e3,
+            "records_per_s": buf.n / sec, "entries_per_s": nrec / sec, "samples_per_s": buf.samples / sec,
+            "host_threads": min(16, os.cpu_count() or 1)}
+
+
 def workload_config(args, s, tr, world):
     return {"workload": args.config, "kernels": len(s.n_instr), "sass_instrs": s.P, "samples": tr.N,
             "order": args.order, "reasons": 19, "trace_depth": 64, "parallelism": f"dp{world}",
@@ -497,7 +529,8 @@ def main():
     if world == 1 and not args.no_extras:
         del host_words
         torch.cuda.empty_cache()
-        for name, fn in (("detect_C3", extra_detect_c3), ("C5", extra_c5)):
+        for name, fn in (("detect_C3", extra_detect_c3), ("C5", extra_c5),
+                         ("cupti_C4", lambda g_, pk, st, wu: extra_cupti(g_, s, pk, st, wu))):
             try:
                 extras[name] = fn(g, read_peaks()[0], 10, 3)
             except Exception as e:  # noqa: BLE001

@@ -125,3 +125,59 @@ class Buffer:
         """(n, pointer to uint32 indices, pointer to char* names) for gs_cupti_stall_reasons"""
         self._idx_arr = np.ascontiguousarray(self.idx, dtype=np.uint32)
         return len(self.names), self._idx_arr.ctypes.data, ctypes.addressof(self._cnames)
+
+
+PCDATA_DTYPE = np.dtype({"names": ["size", "cubinCrc", "pcOffset", "functionIndex", "pad", "functionName",
+                                   "stallReasonCount", "stallReason", "correlationId"],
+                         "formats": [np.uint64, np.uint64, np.uint64, np.uint32, np.uint32, np.uint64, np.uint64,
+                                     np.uint64, np.uint32],
+                         "offsets": [0, 8, 16, 24, 28, 32, 40, 48, 56], "itemsize": 64})
+
+
+class FastBuffer:
+    """Bench-size CUPTI buffer (numpy, vectorised): one CUpti_PCSamplingPCData per PC with nonzero
+    counts, all-samples and not-issued counters per nonzero reason, valid records only."""
+
+    def __init__(self, table, names, first_slot, crc: int = 0x1234ABCD5678EF01, key: int = 7):
+        self.idx, self.names = stall_table(key)
+        ix = {n: int(i) for i, n in zip(self.idx, self.names)}
+        all_ix = np.array([ix[PREFIX + r] for r in REASONS], dtype=np.uint32)
+        ni_ix = np.array([ix[PREFIX + r + "_not_issued"] for r in REASONS], dtype=np.uint32)
+        t = np.asarray(table)[:, :R_ACTIVE]
+        first_slot = np.asarray(first_slot, dtype=np.int64)
+        slots, reasons = np.nonzero(t)               # slot-major
+        counts = t[slots, reasons].astype(np.uint64)
+        n_ent = 2 * len(slots)
+        ents = np.zeros((n_ent, 2), dtype=np.uint32)
+        ents[0::2, 0] = all_ix[reasons]
+        ents[0::2, 1] = counts
+        ents[1::2, 0] = ni_ix[reasons]
+        ents[1::2, 1] = counts // 4                  # not-issued: a subset of the same samples
+        self.skipped = int((counts // 4).sum())
+        self.samples = int(counts.sum())
+        self.ents = ents
+        pcs, start = np.unique(slots, return_index=True)
+        per = np.diff(np.append(start, len(slots))) * 2
+        kern = np.searchsorted(first_slot, pcs, side="right") - 1
+        self._names = [ctypes.create_string_buffer(n.encode()) for n in names]
+        name_addr = np.array([ctypes.addressof(b) for b in self._names], dtype=np.uint64)
+        rec = np.zeros(len(pcs), dtype=PCDATA_DTYPE)
+        rec["size"] = PCDATA_SIZE
+        rec["cubinCrc"] = crc
+        rec["pcOffset"] = 16 * (pcs - first_slot[kern])
+        rec["functionIndex"] = kern
+        rec["functionName"] = name_addr[kern]
+        rec["stallReasonCount"] = per
+        rec["stallReason"] = ents.ctypes.data + 16 * start.astype(np.uint64)  # 2 entries (8 B each) per bin
+        self.rec = rec
+        self.crc = crc
+        self.n = len(rec)
+        self.n_entries = n_ent
+        self._cnames = (ctypes.c_char_p * len(self.names))(*[n.encode() for n in self.names])
+
+    def ptr(self) -> int:
+        return self.rec.ctypes.data
+
+    def table_ptrs(self):
+        self._idx_arr = np.ascontiguousarray(self.idx, dtype=np.uint32)
+        return len(self.names), self._idx_arr.ctypes.data, ctypes.addressof(self._cnames)

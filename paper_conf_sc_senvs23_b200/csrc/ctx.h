@@ -11,7 +11,10 @@
 
 namespace gs {
 
-constexpr uint32_t kWin = 256;  // instructions per detection window (never crosses a kernel)
+#ifndef GS_KWIN
+#define GS_KWIN 1024
+#endif
+constexpr uint32_t kWin = GS_KWIN;  // instructions per detection window (never crosses a kernel)
 
 // A device buffer that only grows; freed with the context.
 struct DevBuf {

@@ -39,6 +39,11 @@ __device__ __forceinline__ Rec ld_rec(const Rec* r, uint64_t i) {
   return o;
 }
 __device__ __forceinline__ uint32_t reg_cap(uint32_t dst) { return dst < 256 ? 254u : 318u; }
+// The opcode-class table in shared memory: op_class() is a switch that compiles to a branch tree,
+// which a warp of mixed opcodes walks divergently for every record; one LDS replaces it.
+__device__ __forceinline__ void opcls_init(uint16_t* t) {
+  for (uint32_t i = threadIdx.x; i < OP_COUNT; i += blockDim.x) t[i] = (uint16_t)op_class(i);
+}
 
 __device__ __forceinline__ uint32_t hash64(unsigned long long k) {
   k ^= k >> 33; k *= 0xff51afd7ed558ccdull; k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull; k ^= k >> 33;
@@ -77,6 +82,9 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
                                                          uint32_t* __restrict__ tab, int32_t* ldiff, int32_t* wsum,
                                                          uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst) {
   __shared__ uint32_t last[kWarps][kNumRegs];
+  __shared__ uint16_t s_cls[OP_COUNT];
+  opcls_init(s_cls);
+  __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
   if (w >= w0 + nw) return;
@@ -99,7 +107,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
     const bool valid = i < W.len;
     const uint64_t g = (uint64_t)W.start + i;
     const Rec r = rr[u];
-    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), dst2 = r_dst2(r);
+    const uint32_t op = r_op(r), cls = s_cls[op], dst = r_dst(r), dw = r_dstw(r), dst2 = r_dst2(r);
     if (valid && dw && reg_live(dst)) {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
       const uint32_t cap = reg_cap(dst);
@@ -186,6 +194,9 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
                                                          uint32_t* __restrict__ ptrrd, uint32_t* narith, CandArrays ca) {
   __shared__ uint32_t tabS[kWarps][kNumRegs];
   __shared__ uint32_t cm[kWarps][kNumRegs];
+  __shared__ uint16_t s_cls[OP_COUNT];
+  opcls_init(s_cls);
+  __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
   if (w >= w0 + nw) return;
@@ -217,7 +228,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
     const uint64_t gbase = (uint64_t)W.start + b;
     const Rec r = rnext;  // records of the next chunk are loaded while this one is resolved
     rnext = i + 32 < W.len ? ld_rec(rec, g + 32) : Rec{0, 0, 0, 0};
-    const uint32_t op = r_op(r), cls = op_class(op), dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
+    const uint32_t op = r_op(r), cls = s_cls[op], dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
     const bool writes = valid && dw && reg_live(dst);
     const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
     const bool writes2 = reg_live(dst2);
@@ -237,19 +248,22 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
       }
       return T[reg];
     };
-    // loop depth: inclusive prefix of the event differences (R13)
-    int32_t ev = 0;
-    if (has_ev && valid) {
-      ev = ldiff[g];
-      if (ev) ldiff[g] = 0;  // keep the difference array zero for the next call
+    // loop depth: inclusive prefix of the event differences (R13); a window without loop events
+    // (warp-uniform) keeps its carried depth
+    int32_t depth = lcarry;
+    if (has_ev) {
+      int32_t pre = 0;
+      if (valid) {
+        pre = ldiff[g];
+        if (pre) ldiff[g] = 0;  // keep the difference array zero for the next call
+      }
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t x = __shfl_up_sync(0xffffffffu, pre, o);
+        if (lane >= o) pre += x;
+      }
+      depth = lcarry + pre;
+      lcarry += __shfl_sync(0xffffffffu, pre, 31);
     }
-    int32_t pre = ev;
-    for (int o = 1; o < 32; o <<= 1) {
-      const int32_t x = __shfl_up_sync(0xffffffffu, pre, o);
-      if (lane >= o) pre += x;
-    }
-    const int32_t depth = lcarry + pre;
-    lcarry += __shfl_sync(0xffffffffu, pre, 31);
     if (valid && r_pk(r) == PK_REG) ptrrd[g] = RD(r_ptr(r)) >> 1;
     const bool iscand = valid && (cls & (C_TRACED | C_CONV));
     const uint32_t cmask = __ballot_sync(0xffffffffu, iscand);
@@ -403,7 +417,7 @@ struct TraceOut {
 // Bounded backward trace (R7). `emit` receives each chain element (kernel-local).
 template <typename Emit>
 __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restrict__ ptrrd, const KDesc& K,
-                          uint32_t base, uint32_t base_rd, uint32_t D, Emit emit) {
+                          uint32_t base, uint32_t base_rd, uint32_t D, const uint16_t* __restrict__ cls_tab, Emit emit) {
   TraceOut o{GS_T_IMM, 0, 0};
   if (!reg_live(base) || base_rd == 0xffffffffu) return o;
   uint32_t r = base, v = base_rd, depth = 0;
@@ -414,7 +428,7 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restric
     depth++;
     emit(j - K.first);
     const Rec rj = ld_rec(rec, j);
-    const uint32_t cj = op_class(r_op(rj));
+    const uint32_t cj = cls_tab[r_op(rj)];
     if (cj & C_CONSTLOAD) {
       const int32_t off = r_imm(rj) + 4 * (int32_t)(r - r_dst(rj));
       const uint32_t bank = r_cbank(rj);
@@ -445,13 +459,16 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restric
 __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
                         uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, OffsetSet os, RootSet rs,
                         gs_kernel_stats* kst) {
+  __shared__ uint16_t s_cls[OP_COUNT];
+  opcls_init(s_cls);
+  __syncthreads();
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (t >= 2 * nc) return;
   const bool groups = t >= nc;
   const uint64_t c = groups ? t - nc : t;
   const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
   const Rec ri = ld_rec(rec, g);
-  const uint32_t op = r_op(ri), cls = op_class(op);
+  const uint32_t op = r_op(ri), cls = s_cls[op];
   const bool traced = (cls & C_TRACED) && (r_flags(ri) & F_HASMEM);
   const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
   if (groups) {
@@ -482,7 +499,7 @@ __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ k
     return;
   }
   const KDesc K = kd[kernel];
-  const TraceOut tr = chase(rec, ptrrd, K, base, brd, D, [](uint32_t) {});
+  const TraceOut tr = chase(rec, ptrrd, K, base, brd, D, s_cls, [](uint32_t) {});
   ca.tk[c] = (uint8_t)tr.tk;
   ca.tv[c] = tr.tv;
   ca.depth[c] = (uint8_t)tr.depth;
@@ -498,8 +515,8 @@ struct RuleCfg {
 };
 
 __device__ uint32_t eval_rules(const Rec& ri, uint64_t c, const CandArrays& ca, const GroupTable& gt,
-                               const RootSet& rs, const uint32_t* narith, RuleCfg rc) {
-  const uint32_t op = r_op(ri), cls = op_class(op), fl = r_flags(ri);
+                               const RootSet& rs, const uint32_t* narith, RuleCfg rc, const uint16_t* cls_tab) {
+  const uint32_t op = r_op(ri), cls = cls_tab[op], fl = r_flags(ri);
   uint32_t f = 0;
   if (!(fl & F_HASMEM) && !(cls & C_CONV)) return 0;
   if (op == OP_LDG && (fl & F_HASMEM)) {
@@ -560,11 +577,14 @@ __device__ __forceinline__ unsigned long long site_chain(uint32_t f, uint32_t de
 __global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca, GroupTable gt,
                                                RootSet rs, const uint32_t* __restrict__ narith, RuleCfg rc,
                                                unsigned long long* __restrict__ tsum) {
+  __shared__ uint16_t s_cls[OP_COUNT];
+  opcls_init(s_cls);
+  __syncthreads();
   const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
   unsigned long long v = 0;
   if (c < nc) {
     const Rec ri = ld_rec(rec, ca.idx[c]);
-    const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc);
+    const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc, s_cls);
     ca.flags[c] = (uint8_t)f;
     v = site_chain(f, ca.depth[c]);
   }
@@ -607,6 +627,8 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
                                                uint32_t* __restrict__ chain, uint64_t site_cap, uint64_t chain_cap) {
   // Launched before the host knows the totals: writes past the buffers' current capacities are
   // skipped, and the host relaunches after growing them when a total exceeds its capacity.
+  __shared__ uint16_t s_cls[OP_COUNT];
+  opcls_init(s_cls);  // (block_excl64 below synchronises the CTA before the first use)
   const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
   const uint32_t f = c < nc ? ca.flags[c] : 0u;
   unsigned long long tot;
@@ -619,7 +641,7 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
   // chain: re-chase and store kernel-local indices
   uint32_t n = 0;
   if (ca.depth[c] && coff + ca.depth[c] <= chain_cap)
-    chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, [&](uint32_t j) { chain[coff + n++] = j; });
+    chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, s_cls, [&](uint32_t j) { chain[coff + n++] = j; });
   uint64_t so = pre_s[blockIdx.x] + (ex & 0xffffffffull);
   for (uint32_t rule = 0; rule < 7; rule++) {
     if (!((f >> rule) & 1u)) continue;

@@ -13,9 +13,13 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--scale", type=float, default=1.0)
 ap.add_argument("--steps", type=int, default=10)
 ap.add_argument("--cpu-scale", type=float, default=0.02)
+ap.add_argument("--lib", default=None, help="another build of the library (diagnostic variants)")
 a = ap.parse_args()
 import torch
 import paper_conf_sc_senvs23_b200 as g
+if a.lib:
+    from paper_conf_sc_senvs23_b200 import binding
+    binding.load_library(a.lib)
 from gen import sass as gsass
 t = time.perf_counter()
 s = gsass.config_sass("C3", scale=a.scale)

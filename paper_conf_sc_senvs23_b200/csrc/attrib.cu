@@ -333,20 +333,21 @@ __device__ void flush(uint32_t* tab, uint32_t ws, uint32_t nr, uint32_t row, uin
 // uint4; rng[c] = (head << 32) | stolen counts tiles taken from the front by the owner and from the
 // back by CTAs that finished their own chunk (work stealing: every SM stays busy to the end while
 // each CTA still walks its own chunk front to back, so windows change rarely).
-__device__ __forceinline__ uint32_t n_tiles(uint64_t c, uint64_t chunk, uint64_t n) {
-  const uint64_t a4 = c * chunk / 4, e = (c + 1) * chunk < n ? (c + 1) * chunk : n, e4 = e / 4;
+// chunk c of the stream = uint4 range [bnd[c], bnd[c + 1]) (k_plan balances the chunks' cost)
+__device__ __forceinline__ uint32_t n_tiles(uint64_t c, const unsigned long long* __restrict__ bnd) {
+  const uint64_t a4 = bnd[c], e4 = bnd[c + 1];
   return e4 > a4 ? (uint32_t)((e4 - a4 + kTile4 - 1) / kTile4) : 0u;
 }
 // Called by the whole producer warp (result broadcast). Own chunk: lane 0 takes the next tile from
 // the front. Stealing: the 32 lanes read the queue words of all chunks in parallel (a serial scan
 // by one lane took longer than the tiles it was meant to rebalance), pick the chunk with the most
 // tiles left and take its last tile with one CAS.
-__device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, uint32_t grid, uint64_t chunk,
-                                        uint64_t n) {
+__device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, uint32_t grid,
+                                        const unsigned long long* __restrict__ bnd) {
   const uint32_t lane = threadIdx.x & 31u;
   unsigned long long got = ~0ull;
   if (lane == 0) {
-    const uint32_t mine = n_tiles(me, chunk, n);
+    const uint32_t mine = n_tiles(me, bnd);
     for (;;) {  // own chunk, front to back
       const unsigned long long o = *(volatile unsigned long long*)(rng + me);
       const uint32_t head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
@@ -360,7 +361,7 @@ __device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, ui
     uint32_t best = grid, best_left = 0;
     for (uint32_t v = lane; v < grid; v += 32) {
       const unsigned long long o = *(volatile unsigned long long*)(rng + v);
-      const uint32_t nt = n_tiles(v, chunk, n), used = (uint32_t)(o >> 32) + (uint32_t)o;
+      const uint32_t nt = n_tiles(v, bnd), used = (uint32_t)(o >> 32) + (uint32_t)o;
       if (nt > used && nt - used > best_left) { best_left = nt - used; best = v; }
     }
     const uint32_t mx = __reduce_max_sync(0xffffffffu, best_left);
@@ -368,7 +369,7 @@ __device__ unsigned long long grab_tile(unsigned long long* rng, uint32_t me, ui
     const uint32_t cand = __reduce_min_sync(0xffffffffu, best_left == mx ? best : 0xffffffffu);
     if (lane == 0) {
       const unsigned long long o = *(volatile unsigned long long*)(rng + cand);
-      const uint32_t nt = n_tiles(cand, chunk, n), head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
+      const uint32_t nt = n_tiles(cand, bnd), head = (uint32_t)(o >> 32), stolen = (uint32_t)o;
       if (head + stolen < nt && atomicCAS(rng + cand, o, o + 1ull) == o)
         got = ((unsigned long long)cand << 32) | (nt - 1 - stolen);
     }
@@ -641,9 +642,10 @@ struct Item {
 template <bool P16>
 __global__ void __launch_bounds__(kThreads, 1)
     k_hist_window(const uint32_t* __restrict__ s, uint64_t n, uint32_t P, uint32_t nr, Div dv,
-                  const KDesc* __restrict__ kd, uint32_t nk, uint64_t chunk, uint32_t one, int32_t* __restrict__ H,
+                  const KDesc* __restrict__ kd, uint32_t nk, uint32_t one, int32_t* __restrict__ H,
                   unsigned long long* d_n_invalid, unsigned long long* rng, uint32_t* __restrict__ defer_ring,
                   uint32_t tw) {
+  const unsigned long long* __restrict__ bnd = rng + gridDim.x;  // chunk bounds (k_plan)
   extern __shared__ uint32_t tab[];  // tw counter words + 32 spare words
   __shared__ Item items[kItems];
   __shared__ __align__(8) uint64_t full[kItems], empty[kItems];
@@ -662,10 +664,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
 
   const auto span = [&](unsigned long long tile, uint64_t& a4, uint64_t& b4) {
-    const uint64_t c = tile >> 32, ca4 = c * chunk / 4;
-    const uint64_t ce = (c + 1) * chunk < n ? (c + 1) * chunk : n;
-    a4 = ca4 + (uint64_t)(uint32_t)tile * kTile4;
-    b4 = a4 + kTile4 < ce / 4 ? a4 + kTile4 : ce / 4;
+    const uint64_t c = tile >> 32, ce4 = bnd[c + 1];
+    a4 = bnd[c] + (uint64_t)(uint32_t)tile * kTile4;
+    b4 = a4 + kTile4 < ce4 ? a4 + kTile4 : ce4;
   };
 
   if (threadIdx.x < 32) {  // ------------------------------------------------ producer
@@ -681,7 +682,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       j++;
     };
     for (;;) {
-      const unsigned long long tile = grab_tile(rng, blockIdx.x, gridDim.x, chunk, n);
+      const unsigned long long tile = grab_tile(rng, blockIdx.x, gridDim.x, bnd);
       if (tile == ~0ull) break;
       uint64_t a4, b4;
       span(tile, a4, b4);
@@ -806,6 +807,88 @@ __global__ void __launch_bounds__(kThreads, 1)
 #else
   (void)d_f0;
 #endif
+}
+
+// Chunk planning for WINDOW: the CTAs' contiguous chunks are cut at equal COST, not at equal
+// sample counts. A chunk costs its samples plus, per window switch, the flush of a whole window
+// (~15K SM cycles ~ kSwitchCost samples at the counting rate): Zipf-distributed kernel weights put
+// many small kernels (many switches) into the last chunks of a trace, which otherwise finish last
+// (per-CTA timeline, GS_DIAG=11). kPlanProbes probe samples estimate where the windows change;
+// the queue words are zeroed here too.
+#ifndef GS_SWITCH_COST
+#define GS_SWITCH_COST 96000
+#endif
+constexpr uint32_t kPlanProbes = 4096;
+__global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, uint64_t n, uint32_t pnr, Div dv,
+                                               uint32_t nslots, uint32_t chunks, unsigned long long* __restrict__ q) {
+  __shared__ unsigned long long pre[kPlanProbes];
+  __shared__ unsigned long long wsum[32];
+  const uint64_t n4 = n / 4;
+  const uint32_t t = threadIdx.x;
+  constexpr uint32_t kPer = kPlanProbes / 1024;
+  // probe p sits at uint4 position pos(p) = p * n4 / NP; interval p = [pos(p), pos(p + 1))
+  uint32_t win[kPer + 1];
+#pragma unroll
+  for (uint32_t u = 0; u <= kPer; u++) {
+    const uint64_t p = (uint64_t)t * kPer + u;
+    const uint64_t pos = p * n4 / kPlanProbes;
+    const uint32_t w = (p < kPlanProbes && pos < n4) ? __ldg(s + 4 * pos) : 0xffffffffu;
+    win[u] = w < pnr ? divq(w, dv) / nslots : 0xffffffffu;  // window-sized slot block of the probe
+  }
+  unsigned long long loc = 0;
+  unsigned long long cst[kPer];
+#pragma unroll
+  for (uint32_t u = 0; u < kPer; u++) {
+    const uint64_t p = (uint64_t)t * kPer + u;
+    const uint64_t a = p * n4 / kPlanProbes, b = (p + 1) * n4 / kPlanProbes;
+    const bool sw = win[u] != 0xffffffffu && win[u + 1] != 0xffffffffu && win[u] != win[u + 1];
+    cst[u] = 4 * (b - a) + (sw ? (unsigned long long)GS_SWITCH_COST : 0ull);
+    loc += cst[u];
+  }
+  // inclusive scan of the per-thread sums over the CTA
+  const uint32_t lane = t & 31u, warp = t >> 5;
+  unsigned long long v = loc;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long x = __shfl_up_sync(0xffffffffu, v, o);
+    if ((int)lane >= o) v += x;
+  }
+  if (lane == 31) wsum[warp] = v;
+  __syncthreads();
+  if (warp == 0) {
+    unsigned long long x = wsum[lane];
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+      if ((int)lane >= o) x += y;
+    }
+    wsum[lane] = x;
+  }
+  __syncthreads();
+  unsigned long long run = (warp ? wsum[warp - 1] : 0ull) + v - loc;  // exclusive prefix of this thread
+#pragma unroll
+  for (uint32_t u = 0; u < kPer; u++) {
+    run += cst[u];
+    pre[t * kPer + u] = run;  // cost up to the end of interval p
+  }
+  __syncthreads();
+  const unsigned long long total = pre[kPlanProbes - 1];
+  unsigned long long* bnd = q + chunks;
+  for (uint32_t c = t; c <= chunks; c += blockDim.x) {
+    if (c < chunks) q[c] = 0ull;
+    uint64_t b;
+    if (c == 0) b = 0;
+    else if (c == chunks) b = n4;
+    else {  // the end of the first interval whose cost prefix reaches c / chunks of the total
+      const unsigned long long target = total * c / chunks;
+      uint32_t lo = 0, hi = kPlanProbes - 1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (pre[mid] >= target) hi = mid;
+        else lo = mid + 1;
+      }
+      b = (uint64_t)(lo + 1) * n4 / kPlanProbes;
+    }
+    bnd[c] = b;
+  }
 }
 
 // ---------------------------------------------------------------------- PARTITION
@@ -1251,10 +1334,13 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   uint64_t chunk = (n + chunks - 1) / chunks;
   chunk = (chunk + 3) & ~3ull;
   chunks = (n + chunk - 1) / chunk;
-  if (dyn) {  // work-stealing tile queue, one 64-bit word per chunk; two deferral ring halves per CTA
-    GS_CUDA(c, dev_grow(&c->d_tileq, &c->tileq_cap, chunks));
-    GS_CUDA(c, cudaMemsetAsync(c->d_tileq, 0, chunks * 8, st));
+  if (dyn) {  // work-stealing tile queue (one 64-bit word per chunk) + chunk bounds (k_plan); two
+              // deferral ring halves per CTA
+    GS_CUDA(c, dev_grow(&c->d_tileq, &c->tileq_cap, 2 * chunks + 1));
     GS_CUDA(c, dev_grow(&c->d_defer, &c->defer_cap, chunks * 2 * kDeferCap));
+    const uint32_t nslots = (uint32_t)std::max<uint64_t>(1, (bits == 16 ? 2ull * tw : (uint64_t)tw) / nr);
+    k_plan<<<1, 1024, 0, st>>>(d_words, n, P * nr, dv, nslots, (uint32_t)chunks, c->d_tileq);
+    count_launch();
   }
   const auto prep = [&](auto kern) -> gs_status {
     GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -1265,7 +1351,7 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     const auto kern = bits == 16 ? k_hist_window<true> : k_hist_window<false>;
     ls = prep(kern);
     if (ls == GS_OK)
-      kern<<<(uint32_t)chunks, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, chunk, 1u, d_hist,
+      kern<<<(uint32_t)chunks, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, 1u, d_hist,
                                                      d_n_invalid, c->d_tileq, c->d_defer, tw);
   } else {
     const auto kern = bits == 16 ? k_hist_smem<true> : k_hist_smem<false>;

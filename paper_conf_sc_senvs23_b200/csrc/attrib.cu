@@ -906,9 +906,25 @@ constexpr uint32_t kPMaxBuckets = 2048;
 constexpr uint32_t kPTile = kPT * 8;       // samples per scatter tile
 
 __device__ __forceinline__ uint32_t bucket_of(uint32_t w, Div dv, uint32_t bshift) { return divq(w, dv) >> bshift; }
+// bucket = w / (R << bshift) exactly for every 32-bit w, as one multiply-high (division by an
+// invariant integer, Granlund & Montgomery 1994, Fig. 4.1): l = ceil(log2 D), m = floor(2^32 (2^l - D) / D) + 1,
+// t = mulhi(m, w), q = (t + ((w - t) >> 1)) >> (l - 1); D >= 2
+struct BDiv {
+  uint32_t m, sh;
+};
+inline BDiv make_bdiv(uint32_t nr, uint32_t bshift) {
+  const uint64_t D = (uint64_t)nr << bshift;
+  uint32_t l = 0;
+  while ((1ull << l) < D) l++;
+  return BDiv{(uint32_t)((((1ull << 32) * ((1ull << l) - D)) / D) + 1), l - 1};
+}
+__device__ __forceinline__ uint32_t bucket_m(uint32_t w, BDiv b) {
+  const uint32_t t = __umulhi(b.m, w);
+  return (t + ((w - t) >> 1)) >> b.sh;
+}
 
 __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
-                                                uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
+                                                uint32_t pnr, BDiv dv, uint32_t B,
                                                 uint32_t* __restrict__ cnt, unsigned long long* d_n_invalid) {
   __shared__ uint32_t h[kPMaxBuckets];
   for (uint32_t b = threadIdx.x; b < B; b += kPT) h[b] = 0;
@@ -927,7 +943,7 @@ __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, 
       const uint32_t w[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        if (w[q] < pnr) atomicAdd(&h[bucket_of(w[q], dv, bshift)], 1u);
+        if (w[q] < pnr) atomicAdd(&h[bucket_m(w[q], dv)], 1u);
         else bad++;
       }
     }
@@ -937,12 +953,12 @@ __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, 
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      if (w[q] < pnr) atomicAdd(&h[bucket_of(w[q], dv, bshift)], 1u);
+      if (w[q] < pnr) atomicAdd(&h[bucket_m(w[q], dv)], 1u);
       else bad++;
     }
   }
   for (uint64_t j = e4 * 4 + threadIdx.x; j < e; j += kPT) {  // the stream's last < 4 words
-    if (s[j] < pnr) atomicAdd(&h[bucket_of(s[j], dv, bshift)], 1u);
+    if (s[j] < pnr) atomicAdd(&h[bucket_m(s[j], dv)], 1u);
     else bad++;
   }
   count_invalid(bad, d_n_invalid);
@@ -1016,7 +1032,7 @@ __device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t
 // sample's bucket and reads its destination base dst[b] = cursor - tile offset.
 template <int NT>
 __global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
-                                                  uint32_t pnr, Div dv, uint32_t bshift, uint32_t B,
+                                                  uint32_t pnr, BDiv dv, uint32_t B,
                                                   const uint32_t* __restrict__ off,
                                                   const unsigned long long* __restrict__ bstart,
                                                   uint32_t* __restrict__ out) {
@@ -1042,7 +1058,10 @@ __global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s,
     for (int q = 0; q < 8; q++) w[q] = nw[q];
     if (t0 + kTile < e) load8(s, t0 + kTile, e, nw);  // next tile in flight during this one
 #pragma unroll
-    for (int q = 0; q < 8; q++) bk[q] = w[q] < pnr ? bucket_of(w[q], dv, bshift) : 0xffffffffu;
+    for (int q = 0; q < 8; q++) {  // branch-free: the bucket of every word, then the validity select
+      const uint32_t b = bucket_m(w[q], dv);
+      bk[q] = w[q] < pnr ? b : 0xffffffffu;
+    }
     // ranks within the tile's buckets: one shared atomic per sample, and one per warp when the
     // whole warp holds a single bucket (trace order)
     const uint32_t bk_lane0 = __shfl_sync(0xffffffffu, bk[0], 0);  // outside any condition (all lanes)
@@ -1116,7 +1135,7 @@ __global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s,
     const uint32_t nv = nv_sh;
     for (uint32_t p = threadIdx.x; p < nv; p += NT) {  // the bucket is recomputed (ALU, not smem)
       const uint32_t x = stage[p];
-      out[dst[bucket_of(x, dv, bshift)] + p] = x;
+      out[dst[bucket_m(x, dv)] + p] = x;
     }
   }
 }
@@ -1241,12 +1260,13 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   unsigned long long* bstart = reinterpret_cast<unsigned long long*>(p);
   p += ((B + 1) * 8 + 255) / 256 * 256;
   uint32_t* ps = reinterpret_cast<uint32_t*>(p);
-  k_pcount<<<(unsigned)nch, kPT, 0, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, d_n_invalid);
+  const BDiv bd = make_bdiv(nr, bshift);
+  k_pcount<<<(unsigned)nch, kPT, 0, st>>>(d_words, n, chunk, P * nr, bd, B, cnt, d_n_invalid);
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaFuncSetAttribute(k_pscatter<kPST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSTile * 4)));
-  k_pscatter<kPST><<<(unsigned)nch, kPST, kSTile * 4, st>>>(d_words, n, chunk, P * nr, dv, bshift, B, cnt, bstart, ps);
+  k_pscatter<kPST><<<(unsigned)nch, kPST, kSTile * 4, st>>>(d_words, n, chunk, P * nr, bd, B, cnt, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4

@@ -126,6 +126,7 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   free_loaded(c);
   c->n_kernels = (uint32_t)ks.size();
   c->n_instr = P;
+  c->win = P >= kBigModule ? kWinBig : kWinSmall;
   c->names.clear();
   c->kd_h.assign(ks.size(), KDesc{});
   c->wd_h.clear();
@@ -148,8 +149,8 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     K.n = (uint32_t)pk.recs.size();
     K.param_base = pk.param_base | (std::min<uint32_t>(pk.nregs, 255u) << 16);
     K.win0 = (uint32_t)c->wd_h.size();
-    for (uint32_t s = 0; s < K.n; s += kWin) {
-      WDesc W{(uint32_t)k, slot + s, std::min(kWin, K.n - s), 0};
+    for (uint32_t s = 0; s < K.n; s += c->win) {
+      WDesc W{(uint32_t)k, slot + s, std::min(c->win, K.n - s), 0};
       uint32_t nc = 0;
       for (uint32_t i = 0; i < W.len; i++) {  // candidates per window: static opcode classes
         const Rec& r = pk.recs[s + i];

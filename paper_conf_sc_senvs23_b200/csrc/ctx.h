@@ -11,10 +11,11 @@
 
 namespace gs {
 
-#ifndef GS_KWIN
-#define GS_KWIN 1024
-#endif
-constexpr uint32_t kWin = GS_KWIN;  // instructions per detection window (never crosses a kernel)
+// instructions per detection window (never crosses a kernel): 256, or 1024 for modules of at least
+// kBigModule instructions (fewer, longer windows: smaller carry tables; a small module needs the
+// short windows to fill the GPU with warps)
+constexpr uint32_t kWinSmall = 256, kWinBig = 1024;
+constexpr uint64_t kBigModule = 16ull << 20;
 
 // A device buffer that only grows; freed with the context.
 struct DevBuf {
@@ -68,6 +69,7 @@ struct gs_ctx {
   uint32_t n_lgroups = 0;             // source-line groups (kernel, file, line), 0 without line info
   std::vector<uint32_t> use_off_h;     // register-pressure inputs (R36), uploaded on first use:
   std::vector<uint8_t> use_reg_h;      //   GPR uses per slot (CSR, global offsets), branch targets
+  uint32_t win = gs::kWinSmall;        // detection window length of the loaded module
   std::vector<int32_t> tgt_h;          //   (kernel-local index, -1 none, -2 - x indirect-branch list x)
   std::vector<uint32_t> xoff_h;        // indirect-branch successor lists (R38i, CSR over x)
   std::vector<int32_t> xtgt_h;

@@ -1,6 +1,6 @@
 // detect.cu — SASS detection on the GPU (SURVEY §8a rows a-2 .. a-7; paper §4).
 //
-// Data layout: records (16 B each, one uint4 per lane) are processed in windows of kWin
+// Data layout: records (16 B each, one uint4 per lane) are processed in windows of c->win
 // instructions that never cross a kernel. One warp owns one window.
 //
 //   k_summary  per window: last writer of every register inside the window (R5), loop events of
@@ -80,7 +80,8 @@ __device__ __forceinline__ unsigned long long group_key(uint32_t base, uint32_t 
 __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
                                                          uint32_t* __restrict__ tab, int32_t* ldiff, int32_t* wsum,
-                                                         uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst) {
+                                                         uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst,
+                                                         uint32_t win) {
   __shared__ uint32_t last[kWarps][kNumRegs];
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
@@ -119,13 +120,13 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
     if (valid && op == OP_BRA && (r_flags(r) & F_BRA_OK)) {
       const uint32_t t = (uint32_t)r_imm(r);           // loop [t, b] in kernel-local indices
       atomicAdd(ldiff + K.first + t, 1);
-      atomicAdd(wsum + K.win0 + t / kWin, 1);
-      atomicAdd(wev + K.win0 + t / kWin, 1u);
+      atomicAdd(wsum + K.win0 + t / win, 1);
+      atomicAdd(wev + K.win0 + t / win, 1u);
       const uint32_t b1 = (uint32_t)(g - K.first) + 1;
       if (b1 < K.n) {
         atomicAdd(ldiff + K.first + b1, -1);
-        atomicAdd(wsum + K.win0 + b1 / kWin, -1);
-        atomicAdd(wev + K.win0 + b1 / kWin, 1u);
+        atomicAdd(wsum + K.win0 + b1 / win, -1);
+        atomicAdd(wev + K.win0 + b1 / win, 1u);
       }
     }
     if (valid) {
@@ -155,11 +156,11 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
 
 // ------------------------------------------------------------------------------------------ B
 __global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, uint32_t* tab,
-                        const int32_t* __restrict__ wsum, int32_t* wloop) {
+                        const int32_t* __restrict__ wsum, int32_t* wloop, uint32_t win) {
   const uint32_t k = kb + blockIdx.x;
   if (k >= ke) return;
   const KDesc K = kd[k];
-  const uint32_t nwk = (K.n + kWin - 1) / kWin;
+  const uint32_t nwk = (K.n + win - 1) / win;
   for (int r = threadIdx.x; r <= kNumRegs; r += blockDim.x) {
     if (r < kNumRegs) {
       uint32_t state = 0;
@@ -839,9 +840,9 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       GS_CUDA(c, cudaMemsetAsync(c->d_wev + w0, 0, (uint64_t)nw * 4, st));
       const uint32_t grid = (nw + kWarps - 1) / kWarps;
       k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
-                                             c->d_wev, c->d_narith, c->d_kstats); count_launch();
+                                             c->d_wev, c->d_narith, c->d_kstats, c->win); count_launch();
       GS_CUDA(c, cudaGetLastError());
-      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop); count_launch();
+      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win); count_launch();
       GS_CUDA(c, cudaGetLastError());
       // candidate arrays are indexed relative to c0
       k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,

@@ -645,3 +645,35 @@ def test_cupti_records_equal_count_table():
     for slot, r, w in buf.foreign_crc_bins:
         want[(slot, r)] = want.get((slot, r), 0) + w
     assert c0.H == want and c0.N["invalid"] == str(buf.invalid_any)
+
+
+def test_join_and_rank_closed_form_multi_kernel():
+    """The same closed form on a module of several kernels (C2: three kernels; the cubin's five
+    kernels): every R line's rel/tot/ktot come from the count table rows of the site's own slot and
+    the sum over ITS kernel's slots (first_slot offsets), and the order is Python's sort of the
+    R20 key — pins the kernel totals beyond the first kernel and the slot mapping of later kernels."""
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C2")
+    tab = gsm.table_class_weighted(s.cls, 500_000, key=21)
+    raw = gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=21).raw()
+    c = Canon(orc.run(s.text, samples=raw))
+    first = np.asarray(s.first_slot, dtype=np.int64)
+    n = np.asarray(s.n_instr, dtype=np.int64)
+    ktot = [int(tab[first[k]:first[k] + n[k]].sum()) for k in range(len(n))]
+    assert len(set(ktot)) == len(ktot) and len(ktot) == 3
+    rel_sets = {"VEC": [6], "SPILL": [5, 6], "SHMEM": [6], "GATOM": [5], "RO": [6], "TEX": [6, 16],
+                "CONV": list(range(32))}
+    order = ["VEC", "SPILL", "SHMEM", "GATOM", "RO", "TEX", "CONV"]
+    rows = []
+    for st in c.sites():
+        h = tab[first[st["k"]] + st["idx"]]
+        rows.append((-int(h[rel_sets[st["rule"]]].sum()), -int(h.sum()), st["k"], st["idx"], order.index(st["rule"])))
+    rows.sort()
+    got = [r.split() for r in c.R]
+    assert len(got) == len(rows) and {w[2] for w in rows} == {0, 1, 2}
+    for q, (g, w) in enumerate(zip(got, rows)):
+        assert g[:5] == ["R", str(q), str(w[2]), str(w[3]), order[w[4]]]
+        assert g[5:8] == [f"rel={-w[0]}", f"tot={-w[1]}", f"ktot={ktot[w[2]]}"]
+        h = tab[first[w[2]] + w[3]][:19]
+        assert g[8] == "h=" + ",".join(str(int(x)) for x in h)

@@ -816,7 +816,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 // (per-CTA timeline, GS_DIAG=11). kPlanProbes probe samples estimate where the windows change;
 // the queue words are zeroed here too.
 #ifndef GS_SWITCH_COST
-#define GS_SWITCH_COST 96000
+#define GS_SWITCH_COST 160000
 #endif
 constexpr uint32_t kPlanProbes = 4096;
 __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, uint64_t n, uint32_t pnr, Div dv,
@@ -825,6 +825,13 @@ __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, u
   __shared__ unsigned long long wsum[32];
   const uint64_t n4 = n / 4;
   const uint32_t t = threadIdx.x;
+#ifdef GS_PLAN_UNIFORM  // diagnostic: equal-sample chunks (the cost of the probes)
+  for (uint32_t c = t; c <= chunks; c += blockDim.x) {
+    if (c < chunks) q[c] = 0ull;
+    q[chunks + c] = (uint64_t)c * n4 / chunks;
+  }
+  return;
+#endif
   constexpr uint32_t kPer = kPlanProbes / 1024;
   // probe p sits at uint4 position pos(p) = p * n4 / NP; interval p = [pos(p), pos(p + 1))
   uint32_t win[kPer + 1];

@@ -476,9 +476,20 @@ static_assert(kNct * 4 * kVec < 0x8000, "16-bit counters: too many increments in
 
 // the rare part of one batch of nv uint4 at s4[i + u * kNct], re-read from L1/L2: outside the
 // window (deferred / invalid), or a 16-bit half that needs draining. Returns the invalid count.
+// Hot words of an item (skew, e.g. C5: 90% of the samples on 10 PCs): samples equal to one of them
+// are counted in registers and added to H once per item, instead of hammering one shared counter
+// with same-address atomics (the north star's warp aggregation, for the case where it pays).
+struct Hot {
+  uint32_t w[3];  // the first n are hot words (every 32-bit value is a possible sample word: no sentinel)
+  uint32_t n;
+};
+__device__ __forceinline__ bool is_hot(uint32_t x, const Hot& h) {
+  return (h.n > 0 && x == h.w[0]) || (h.n > 1 && x == h.w[1]) || (h.n > 2 && x == h.w[2]);
+}
+
 template <bool P16, uint32_t NCT>
 __device__ __noinline__ uint32_t rare_w(const uint4* __restrict__ s4, uint64_t i, uint32_t nv, Win W, uint32_t* tab,
-                                        uint32_t flag, uint32_t am, const Spill* sS) {
+                                        uint32_t flag, uint32_t am, const Spill* sS, Hot hot) {
   const Spill S = *sS;
   uint32_t bad = 0;
   for (uint32_t u = 0; u < nv; u++) {
@@ -486,9 +497,10 @@ __device__ __noinline__ uint32_t rare_w(const uint4* __restrict__ s4, uint64_t i
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      const uint32_t off = w[q] - W.wb;
-      out_of_window<OUT_DEFER>(am, off >= W.lim, w[q], S, bad);
-      if (P16 && flag && off < W.lim && ((tab[off >> 1] >> ((off & 1u) << 4)) & 0x8000u))
+      const uint32_t off = is_hot(w[q], hot) ? 0u : w[q] - W.wb;  // hot words: counted in registers
+      const bool hw = is_hot(w[q], hot);
+      out_of_window<OUT_DEFER>(am, !hw && off >= W.lim, w[q], S, bad);
+      if (P16 && flag && !hw && off < W.lim && ((tab[off >> 1] >> ((off & 1u) << 4)) & 0x8000u))
         drain16(tab, off >> 1, (off & 1u) << 4, w[q], S.dv, S.H);
     }
   }
@@ -514,10 +526,45 @@ __device__ __forceinline__ uint32_t hot_w(const uint32_t (&w)[N], Win W, uint32_
   return flag;
 }
 
-template <bool P16, uint32_t NCT = kNct>
+// shared-memory atomic add executed only when p (a predicated ATOMS, no branch); 0 otherwise
+__device__ __forceinline__ uint32_t atoms_add_if(bool p, uint32_t* addr, uint32_t v) {
+  uint32_t r = 0;
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.u32 q, %3, 0;\n @q atom.shared.add.u32 %0, [%1], %2;\n}"
+      : "+r"(r)
+      : "r"((uint32_t)__cvta_generic_to_shared(addr)), "r"(v), "r"(p ? 1u : 0u)
+      : "memory");
+  return r;
+}
+
+// the fast path with hot words: a hot sample adds to its register counter and issues no atomic
+template <bool P16, int N>
+__device__ __forceinline__ uint32_t hot_w_skew(const uint32_t (&w)[N], Win W, uint32_t* tab, uint32_t spare,
+                                               const Hot& h, uint32_t& c) {
+  uint32_t flag = 0;
+#pragma unroll
+  for (int q = 0; q < N; q++) {
+    const bool m0 = h.n > 0 && w[q] == h.w[0], m1 = h.n > 1 && w[q] == h.w[1], m2 = h.n > 2 && w[q] == h.w[2];
+    c += (m0 ? 1u : 0u) + (m1 ? 1u << 10 : 0u) + (m2 ? 1u << 20 : 0u);  // three 10-bit counters, one register
+    const bool cold = !(m0 | m1 | m2);
+    const uint32_t off = w[q] - W.wb;
+    const bool in = off < W.lim;
+    if (P16) {
+      const uint32_t inc = 1u << ((off & 1u) << 4);
+      flag |= atoms_add_if(cold, tab + (in ? off >> 1 : spare), in ? inc : 2u) & (in ? inc << 15 : 0xffffffffu);
+    } else {
+      atoms_add_if(cold, tab + (in ? off : spare), 1u);
+      flag |= (cold && !in) ? 1u : 0u;
+    }
+  }
+  return flag;
+}
+
+template <bool P16, uint32_t NCT = kNct, bool HOT = false>
 __device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, uint64_t i0, uint64_t i1, uint32_t ct,
-                                                 Win W, uint32_t* tab, uint32_t spare, const Spill* sS) {
-  uint32_t bad = 0;
+                                                 Win W, uint32_t* tab, uint32_t spare, const Spill* sS,
+                                                 Hot hot = Hot{{0u, 0u, 0u}, 0u}) {
+  uint32_t bad = 0, c = 0;  // HOT: packed counters of the 3 hot words (< 1024 per item and thread)
   uint64_t i = i0 + ct;
   for (; i + (kVec - 1) * NCT < i1; i += kVec * NCT) {
     uint32_t w[4 * kVec];
@@ -526,16 +573,24 @@ __device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, u
       const uint4 v = __ldg(s4 + i + u * NCT);
       w[4 * u] = v.x; w[4 * u + 1] = v.y; w[4 * u + 2] = v.z; w[4 * u + 3] = v.w;
     }
-    const uint32_t flag = hot_w<P16>(w, W, tab, spare);
+    const uint32_t flag = HOT ? hot_w_skew<P16>(w, W, tab, spare, hot, c) : hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, kVec, W, tab, flag, am, sS);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, kVec, W, tab, flag, am, sS, hot);
   }
   for (; i < i1; i += NCT) {
     const uint4 v = __ldg(s4 + i);
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-    const uint32_t flag = hot_w<P16>(w, W, tab, spare);
+    const uint32_t flag = HOT ? hot_w_skew<P16>(w, W, tab, spare, hot, c) : hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, 1, W, tab, flag, am, sS);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, 1, W, tab, flag, am, sS, hot);
+  }
+  if (HOT) {  // the item's hot counts, one L2 reduction per hot word and thread
+    const Spill S = *sS;
+#pragma unroll
+    for (int j = 0; j < 3; j++) {
+      const uint32_t cj = (c >> (10 * j)) & 1023u;
+      if (cj && (uint32_t)j < hot.n) atomicAdd(S.H + hidx(hot.w[j], S.dv), (int32_t)cj);
+    }
   }
   return bad;
 }
@@ -621,7 +676,12 @@ struct Item {
   uint64_t a4, b4;  // uint4 range of the stream
   uint32_t ws;      // window (first slot) for the range
   uint32_t last;    // 1: no more work
+  Hot hot;          // hot words of the tile (hot.n of them)
 };
+// a probe word seen in at least kHotMin of the tile's 32 probes is a hot word of the tile
+#ifndef GS_HOT_MIN
+#define GS_HOT_MIN 3
+#endif
 
 // One persistent CTA per SM. Warp 0 (producer) grabs tiles from the work-stealing queue, picks
 // each tile's window(s) from 32 probe samples and publishes (range, window) items through an
@@ -671,11 +731,12 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (threadIdx.x < 32) {  // ------------------------------------------------ producer
     uint32_t pws = kNoWindow, j = 0;
+    Hot hot{{0u, 0u, 0u}, 0u};
     const auto publish = [&](uint64_t a4, uint64_t b4, uint32_t ws, uint32_t last) {
       const uint32_t k = j % kItems;
       if (lane == 0) {
         mbar_wait_backoff(&empty[k], ((j / kItems) & 1u) ^ 1u);
-        items[k] = Item{a4, b4, ws, last};
+        items[k] = Item{a4, b4, ws, last, hot};
         mbar_arrive(&full[k]);
       }
       __syncwarp();
@@ -692,6 +753,21 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t slot = ok ? divq(w, dv) : 0xffffffffu;
       const uint32_t k = ok ? kernel_of(slot, kd, nk) : 0xffffffffu;
       const uint32_t okm = __ballot_sync(0xffffffffu, ok);
+      {  // hot words: the most frequent valid probe words seen >= GS_HOT_MIN times (at most 3)
+        const uint32_t mm = __match_any_sync(0xffffffffu, w);
+        uint32_t cnt = (ok && (uint32_t)(__ffs(mm) - 1) == lane) ? (uint32_t)__popc(mm) : 0u;
+        hot.n = 0;
+#pragma unroll
+        for (int q = 0; q < 3; q++) {
+          const uint32_t key = cnt >= GS_HOT_MIN ? (cnt << 5) | lane : 0u;
+          const uint32_t best = __reduce_max_sync(0xffffffffu, key);
+          const uint32_t bl = best & 31u;
+          const uint32_t bw = __shfl_sync(0xffffffffu, w, bl);
+          hot.w[q] = bw;
+          hot.n += best ? 1u : 0u;  // keys are taken in decreasing order: the hot words come first
+          if (best && lane == bl) cnt = 0;
+        }
+      }
       const uint32_t k0 = __reduce_min_sync(0xffffffffu, k), k1 = __reduce_max_sync(0xffffffffu, ok ? k : 0u);
       const uint32_t m0 = __ballot_sync(0xffffffffu, ok && k == k0), m1 = __ballot_sync(0xffffffffu, ok && k == k1);
       // one window for the probes of mask pm, given the window before them
@@ -776,7 +852,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (ct == 0) sh_S = S;
       bar_counters();
     }
-    GS_T(d_count, bad += count_span_w<P16>(s4, it.a4, it.b4, ct, W, tab, spare, &sh_S));
+    if (it.hot.n) {
+      GS_T(d_count, bad += count_span_w<P16, kNct, true>(s4, it.a4, it.b4, ct, W, tab, spare, &sh_S, it.hot));
+    } else {
+      GS_T(d_count, bad += count_span_w<P16>(s4, it.a4, it.b4, ct, W, tab, spare, &sh_S));
+    }
 #if defined(GS_DIAG) && GS_DIAG == 11
     d_items++;
     d_words += 4 * (it.b4 - it.a4);

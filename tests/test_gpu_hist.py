@@ -135,3 +135,51 @@ def test_small_and_ragged_streams_all_modes(gs, n, nr):
             assert int(ninv.item()) == bad, (mode, row)
             assert np.array_equal(got, want_c), (mode, row, n)
             ctx.close()
+
+
+def test_c5_trace_order_hot_words(gs):
+    """C5 in trace order (90% of 200M samples on 10 PCs, grouped by kernel): tiles whose probes
+    repeat a word count those hot words in registers and add them to H once per item (WINDOW); the
+    histogram equals the count table in every strategy, both counter widths and row layouts."""
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass("C5")
+    hot = [int(f) + 40 for f in s.first_slot[:10]]
+    tab = gsm.table_c5(s.cls, hot, 200_000_000, key=0x6E5C0005)
+    tr = gsm.Trace(tab, s.first_slot, s.n_instr, order="trace", seed=2)
+    _check(gs, s, tr, [0, 3, 4])
+
+
+def test_hot_words_with_invalid_and_foreign_words(gs):
+    """Hot-word edge cases: a tile whose most frequent probe word is INVALID (never hot: it must
+    still be counted as invalid), hot words of another kernel than the tile's window, and the
+    word 0xFFFFFFFF itself frequent. Exact histogram and invalid count in every strategy."""
+    import torch
+    from gen import sass as gsass
+    s = gsass.config_sass("C4", scale=0.02)
+    P, R = int(sum(s.n_instr)), 19
+    n = 6_000_000
+    g = torch.Generator(device="cuda").manual_seed(5)
+    idx = torch.arange(n, device="cuda")
+    k0 = int(s.first_slot[1]) * R                       # kernel 1's first bin
+    base = torch.randint(0, int(s.n_instr[0]) * R, (n,), device="cuda", generator=g)   # kernel 0
+    words = torch.where(idx % 7 == 0, torch.full_like(base, k0 + 5), base)           # a foreign hot word
+    words = torch.where(idx % 11 == 0, torch.full_like(base, P * R + 3), words)        # a frequent invalid word
+    words = torch.where(idx % 13 == 0, torch.full_like(base, -1), words)               # 0xFFFFFFFF, frequent
+    words = words.to(torch.int32)
+    w64 = words.to(torch.int64) & 0xFFFFFFFF
+    valid = w64 < P * R
+    want_inv = int((~valid).sum().item())
+    for row in (32, 19):
+        want = torch.zeros(P * row, dtype=torch.int64, device="cuda")
+        vw = w64[valid]
+        want.index_add_(0, (vw // R) * row + vw % R, torch.ones_like(vw))
+        for mode in (0, 3, 4):
+            for bits in ((16, 32) if mode in (0, 3) else (0,)):
+                ctx = gs.Context(hist_mode=mode, hist_counter_bits=bits, hist_row=row)
+                ctx.load_sass(s.text)
+                hist, ninv = ctx.attribute_samples(words)
+                torch.cuda.synchronize()
+                assert int(ninv.item()) == want_inv, (mode, bits, row)
+                assert torch.equal(hist.to(torch.int64), want), (mode, bits, row)
+                ctx.close()

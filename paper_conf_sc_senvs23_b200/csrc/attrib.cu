@@ -900,9 +900,20 @@ __global__ void __launch_bounds__(kThreads, 1)
 #endif
 constexpr uint32_t kPlanProbes = 4096;
 __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, uint64_t n, uint32_t pnr, Div dv,
-                                               uint32_t nslots, uint32_t chunks, unsigned long long* __restrict__ q) {
+                                               uint32_t nslots, uint32_t chunks, unsigned long long* __restrict__ q,
+                                               int32_t* __restrict__ zero_h, uint64_t zero_n) {
   __shared__ unsigned long long pre[kPlanProbes];
   __shared__ unsigned long long wsum[32];
+  // the histogram's zeroing (instead of a separate memset node): every CTA zeroes a grid-strided
+  // share with 128-bit stores; CTA 0 then plans (zero_h is 16-byte aligned, zero_n words)
+  if (zero_h) {
+    uint4* h4 = reinterpret_cast<uint4*>(zero_h);
+    const uint64_t n4w = zero_n / 4;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n4w; i += (uint64_t)gridDim.x * blockDim.x)
+      h4[i] = make_uint4(0, 0, 0, 0);
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (zero_n & 3)) zero_h[n4w * 4 + threadIdx.x] = 0;
+  }
+  if (blockIdx.x != 0) return;
   const uint64_t n4 = n / 4;
   const uint32_t t = threadIdx.x;
 #ifdef GS_PLAN_UNIFORM  // diagnostic: equal-sample chunks (the cost of the probes)
@@ -1374,21 +1385,12 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   cudaStream_t st = c->stream;
   const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
   const Div dv = make_div(nr, c->cfg.hist_row);
-  if (zero_first && !accumulate) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, (uint64_t)P * c->cfg.hist_row * 4, st));
-  if (!n) return GS_OK;
+  const uint64_t hbins = (uint64_t)P * c->cfg.hist_row;
   if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
   int dev_sms = 148;
   cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
   // peel the words before the first 16-byte boundary so the main kernels use 128-bit loads
   const uint64_t head = std::min<uint64_t>(n, ((16u - (reinterpret_cast<uintptr_t>(d_words) & 15u)) & 15u) / 4u);
-  if (head) {
-    k_hist_global<<<1, 32, 0, st>>>(d_words, head, P * nr, dv, d_hist, d_n_invalid);
-    count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    d_words += head;
-    n -= head;
-    if (!n) return GS_OK;
-  }
   const uint32_t nslots32 = kTableWords / nr, nslots16 = 2 * kTableWords / nr;  // whole slots per window
   const auto ranges = [&](uint32_t ns) { return (uint32_t)std::max<uint64_t>(1, ((uint64_t)P + ns - 1) / ns); };
   uint32_t max_kn = 0;
@@ -1400,6 +1402,28 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     else mode = GS_HIST_WINDOW;
   }
   if (!bits) bits = (mode == GS_HIST_WINDOW && max_kn > nslots32) ? 16 : 32;  // whole kernels per window
+  // the histogram's zeroing: folded into k_plan for the WINDOW strategy (one launch instead of a
+  // memset node + k_plan), else a memset; the head words go in after it
+  const bool zero = zero_first && !accumulate && hbins;
+  const bool fold_zero = zero && n > head && mode == GS_HIST_WINDOW && (reinterpret_cast<uintptr_t>(d_hist) & 15u) == 0 &&
+                         (n - head) / (2ull * kMinTableWords) + 1 > 1;
+  if (zero && !fold_zero) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, hbins * 4, st));
+  const uint32_t* const d_head = d_words;
+  const auto peel = [&, d_head]() -> gs_status {
+    if (head) {
+      k_hist_global<<<1, 32, 0, st>>>(d_head, head, P * nr, dv, d_hist, d_n_invalid);
+      count_launch();
+      GS_CUDA(c, cudaGetLastError());
+    }
+    return GS_OK;
+  };
+  if (!fold_zero) {
+    const gs_status ps = peel();
+    if (ps != GS_OK) return ps;
+  }
+  d_words += head;
+  n -= head;
+  if (!n) return GS_OK;
   const uint32_t n_ranges = ranges(bits == 16 ? nslots16 : nslots32);
   if (mode == GS_HIST_PRIVATE && n_ranges > 64) mode = GS_HIST_WINDOW;
   c->last_hist_mode = (int)mode;
@@ -1446,8 +1470,13 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
     GS_CUDA(c, dev_grow(&c->d_tileq, &c->tileq_cap, 2 * chunks + 1));
     GS_CUDA(c, dev_grow(&c->d_defer, &c->defer_cap, chunks * 2 * kDeferCap));
     const uint32_t nslots = (uint32_t)std::max<uint64_t>(1, (bits == 16 ? 2ull * tw : (uint64_t)tw) / nr);
-    k_plan<<<1, 1024, 0, st>>>(d_words, n, P * nr, dv, nslots, (uint32_t)chunks, c->d_tileq);
+    k_plan<<<fold_zero ? (uint32_t)dev_sms : 1u, 1024, 0, st>>>(d_words, n, P * nr, dv, nslots, (uint32_t)chunks,
+                                                               c->d_tileq, fold_zero ? d_hist : nullptr, hbins);
     count_launch();
+    if (fold_zero) {
+      const gs_status ps = peel();
+      if (ps != GS_OK) return ps;
+    }
   }
   const auto prep = [&](auto kern) -> gs_status {
     GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

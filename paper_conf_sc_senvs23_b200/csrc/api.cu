@@ -29,6 +29,12 @@ gs_status cuda_fail(gs_ctx* c, cudaError_t e, const char* what) {
 
 namespace {
 
+uint64_t pow2_ceil(uint64_t n) {
+  uint64_t c = 1;
+  while (c < n) c <<= 1;
+  return c;
+}
+
 void free_loaded(gs_ctx* c) {
   detect_free(c);
   rank_reset_graph(c);
@@ -139,6 +145,8 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   c->xoff_h.assign(1, 0);
   c->xtgt_h.clear();
   c->n_cand = c->n_ldg = c->n_store = 0;
+  c->kh_h.assign(ks.size(), KHash{});
+  c->grp.gtot = c->grp.rtot = 0;
   std::vector<Rec> recs;
   recs.reserve(P);
   uint32_t slot = 0;
@@ -149,6 +157,7 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     K.n = (uint32_t)pk.recs.size();
     K.param_base = pk.param_base | (std::min<uint32_t>(pk.nregs, 255u) << 16);
     K.win0 = (uint32_t)c->wd_h.size();
+    const uint64_t ldg0 = c->n_ldg, st0 = c->n_store;
     for (uint32_t s = 0; s < K.n; s += c->win) {
       WDesc W{(uint32_t)k, slot + s, std::min(c->win, K.n - s), 0};
       uint32_t nc = 0;
@@ -162,6 +171,16 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
       c->cbase_h.push_back((uint32_t)c->n_cand);
       c->n_cand += nc;
       c->wd_h.push_back(W);
+    }
+    {  // the kernel's hash-table regions: a power of two >= 2x its global loads / stores
+      KHash& H = c->kh_h[k];
+      const uint64_t gcap = pow2_ceil(2 * (c->n_ldg - ldg0) + 2), rcap = pow2_ceil(2 * (c->n_store - st0) + 2);
+      H.gofs = c->grp.gtot;
+      H.rofs = c->grp.rtot;
+      H.gmask = (uint32_t)(gcap - 1);
+      H.rmask = (uint32_t)(rcap - 1);
+      c->grp.gtot += gcap;
+      c->grp.rtot += rcap;
     }
     slot += K.n;
     recs.insert(recs.end(), pk.recs.begin(), pk.recs.end());

@@ -26,27 +26,40 @@ struct DevBuf {
 // Candidate arrays: one entry per traced memory instruction or conversion.
 struct CandArrays {
   uint32_t *idx = nullptr, *kernel = nullptr, *base_rd = nullptr, *data_rd = nullptr, *tv = nullptr,
-           *grp = nullptr, *nsite = nullptr, *soff = nullptr;
+           *grp = nullptr,
+           *cont = nullptr;  // a trace left its window: the RD value to resume from (tk = kTCont, tv = register)
   uint8_t *ld = nullptr, *tk = nullptr, *depth = nullptr, *flags = nullptr;
+  Rec* rec = nullptr;  // the candidate's instruction record (later passes read it coalesced, not gathered)
+  uint32_t* chain4 = nullptr;  // the first kChain4 chain elements of the trace (k_write re-traces longer ones)
   unsigned long long* choff = nullptr;  // chain offsets (exclusive scan of chain lengths)
 };
 
-struct GroupTable {  // key-group statistics of global loads (R3)
-  uint32_t cap = 0;  // power of two
-  unsigned long long* key = nullptr;
-  uint32_t *nload = nullptr, *n32 = nullptr, *nall = nullptr, *or3 = nullptr, *and3 = nullptr;
-  int32_t *mn = nullptr, *mx = nullptr;
+// Key-group statistics of global loads (R3), their distinct offsets, and the store roots (R8),
+// as open-addressing hash tables partitioned by kernel: kernel k owns a power-of-two region of each
+// table sized to twice its global loads / stores. Candidates are traced in instruction order, so
+// the regions the resident threads update at any time are a few kernels' worth and stay in L2
+// (one table over the whole module sent every update to a random DRAM sector).
+struct KHash {
+  unsigned long long gofs, rofs;  // first entry of the kernel's group / root region
+  uint32_t gmask, rmask;          // region size - 1 (power of two)
+  uint32_t pad[2];
 };
-
-struct OffsetSet {  // distinct (group, offset) pairs
-  uint32_t cap = 0;
-  unsigned long long* key = nullptr;
-  uint32_t* flags = nullptr;
+struct GEnt {  // one 32-byte sector per group
+  unsigned long long key;
+  uint32_t nload, n32, nall;
+  int32_t mn, mx;
+  uint32_t bits;  // bits 0-1: OR of (offset & 3); bits 2-3: AND of (offset & 3)
 };
-
-struct RootSet {  // store roots per kernel (R8)
-  uint32_t cap = 0;
-  unsigned long long* key = nullptr;
+struct OEnt {  // a (group slot, offset) pair; flags: 1 = seen as a 32-bit load, 2 = seen
+  unsigned long long key;
+  uint32_t flags, pad;
+};
+struct GroupTable {
+  uint64_t gtot = 0, rtot = 0;  // entries of the group / offset tables and of the root table
+  GEnt* g = nullptr;
+  OEnt* o = nullptr;            // the offset table shares the group table's regions
+  unsigned long long* r = nullptr;
+  KHash* kh = nullptr;
 };
 
 }  // namespace gs
@@ -100,8 +113,7 @@ struct gs_ctx {
   uint32_t* d_narith = nullptr; // n_arith per global load (sparse)
   gs::CandArrays cand;
   gs::GroupTable grp;
-  gs::OffsetSet oset;
-  gs::RootSet roots;
+  std::vector<gs::KHash> kh_h;
   gs_kernel_stats* d_kstats = nullptr;
   std::vector<gs_kernel_stats> kstats_h;
   void* d_scan_tmp = nullptr;

@@ -38,6 +38,13 @@ __device__ __forceinline__ Rec ld_rec(const Rec* r, uint64_t i) {
   o.w0 = v.x; o.w1 = v.y; o.w2 = v.z; o.w3 = (int32_t)v.w;
   return o;
 }
+// a record written earlier by the same kernel (not through the read-only path)
+__device__ __forceinline__ Rec ld_rec_rw(const Rec* r, uint64_t i) {
+  const uint4 v = reinterpret_cast<const uint4*>(r)[i];
+  Rec o;
+  o.w0 = v.x; o.w1 = v.y; o.w2 = v.z; o.w3 = (int32_t)v.w;
+  return o;
+}
 __device__ __forceinline__ uint32_t reg_cap(uint32_t dst) { return dst < 256 ? 254u : 318u; }
 // The opcode-class table in shared memory: op_class() is a switch that compiles to a branch tree,
 // which a warp of mixed opcodes walks divergently for every record; one LDS replaces it.
@@ -49,21 +56,24 @@ __device__ __forceinline__ uint32_t hash64(unsigned long long k) {
   k ^= k >> 33; k *= 0xff51afd7ed558ccdull; k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull; k ^= k >> 33;
   return (uint32_t)k;
 }
-__device__ uint32_t hinsert(unsigned long long* keys, uint32_t cap, unsigned long long k) {
-  uint32_t s = hash64(k) & (cap - 1);
+// Open addressing inside one kernel's region [base, base + mask + 1) of a table whose entries are
+// `stride` 8-byte words apart (the key is the entry's first word); returns the region-relative slot.
+template <int kStride>
+__device__ uint32_t hinsert(unsigned long long* tab, uint32_t mask, unsigned long long k) {
+  uint32_t s = hash64(k) & mask;
   for (;;) {
-    unsigned long long prev = atomicCAS(keys + s, kEmpty, k);
+    unsigned long long prev = atomicCAS(tab + (uint64_t)s * kStride, kEmpty, k);
     if (prev == kEmpty || prev == k) return s;
-    s = (s + 1) & (cap - 1);
+    s = (s + 1) & mask;
   }
 }
-__device__ bool hcontains(const unsigned long long* keys, uint32_t cap, unsigned long long k) {
-  uint32_t s = hash64(k) & (cap - 1);
+__device__ bool hcontains(const unsigned long long* keys, uint32_t mask, unsigned long long k) {
+  uint32_t s = hash64(k) & mask;
   for (;;) {
     unsigned long long v = keys[s];
     if (v == k) return true;
     if (v == kEmpty) return false;
-    s = (s + 1) & (cap - 1);
+    s = (s + 1) & mask;
   }
 }
 __device__ __forceinline__ unsigned long long root_key(uint32_t kernel, uint32_t tk, uint32_t tv) {
@@ -111,10 +121,12 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
     const uint32_t op = r_op(r), cls = s_cls[op], dst = r_dst(r), dw = r_dstw(r), dst2 = r_dst2(r);
     if (valid && dw && reg_live(dst)) {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
-      const uint32_t cap = reg_cap(dst);
-      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicMax(&last[warp][dst + q], v);
-      if (reg_live(dst2))  // second quad of a 256-bit load (R38a)
-        for (uint32_t q = 0; q < dw && dst2 + q <= reg_cap(dst2); q++) atomicMax(&last[warp][dst2 + q], v);
+      const uint32_t nq = min(dw, reg_cap(dst) + 1 - dst);
+      for (uint32_t q = 0; q < nq; q++) atomicMax(&last[warp][dst + q], v);
+      if (reg_live(dst2)) {  // second quad of a 256-bit load (R38a)
+        const uint32_t nq2 = min(dw, reg_cap(dst2) + 1 - dst2);
+        for (uint32_t q = 0; q < nq2; q++) atomicMax(&last[warp][dst2 + q], v);
+      }
     }
     if (valid && op == OP_LDG) narith[g] = 0;
     if (valid && op == OP_BRA && (r_flags(r) & F_BRA_OK)) {
@@ -161,8 +173,8 @@ __global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, 
   if (k >= ke) return;
   const KDesc K = kd[k];
   const uint32_t nwk = (K.n + win - 1) / win;
-  for (int r = threadIdx.x; r <= kNumRegs; r += blockDim.x) {
-    if (r < kNumRegs) {
+  for (int r = threadIdx.x; r < kNumRegs; r += blockDim.x) {
+    {
       uint32_t state = 0;
       constexpr uint32_t kB = 8;  // window summaries loaded per batch
       for (uint32_t j0 = 0; j0 < nwk; j0 += kB) {
@@ -176,31 +188,109 @@ __global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, 
           if (v[u]) state = v[u];
         }
       }
-    } else {
-      int32_t acc = 0;
-      for (uint32_t j = 0; j < nwk; j++) {
-        wloop[K.win0 + j] = acc;
-        acc += wsum[K.win0 + j];
+    }
+  }
+  if (threadIdx.x >= kNumRegs && threadIdx.x < kNumRegs + 32) {  // loop-depth carry-in: warp scan
+    const int lane = threadIdx.x & 31;
+    int32_t acc = 0;
+    for (uint32_t j0 = 0; j0 < nwk; j0 += 32) {
+      const uint32_t j = j0 + lane;
+      int32_t x = j < nwk ? wsum[K.win0 + j] : 0;
+      int32_t inc = x;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
       }
+      if (j < nwk) wloop[K.win0 + j] = acc + inc - x;
+      acc += __shfl_sync(0xffffffffu, inc, 31);
     }
   }
 }
 
+// ------------------------------------------------------------------------------------------ D0
+struct TraceOut {
+  uint32_t tk, tv, depth, cont;
+};
+constexpr uint32_t kTCont = 0xFEu;
+constexpr uint32_t kChain4 = 4;  // chain elements kept per candidate  // internal term kind: the trace continues before `lo` (resumed later)
+
+// Bounded backward trace (R7) from the state (register r, its RD value v, steps taken):
+// each step j = v - 1 is emitted (kernel-local) and classified; a step that would read an instruction
+// below `lo` (an earlier window, whose RDs another warp may still be resolving) stops with
+// tk = kTCont, tv = r, cont = v, to be resumed from exactly that state.
+template <typename Emit>
+__device__ TraceOut chase_from(const Rec* __restrict__ rec, const uint32_t* ptrrd, const KDesc& K, uint32_t r,
+                               uint32_t v, uint32_t depth, uint32_t D, uint64_t lo,
+                               const uint16_t* __restrict__ cls_tab, Emit emit) {
+  TraceOut o{GS_T_IMM, 0, 0, 0};
+  for (;;) {
+    if (depth == D) { o.tk = GS_T_TRUNC; break; }
+    if (v == 0) { o.tk = GS_T_ENTRY; o.tv = r; break; }
+    const uint32_t j = v - 1;
+    if (j < lo) { o.tk = kTCont; o.tv = r; o.cont = v; break; }
+    depth++;
+    emit(j - K.first);
+    const Rec rj = ld_rec(rec, j);
+    const uint32_t cj = cls_tab[r_op(rj)];
+    if (cj & C_CONSTLOAD) {
+      const int32_t off = r_imm(rj) + 4 * (int32_t)(r - r_dst(rj));
+      const uint32_t bank = r_cbank(rj);
+      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
+      break;
+    }
+    if (cj & C_SREG) { o.tk = GS_T_SREG; o.tv = j - K.first; break; }
+    if (cj & C_MEMLOAD) { o.tk = GS_T_MEMORY; o.tv = j - K.first; break; }
+    const uint32_t pk = r_pk(rj);
+    if (pk == PK_CONST) {
+      const int32_t off = r_imm(rj);
+      const uint32_t bank = r_cbank(rj);
+      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
+      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
+      break;
+    }
+    if (pk != PK_REG) { o.tk = GS_T_IMM; break; }
+    r = r_ptr(rj);
+    v = ptrrd[j];
+  }
+  o.depth = depth;
+  return o;
+}
+// the whole trace of a candidate with address base `base` and RD(base) = base_rd
+template <typename Emit>
+__device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* ptrrd, const KDesc& K, uint32_t base,
+                          uint32_t base_rd, uint32_t D, const uint16_t* __restrict__ cls_tab, Emit emit) {
+  if (!reg_live(base) || base_rd == 0xffffffffu) return TraceOut{GS_T_IMM, 0, 0, 0};
+  return chase_from(rec, ptrrd, K, base, base_rd, 0, D, 0, cls_tab, emit);
+}
+
 // ------------------------------------------------------------------------------------------ C
+// One warp per window. Per 32-instruction chunk: (1) every lane marks the registers its instruction
+// writes in the chunk's writer bitmasks M; (2) lookups RD(i, reg) = the highest earlier lane of the
+// chunk whose bit is set in M[reg], else the carried table T[reg]; (3) T[reg] = max(T[reg], v) (v
+// grows with the instruction index, so the chunk's last writer wins) and M is cleared. n_arith of
+// loads defined inside the window is counted in shared memory (16-bit halves) and added to the
+// global array once per window. At the end of the window the warp traces the window's candidates
+// while their steps stay inside the window (the RDs of earlier windows belong to other warps);
+// k_trace resumes the others.
+constexpr uint32_t kNarWords = kWinBig / 2;  // 16-bit n_arith counters per window instruction
 __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
-                                                         uint32_t w0, uint32_t nw, const uint32_t* __restrict__ tab,
-                                                         int32_t* ldiff, const int32_t* __restrict__ wloop,
+                                                         const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
+                                                         const uint32_t* __restrict__ tab, int32_t* ldiff,
+                                                         const int32_t* __restrict__ wloop,
                                                          const uint32_t* __restrict__ wev,
                                                          const uint32_t* __restrict__ cbase, uint64_t c0,
-                                                         uint32_t* __restrict__ ptrrd, uint32_t* narith, CandArrays ca) {
+                                                         uint32_t* ptrrd, uint32_t* narith, CandArrays ca, uint32_t D) {
   __shared__ uint32_t tabS[kWarps][kNumRegs];
   __shared__ uint32_t cm[kWarps][kNumRegs];
+  __shared__ uint32_t nar[kWarps][kNarWords];
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
   if (w >= w0 + nw) return;
+  const WDesc W = wd[w];
   {  // the window's carried table: all ten loads of a lane in flight before the first store
     static_assert(kNumRegs % 32 == 0, "registers per lane");
     uint32_t tv[kNumRegs / 32];
@@ -211,53 +301,55 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
       tabS[warp][lane + 32 * u] = tv[u];
       cm[warp][lane + 32 * u] = 0;
     }
+    for (uint32_t q = lane; q < (W.len + 1) / 2; q += 32) nar[warp][q] = 0;
   }
   __syncwarp();
-  const WDesc W = wd[w];
   int32_t lcarry = wloop[w];
   const bool has_ev = wev[w] != 0;
-  uint64_t cb = (uint64_t)cbase[w] - c0;
+  const uint64_t cb0 = (uint64_t)cbase[w] - c0;
+  uint64_t cb = cb0;
   const uint32_t lt = (1u << lane) - 1u;
-  const uint32_t gt = ~((2u << lane) - 1u);
   uint32_t* T = tabS[warp];
   uint32_t* M = cm[warp];
-  Rec rnext = lane < W.len ? ld_rec(rec, (uint64_t)W.start + lane) : Rec{0, 0, 0, 0};
+  uint32_t* NA = nar[warp];
+  // records (and loop events) of the next two chunks load while a chunk resolves
+  Rec rn1 = lane < W.len ? ld_rec(rec, (uint64_t)W.start + lane) : Rec{0, 0, 0, 0};
+  Rec rn2 = lane + 32 < W.len ? ld_rec(rec, (uint64_t)W.start + lane + 32) : Rec{0, 0, 0, 0};
+  int32_t dn1 = has_ev && lane < W.len ? ldiff[(uint64_t)W.start + lane] : 0;
+  int32_t dn2 = has_ev && lane + 32 < W.len ? ldiff[(uint64_t)W.start + lane + 32] : 0;
   for (uint32_t b = 0; b < W.len; b += 32) {
     const uint32_t i = b + lane;
     const bool valid = i < W.len;
     const uint64_t g = (uint64_t)W.start + i;
     const uint64_t gbase = (uint64_t)W.start + b;
-    const Rec r = rnext;  // records of the next chunk are loaded while this one is resolved
-    rnext = i + 32 < W.len ? ld_rec(rec, g + 32) : Rec{0, 0, 0, 0};
-    const uint32_t op = r_op(r), cls = s_cls[op], dst = r_dst(r), dw = r_dstw(r), fl = r_flags(r);
-    const bool writes = valid && dw && reg_live(dst);
+    const Rec r = rn1;
+    const int32_t dcur = dn1;
+    rn1 = rn2;
+    dn1 = dn2;
+    rn2 = i + 64 < W.len ? ld_rec(rec, g + 64) : Rec{0, 0, 0, 0};
+    if (has_ev) dn2 = i + 64 < W.len ? ldiff[g + 64] : 0;
+    const uint32_t op = r_op(r), cls = s_cls[op], dst = r_dst(r), fl = r_flags(r);
+    const bool writes = valid && r_dstw(r) && reg_live(dst);
+    const uint32_t nq = writes ? min(r_dstw(r), reg_cap(dst) + 1 - dst) : 0u;
     const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
-    const bool writes2 = reg_live(dst2);
-    const uint32_t cap = reg_cap(dst), cap2 = reg_cap(dst2);
-    if (writes)
-      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) atomicOr(&M[dst + q], 1u << lane);
-    if (writes2)
-      for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++) atomicOr(&M[dst2 + q], 1u << lane);
+    const uint32_t nq2 = reg_live(dst2) ? min(r_dstw(r), reg_cap(dst2) + 1 - dst2) : 0u;
+    for (uint32_t q = 0; q < nq; q++) atomicOr(&M[dst + q], 1u << lane);
+    for (uint32_t q = 0; q < nq2; q++) atomicOr(&M[dst2 + q], 1u << lane);
     const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
     __syncwarp();
     // RD value: ((def + 1) << 1) | def_is_global_load, or 0 for ENTRY
     auto RD = [&](uint32_t reg) -> uint32_t {
       const uint32_t m = M[reg] & lt;
-      if (m) {
-        const uint32_t j = 31u - __clz(m);
-        return (uint32_t)((gbase + j + 1) << 1) | ((ldgmask >> j) & 1u);
-      }
-      return T[reg];
+      const uint32_t t = T[reg];
+      const uint32_t j = 31u - __clz(m);
+      return m ? (uint32_t)((gbase + j + 1) << 1) | ((ldgmask >> j) & 1u) : t;
     };
     // loop depth: inclusive prefix of the event differences (R13); a window without loop events
     // (warp-uniform) keeps its carried depth
     int32_t depth = lcarry;
     if (has_ev) {
-      int32_t pre = 0;
-      if (valid) {
-        pre = ldiff[g];
-        if (pre) ldiff[g] = 0;  // keep the difference array zero for the next call
-      }
+      int32_t pre = dcur;
+      if (pre) ldiff[g] = 0;  // keep the difference array zero for the next call
       for (int o = 1; o < 32; o <<= 1) {
         const int32_t x = __shfl_up_sync(0xffffffffu, pre, o);
         if (lane >= o) pre += x;
@@ -272,6 +364,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
       const uint64_t c = cb + __popc(cmask & lt);
       ca.idx[c] = (uint32_t)g;
       ca.kernel[c] = W.kernel;
+      reinterpret_cast<uint4*>(ca.rec)[c] = make_uint4(r.w0, r.w1, r.w2, (uint32_t)r.w3);
       const uint32_t base = r_s0(r);
       ca.base_rd[c] = ((fl & F_HASMEM) && reg_live(base)) ? (RD(base) >> 1) : 0xffffffffu;
       const uint32_t data = r_s1(r);
@@ -280,36 +373,63 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
     }
     cb += __popc(cmask);
     if (valid && (cls & C_ARITH)) {  // n_arith (R29): count each defining load once
-      uint32_t defs[4];
-      int nd = 0;
       const uint32_t src[4] = {r_s0(r), r_s1(r), r_s2(r), r_s3(r)};
+      uint32_t d[4];
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        if (!reg_live(src[q])) continue;
-        const uint32_t v = RD(src[q]);
-        if (!(v & 1u)) continue;
-        const uint32_t d = (v >> 1) - 1u;
-        bool dup = false;
-        for (int t = 0; t < nd; t++) dup |= defs[t] == d;
-        if (!dup) defs[nd++] = d;
+        const uint32_t v = reg_live(src[q]) ? RD(src[q]) : 0u;
+        d[q] = (v & 1u) ? (v >> 1) - 1u : ~0u;  // the defining load, ~0u if none
       }
-      for (int t = 0; t < nd; t++) atomicAdd(narith + defs[t], 1u);
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        bool dup = d[q] == ~0u;
+#pragma unroll
+        for (int t = 0; t < q; t++) dup |= d[t] == d[q];
+        if (dup) continue;
+        const uint32_t off = d[q] - (uint32_t)W.start;  // loads of this window: shared counters
+        if (off < W.len) atomicAdd(NA + (off >> 1), 1u << ((off & 1u) << 4));
+        else atomicAdd(narith + d[q], 1u);
+      }
     }
     __syncwarp();
-    if (writes) {
+    {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
-      for (uint32_t q = 0; q < dw && dst + q <= cap; q++)
-        if ((M[dst + q] & gt) == 0) T[dst + q] = v;
-      if (writes2)
-        for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++)
-          if ((M[dst2 + q] & gt) == 0) T[dst2 + q] = v;
+      for (uint32_t q = 0; q < nq; q++) { atomicMax(&T[dst + q], v); M[dst + q] = 0; }
+      for (uint32_t q = 0; q < nq2; q++) { atomicMax(&T[dst2 + q], v); M[dst2 + q] = 0; }
     }
     __syncwarp();
-    if (writes)
-      for (uint32_t q = 0; q < dw && dst + q <= cap; q++) M[dst + q] = 0;
-    if (writes2)
-      for (uint32_t q = 0; q < dw && dst2 + q <= cap2; q++) M[dst2 + q] = 0;
-    __syncwarp();
+  }
+  // n_arith of the window's loads (k_summary zeroed their entries; later windows add theirs)
+  for (uint32_t i = lane; i < W.len; i += 32) {
+    const uint32_t n = (NA[i >> 1] >> ((i & 1u) << 4)) & 0xffffu;
+    if (n) atomicAdd(narith + W.start + i, n);
+  }
+  // in-window traces of the window's candidates (ptrrd of the window is complete and visible to
+  // the warp after the __syncwarp above)
+  const KDesc K = kd[W.kernel];
+  for (uint64_t c = cb0 + lane; c < cb; c += 32) {
+    const Rec ri = ld_rec_rw(ca.rec, c);
+    const uint32_t cls = s_cls[r_op(ri)];
+    TraceOut tr{GS_T_NONE, 0, 0, 0};
+    uint32_t e0 = 0, e1 = 0, e2 = 0, e3 = 0, n = 0;  // the first chain elements (k_write copies them)
+    if ((cls & C_TRACED) && (r_flags(ri) & F_HASMEM)) {
+      const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
+      tr = reg_live(base) && brd != 0xffffffffu
+               ? chase_from(rec, ptrrd, K, base, brd, 0, D, W.start, s_cls,
+                            [&](uint32_t j) {
+                              e0 = n == 0 ? j : e0;
+                              e1 = n == 1 ? j : e1;
+                              e2 = n == 2 ? j : e2;
+                              e3 = n == 3 ? j : e3;
+                              n++;
+                            })
+               : TraceOut{GS_T_IMM, 0, 0, 0};
+      reinterpret_cast<uint4*>(ca.chain4)[c] = make_uint4(e0, e1, e2, e3);
+    }
+    ca.tk[c] = (uint8_t)tr.tk;
+    ca.tv[c] = tr.tv;
+    ca.depth[c] = (uint8_t)tr.depth;
+    ca.cont[c] = tr.cont;
   }
 }
 
@@ -411,55 +531,11 @@ __global__ void k_cons_fill(uint64_t s0, uint64_t n, const uint32_t* __restrict_
 }
 
 // ------------------------------------------------------------------------------------------ D
-struct TraceOut {
-  uint32_t tk, tv, depth;
-};
-
-// Bounded backward trace (R7). `emit` receives each chain element (kernel-local).
-template <typename Emit>
-__device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* __restrict__ ptrrd, const KDesc& K,
-                          uint32_t base, uint32_t base_rd, uint32_t D, const uint16_t* __restrict__ cls_tab, Emit emit) {
-  TraceOut o{GS_T_IMM, 0, 0};
-  if (!reg_live(base) || base_rd == 0xffffffffu) return o;
-  uint32_t r = base, v = base_rd, depth = 0;
-  for (;;) {
-    if (depth == D) { o.tk = GS_T_TRUNC; break; }
-    if (v == 0) { o.tk = GS_T_ENTRY; o.tv = r; break; }
-    const uint32_t j = v - 1;
-    depth++;
-    emit(j - K.first);
-    const Rec rj = ld_rec(rec, j);
-    const uint32_t cj = cls_tab[r_op(rj)];
-    if (cj & C_CONSTLOAD) {
-      const int32_t off = r_imm(rj) + 4 * (int32_t)(r - r_dst(rj));
-      const uint32_t bank = r_cbank(rj);
-      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
-      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
-      break;
-    }
-    if (cj & C_SREG) { o.tk = GS_T_SREG; o.tv = j - K.first; break; }
-    if (cj & C_MEMLOAD) { o.tk = GS_T_MEMORY; o.tv = j - K.first; break; }
-    const uint32_t pk = r_pk(rj);
-    if (pk == PK_CONST) {
-      const int32_t off = r_imm(rj);
-      const uint32_t bank = r_cbank(rj);
-      if (bank == 0 && off >= (int32_t)kd_param_base(K)) { o.tk = GS_T_PARAM; o.tv = (uint32_t)off; }
-      else { o.tk = GS_T_CONST; o.tv = (bank << 16) | ((uint32_t)off & 0xffffu); }
-      break;
-    }
-    if (pk != PK_REG) { o.tk = GS_T_IMM; break; }
-    r = r_ptr(rj);
-    v = ptrrd[j];
-  }
-  o.depth = depth;
-  return o;
-}
-
-// Threads [0, nc) trace candidate c; threads [nc, 2nc) update the key-group statistics of
+// Threads [0, nc) finish candidate c's trace if it left its window (k_resolve traced the in-window
+// steps) and record store roots (R8); threads [nc, 2nc) update the key-group statistics of
 // candidate c - nc (two independent latency chains per candidate run on different threads).
 __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
-                        uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, OffsetSet os, RootSet rs,
-                        gs_kernel_stats* kst) {
+                        uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, gs_kernel_stats* kst) {
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
   __syncthreads();
@@ -467,46 +543,63 @@ __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ k
   if (t >= 2 * nc) return;
   const bool groups = t >= nc;
   const uint64_t c = groups ? t - nc : t;
-  const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
-  const Rec ri = ld_rec(rec, g);
+  if (!groups) {
+    uint32_t tk = ca.tk[c];
+    if (tk == GS_T_NONE) return;
+    const uint32_t kernel = ca.kernel[c];
+    const uint32_t op = r_op(ld_rec(ca.rec, c)), cls = s_cls[op];
+    uint32_t tv = ca.tv[c];
+    if (tk == kTCont) {
+      const KDesc K = kd[kernel];
+      uint32_t n = ca.depth[c];
+      const TraceOut tr = chase_from(rec, ptrrd, K, tv, ca.cont[c], n, D, 0, s_cls, [&](uint32_t j) {
+        if (n < kChain4) ca.chain4[c * kChain4 + n] = j;
+        n++;
+      });
+      tk = tr.tk;
+      tv = tr.tv;
+      ca.tk[c] = (uint8_t)tk;
+      ca.tv[c] = tv;
+      ca.depth[c] = (uint8_t)tr.depth;
+    }
+    if (cls & C_STORE) {  // store roots (R8, R27)
+      if (tk == GS_T_PARAM || tk == GS_T_ENTRY) {
+        const KHash H = gt.kh[kernel];
+        hinsert<1>(gt.r + H.rofs, H.rmask, root_key(kernel, tk, tv));
+      } else {
+        atomicAdd(&kst[kernel].n_unresolved_stores, 1u);
+      }
+    }
+    return;
+  }
+  const uint32_t kernel = ca.kernel[c];
+  const Rec ri = ld_rec(ca.rec, c);
   const uint32_t op = r_op(ri), cls = s_cls[op];
   const bool traced = (cls & C_TRACED) && (r_flags(ri) & F_HASMEM);
   const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
-  if (groups) {
-    if (!traced || op != OP_LDG) {
-      ca.grp[c] = 0xffffffffu;
-      return;
-    }
-    // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max, contiguity
-    const uint32_t slot = hinsert(gt.key, gt.cap, group_key(base, brd, kernel));
-    ca.grp[c] = slot;
-    atomicAdd(gt.nload + slot, 1u);
-    const int32_t off = r_imm(ri);
-    const bool is32 = r_aw(ri) == AW_32;
-    const uint32_t os_slot = hinsert(os.key, os.cap, ((unsigned long long)slot << 32) | (uint32_t)off);
-    const uint32_t prev = atomicOr(os.flags + os_slot, is32 ? 3u : 2u);
-    if (!(prev & 2u)) atomicAdd(gt.nall + slot, 1u);
-    if (is32 && !(prev & 1u)) {
-      atomicAdd(gt.n32 + slot, 1u);
-      atomicMin(gt.mn + slot, off);
-      atomicMax(gt.mx + slot, off);
-      atomicOr(gt.or3 + slot, (uint32_t)off & 3u);
-      atomicAnd(gt.and3 + slot, (uint32_t)off & 3u);
-    }
+  if (!traced || op != OP_LDG) {
+    ca.grp[c] = 0xffffffffu;
     return;
   }
-  if (!traced) {
-    ca.tk[c] = GS_T_NONE; ca.tv[c] = 0; ca.depth[c] = 0;
-    return;
-  }
-  const KDesc K = kd[kernel];
-  const TraceOut tr = chase(rec, ptrrd, K, base, brd, D, s_cls, [](uint32_t) {});
-  ca.tk[c] = (uint8_t)tr.tk;
-  ca.tv[c] = tr.tv;
-  ca.depth[c] = (uint8_t)tr.depth;
-  if (cls & C_STORE) {  // store roots (R8, R27)
-    if (tr.tk == GS_T_PARAM || tr.tk == GS_T_ENTRY) hinsert(rs.key, rs.cap, root_key(kernel, tr.tk, tr.tv));
-    else atomicAdd(&kst[kernel].n_unresolved_stores, 1u);
+  // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max, contiguity
+  const KHash H = gt.kh[kernel];
+  GEnt* G = gt.g + H.gofs;
+  const uint32_t slot = hinsert<4>(&G->key, H.gmask, group_key(base, brd, kernel));
+  ca.grp[c] = (uint32_t)(H.gofs + slot);
+  GEnt* e = G + slot;
+  atomicAdd(&e->nload, 1u);
+  const int32_t off = r_imm(ri);
+  const bool is32 = r_aw(ri) == AW_32;
+  OEnt* O = gt.o + H.gofs;
+  const uint32_t os_slot = hinsert<2>(&O->key, H.gmask, ((unsigned long long)slot << 32) | (uint32_t)off);
+  const uint32_t prev = atomicOr(&O[os_slot].flags, is32 ? 3u : 2u);
+  if (!(prev & 2u)) atomicAdd(&e->nall, 1u);
+  if (is32 && !(prev & 1u)) {
+    atomicAdd(&e->n32, 1u);
+    atomicMin(&e->mn, off);
+    atomicMax(&e->mx, off);
+    atomicOr(&e->bits, (uint32_t)off & 3u);
+    atomicAnd(&e->bits, ((((uint32_t)off & 3u) << 2) | 3u));
   }
 }
 
@@ -516,18 +609,22 @@ struct RuleCfg {
 };
 
 __device__ uint32_t eval_rules(const Rec& ri, uint64_t c, const CandArrays& ca, const GroupTable& gt,
-                               const RootSet& rs, const uint32_t* narith, RuleCfg rc, const uint16_t* cls_tab) {
+                               const uint32_t* narith, RuleCfg rc, const uint16_t* cls_tab) {
   const uint32_t op = r_op(ri), cls = cls_tab[op], fl = r_flags(ri);
   uint32_t f = 0;
   if (!(fl & F_HASMEM) && !(cls & C_CONV)) return 0;
   if (op == OP_LDG && (fl & F_HASMEM)) {
-    const uint32_t s = ca.grp[c];
-    const uint32_t n32 = gt.n32[s], nall = gt.nall[s], nload = gt.nload[s];
+    const GEnt& e = gt.g[ca.grp[c]];
+    const uint32_t n32 = e.n32, nall = e.nall, nload = e.nload;
     if (r_aw(ri) == AW_32 && n32 >= 2) f |= 1u << GS_VEC;                                // O6
     if (narith[ca.idx[c]] >= rc.TA && (nload >= rc.TL || ca.ld[c] >= 1)) f |= 1u << GS_SHMEM;  // O8
     const uint32_t tk = ca.tk[c];
-    const bool ro = !(fl & F_CONSTANT) && (tk == GS_T_PARAM || tk == GS_T_ENTRY) &&
-                    !hcontains(rs.key, rs.cap, root_key(ca.kernel[c], tk, ca.tv[c]));   // O10
+    bool ro = !(fl & F_CONSTANT) && (tk == GS_T_PARAM || tk == GS_T_ENTRY);
+    if (ro) {
+      const uint32_t k = ca.kernel[c];
+      const KHash H = gt.kh[k];
+      ro = !hcontains(gt.r + H.rofs, H.rmask, root_key(k, tk, ca.tv[c]));              // O10
+    }
     if (ro) f |= 1u << GS_RO;
     if (ro && nall >= 2) f |= 1u << GS_TEX;                                              // O11
   }
@@ -576,7 +673,7 @@ __device__ __forceinline__ unsigned long long site_chain(uint32_t f, uint32_t de
 }
 
 __global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint64_t nc, CandArrays ca, GroupTable gt,
-                                               RootSet rs, const uint32_t* __restrict__ narith, RuleCfg rc,
+                                               const uint32_t* __restrict__ narith, RuleCfg rc,
                                                unsigned long long* __restrict__ tsum) {
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
@@ -584,8 +681,8 @@ __global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint
   const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
   unsigned long long v = 0;
   if (c < nc) {
-    const Rec ri = ld_rec(rec, ca.idx[c]);
-    const uint32_t f = eval_rules(ri, c, ca, gt, rs, narith, rc, s_cls);
+    const Rec ri = ld_rec(ca.rec, c);
+    const uint32_t f = eval_rules(ri, c, ca, gt, narith, rc, s_cls);
     ca.flags[c] = (uint8_t)f;
     v = site_chain(f, ca.depth[c]);
   }
@@ -637,12 +734,23 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
   if (!f) return;
   const uint32_t g = ca.idx[c], kernel = ca.kernel[c];
   const KDesc K = kd[kernel];
-  const Rec ri = ld_rec(rec, g);
+  const Rec ri = ld_rec(ca.rec, c);
   const unsigned long long coff = pre_c[blockIdx.x] + (ex >> 32);
-  // chain: re-chase and store kernel-local indices
-  uint32_t n = 0;
-  if (ca.depth[c] && coff + ca.depth[c] <= chain_cap)
-    chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, s_cls, [&](uint32_t j) { chain[coff + n++] = j; });
+  // chain (kernel-local indices): the first kChain4 elements were kept by the trace; longer chains
+  // are traced again
+  const uint32_t dep = ca.depth[c];
+  if (dep && coff + dep <= chain_cap) {
+    if (dep <= kChain4) {
+      const uint4 e = reinterpret_cast<const uint4*>(ca.chain4)[c];
+      chain[coff] = e.x;
+      if (dep > 1) chain[coff + 1] = e.y;
+      if (dep > 2) chain[coff + 2] = e.z;
+      if (dep > 3) chain[coff + 3] = e.w;
+    } else {
+      uint32_t n = 0;
+      chase(rec, ptrrd, K, r_s0(ri), ca.base_rd[c], D, s_cls, [&](uint32_t j) { chain[coff + n++] = j; });
+    }
+  }
   uint64_t so = pre_s[blockIdx.x] + (ex & 0xffffffffull);
   for (uint32_t rule = 0; rule < 7; rule++) {
     if (!((f >> rule) & 1u)) continue;
@@ -657,10 +765,10 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
     s.chain_off = (uint32_t)coff;
     s.a0 = s.a1 = s.a2 = 0;
     if (rule == GS_VEC) {
-      const uint32_t sl = ca.grp[c];
-      const uint32_t n32 = gt.n32[sl];
-      const int32_t mn = gt.mn[sl], mx = gt.mx[sl];
-      const bool contig = (int64_t)mx - (int64_t)mn == 4ll * ((int64_t)n32 - 1) && gt.or3[sl] == gt.and3[sl];
+      const GEnt& e = gt.g[ca.grp[c]];
+      const uint32_t n32 = e.n32;
+      const int32_t mn = e.mn, mx = e.mx;
+      const bool contig = (int64_t)mx - (int64_t)mn == 4ll * ((int64_t)n32 - 1) && (e.bits & 3u) == (e.bits >> 2);
       s.a0 = (int32_t)(n32 | (contig ? (1u << 30) : 0u));
       s.a1 = mn;
       s.a2 = mx;
@@ -674,10 +782,10 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
         s.a1 = -2;
       }
     } else if (rule == GS_SHMEM) {
-      s.a0 = (int32_t)gt.nload[ca.grp[c]];
+      s.a0 = (int32_t)gt.g[ca.grp[c]].nload;
       s.a1 = (int32_t)narith[g];
     } else if (rule == GS_TEX) {
-      s.a0 = (int32_t)gt.nall[ca.grp[c]];
+      s.a0 = (int32_t)gt.g[ca.grp[c]].nall;
     }
     if (rule == GS_CONV) { s.depth = 0; s.term_kind = GS_T_NONE; s.term_value = 0; }
     if (so < site_cap) sites[so] = s;
@@ -685,23 +793,24 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
   }
 }
 
-__global__ void k_init_groups(GroupTable gt, OffsetSet os, RootSet rs) {
+// entries [g0, g1) of the group and offset tables, [r0, r1) of the root table (the regions of the
+// detected kernels)
+__global__ void k_init_groups(GroupTable gt, uint64_t g0, uint64_t g1, uint64_t r0, uint64_t r1) {
   const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-  if (i < gt.cap) {
-    gt.key[i] = kEmpty;
-    gt.nload[i] = gt.n32[i] = gt.nall[i] = gt.or3[i] = 0;
-    gt.and3[i] = 3u;
-    gt.mn[i] = INT_MAX;
-    gt.mx[i] = INT_MIN;
+  if (g0 + i < g1) {
+    GEnt e;
+    e.key = kEmpty;
+    e.nload = e.n32 = e.nall = 0;
+    e.mn = INT_MAX;
+    e.mx = INT_MIN;
+    e.bits = 3u << 2;
+    gt.g[g0 + i] = e;
+    OEnt o;
+    o.key = kEmpty;
+    o.flags = o.pad = 0;
+    gt.o[g0 + i] = o;
   }
-  if (i < os.cap) { os.key[i] = kEmpty; os.flags[i] = 0; }
-  if (i < rs.cap) rs.key[i] = kEmpty;
-}
-
-uint32_t pow2_at_least(uint64_t n) {
-  uint64_t c = 16;
-  while (c < n) c <<= 1;
-  return (uint32_t)c;
+  if (r0 + i < r1) gt.r[r0 + i] = kEmpty;
 }
 
 }  // namespace
@@ -709,9 +818,8 @@ uint32_t pow2_at_least(uint64_t n) {
 void detect_free(gs_ctx* c) {
   void* ps[] = {c->d_tab, c->d_ldiff, c->d_wsum, c->d_wloop, c->d_wev, c->d_ptrrd, c->d_narith,
                 c->cand.idx, c->cand.kernel, c->cand.base_rd, c->cand.data_rd, c->cand.tv, c->cand.grp,
-                c->cand.nsite, c->cand.soff, c->cand.ld, c->cand.tk, c->cand.depth, c->cand.flags,
-                c->cand.choff, c->grp.key, c->grp.nload, c->grp.n32, c->grp.nall, c->grp.or3, c->grp.and3,
-                c->grp.mn, c->grp.mx, c->oset.key, c->oset.flags, c->roots.key, c->d_kstats, c->d_sites,
+                c->cand.cont, c->cand.rec, c->cand.chain4, c->cand.ld, c->cand.tk, c->cand.depth, c->cand.flags,
+                c->cand.choff, c->grp.g, c->grp.o, c->grp.r, c->grp.kh, c->d_kstats, c->d_sites,
                 c->d_chain, c->d_scan_tmp};
   for (void* p : ps)
     if (p) cudaFree(p);
@@ -719,8 +827,6 @@ void detect_free(gs_ctx* c) {
   c->d_ptrrd = nullptr; c->d_narith = nullptr;
   c->cand = CandArrays();
   c->grp = GroupTable();
-  c->oset = OffsetSet();
-  c->roots = RootSet();
   c->d_kstats = nullptr;
   c->d_sites = nullptr; c->sites_cap = 0; c->n_sites = 0;
   c->d_chain = nullptr; c->chain_cap = 0; c->n_chain = 0;
@@ -782,20 +888,16 @@ gs_status detect_alloc(gs_ctx* c) {
   A(c->d_ptrrd, P * 4);
   A(c->d_narith, P * 4);
   A(c->cand.idx, NC * 4); A(c->cand.kernel, NC * 4); A(c->cand.base_rd, NC * 4); A(c->cand.data_rd, NC * 4);
-  A(c->cand.tv, NC * 4); A(c->cand.grp, NC * 4); A(c->cand.nsite, NC * 4); A(c->cand.soff, NC * 4 + 4);
+  A(c->cand.tv, NC * 4); A(c->cand.grp, NC * 4); A(c->cand.cont, NC * 4); A(c->cand.rec, NC * sizeof(Rec)); A(c->cand.chain4, NC * 16);
   A(c->cand.ld, NC); A(c->cand.tk, NC); A(c->cand.depth, NC); A(c->cand.flags, NC);
   A(c->cand.choff, 24 * ((NC + kCT - 1) / kCT) + 16);  // tile sums, prefixes, totals (k_rules / k_write)
-  c->grp.cap = pow2_at_least(2 * c->n_ldg + 16);
-  A(c->grp.key, (uint64_t)c->grp.cap * 8);
-  A(c->grp.nload, (uint64_t)c->grp.cap * 4); A(c->grp.n32, (uint64_t)c->grp.cap * 4);
-  A(c->grp.nall, (uint64_t)c->grp.cap * 4); A(c->grp.or3, (uint64_t)c->grp.cap * 4);
-  A(c->grp.and3, (uint64_t)c->grp.cap * 4); A(c->grp.mn, (uint64_t)c->grp.cap * 4);
-  A(c->grp.mx, (uint64_t)c->grp.cap * 4);
-  c->oset.cap = pow2_at_least(2 * c->n_ldg + 16);
-  A(c->oset.key, (uint64_t)c->oset.cap * 8);
-  A(c->oset.flags, (uint64_t)c->oset.cap * 4);
-  c->roots.cap = pow2_at_least(2 * c->n_store + 16);
-  A(c->roots.key, (uint64_t)c->roots.cap * 8);
+  A(c->grp.g, c->grp.gtot * sizeof(GEnt));
+  A(c->grp.o, c->grp.gtot * sizeof(OEnt));
+  A(c->grp.r, c->grp.rtot * 8);
+  A(c->grp.kh, (uint64_t)c->kh_h.size() * sizeof(KHash));
+  if (!c->kh_h.empty())
+    GS_CUDA(c, cudaMemcpyAsync(c->grp.kh, c->kh_h.data(), c->kh_h.size() * sizeof(KHash), cudaMemcpyHostToDevice,
+                               c->stream));
   A(c->d_kstats, (uint64_t)(c->n_kernels ? c->n_kernels : 1) * sizeof(gs_kernel_stats));
 #undef A
   return GS_OK;
@@ -845,8 +947,9 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win); count_launch();
       GS_CUDA(c, cudaGetLastError());
       // candidate arrays are indexed relative to c0
-      k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop, c->d_wev,
-                                             c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand); count_launch();
+      k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop,
+                                             c->d_wev, c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand, D);
+      count_launch();
       GS_CUDA(c, cudaGetLastError());
     }
     if (cons) {
@@ -854,14 +957,18 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       if (cs != GS_OK) return cs;
     }
     if (nc) {
-      const uint32_t gcap = std::max(c->grp.cap, std::max(c->oset.cap, c->roots.cap));
-      k_init_groups<<<(gcap + 255) / 256, 256, 0, st>>>(c->grp, c->oset, c->roots); count_launch();
+      // the hash-table regions of kernels [kb, ke)
+      const uint64_t g0 = c->kh_h[kb].gofs, r0 = c->kh_h[kb].rofs;
+      const uint64_t g1 = ke < c->n_kernels ? c->kh_h[ke].gofs : c->grp.gtot;
+      const uint64_t r1 = ke < c->n_kernels ? c->kh_h[ke].rofs : c->grp.rtot;
+      const uint64_t ni = std::max(g1 - g0, r1 - r0);
+      k_init_groups<<<(uint32_t)((ni + 255) / 256), 256, 0, st>>>(c->grp, g0, g1, r0, r1); count_launch();
       GS_CUDA(c, cudaGetLastError());
       const uint32_t gridc = (uint32_t)((nc + 255) / 256);
-      k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->oset, c->roots,
-                                         c->d_kstats); count_launch();
+      k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->d_kstats);
+      count_launch();
       GS_CUDA(c, cudaGetLastError());
-      k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->roots, c->d_narith,
+      k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->d_narith,
                                                RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum);
       count_launch();
       k_tile_prefix<<<1, 1024, 0, st>>>(d_tsum, ntile, d_pre_s, d_pre_c, d_tot); count_launch();

@@ -14,6 +14,8 @@
 #include <cstring>
 #include <map>
 #include <string>
+#include <string_view>
+#include <unordered_map>
 #include <thread>
 #include <utility>
 #include <vector>
@@ -26,7 +28,9 @@ namespace {
 struct Sv {  // non-owning text span
   const char* p = nullptr;
   size_t n = 0;
-  bool eq(const char* s) const { size_t m = strlen(s); return m == n && memcmp(p, s, n) == 0; }
+  template <size_t N>  // literals: length known at compile time (the parser compares thousands per line)
+  bool eq(const char (&s)[N]) const { return n == N - 1 && memcmp(p, s, N - 1) == 0; }
+  bool eqz(const char* s) const { size_t m = strlen(s); return m == n && memcmp(p, s, n) == 0; }
   char operator[](size_t i) const { return p[i]; }
 };
 
@@ -37,13 +41,15 @@ inline Sv trim(Sv s) {
   return s;
 }
 inline bool contains(Sv s, const char* needle, size_t* at = nullptr) {
-  size_t m = strlen(needle);
+  const size_t m = strlen(needle);
   if (m > s.n) return false;
-  for (size_t i = 0; i + m <= s.n; i++)
-    if (memcmp(s.p + i, needle, m) == 0) { if (at) *at = i; return true; }
-  return false;
+  const void* f = memmem(s.p, s.n, needle, m);
+  if (!f) return false;
+  if (at) *at = (size_t)((const char*)f - s.p);
+  return true;
 }
-inline bool starts(Sv s, const char* pre) { size_t m = strlen(pre); return s.n >= m && memcmp(s.p, pre, m) == 0; }
+template <size_t N>
+inline bool starts(Sv s, const char (&pre)[N]) { return s.n >= N - 1 && memcmp(s.p, pre, N - 1) == 0; }
 inline int hexv(char c) {
   if (c >= '0' && c <= '9') return c - '0';
   if (c >= 'a' && c <= 'f') return c - 'a' + 10;
@@ -204,9 +210,13 @@ const OpName kOps[] = {
 };
 
 uint8_t op_lookup(Sv m) {
-  for (const auto& o : kOps)
-    if (m.eq(o.s)) return o.id;
-  return OP_OTHER;
+  static const std::unordered_map<std::string_view, uint8_t> tab = [] {
+    std::unordered_map<std::string_view, uint8_t> t;
+    for (const auto& o : kOps) t.emplace(o.s, o.id);
+    return t;
+  }();
+  const auto it = tab.find(std::string_view(m.p, m.n));
+  return it == tab.end() ? (uint8_t)OP_OTHER : it->second;
 }
 
 struct Line {
@@ -230,12 +240,12 @@ struct LiveOut {
 inline bool is64type(Sv m) { return m.eq("F64") || m.eq("S64") || m.eq("U64"); }
 inline bool isinttype(Sv m) {
   static const char* k[] = {"S64", "U64", "S32", "U32", "S16", "U16", "S8", "U8"};
-  for (auto* x : k) if (m.eq(x)) return true;
+  for (auto* x : k) if (m.eqz(x)) return true;
   return false;
 }
 inline bool isfloattype(Sv m) {
   static const char* k[] = {"F64", "F32", "F16", "BF16", "TF32", "E4M3", "E5M2"};
-  for (auto* x : k) if (m.eq(x)) return true;
+  for (auto* x : k) if (m.eqz(x)) return true;
   return false;
 }
 
@@ -297,7 +307,7 @@ bool pack_line(Sv body, long lineno, size_t index, Rec* out, std::string* msg, L
     mods[nm++] = Sv{opc.p + d + 1, e - d - 1};
     d = e;
   }
-  auto has = [&](const char* m) { for (int q = 0; q < nm; q++) if (mods[q].eq(m)) return true; return false; };
+  auto has = [&](const auto& m) { for (int q = 0; q < nm; q++) if (mods[q].eq(m)) return true; return false; };
   uint32_t op = op_lookup(mn);
   if (op == OP_IMAD && nm > 0 && mods[0].eq("MOV")) op = OP_IMAD_MOV;
   // operands: top-level commas

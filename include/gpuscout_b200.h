@@ -5,7 +5,7 @@
  *     each flagged memory instruction carrying a bounded backward def-use trace;
  *   - warp-stall attribution: PC samples with stall reasons aggregated per PC and
  *     attributed "to the instruction detected by the SASS Analysis engine".
- * Readings of the paper where it is silent are numbered R1..R38 in DESIGN.md §3.
+ * Readings of the paper where it is silent are numbered R1..R39 in DESIGN.md §3.
  *
  * Conventions (all entry points):
  *   - Every call returns a gs_status; no exception or abort crosses the ABI. On error the message
@@ -230,6 +230,14 @@ uint64_t gs_launch_count(void);
 
 /* Histogram strategy actually used by the last gs_attribute_samples (GS_HIST_*). */
 int gs_last_hist_mode(const gs_ctx *ctx);
+
+/* GPU time in milliseconds of the device work of the last gs_attribute_samples call with device
+ * input (histogram zeroing, planning and counting kernels): two CUDA events recorded on the
+ * context's stream, the first after the call's host-side preparation and before its first
+ * enqueue, the second after its last enqueue, so host launch gaps before the pass are excluded.
+ * Waits for the second event. GS_E_STATE if there was no such call (or the last one had host
+ * input). A measurement aid for harnesses (bench.py's roofline); computes nothing. */
+gs_status gs_last_attribute_ms(gs_ctx *ctx, float *ms);
 
 #ifdef __cplusplus
 }

@@ -47,7 +47,7 @@ _lib = None
 EXPORTS = ["gs_create", "gs_destroy", "gs_last_error", "gs_version", "gs_load_sass", "gs_kernel_table",
            "gs_kernel_name", "gs_instr_lines", "gs_detect", "gs_sites", "gs_sites_host", "gs_kernel_stats_get", "gs_pack_samples",
            "gs_attribute_samples", "gs_attribute_counts", "gs_cupti_stall_reasons", "gs_attribute_cupti", "gs_register_pressure", "gs_rank_sites",
-           "gs_rank_sites_slice", "gs_last_hist_mode", "gs_launch_count"]
+           "gs_rank_sites_slice", "gs_last_hist_mode", "gs_last_attribute_ms", "gs_launch_count"]
 
 
 def launch_count() -> int:
@@ -86,6 +86,7 @@ def load_library(path: str = LIB_PATH):
         "gs_rank_sites": (I32, [P, P, U64, P, ctypes.POINTER(U64)]),
         "gs_rank_sites_slice": (I32, [P, P, U64, U64, U64, P, ctypes.POINTER(U64)]),
         "gs_last_hist_mode": (I32, [P]),
+        "gs_last_attribute_ms": (I32, [P, ctypes.POINTER(ctypes.c_float)]),
         "gs_launch_count": (U64, []),
     }
     for name, (res, args) in sig.items():
@@ -278,6 +279,12 @@ class Context:
 
     def last_hist_mode(self) -> int:
         return self.L.gs_last_hist_mode(self.h)
+
+    def last_attribute_ms(self) -> float:
+        """GPU time of the last device-input attribute_samples call (events around its kernels)."""
+        ms = ctypes.c_float()
+        self._check(self.L.gs_last_attribute_ms(self.h, ctypes.byref(ms)), "gs_last_attribute_ms")
+        return ms.value
 
     # ---- a-11, a-12
     def rank_sites(self, hist, k: int | None = None, out=None, slot_begin: int = 0,

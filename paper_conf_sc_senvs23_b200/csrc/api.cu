@@ -2,6 +2,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -112,6 +115,12 @@ void gs_destroy(gs_ctx* c) {
   rank_free(c);
   cupti_free(c);
   if (c->h_pin) cudaFreeHost(c->h_pin);
+  if (c->side_stream) {
+    cudaStreamSynchronize(c->side_stream);
+    cudaStreamDestroy(c->side_stream);
+  }
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
   delete c;
 }
 
@@ -124,7 +133,12 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   std::vector<ParsedKernel> ks;
   std::string err;
   const int nt = (int)std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  // GS_TIMING=1: host phase times of the load on stderr (parse | pack tables | upload | scratch)
+  static const bool timing = getenv("GS_TIMING") != nullptr;
+  using clk = std::chrono::steady_clock;
+  const auto t0 = clk::now();
   if (!parse_sass(text, len, nt, &ks, &err)) return fail(c, GS_E_PARSE, err);
+  const auto t1 = clk::now();
   uint64_t P = 0;
   for (auto& k : ks) P += k.recs.size();
   if (P > 0x7ffffffeull) return fail(c, GS_E_RANGE, "more than 2^31-2 instructions");
@@ -147,55 +161,95 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   c->n_cand = c->n_ldg = c->n_store = 0;
   c->kh_h.assign(ks.size(), KHash{});
   c->grp.gtot = c->grp.rtot = 0;
-  std::vector<Rec> recs;
-  recs.reserve(P);
-  uint32_t slot = 0;
-  for (size_t k = 0; k < ks.size(); k++) {
-    ParsedKernel& pk = ks[k];
-    KDesc& K = c->kd_h[k];
-    K.first = slot;
-    K.n = (uint32_t)pk.recs.size();
-    K.param_base = pk.param_base | (std::min<uint32_t>(pk.nregs, 255u) << 16);
-    K.win0 = (uint32_t)c->wd_h.size();
-    const uint64_t ldg0 = c->n_ldg, st0 = c->n_store;
-    for (uint32_t s = 0; s < K.n; s += c->win) {
-      WDesc W{(uint32_t)k, slot + s, std::min(c->win, K.n - s), 0};
-      uint32_t nc = 0;
-      for (uint32_t i = 0; i < W.len; i++) {  // candidates per window: static opcode classes
-        const Rec& r = pk.recs[s + i];
-        const uint32_t cls = op_class(r_op(r));
-        if (cls & (C_TRACED | C_CONV)) nc++;
-        if (r_op(r) == OP_LDG) c->n_ldg++;
-        if (cls & C_STORE) c->n_store++;
+  // per-kernel offsets (sequential, O(kernels)), then the kernels' records and tables are copied
+  // into the module arrays in parallel
+  const size_t K = ks.size();
+  std::vector<uint64_t> use_base(K + 1, 0), xl_base(K + 1, 0), xt_base(K + 1, 0);
+  uint32_t slot = 0, nwin = 0;
+  for (size_t k = 0; k < K; k++) {
+    const ParsedKernel& pk = ks[k];
+    KDesc& Kd = c->kd_h[k];
+    Kd.first = slot;
+    Kd.n = (uint32_t)pk.recs.size();
+    Kd.param_base = pk.param_base | (std::min<uint32_t>(pk.nregs, 255u) << 16);
+    Kd.win0 = nwin;
+    nwin += (Kd.n + c->win - 1) / c->win;
+    slot += Kd.n;
+    use_base[k + 1] = use_base[k] + pk.use_reg.size();
+    xl_base[k + 1] = xl_base[k] + (pk.xtgt_off.empty() ? 0 : pk.xtgt_off.size() - 1);
+    xt_base[k + 1] = xt_base[k] + pk.xtgt.size();
+  }
+  std::vector<Rec> recs(P);
+  c->lines_h.resize(P);
+  c->use_off_h.assign(P + 1, 0);
+  c->use_reg_h.resize(use_base[K]);
+  c->tgt_h.resize(P);
+  c->xoff_h.assign(xl_base[K] + 1, 0);
+  c->xtgt_h.resize(xt_base[K]);
+  c->wd_h.resize(nwin);
+  std::vector<uint32_t> wcand(nwin, 0);
+  std::vector<uint64_t> kldg(K, 0), kst(K, 0);
+  {
+    std::atomic<size_t> next(0);
+    auto fill = [&]() {
+      for (;;) {
+        const size_t k = next.fetch_add(1);
+        if (k >= K) return;
+        const ParsedKernel& pk = ks[k];
+        const KDesc& Kd = c->kd_h[k];
+        std::copy(pk.recs.begin(), pk.recs.end(), recs.begin() + Kd.first);
+        std::copy(pk.lines.begin(), pk.lines.end(), c->lines_h.begin() + Kd.first);
+        std::copy(pk.use_reg.begin(), pk.use_reg.end(), c->use_reg_h.begin() + use_base[k]);
+        for (size_t i = 1; i < pk.use_off.size(); i++)  // register-pressure inputs, offsets made global
+          c->use_off_h[Kd.first + i] = (uint32_t)(use_base[k] + pk.use_off[i]);
+        const int32_t x0 = (int32_t)xl_base[k];  // indirect-branch lists: global list ids
+        for (size_t i = 0; i < pk.tgt.size(); i++) {
+          const int32_t t = pk.tgt[i];
+          c->tgt_h[Kd.first + i] = t <= -2 ? t - x0 : t;
+        }
+        for (size_t x = 1; x < pk.xtgt_off.size(); x++)
+          c->xoff_h[xl_base[k] + x] = (uint32_t)(xt_base[k] + pk.xtgt_off[x]);
+        std::copy(pk.xtgt.begin(), pk.xtgt.end(), c->xtgt_h.begin() + xt_base[k]);
+        uint64_t nl = 0, ns = 0;
+        for (uint32_t s0 = 0, w = Kd.win0; s0 < Kd.n; s0 += c->win, w++) {
+          const WDesc W{(uint32_t)k, Kd.first + s0, std::min(c->win, Kd.n - s0), 0};
+          uint32_t nc = 0;
+          for (uint32_t i = 0; i < W.len; i++) {  // candidates per window: static opcode classes
+            const Rec& r = pk.recs[s0 + i];
+            const uint32_t cls = op_class(r_op(r));
+            if (cls & (C_TRACED | C_CONV)) nc++;
+            if (r_op(r) == OP_LDG) nl++;
+            if (cls & C_STORE) ns++;
+          }
+          c->wd_h[w] = W;
+          wcand[w] = nc;
+        }
+        kldg[k] = nl;
+        kst[k] = ns;
       }
-      c->cbase_h.push_back((uint32_t)c->n_cand);
-      c->n_cand += nc;
-      c->wd_h.push_back(W);
-    }
-    {  // the kernel's hash-table regions: a power of two >= 2x its global loads / stores
-      KHash& H = c->kh_h[k];
-      const uint64_t gcap = pow2_ceil(2 * (c->n_ldg - ldg0) + 2), rcap = pow2_ceil(2 * (c->n_store - st0) + 2);
-      H.gofs = c->grp.gtot;
-      H.rofs = c->grp.rtot;
-      H.gmask = (uint32_t)(gcap - 1);
-      H.rmask = (uint32_t)(rcap - 1);
-      c->grp.gtot += gcap;
-      c->grp.rtot += rcap;
-    }
-    slot += K.n;
-    recs.insert(recs.end(), pk.recs.begin(), pk.recs.end());
-    {  // register-pressure inputs, offsets made global
-      const uint32_t base = (uint32_t)c->use_reg_h.size();
-      for (size_t i = 1; i < pk.use_off.size(); i++) c->use_off_h.push_back(base + pk.use_off[i]);
-      c->use_reg_h.insert(c->use_reg_h.end(), pk.use_reg.begin(), pk.use_reg.end());
-      const int32_t x0 = (int32_t)c->xoff_h.size() - 1;  // indirect-branch lists: global list ids
-      for (int32_t t : pk.tgt) c->tgt_h.push_back(t <= -2 ? t - x0 : t);
-      const uint32_t xbase = (uint32_t)c->xtgt_h.size();
-      for (size_t x = 1; x < pk.xtgt_off.size(); x++) c->xoff_h.push_back(xbase + pk.xtgt_off[x]);
-      c->xtgt_h.insert(c->xtgt_h.end(), pk.xtgt.begin(), pk.xtgt.end());
-    }
-    c->lines_h.insert(c->lines_h.end(), pk.lines.begin(), pk.lines.end());
-    c->names.push_back(std::move(pk.name));
+    };
+    std::vector<std::thread> th;
+    for (int t = 1; t < nt; t++) th.emplace_back(fill);
+    fill();
+    for (auto& t : th) t.join();
+  }
+  c->cbase_h.resize(nwin);
+  for (uint32_t w = 0; w < nwin; w++) {
+    c->cbase_h[w] = (uint32_t)c->n_cand;
+    c->n_cand += wcand[w];
+  }
+  for (size_t k = 0; k < K; k++) {  // the kernel's hash-table regions: a power of two >= 2x its loads / stores
+    KHash& H = c->kh_h[k];
+    const uint64_t gcap = pow2_ceil(2 * kldg[k] + 2), rcap = pow2_ceil(2 * kst[k] + 2);
+    H.gofs = c->grp.gtot;
+    H.rofs = c->grp.rtot;
+    H.gmask = (uint32_t)(gcap - 1);
+    H.rmask = (uint32_t)(rcap - 1);
+    c->grp.gtot += gcap;
+    c->grp.rtot += rcap;
+    c->n_ldg += kldg[k];
+    c->n_store += kst[k];
+    c->names.push_back(std::move(ks[k].name));
   }
   c->cbase_h.push_back((uint32_t)c->n_cand);
   c->n_win = (uint32_t)c->wd_h.size();
@@ -227,6 +281,7 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
   GS_CUDA(c, cudaMalloc((void**)&c->d_kd, std::max<size_t>(ks.size(), 1) * sizeof(KDesc)));
   GS_CUDA(c, cudaMalloc((void**)&c->d_wd, std::max<size_t>(c->wd_h.size(), 1) * sizeof(WDesc)));
   GS_CUDA(c, cudaMalloc((void**)&c->d_cbase, c->cbase_h.size() * 4));
+  const auto t2 = clk::now();
   if (P) GS_CUDA(c, cudaMemcpyAsync(c->d_rec, recs.data(), P * sizeof(Rec), cudaMemcpyHostToDevice, c->stream));
   if (!ks.empty())
     GS_CUDA(c, cudaMemcpyAsync(c->d_kd, c->kd_h.data(), ks.size() * sizeof(KDesc), cudaMemcpyHostToDevice, c->stream));
@@ -243,10 +298,17 @@ gs_status gs_load_sass(gs_ctx* c, const char* text, size_t len, uint32_t* n_kern
     if (!gslot.empty())
       GS_CUDA(c, cudaMemcpyAsync(c->d_gslot, gslot.data(), gslot.size() * 4, cudaMemcpyHostToDevice, c->stream));
   }
+  const auto t3 = clk::now();
   gs_status s = detect_alloc(c);
   if (s != GS_OK) return s;
   // pageable source buffers: wait for the copies before they go out of scope
   GS_CUDA(c, cudaStreamSynchronize(c->stream));
+  if (timing) {
+    const auto t4 = clk::now();
+    const auto sec = [](clk::duration d) { return std::chrono::duration<double>(d).count(); };
+    fprintf(stderr, "gs_load_sass: parse %.3f s, tables %.3f s, upload %.3f s, scratch+sync %.3f s (%u threads)\n",
+            sec(t1 - t0), sec(t2 - t1), sec(t3 - t2), sec(t4 - t3), (unsigned)nt);
+  }
   c->loaded = true;
   if (n_kernels) *n_kernels = c->n_kernels;
   if (n_instr) *n_instr = P;
@@ -332,7 +394,14 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
   if (!d_hist && c->n_instr) return fail(c, GS_E_INVAL, "null histogram");
   if (c->n_instr >= (1ull << 27)) return fail(c, GS_E_RANGE, "packed samples address at most 2^27 slots");
   GS_CUDA(c, cudaSetDevice(c->device));
-  if (!n || is_device_ptr(samples)) return hist_run(c, samples, n, d_hist, d_n_invalid, accumulate, true);
+  if (!n || is_device_ptr(samples)) {
+    const gs_status hs = hist_run(c, samples, n, d_hist, d_n_invalid, accumulate, true);
+    if (hs == GS_OK && c->ev_pass[1]) {  // hist_run recorded ev_pass[0] before its first enqueue
+      GS_CUDA(c, cudaEventRecord(c->ev_pass[1], c->stream));
+      c->pass_timed = true;
+    }
+    return hs;
+  }
   // host input: chunks through two device staging buffers; the H2D copy of chunk i+1 runs on a
   // copy stream (copy engine) while the histogram of chunk i runs on the context's stream
   const size_t chunk = size_t(16) << 20;  // words
@@ -436,5 +505,13 @@ gs_status gs_rank_sites(gs_ctx* c, const int32_t* d_hist, uint64_t k, gs_ranked_
 uint64_t gs_launch_count(void) { return gs::g_launches.load(); }
 
 int gs_last_hist_mode(const gs_ctx* c) { return c ? c->last_hist_mode : -1; }
+
+gs_status gs_last_attribute_ms(gs_ctx* c, float* ms) {
+  if (!c || !ms) return GS_E_INVAL;
+  if (!c->pass_timed) return fail(c, GS_E_STATE, "no timed gs_attribute_samples call (device input) yet");
+  GS_CUDA(c, cudaEventSynchronize(c->ev_pass[1]));
+  GS_CUDA(c, cudaEventElapsedTime(ms, c->ev_pass[0], c->ev_pass[1]));
+  return GS_OK;
+}
 
 }  // extern "C"

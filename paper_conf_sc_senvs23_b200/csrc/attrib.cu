@@ -1395,8 +1395,15 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   const Div dv = make_div(nr, c->cfg.hist_row);
   const uint64_t hbins = (uint64_t)P * c->cfg.hist_row;
   if (reinterpret_cast<uintptr_t>(d_words) & 3u) return fail(c, GS_E_INVAL, "sample pointer must be 4-byte aligned");
-  int dev_sms = 148;
-  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+  if (!c->dev_sms) GS_CUDA(c, cudaDeviceGetAttribute(&c->dev_sms, cudaDevAttrMultiProcessorCount, c->device));
+  const int dev_sms = c->dev_sms;
+  // the pass's GPU time (gs_last_attribute_ms): from here to the end of its enqueued work
+  if (!c->ev_pass[0]) {
+    GS_CUDA(c, cudaEventCreate(&c->ev_pass[0]));
+    GS_CUDA(c, cudaEventCreate(&c->ev_pass[1]));
+  }
+  c->pass_timed = false;
+  GS_CUDA(c, cudaEventRecord(c->ev_pass[0], st));
   // peel the words before the first 16-byte boundary so the main kernels use 128-bit loads
   const uint64_t head = std::min<uint64_t>(n, ((16u - (reinterpret_cast<uintptr_t>(d_words) & 15u)) & 15u) / 4u);
   const uint32_t nslots32 = kTableWords / nr, nslots16 = 2 * kTableWords / nr;  // whole slots per window
@@ -1486,8 +1493,17 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
       if (ps != GS_OK) return ps;
     }
   }
-  const auto prep = [&](auto kern) -> gs_status {
+  const auto prep = [&](auto kern) -> gs_status {  // the dynamic smem limit, raised once per kernel and size
+    const void* fn = reinterpret_cast<const void*>(kern);
+    int slot = -1;
+    for (int q = 0; q < 4 && slot < 0; q++)
+      if (c->smem_fn[q] == fn || !c->smem_fn[q]) slot = q;
+    if (slot >= 0 && c->smem_fn[slot] == fn && c->smem_set[slot] >= smem) return GS_OK;
     GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (slot >= 0) {
+      c->smem_fn[slot] = fn;
+      c->smem_set[slot] = smem;
+    }
     return GS_OK;
   };
   gs_status ls = GS_OK;
@@ -1524,6 +1540,8 @@ void attrib_free(gs_ctx* c) {
     if (c->h_stage[b]) cudaFreeHost(c->h_stage[b]);
     if (c->d_stage[b]) cudaFree(c->d_stage[b]);
     if (c->ev_stage[b]) cudaEventDestroy(c->ev_stage[b]);
+    if (c->ev_pass[b]) cudaEventDestroy(c->ev_pass[b]);
+    c->ev_pass[b] = nullptr;
     if (c->ev_copied[b]) cudaEventDestroy(c->ev_copied[b]);
     c->h_stage[b] = nullptr;
     c->d_stage[b] = nullptr;

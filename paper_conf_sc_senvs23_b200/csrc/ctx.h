@@ -181,6 +181,15 @@ struct gs_ctx {
   cudaEvent_t ev_stage[2] = {nullptr, nullptr};   // histogram of staging buffer b done (ctx stream)
   cudaEvent_t ev_copied[2] = {nullptr, nullptr};  // H2D into staging buffer b done (copy stream)
   cudaStream_t copy_stream = nullptr;             // host input: H2D copies overlap the histogram
+  // detection: hash-table zeroing on a side stream, forked from and joined into the context's stream
+  cudaStream_t side_stream = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  // GPU time of the last device-input gs_attribute_samples (events around its enqueued work)
+  cudaEvent_t ev_pass[2] = {nullptr, nullptr};
+  bool pass_timed = false;
+  int dev_sms = 0;                   // cached multiprocessor count
+  const void* smem_fn[4] = {nullptr, nullptr, nullptr, nullptr};  // kernels whose dynamic smem limit
+  size_t smem_set[4] = {0, 0, 0, 0};                               // was raised, and to what
   size_t stage_words = 0;
 };
 

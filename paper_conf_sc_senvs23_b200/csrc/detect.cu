@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 
 #include <climits>
+#include <cstring>
 #include <cstdio>
 
 #include "ctx.h"
@@ -50,6 +51,17 @@ __device__ __forceinline__ uint32_t reg_cap(uint32_t dst) { return dst < 256 ? 2
 // which a warp of mixed opcodes walks divergently for every record; one LDS replaces it.
 __device__ __forceinline__ void opcls_init(uint16_t* t) {
   for (uint32_t i = threadIdx.x; i < OP_COUNT; i += blockDim.x) t[i] = (uint16_t)op_class(i);
+}
+
+// f(q < nq, base + q) for the first four registers of a destination (unrolled: no divergent loop
+// for the usual widths 1, 2, 4; k_summary 262 -> 235 us on C3), a loop for wider destinations
+template <typename F>
+__device__ __forceinline__ void for_regs(uint32_t base, uint32_t nq, F f) {
+  f(nq > 0, base);
+  f(nq > 1, base + 1);
+  f(nq > 2, base + 2);
+  f(nq > 3, base + 3);
+  for (uint32_t q = 4; q < nq; q++) f(true, base + q);
 }
 
 __device__ __forceinline__ uint32_t hash64(unsigned long long k) {
@@ -87,7 +99,7 @@ __device__ __forceinline__ unsigned long long group_key(uint32_t base, uint32_t 
 }
 
 // ------------------------------------------------------------------------------------------ A
-__global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+__global__ void __launch_bounds__(kWarps * 32, 5) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
                                                          uint32_t* __restrict__ tab, int32_t* ldiff, int32_t* wsum,
                                                          uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst,
@@ -122,10 +134,10 @@ __global__ void __launch_bounds__(kWarps * 32) k_summary(const Rec* __restrict__
     if (valid && dw && reg_live(dst)) {
       const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
       const uint32_t nq = min(dw, reg_cap(dst) + 1 - dst);
-      for (uint32_t q = 0; q < nq; q++) atomicMax(&last[warp][dst + q], v);
+      for_regs(dst, nq, [&](bool p, uint32_t x) { if (p) atomicMax(&last[warp][x], v); });
       if (reg_live(dst2)) {  // second quad of a 256-bit load (R38a)
         const uint32_t nq2 = min(dw, reg_cap(dst2) + 1 - dst2);
-        for (uint32_t q = 0; q < nq2; q++) atomicMax(&last[warp][dst2 + q], v);
+        for_regs(dst2, nq2, [&](bool p, uint32_t x) { if (p) atomicMax(&last[warp][x], v); });
       }
     }
     if (valid && op == OP_LDG) narith[g] = 0;
@@ -274,15 +286,14 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* ptrrd, co
 // while their steps stay inside the window (the RDs of earlier windows belong to other warps);
 // k_trace resumes the others.
 constexpr uint32_t kNarWords = kWinBig / 2;  // 16-bit n_arith counters per window instruction
-__global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+__global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
                                                          const uint32_t* __restrict__ tab, int32_t* ldiff,
                                                          const int32_t* __restrict__ wloop,
                                                          const uint32_t* __restrict__ wev,
                                                          const uint32_t* __restrict__ cbase, uint64_t c0,
                                                          uint32_t* ptrrd, uint32_t* narith, CandArrays ca, uint32_t D) {
-  __shared__ uint32_t tabS[kWarps][kNumRegs];
-  __shared__ uint32_t cm[kWarps][kNumRegs];
+  __shared__ uint2 mtS[kWarps][kNumRegs];  // per register: {writer lanes of the chunk M, carried table T}
   __shared__ uint32_t nar[kWarps][kNarWords];
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
@@ -297,10 +308,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
 #pragma unroll
     for (int u = 0; u < kNumRegs / 32; u++) tv[u] = __ldg(tab + (uint64_t)w * kNumRegs + lane + 32 * u);
 #pragma unroll
-    for (int u = 0; u < kNumRegs / 32; u++) {
-      tabS[warp][lane + 32 * u] = tv[u];
-      cm[warp][lane + 32 * u] = 0;
-    }
+    for (int u = 0; u < kNumRegs / 32; u++) mtS[warp][lane + 32 * u] = make_uint2(0u, tv[u]);
     for (uint32_t q = lane; q < (W.len + 1) / 2; q += 32) nar[warp][q] = 0;
   }
   __syncwarp();
@@ -309,8 +317,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
   const uint64_t cb0 = (uint64_t)cbase[w] - c0;
   uint64_t cb = cb0;
   const uint32_t lt = (1u << lane) - 1u;
-  uint32_t* T = tabS[warp];
-  uint32_t* M = cm[warp];
+  uint2* MT = mtS[warp];
   uint32_t* NA = nar[warp];
   // records (and loop events) of the next two chunks load while a chunk resolves
   Rec rn1 = lane < W.len ? ld_rec(rec, (uint64_t)W.start + lane) : Rec{0, 0, 0, 0};
@@ -320,8 +327,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
   for (uint32_t b = 0; b < W.len; b += 32) {
     const uint32_t i = b + lane;
     const bool valid = i < W.len;
-    const uint64_t g = (uint64_t)W.start + i;
-    const uint64_t gbase = (uint64_t)W.start + b;
+    const uint32_t g = W.start + i, gbase = W.start + b;  // slots < 2^31: RD values fit 32 bits
     const Rec r = rn1;
     const int32_t dcur = dn1;
     rn1 = rn2;
@@ -333,17 +339,10 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
     const uint32_t nq = writes ? min(r_dstw(r), reg_cap(dst) + 1 - dst) : 0u;
     const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
     const uint32_t nq2 = reg_live(dst2) ? min(r_dstw(r), reg_cap(dst2) + 1 - dst2) : 0u;
-    for (uint32_t q = 0; q < nq; q++) atomicOr(&M[dst + q], 1u << lane);
-    for (uint32_t q = 0; q < nq2; q++) atomicOr(&M[dst2 + q], 1u << lane);
+    for (uint32_t q = 0; q < nq; q++) atomicOr(&MT[dst + q].x, 1u << lane);
+    for (uint32_t q = 0; q < nq2; q++) atomicOr(&MT[dst2 + q].x, 1u << lane);
     const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
     __syncwarp();
-    // RD value: ((def + 1) << 1) | def_is_global_load, or 0 for ENTRY
-    auto RD = [&](uint32_t reg) -> uint32_t {
-      const uint32_t m = M[reg] & lt;
-      const uint32_t t = T[reg];
-      const uint32_t j = 31u - __clz(m);
-      return m ? (uint32_t)((gbase + j + 1) << 1) | ((ldgmask >> j) & 1u) : t;
-    };
     // loop depth: inclusive prefix of the event differences (R13); a window without loop events
     // (warp-uniform) keeps its carried depth
     int32_t depth = lcarry;
@@ -357,12 +356,20 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
       depth = lcarry + pre;
       lcarry += __shfl_sync(0xffffffffu, pre, 31);
     }
+    // RD value: ((def + 1) << 1) | def_is_global_load, or 0 for ENTRY (a flat, predicated form of
+    // the lookups measured slower: 962 vs 915 us on C3, more instructions)
+    auto RD = [&](uint32_t reg) -> uint32_t {
+      const uint2 mt = MT[reg];
+      const uint32_t m = mt.x & lt;
+      const uint32_t j = 31u - __clz(m);
+      return m ? ((gbase + j + 1) << 1) | ((ldgmask >> j) & 1u) : mt.y;
+    };
     if (valid && r_pk(r) == PK_REG) ptrrd[g] = RD(r_ptr(r)) >> 1;
     const bool iscand = valid && (cls & (C_TRACED | C_CONV));
     const uint32_t cmask = __ballot_sync(0xffffffffu, iscand);
     if (iscand) {
       const uint64_t c = cb + __popc(cmask & lt);
-      ca.idx[c] = (uint32_t)g;
+      ca.idx[c] = g;
       ca.kernel[c] = W.kernel;
       reinterpret_cast<uint4*>(ca.rec)[c] = make_uint4(r.w0, r.w1, r.w2, (uint32_t)r.w3);
       const uint32_t base = r_s0(r);
@@ -386,16 +393,16 @@ __global__ void __launch_bounds__(kWarps * 32) k_resolve(const Rec* __restrict__
 #pragma unroll
         for (int t = 0; t < q; t++) dup |= d[t] == d[q];
         if (dup) continue;
-        const uint32_t off = d[q] - (uint32_t)W.start;  // loads of this window: shared counters
+        const uint32_t off = d[q] - W.start;  // loads of this window: shared counters
         if (off < W.len) atomicAdd(NA + (off >> 1), 1u << ((off & 1u) << 4));
         else atomicAdd(narith + d[q], 1u);
       }
     }
     __syncwarp();
     {
-      const uint32_t v = (uint32_t)((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
-      for (uint32_t q = 0; q < nq; q++) { atomicMax(&T[dst + q], v); M[dst + q] = 0; }
-      for (uint32_t q = 0; q < nq2; q++) { atomicMax(&T[dst2 + q], v); M[dst2 + q] = 0; }
+      const uint32_t v = ((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
+      for (uint32_t q = 0; q < nq; q++) { atomicMax(&MT[dst + q].y, v); MT[dst + q].x = 0; }
+      for (uint32_t q = 0; q < nq2; q++) { atomicMax(&MT[dst2 + q].y, v); MT[dst2 + q].x = 0; }
     }
     __syncwarp();
   }
@@ -692,28 +699,58 @@ __global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint
 }
 
 // one CTA: exclusive prefixes of the tile sums, sites and chains as separate u64 counters;
-// tot[0] = chain-pool entries, tot[1] = sites
+// tot[0] = chain-pool entries, tot[1] = sites. Warp w owns a contiguous segment of the tiles: its
+// lanes sum the segment with coalesced loads, one warp scans the 32 segment totals, then each
+// warp re-reads its segment 32 tiles at a time and writes the prefixes (warp scans, no barriers
+// per tile group).
+__device__ __forceinline__ void warp_incl_pair(unsigned long long& a, unsigned long long& b) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long x = __shfl_up_sync(0xffffffffu, a, o), y = __shfl_up_sync(0xffffffffu, b, o);
+    if (lane >= o) { a += x; b += y; }
+  }
+}
 __global__ void __launch_bounds__(1024) k_tile_prefix(const unsigned long long* __restrict__ tsum, uint64_t nt,
                                                       unsigned long long* __restrict__ pre_s,
                                                       unsigned long long* __restrict__ pre_c,
                                                       unsigned long long* __restrict__ tot) {
-  unsigned long long cs = 0, cc = 0;
-  for (uint64_t b = 0; b < nt; b += 1024) {
-    const uint64_t i = b + threadIdx.x;
-    const unsigned long long v = i < nt ? tsum[i] : 0;
-    unsigned long long ts, tc;
-    const unsigned long long es = block_excl64<1024>(v & 0xffffffffull, &ts);
-    const unsigned long long ec = block_excl64<1024>(v >> 32, &tc);
-    if (i < nt) {
-      pre_s[i] = cs + es;
-      pre_c[i] = cc + ec;
-    }
-    cs += ts;
-    cc += tc;
+  __shared__ unsigned long long ws[32], wc[32];
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  const uint64_t seg = (nt + 31) / 32, a = min(nt, warp * seg), e = min(nt, a + seg);
+  unsigned long long ls = 0, lc = 0;
+  for (uint64_t i = a + lane; i < e; i += 32) {
+    const unsigned long long v = tsum[i];
+    ls += v & 0xffffffffull;
+    lc += v >> 32;
   }
-  if (threadIdx.x == 0) {
-    tot[0] = cc;
-    tot[1] = cs;
+  for (int o = 16; o; o >>= 1) {
+    ls += __shfl_xor_sync(0xffffffffu, ls, o);
+    lc += __shfl_xor_sync(0xffffffffu, lc, o);
+  }
+  if (lane == 0) { ws[warp] = ls; wc[warp] = lc; }
+  __syncthreads();
+  if (warp == 0) {
+    unsigned long long x = ws[lane], y = wc[lane];
+    const unsigned long long x0 = x, y0 = y;
+    warp_incl_pair(x, y);
+    ws[lane] = x - x0;  // exclusive prefix of segment `lane`
+    wc[lane] = y - y0;
+    if (lane == 31) { tot[0] = y; tot[1] = x; }
+  }
+  __syncthreads();
+  unsigned long long rs = ws[warp], rc = wc[warp];  // running prefix of this warp's segment
+  for (uint64_t i0 = a; i0 < e; i0 += 32) {
+    const uint64_t i = i0 + lane;
+    const unsigned long long v = i < e ? tsum[i] : 0ull;
+    unsigned long long s_ = v & 0xffffffffull, c_ = v >> 32;
+    warp_incl_pair(s_, c_);
+    if (i < e) {
+      pre_s[i] = rs + s_ - (v & 0xffffffffull);
+      pre_c[i] = rc + c_ - (v >> 32);
+    }
+    rs += __shfl_sync(0xffffffffu, s_, 31);
+    rc += __shfl_sync(0xffffffffu, c_, 31);
   }
 }
 
@@ -788,13 +825,21 @@ __global__ void __launch_bounds__(kCT) k_write(const Rec* __restrict__ rec, cons
       s.a0 = (int32_t)gt.g[ca.grp[c]].nall;
     }
     if (rule == GS_CONV) { s.depth = 0; s.term_kind = GS_T_NONE; s.term_value = 0; }
-    if (so < site_cap) sites[so] = s;
+    if (so < site_cap) {  // two 16-byte stores (gs_site is 32 bytes, 32-byte aligned)
+      static_assert(sizeof(gs_site) == 32, "site layout");
+      uint4 v[2];
+      memcpy(v, &s, 32);
+      uint4* d = reinterpret_cast<uint4*>(sites + so);
+      d[0] = v[0];
+      d[1] = v[1];
+    }
     so++;
   }
 }
 
+
 // entries [g0, g1) of the group and offset tables, [r0, r1) of the root table (the regions of the
-// detected kernels)
+// detected kernels); runs on a side stream, concurrently with k_summary .. k_resolve
 __global__ void k_init_groups(GroupTable gt, uint64_t g0, uint64_t g1, uint64_t r0, uint64_t r1) {
   const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   if (g0 + i < g1) {
@@ -912,6 +957,11 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   const uint32_t D = c->cfg.trace_depth;
   c->detected = false;
   const bool cons = c->cfg.join_mode == GS_JOIN_CONSUMER;
+  if (!c->side_stream) {
+    GS_CUDA(c, cudaStreamCreateWithFlags(&c->side_stream, cudaStreamNonBlocking));
+    GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+  }
   // tile sums, their exclusive prefixes (sites, chains) and the two totals, carved from cand.choff
   // (3 x ceil(NC / 256) u64 + 2)
   const uint64_t ntile = (nc + kCT - 1) / kCT;
@@ -936,6 +986,18 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   };
   // everything up to the speculative write and the read-backs (no allocation in here)
   const auto enqueue = [&]() -> gs_status {
+    if (nc) {  // the hash-table regions of kernels [kb, ke), zeroed on a side stream meanwhile
+      const uint64_t g0 = c->kh_h[kb].gofs, r0 = c->kh_h[kb].rofs;
+      const uint64_t g1 = ke < c->n_kernels ? c->kh_h[ke].gofs : c->grp.gtot;
+      const uint64_t r1 = ke < c->n_kernels ? c->kh_h[ke].rofs : c->grp.rtot;
+      const uint64_t ni = std::max(g1 - g0, r1 - r0);
+      GS_CUDA(c, cudaEventRecord(c->ev_fork, st));
+      GS_CUDA(c, cudaStreamWaitEvent(c->side_stream, c->ev_fork, 0));
+      k_init_groups<<<(uint32_t)((ni + 255) / 256), 256, 0, c->side_stream>>>(c->grp, g0, g1, r0, r1);
+      count_launch();
+      GS_CUDA(c, cudaGetLastError());
+      GS_CUDA(c, cudaEventRecord(c->ev_join, c->side_stream));
+    }
     GS_CUDA(c, cudaMemsetAsync(c->d_kstats, 0, (uint64_t)c->n_kernels * sizeof(gs_kernel_stats), st));
     if (nw) {
       GS_CUDA(c, cudaMemsetAsync(c->d_wsum + w0, 0, (uint64_t)nw * 4, st));
@@ -944,7 +1006,8 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
                                              c->d_wev, c->d_narith, c->d_kstats, c->win); count_launch();
       GS_CUDA(c, cudaGetLastError());
-      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win); count_launch();
+      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win);
+      count_launch();
       GS_CUDA(c, cudaGetLastError());
       // candidate arrays are indexed relative to c0
       k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop,
@@ -957,13 +1020,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       if (cs != GS_OK) return cs;
     }
     if (nc) {
-      // the hash-table regions of kernels [kb, ke)
-      const uint64_t g0 = c->kh_h[kb].gofs, r0 = c->kh_h[kb].rofs;
-      const uint64_t g1 = ke < c->n_kernels ? c->kh_h[ke].gofs : c->grp.gtot;
-      const uint64_t r1 = ke < c->n_kernels ? c->kh_h[ke].rofs : c->grp.rtot;
-      const uint64_t ni = std::max(g1 - g0, r1 - r0);
-      k_init_groups<<<(uint32_t)((ni + 255) / 256), 256, 0, st>>>(c->grp, g0, g1, r0, r1); count_launch();
-      GS_CUDA(c, cudaGetLastError());
+      GS_CUDA(c, cudaStreamWaitEvent(st, c->ev_join, 0));
       const uint32_t gridc = (uint32_t)((nc + 255) / 256);
       k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->d_kstats);
       count_launch();

@@ -698,22 +698,102 @@ bool is_instr_line(Sv t) {
   return false;
 }
 
+// Pass 1 in parallel: only lines containing one of these can change the segment state (the
+// header state machine below), plus the first instruction line of a module without headers.
+struct Cand {
+  size_t b, e;  // line [b, e)
+  long lineno;  // 1-based
+};
+void find_candidates(const char* text, size_t b0, size_t e0, std::vector<Cand>* out, long* nlines) {
+  static const char* const pats[] = {"Function", "REG:", "code for sm_", ".target", ".text."};
+  std::vector<size_t> hits;
+  for (const char* pt : pats) {
+    const size_t m = strlen(pt);
+    size_t q = b0;
+    while (q < e0) {
+      const void* f = memmem(text + q, e0 - q, pt, m);
+      if (!f) break;
+      const size_t at = (size_t)((const char*)f - text);
+      hits.push_back(at);
+      q = at + 1;
+    }
+  }
+  // the first instruction line of the range (a module whose instructions precede any header)
+  for (size_t q = b0; q < e0;) {
+    const char* nl = (const char*)memchr(text + q, '\n', e0 - q);
+    const size_t e = nl ? (size_t)(nl - text) : e0;
+    Sv t = trim(Sv{text + q, e - q});
+    if (t.n && !starts(t, "//##") && is_instr_line(t)) { hits.push_back(q); break; }
+    q = e + 1;
+  }
+  std::sort(hits.begin(), hits.end());
+  // lines of the hits (deduplicated), with line numbers relative to b0
+  long line = 0;
+  size_t pos = b0, lb = b0;  // lb: start of the line holding pos
+  size_t last_b = ~(size_t)0;
+  for (size_t h : hits) {
+    while (pos < h) {  // advance to the line of h, counting newlines
+      const char* nl = (const char*)memchr(text + pos, '\n', h - pos);
+      if (!nl) { pos = h; break; }
+      line++;
+      pos = (size_t)(nl - text) + 1;
+      lb = pos;
+    }
+    if (lb == last_b) continue;
+    const char* nl = (const char*)memchr(text + lb, '\n', e0 - lb);
+    out->push_back(Cand{lb, nl ? (size_t)(nl - text) : e0, line});
+    last_b = lb;
+  }
+  // total lines of the range: newlines after pos
+  for (size_t q = pos; q < e0;) {
+    const char* nl = (const char*)memchr(text + q, '\n', e0 - q);
+    if (!nl) break;
+    line++;
+    q = (size_t)(nl - text) + 1;
+  }
+  *nlines = line;
+}
+
 }  // namespace
 
 bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedKernel>* out, std::string* err) {
-  // pass 1: segments
+  // pass 1: segments. The ranges (cut after a newline) are scanned in parallel for candidate
+  // lines; the header state machine then runs over the candidates in text order, exactly as it
+  // would over every line (the other lines take none of its branches).
+  // ranges of at least 1 MB (GS_PARSE_RANGE_BYTES overrides it: tests cut tiny inputs finely)
+  static const size_t min_range = [] {
+    const char* v = getenv("GS_PARSE_RANGE_BYTES");
+    return v && atoll(v) > 0 ? (size_t)atoll(v) : (size_t)1 << 20;
+  }();
+  const int nr = (int)std::max<size_t>(1, std::min<size_t>((size_t)n_threads, len / min_range + 1));
+  std::vector<size_t> cut(nr + 1, len);
+  cut[0] = 0;
+  for (int r = 1; r < nr; r++) {
+    size_t q = std::max(cut[r - 1], len * (size_t)r / (size_t)nr);
+    const char* nl = q < len ? (const char*)memchr(text + q, '\n', len - q) : nullptr;
+    cut[r] = nl ? (size_t)(nl - text) + 1 : len;
+  }
+  std::vector<std::vector<Cand>> cands(nr);
+  std::vector<long> nlines(nr, 0);
+  {
+    std::vector<std::thread> th;
+    for (int r = 1; r < nr; r++)
+      th.emplace_back([&, r]() { find_candidates(text, cut[r], cut[r + 1], &cands[r], &nlines[r]); });
+    find_candidates(text, cut[0], cut[1], &cands[0], &nlines[0]);
+    for (auto& t : th) t.join();
+  }
   std::vector<Segment> segs;
   std::map<std::string, int> res_regs;  // cuobjdump -res-usage: " Function <name>:" / "  REG:N ..." (R38k)
   std::string res_fn;
   int sm = 100;
-  long lineno = 1;
-  size_t p = 0;
-  while (p < len) {
-    const char* nl = (const char*)memchr(text + p, '\n', len - p);
-    size_t e = nl ? (size_t)(nl - text) : len;
-    Sv t = trim(Sv{text + p, e - p});
-    size_t at;
-    if (t.n) {
+  long line0 = 1;  // line number of the first line of range r
+  for (int r = 0; r < nr; r++) {
+    for (const Cand& cd : cands[r]) {
+      const size_t p = cd.b, e = cd.e;
+      const long lineno = line0 + cd.lineno;
+      Sv t = trim(Sv{text + p, e - p});
+      size_t at;
+      if (!t.n) continue;
       if (starts(t, "Function ") && t[t.n - 1] == ':' && !contains(t, "Function :")) {
         res_fn.assign(t.p + 9, t.n - 10);
       } else if (!res_fn.empty() && starts(t, "REG:")) {
@@ -725,31 +805,30 @@ bool parse_sass(const char* text, size_t len, int n_threads, std::vector<ParsedK
         sm = atoi(std::string(t.p + at + 3, t.n - at - 3).c_str());
       } else if (contains(t, "Function :", &at) || is_fn_label(t)) {
         if (!segs.empty()) segs.back().end = p;
-        Segment s;
-        s.begin = e + 1 > len ? len : e + 1;
-        s.end = len;
-        s.first_line = lineno + 1;
-        s.sm = sm;
+        Segment sg;
+        sg.begin = e + 1 > len ? len : e + 1;
+        sg.end = len;
+        sg.first_line = lineno + 1;
+        sg.sm = sm;
         Sv nm = is_fn_label(t) ? Sv{t.p + 6, t.n - 7} : trim(Sv{t.p + at + 10, t.n - at - 10});
-        s.name.assign(nm.p, nm.n);
-        s.header = true;
-        auto rr = res_regs.find(s.name);
-        s.regcount = rr == res_regs.end() ? -1 : rr->second;
-        segs.push_back(s);
+        sg.name.assign(nm.p, nm.n);
+        sg.header = true;
+        auto rr = res_regs.find(sg.name);
+        sg.regcount = rr == res_regs.end() ? -1 : rr->second;
+        segs.push_back(sg);
       } else if (segs.empty() && !starts(t, "//##") && is_instr_line(t)) {
-        Segment s;  // instructions before any Function header: one anonymous kernel
-        s.begin = 0;
-        s.end = len;
-        s.first_line = 1;
-        s.sm = sm;
-        s.name = "<anonymous>";
-        s.header = false;
-        s.regcount = -1;
-        segs.push_back(s);
+        Segment sg;  // instructions before any Function header: one anonymous kernel
+        sg.begin = 0;
+        sg.end = len;
+        sg.first_line = 1;
+        sg.sm = sm;
+        sg.name = "<anonymous>";
+        sg.header = false;
+        sg.regcount = -1;
+        segs.push_back(sg);
       }
     }
-    p = e + 1;
-    lineno++;
+    line0 += nlines[r];
   }
   // a later "code for"/".target" line inside a segment applies to the next Function only; the
   // per-segment sm was captured when its header was seen.

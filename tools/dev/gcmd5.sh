@@ -1,0 +1,5 @@
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_multirank.py -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1; echo TESTS $? >> gpurun_out/gpu_tests.log
+GS_TIMING=1 python tools/bench_detect.py --cpu-scale 0.001 > gpurun_out/detect.log 2>&1
+timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,smsp__inst_executed.sum --clock-control none -k regex:"k_" -c 12 --csv --log-file gpurun_out/det_launch4.csv python tools/bench_detect.py --steps 1 --cpu-scale 0.001 > gpurun_out/ncu_det.log 2>&1
+tail -3 gpurun_out/gpu_tests.log; grep gs_load gpurun_out/detect.log; tail -1 gpurun_out/detect.log | cut -c1-200

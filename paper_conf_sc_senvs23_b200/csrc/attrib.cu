@@ -489,8 +489,9 @@ __device__ __forceinline__ bool is_hot(uint32_t x, const Hot& h) {
 
 template <bool P16, uint32_t NCT>
 __device__ __noinline__ uint32_t rare_w(const uint4* __restrict__ s4, uint64_t i, uint32_t nv, Win W, uint32_t* tab,
-                                        uint32_t flag, uint32_t am, const Spill* sS, Hot hot) {
-  const Spill S = *sS;
+                                        uint32_t flag, uint32_t am, const Spill S, Hot hot) {
+  // (S by value: with the pointer, nvcc specialised the call to the one shared-memory state of its
+  // single caller and the WINDOW kernel's register allocation came out 4% slower on C4)
   uint32_t bad = 0;
   for (uint32_t u = 0; u < nv; u++) {
     const uint4 v = __ldg(s4 + i + (uint64_t)u * NCT);
@@ -583,14 +584,14 @@ __device__ __forceinline__ uint32_t count_span_w(const uint4* __restrict__ s4, u
     }
     const uint32_t flag = HOT ? hot_w_skew<P16>(w, W, tab, spare, hot, c) : hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, kVec, W, tab, flag, am, sS, hot);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, kVec, W, tab, flag, am, *sS, hot);
   }
   for (; i < i1; i += NCT) {
     const uint4 v = __ldg(s4 + i);
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
     const uint32_t flag = HOT ? hot_w_skew<P16>(w, W, tab, spare, hot, c) : hot_w<P16>(w, W, tab, spare);
     const uint32_t am = __activemask();
-    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, 1, W, tab, flag, am, sS, hot);
+    if (__any_sync(am, flag)) bad += rare_w<P16, NCT>(s4, i, 1, W, tab, flag, am, *sS, hot);
   }
   if (HOT) {  // the item's hot counts, one L2 reduction per hot word and thread
     const Spill S = *sS;
@@ -1000,38 +1001,46 @@ __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, u
 // ---------------------------------------------------------------------- PARTITION
 // For streams without locality (e.g. samples in random order): a WINDOW would see most samples
 // outside any window (L2 atomics, ~0.12 T samples/s). Instead the samples are first partitioned by
-// bucket = slot >> bshift (2^bshift slots, one shared-memory table), then every bucket is counted
-// with its own window, where every sample is inside:
+// bucket = compact bin >> kPBits (2^kPBits bins, one shared-memory table of 32-bit counters), then
+// every bucket is counted in its own table, where every sample is inside. The partitioned copy
+// holds only the bin's offset inside its bucket, 16 bits per sample, so the two passes after the
+// count move 4 + 2 + 2 bytes per sample instead of 4 + 4 + 4:
 //   k_pcount   per CTA chunk: samples per bucket (shared counters), invalid words counted
-//   k_pscan    one CTA: bucket regions (4-word aligned starts) and each chunk's offset per bucket
-//   k_pscatter per CTA chunk, tiles of 8K samples: counting sort of the tile in shared memory by
-//              bucket, runs written to the bucket regions (coalesced within a run)
-//   k_pcount_hist  per CTA a contiguous share of the partitioned array, bucket by bucket
-constexpr int kPT = 1024;                  // threads of the partition kernels
-constexpr uint32_t kPMaxBuckets = 2048;
-constexpr uint32_t kPTile = kPT * 8;       // samples per scatter tile
+//   k_pscan    one CTA: bucket regions (8-entry aligned starts, padding 0xFFFF) and each chunk's
+//              offset per bucket
+//   k_pscatter per CTA chunk, tiles of NT x 8 samples: counting sort of the tile in shared memory
+//              by bucket, the 16-bit offsets written to the bucket regions (coalesced within a run)
+//   k_pbucket_hist  per CTA a contiguous share of the partitioned array, bucket by bucket: one
+//              non-returning shared atomic per sample, the table flushed into H at bucket switches
+#ifndef GS_PBITS
+#define GS_PBITS 15
+#endif
+constexpr uint32_t kPBits = GS_PBITS;          // bins per bucket = 2^kPBits (offsets fit 16 bits)
+static_assert(kPBits <= 15, "bucket offsets are 16-bit, 0xFFFF is the padding");
+constexpr uint32_t kPBins = 1u << kPBits;
+constexpr uint16_t kPPad = 0xffffu;            // padding entry (>= kPBins when kPBits < 16: never counted)
+constexpr int kPT = 1024;                      // threads of k_pcount / k_pscan
+constexpr uint32_t kPMaxBuckets = 1024;        // B < kPMaxBuckets (+1 for the invalid words): P * R < 2^25 at kPBits = 15
+constexpr uint32_t kPSub = 4;                  // rank counters per bucket (k_pscatter)
+#ifndef GS_PST
+#define GS_PST 1024
+#endif
+constexpr int kPST = GS_PST;                   // threads of k_pscatter
+#ifndef GS_PV
+#define GS_PV 16
+#endif
+constexpr uint32_t kPV = GS_PV;                // samples per thread per scatter tile
+constexpr uint32_t kSTile = kPST * kPV;        // samples per scatter tile
+#ifndef GS_PHT
+#define GS_PHT 1024
+#endif
+constexpr int kPHT = GS_PHT;                   // threads of k_pbucket_hist
 
-__device__ __forceinline__ uint32_t bucket_of(uint32_t w, Div dv, uint32_t bshift) { return divq(w, dv) >> bshift; }
-// bucket = w / (R << bshift) exactly for every 32-bit w, as one multiply-high (division by an
-// invariant integer, Granlund & Montgomery 1994, Fig. 4.1): l = ceil(log2 D), m = floor(2^32 (2^l - D) / D) + 1,
-// t = mulhi(m, w), q = (t + ((w - t) >> 1)) >> (l - 1); D >= 2
-struct BDiv {
-  uint32_t m, sh;
-};
-inline BDiv make_bdiv(uint32_t nr, uint32_t bshift) {
-  const uint64_t D = (uint64_t)nr << bshift;
-  uint32_t l = 0;
-  while ((1ull << l) < D) l++;
-  return BDiv{(uint32_t)((((1ull << 32) * ((1ull << l) - D)) / D) + 1), l - 1};
-}
-__device__ __forceinline__ uint32_t bucket_m(uint32_t w, BDiv b) {
-  const uint32_t t = __umulhi(b.m, w);
-  return (t + ((w - t) >> 1)) >> b.sh;
-}
+__device__ __forceinline__ uint32_t pbucket(uint32_t w) { return w >> kPBits; }
 
 __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
-                                                uint32_t pnr, BDiv dv, uint32_t B,
-                                                uint32_t* __restrict__ cnt, unsigned long long* d_n_invalid) {
+                                                uint32_t pnr, uint32_t B, uint32_t* __restrict__ cnt,
+                                                unsigned long long* d_n_invalid) {
   __shared__ uint32_t h[kPMaxBuckets];
   for (uint32_t b = threadIdx.x; b < B; b += kPT) h[b] = 0;
   __syncthreads();
@@ -1043,14 +1052,15 @@ __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, 
   for (; i + 3 * kPT < e4; i += 4 * kPT) {
     uint4 v[4];
 #pragma unroll
-    for (int u = 0; u < 4; u++) v[u] = __ldg(s4 + i + u * kPT);
+    for (int u = 0; u < 4; u++) v[u] = ld_stream(s4 + i + u * kPT);
 #pragma unroll
     for (int u = 0; u < 4; u++) {
       const uint32_t w[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        if (w[q] < pnr) atomicAdd(&h[bucket_m(w[q], dv)], 1u);
-        else bad++;
+        const bool ok = w[q] < pnr;
+        if (ok) atomicAdd(&h[pbucket(w[q])], 1u);
+        bad += ok ? 0u : 1u;
       }
     }
   }
@@ -1059,12 +1069,12 @@ __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, 
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      if (w[q] < pnr) atomicAdd(&h[bucket_m(w[q], dv)], 1u);
+      if (w[q] < pnr) atomicAdd(&h[pbucket(w[q])], 1u);
       else bad++;
     }
   }
   for (uint64_t j = e4 * 4 + threadIdx.x; j < e; j += kPT) {  // the stream's last < 4 words
-    if (s[j] < pnr) atomicAdd(&h[bucket_m(s[j], dv)], 1u);
+    if (s[j] < pnr) atomicAdd(&h[pbucket(s[j])], 1u);
     else bad++;
   }
   count_invalid(bad, d_n_invalid);
@@ -1072,10 +1082,10 @@ __global__ void __launch_bounds__(kPT) k_pcount(const uint32_t* __restrict__ s, 
   for (uint32_t b = threadIdx.x; b < B; b += kPT) cnt[(uint64_t)blockIdx.x * B + b] = h[b];
 }
 
-// bstart[b]: first word of bucket b's region (4-aligned), bstart[B] = end; off[c][b] = where chunk c
-// writes its bucket-b samples (in place of cnt)
+// bstart[b]: first entry of bucket b's region (8-aligned: whole uint4 of 16-bit entries),
+// bstart[B] = end; off[c][b] = where chunk c writes its bucket-b samples (in place of cnt)
 __global__ void __launch_bounds__(kPT) k_pscan(uint32_t* __restrict__ cnt, uint32_t nchunk, uint32_t B,
-                                               unsigned long long* __restrict__ bstart, uint32_t* __restrict__ out) {
+                                               unsigned long long* __restrict__ bstart, uint16_t* __restrict__ out) {
   __shared__ unsigned long long tot[kPMaxBuckets], pre[kPMaxBuckets];
   for (uint32_t b = threadIdx.x; b < B; b += kPT) {
     unsigned long long t = 0;
@@ -1084,12 +1094,12 @@ __global__ void __launch_bounds__(kPT) k_pscan(uint32_t* __restrict__ cnt, uint3
     tot[b] = t;
   }
   __syncthreads();
-  if (threadIdx.x < 32) {  // warp scan of the 4-aligned region sizes, 64 buckets per lane at most
+  if (threadIdx.x < 32) {  // warp scan of the 8-aligned region sizes, 64 buckets per lane at most
     const uint32_t lane = threadIdx.x, per = (B + 31) / 32;
     unsigned long long sum = 0;
     for (uint32_t q = 0; q < per; q++) {
       const uint32_t b = lane * per + q;
-      if (b < B) sum += (tot[b] + 3) & ~3ull;
+      if (b < B) sum += (tot[b] + 7) & ~7ull;
     }
     unsigned long long inc = sum;
     for (int o = 1; o < 32; o <<= 1) {
@@ -1102,15 +1112,15 @@ __global__ void __launch_bounds__(kPT) k_pscan(uint32_t* __restrict__ cnt, uint3
       if (b < B) {
         pre[b] = p;
         bstart[b] = p;
-        p += (tot[b] + 3) & ~3ull;
+        p += (tot[b] + 7) & ~7ull;
       }
     }
     if (lane == 31) bstart[B] = inc;
   }
   __syncthreads();
   for (uint32_t b = threadIdx.x; b < B; b += kPT) {
-    const unsigned long long e = pre[b] + tot[b], e4 = b + 1 < B ? pre[b + 1] : (e + 3) & ~3ull;
-    for (unsigned long long q = e; q < e4; q++) out[q] = 0xffffffffu;  // padding: invalid words
+    const unsigned long long e = pre[b] + tot[b], e8 = (e + 7) & ~7ull;
+    for (unsigned long long q = e; q < e8; q++) out[q] = kPPad;  // padding entries
     unsigned long long p = 0;
     for (uint32_t c = 0; c < nchunk; c++) {
       const uint32_t x = cnt[(uint64_t)c * B + b];
@@ -1120,86 +1130,99 @@ __global__ void __launch_bounds__(kPT) k_pscan(uint32_t* __restrict__ cnt, uint3
   }
 }
 
-// the 8 contiguous words of thread t in the tile at t0 (two 128-bit loads when the tile is whole)
-__device__ __forceinline__ void load8(const uint32_t* __restrict__ s, uint64_t t0, uint64_t e, uint32_t (&w)[8]) {
-  const uint64_t base = t0 + (uint64_t)threadIdx.x * 8;
-  if (base + 8 <= e) {
-    const uint4 v0 = __ldg(reinterpret_cast<const uint4*>(s + base));
-    const uint4 v1 = __ldg(reinterpret_cast<const uint4*>(s + base) + 1);
-    w[0] = v0.x; w[1] = v0.y; w[2] = v0.z; w[3] = v0.w; w[4] = v1.x; w[5] = v1.y; w[6] = v1.z; w[7] = v1.w;
-  } else {
-#pragma unroll
-    for (int q = 0; q < 8; q++) w[q] = base + q < e ? s[base + q] : 0xffffffffu;
+// Counting sort of each tile of kSTile samples by bucket. The tiles of the CTA's chunk arrive in
+// shared memory by TMA bulk copies (cp.async.bulk, double-buffered: the copy of tile i + 1 runs
+// while tile i is sorted; no registers hold the next tile). Three barriers per tile: ranks | scan
+// (resets the rank counters, advances the bucket cursors) | stage | write-out. The write-out reads
+// each staged word, its bucket's destination base dst[b] = cursor - tile offset, and stores the
+// 16-bit offset (consecutive threads of a run store consecutive entries).
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  if (!bytes) {  // a tile of < 4 words: nothing to copy, complete the phase
+    mbar_arrive(bar);
+    return;
   }
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
 }
-
-// Four barriers per tile: ranks | scan (also resets the rank counters and advances the bucket
-// cursors by the previous tile's counts) | stage | write-out. The write-out recomputes each
-// sample's bucket and reads its destination base dst[b] = cursor - tile offset.
-template <int NT>
-__global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
-                                                  uint32_t pnr, BDiv dv, uint32_t B,
-                                                  const uint32_t* __restrict__ off,
-                                                  const unsigned long long* __restrict__ bstart,
-                                                  uint32_t* __restrict__ out) {
-  __shared__ unsigned long long dst[kPMaxBuckets];   // cursor of bucket b minus its tile offset
-  __shared__ uint32_t th[kPMaxBuckets], tcnt[kPMaxBuckets];
-  extern __shared__ uint32_t stage[];  // kPTile words (dynamic)
-  constexpr uint32_t kTile = NT * 8, BPT = kPMaxBuckets / NT;  // samples per tile, buckets per thread
+// Off: uint32_t when the partitioned array has < 2^32 entries (a 64-bit dst[] doubles the bank
+// conflicts of the write-out's random lookups), else unsigned long long.
+template <int NT, typename Off>
+__global__ void __launch_bounds__(NT, 1) k_pscatter(const uint32_t* __restrict__ s, uint64_t n, uint64_t chunk,
+                                                     uint32_t pnr, uint32_t B, const uint32_t* __restrict__ off,
+                                                     const unsigned long long* __restrict__ bstart,
+                                                     uint16_t* __restrict__ out) {
+  // Rank counters: kPSub per bucket, lane % kPSub picks one, so lanes of a warp that hold the same
+  // (Zipf-hot) bucket mostly hit different words and banks (one counter per bucket measured 6.6
+  // shared-memory wavefronts per warp-level rank atomic on C4-shuffled). Thread t scans bucket t.
+  static_assert(NT == kPMaxBuckets, "one bucket per scanning thread");
+  __shared__ uint32_t th[kPMaxBuckets * kPSub];
+  __shared__ uint16_t tcnt[kPMaxBuckets * kPSub];  // tile offset of (bucket, sub); < 2^16
+  __shared__ Off dst[kPMaxBuckets];                // cursor of bucket b minus its tile offset (mod 2^bits(Off))
   __shared__ uint32_t wsum[NT / 32];
-  __shared__ uint32_t nv_sh;
-  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-  const uint32_t bb = BPT * threadIdx.x;  // the buckets this thread scans: [bb, bb + BPT)
-  unsigned long long cur[BPT];            // their cursors (registers)
-#pragma unroll
-  for (uint32_t j = 0; j < BPT; j++) cur[j] = bb + j < B ? bstart[bb + j] + off[(uint64_t)blockIdx.x * B + bb + j] : 0;
-  for (uint32_t b = threadIdx.x; b < B; b += NT) th[b] = 0;
+  __shared__ __align__(8) uint64_t full[2];
+  constexpr uint32_t kTile = NT * kPV;  // samples per tile
+  static_assert(kPV % 8 == 0, "write-out in groups of eight, uint4 reads");
+  static_assert(kTile < 65536 && kPMaxBuckets * kPSub <= 65536, "packed counter/rank, 16-bit tile offsets");
+  extern __shared__ __align__(16) uint32_t dyn[];    // raw[2][kTile] (TMA destinations), stage[kTile]
+  uint32_t* const raw0 = dyn;
+  uint32_t* const stage = dyn + 2 * kTile;
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, sub = lane % kPSub;
+  const uint32_t bt = threadIdx.x;  // the bucket this thread scans
+  Off cur = bt < B ? (Off)(bstart[bt] + off[(uint64_t)blockIdx.x * B + bt]) : (Off)0;  // its cursor
+  for (uint32_t i = threadIdx.x; i < (B + 1) * kPSub; i += NT) th[i] = 0;
+  const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);  // a: a multiple of kTile
+  // whole 16-byte units of the tile at t0 go through TMA; the < 4 trailing words of the stream are
+  // read directly
+  const auto tma_words = [&](uint64_t t0) -> uint32_t { return (uint32_t)((min(e, t0 + kTile) - t0) & ~3ull); };
+  if (threadIdx.x == 0) {
+    mbar_init(&full[0], 1);
+    mbar_init(&full[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (a < e) bulk_g2s(raw0, s + a, 4 * tma_words(a), &full[0]);
+  }
   __syncthreads();
-  const uint64_t a = blockIdx.x * chunk, e = min(n, a + chunk);
-  uint32_t nw[8];
-  if (a < e) load8(s, a, e, nw);
-  for (uint64_t t0 = a; t0 < e; t0 += kTile) {
-    uint32_t w[8], bk[8], r[8];
-#pragma unroll
-    for (int q = 0; q < 8; q++) w[q] = nw[q];
-    if (t0 + kTile < e) load8(s, t0 + kTile, e, nw);  // next tile in flight during this one
-#pragma unroll
-    for (int q = 0; q < 8; q++) {  // branch-free: the bucket of every word, then the validity select
-      const uint32_t b = bucket_m(w[q], dv);
-      bk[q] = w[q] < pnr ? b : 0xffffffffu;
+  uint32_t it = 0;
+  for (uint64_t t0 = a; t0 < e; t0 += kTile, it++) {
+    const uint32_t buf = it & 1u;
+    const uint32_t* raw = raw0 + buf * kTile;
+    if (threadIdx.x == 0 && t0 + kTile < e) {  // the next tile into the other buffer (free: every
+      // thread passed barrier D of the previous tile, its last reader)
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      bulk_g2s(raw0 + (buf ^ 1u) * kTile, s + t0 + kTile, 4 * tma_words(t0 + kTile), &full[buf ^ 1u]);
     }
-    // ranks within the tile's buckets: one shared atomic per sample, and one per warp when the
-    // whole warp holds a single bucket (trace order)
-    const uint32_t bk_lane0 = __shfl_sync(0xffffffffu, bk[0], 0);  // outside any condition (all lanes)
-    const bool uni = __all_sync(0xffffffffu, bk[0] == bk[7] && bk[0] == bk_lane0 && bk[0] != 0xffffffffu);
-    bool same = true;
+    const uint32_t nt = tma_words(t0), nall = (uint32_t)(min(e, t0 + kTile) - t0);
+    mbar_wait(&full[buf], (it >> 1) & 1u);
+    // thread's words: uint4 (threadIdx.x + NT * u) of the tile
+    const auto word4 = [&](uint32_t u, uint32_t (&w)[4]) {
+      const uint32_t i = 4 * (threadIdx.x + NT * u);
+      if (i + 4 <= nt) {
+        const uint4 v = *reinterpret_cast<const uint4*>(raw + i);
+        w[0] = v.x; w[1] = v.y; w[2] = v.z; w[3] = v.w;
+      } else {
 #pragma unroll
-    for (int q = 1; q < 8; q++) same &= bk[q] == bk[0];
-    if (uni && __all_sync(0xffffffffu, same)) {
-      uint32_t r0 = 0;
-      if (lane == 0) r0 = atomicAdd(&th[bk[0]], 256u);
-      r0 = __shfl_sync(0xffffffffu, r0, 0) + 8 * lane;
+        for (int q = 0; q < 4; q++) w[q] = i + q < nt ? raw[i + q] : (i + q < nall ? s[t0 + i + q] : 0xffffffffu);
+      }
+    };
+    uint32_t rb[kPV];  // rb = counter << 16 | rank within the counter (invalid words: bucket B)
 #pragma unroll
-      for (int q = 0; q < 8; q++) r[q] = r0 + q;
-    } else if (__all_sync(0xffffffffu, bk[0] != 0xffffffffu && bk[1] != 0xffffffffu && bk[2] != 0xffffffffu &&
-                                          bk[3] != 0xffffffffu && bk[4] != 0xffffffffu && bk[5] != 0xffffffffu &&
-                                          bk[6] != 0xffffffffu && bk[7] != 0xffffffffu)) {
+    for (uint32_t u = 0; u < kPV / 4; u++) {
+      uint32_t w[4];
+      word4(u, w);
 #pragma unroll
-      for (int q = 0; q < 8; q++) r[q] = atomicAdd(&th[bk[q]], 1u);  // branch-free: all valid
-    } else {  // one shared atomic per valid sample
-#pragma unroll
-      for (int q = 0; q < 8; q++) r[q] = bk[q] != 0xffffffffu ? atomicAdd(&th[bk[q]], 1u) : 0u;
+      for (uint32_t q = 0; q < 4; q++) {
+        const uint32_t ci = (w[q] < pnr ? pbucket(w[q]) : B) * kPSub + sub;  // branch-free (a predicated
+        rb[4 * u + q] = (ci << 16) | atomicAdd(&th[ci], 1u);                    // atomic compiled to a branch)
+      }
     }
-    uint32_t vmask = 0;
-#pragma unroll
-    for (int q = 0; q < 8; q++) vmask |= bk[q] != 0xffffffffu ? 1u << q : 0u;
-    const bool allv = __all_sync(0xffffffffu, vmask == 0xffu);
     __syncthreads();  // A: ranks done (and the previous tile's write-out)
-    uint32_t x[BPT], v = 0;
+    uint32_t x[kPSub], v = 0;  // bucket bt's counters ([0, B]: B = the invalid words, staged last)
 #pragma unroll
-    for (uint32_t j = 0; j < BPT; j++) {
+    for (uint32_t j = 0; j < kPSub; j++) {
       x[j] = 0;
-      if (bb + j < B) { x[j] = th[bb + j]; th[bb + j] = 0; }
+      if (bt <= B) { x[j] = th[bt * kPSub + j]; th[bt * kPSub + j] = 0; }
       v += x[j];
     }
     uint32_t inc = v;
@@ -1210,7 +1233,9 @@ __global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s,
     }
     if (lane == 31) wsum[warp] = inc;
     __syncthreads();  // B
-    if (warp == 0) {
+    uint32_t wpre = 0;  // exclusive prefix of this warp's total (every warp scans the NT / 32
+                        // totals itself: no second barrier)
+    {
       const uint32_t y = lane < NT / 32 ? wsum[lane] : 0u;
       uint32_t yi = y;
 #pragma unroll
@@ -1218,82 +1243,121 @@ __global__ void __launch_bounds__(NT) k_pscatter(const uint32_t* __restrict__ s,
         const uint32_t z = __shfl_up_sync(0xffffffffu, yi, o);
         if (lane >= o) yi += z;
       }
-      if (lane < NT / 32) wsum[lane] = yi - y;
-      if (lane == 31) nv_sh = yi;
+      wpre = __shfl_sync(0xffffffffu, yi - y, warp);
     }
-    __syncthreads();  // C
-    uint32_t ex = wsum[warp] + inc - v;  // tile offset of bucket bb
+    uint32_t ex = wpre + inc - v;  // tile offset of bucket bt
+    if (bt <= B) {
+      dst[bt] = cur - (Off)ex;
+      cur += (Off)v;
 #pragma unroll
-    for (uint32_t j = 0; j < BPT; j++) {
-      if (bb + j < B) { tcnt[bb + j] = ex; dst[bb + j] = cur[j] - ex; cur[j] += x[j]; }
-      ex += x[j];
+      for (uint32_t j = 0; j < kPSub; j++) {
+        tcnt[bt * kPSub + j] = (uint16_t)ex;
+        ex += x[j];
+      }
     }
-    __syncthreads();  // D: offsets ready
-    if (allv) {
+    __syncthreads();  // C: offsets ready
 #pragma unroll
-      for (int q = 0; q < 8; q++) stage[tcnt[bk[q]] + r[q]] = w[q];
-    } else {
+    for (uint32_t u = 0; u < kPV / 4; u++) {  // loads of a group before its stores (stage / tcnt
+      uint32_t w[4], tc[4];                   // could alias for the compiler)
+      word4(u, w);
 #pragma unroll
-      for (int q = 0; q < 8; q++)
-        if (bk[q] != 0xffffffffu) stage[tcnt[bk[q]] + r[q]] = w[q];
+      for (uint32_t q = 0; q < 4; q++) tc[q] = tcnt[rb[4 * u + q] >> 16];
+#pragma unroll
+      for (uint32_t q = 0; q < 4; q++) stage[tc[q] + (rb[4 * u + q] & 0xffffu)] = w[q];
     }
-    __syncthreads();  // E: staged
-    const uint32_t nv = nv_sh;
-    for (uint32_t p = threadIdx.x; p < nv; p += NT) {  // the bucket is recomputed (ALU, not smem)
-      const uint32_t x = stage[p];
-      out[dst[bucket_m(x, dv)] + p] = x;
+    __syncthreads();  // D: staged
+    const uint32_t nv = tcnt[B * kPSub];  // the valid words of the tile
+#pragma unroll
+    for (uint32_t k0 = 0; k0 < kPV; k0 += 8) {  // eight entries per thread in flight
+      uint32_t y[8];
+      Off d[8];
+#pragma unroll
+      for (uint32_t k = 0; k < 8; k++) {
+        const uint32_t p = threadIdx.x + NT * (k0 + k);
+        y[k] = p < nv ? stage[p] : 0u;
+      }
+#pragma unroll
+      for (uint32_t k = 0; k < 8; k++) d[k] = dst[pbucket(y[k])];
+#pragma unroll
+      for (uint32_t k = 0; k < 8; k++) {
+        const uint32_t p = threadIdx.x + NT * (k0 + k);
+        if (p < nv) out[(Off)(d[k] + p)] = (uint16_t)(y[k] & (kPBins - 1u));
+      }
     }
   }
 }
 
-// per CTA: uint4 [c0, c1) of the partitioned array, bucket by bucket; every sample of bucket b is
-// inside its window [b << bshift, (b + 1) << bshift) (16-bit counters, drains only)
-template <bool P16>
-__global__ void __launch_bounds__(kPT, 1)
-    k_pcount_hist(const uint32_t* __restrict__ ps, const unsigned long long* __restrict__ bstart, uint32_t B,
-                  uint64_t chunk4, uint32_t P, uint32_t nr, Div dv, uint32_t bshift, int32_t* __restrict__ H,
-                  uint32_t tw) {
-  extern __shared__ uint32_t tab[];
-  __shared__ Spill sh_S;
-  for (uint32_t i = threadIdx.x; i < tw + 32; i += kPT) tab[i] = i < tw ? 0u : 1u;
-  if (threadIdx.x == 0) sh_S = Spill{P * nr, dv, H, nullptr, nullptr, 0};
+// per CTA: uint4 [c0, c1) of the partitioned array (8 entries each, never across buckets), bucket
+// by bucket; bucket b's entries are offsets of bins [b << kPBits, ...) (padding kPPad is counted
+// into a spare word). 32-bit counters: exact, no drains.
+__global__ void __launch_bounds__(kPHT, 1)
+    k_pbucket_hist(const uint16_t* __restrict__ ps, const unsigned long long* __restrict__ bstart, uint32_t B,
+                   uint64_t chunk4, uint32_t pnr, Div dv, int32_t* __restrict__ H) {
+  extern __shared__ uint32_t tab[];  // kPBins counters + 32 spare words
+  for (uint32_t i = threadIdx.x; i < kPBins + 32; i += kPHT) tab[i] = 0;
   __syncthreads();
   const uint4* s4 = reinterpret_cast<const uint4*>(ps);
-  const uint64_t end4 = bstart[B] / 4;
+  const uint64_t end4 = bstart[B] / 8;
   const uint64_t c0 = blockIdx.x * chunk4, c1 = min(end4, c0 + chunk4);
   if (c0 >= c1) return;
-  const uint32_t spare = tw + (threadIdx.x & 31u);
-  // first bucket touching c0: last b with bstart[b] / 4 <= c0
+  const uint32_t spare = kPBins + (threadIdx.x & 31u);
+  // first bucket touching c0: last b with bstart[b] / 8 <= c0
   uint32_t lo = 0, hi = B;
   while (hi - lo > 1) {
     const uint32_t mid = (lo + hi) >> 1;
-    if (bstart[mid] / 4 <= c0) lo = mid;
+    if (bstart[mid] / 8 <= c0) lo = mid;
     else hi = mid;
   }
-  uint32_t ws = 0xffffffffu;
-  Win W{0, 0};
-  uint32_t bad = 0;
+  const auto add8 = [&](const uint4 v) {
+    const uint32_t x[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      const uint32_t o0 = x[q] & 0xffffu, o1 = x[q] >> 16;
+      atomicAdd(tab + (o0 < kPBins ? o0 : spare), 1u);
+      atomicAdd(tab + (o1 < kPBins ? o1 : spare), 1u);
+    }
+  };
   for (uint32_t b = lo; b < B; b++) {
     const unsigned long long bs = bstart[b];
-    if (bs / 4 >= c1) break;
-    const unsigned long long we = bstart[b + 1];  // 4-aligned; the padding words hold ~0u (invalid)
-    const uint64_t a4 = c0 > bs / 4 ? c0 : (uint64_t)(bs / 4), e4 = c1 < we / 4 ? c1 : (uint64_t)(we / 4);
+    if (bs / 8 >= c1) break;
+    const uint64_t a4 = max(c0, (uint64_t)(bs / 8)), e4 = min(c1, (uint64_t)(bstart[b + 1] / 8));
     if (a4 >= e4) continue;
-    const uint32_t nws = b << bshift;
-    if (nws != ws) {
-      __syncthreads();
-      if (ws != 0xffffffffu) flush<P16>(tab, ws, nr, dv.row, W.lim, H, threadIdx.x, kPT);
-      __syncthreads();
-      ws = nws;
-      W = Win{ws * nr, min(1u << bshift, P - ws) * nr};
+    uint64_t i = a4 + threadIdx.x;
+    constexpr int kU = 4;  // 128-bit loads in flight per thread
+    for (; i + (kU - 1) * kPHT < e4; i += kU * kPHT) {
+      uint4 v[kU];
+#pragma unroll
+      for (int u = 0; u < kU; u++) v[u] = ld_stream(s4 + i + u * kPHT);
+#pragma unroll
+      for (int u = 0; u < kU; u++) add8(v[u]);
     }
-    // warps 1..31 count (kNct threads: the 16-bit exactness bound below), warp 0 only flushes
-    if (threadIdx.x >= 32) bad += count_span_w<P16, kNct>(s4, a4, e4, threadIdx.x - 32, W, tab, spare, &sh_S);
+    for (; i < e4; i += kPHT) add8(__ldg(s4 + i));
+    __syncthreads();
+    // flush bucket b into H and zero the table (the bins of bucket b are counted only by the CTAs
+    // whose range overlaps its region: L2 reductions)
+    const uint32_t base = b << kPBits, lim = min(kPBins, pnr - base);
+    if (dv.row == dv.d && (reinterpret_cast<uintptr_t>(H) & 7u) == 0) {  // compact rows: bin pairs
+      unsigned long long* H2 = reinterpret_cast<unsigned long long*>(H + base);  // base is even
+      uint2* t2 = reinterpret_cast<uint2*>(tab);
+      for (uint32_t i2 = threadIdx.x; 2 * i2 < lim; i2 += kPHT) {
+        const uint2 t = t2[i2];
+        if (t.x | t.y) {
+          t2[i2] = make_uint2(0u, 0u);
+          if (2 * i2 + 1 < lim) atomicAdd(H2 + i2, (unsigned long long)t.x | ((unsigned long long)t.y << 32));
+          else atomicAdd(H + base + 2 * i2, (int32_t)t.x);
+        }
+      }
+    } else {
+      for (uint32_t j = threadIdx.x; j < lim; j += kPHT) {
+        const uint32_t t = tab[j];
+        if (t) {
+          tab[j] = 0;
+          atomicAdd(H + hidx(base + j, dv), (int32_t)t);
+        }
+      }
+    }
+    __syncthreads();
   }
-  (void)bad;  // the padding words (~0u) are counted as invalid here and ignored: invalid samples
-              // were counted by k_pcount
-  __syncthreads();
-  if (ws != 0xffffffffu) flush<P16>(tab, ws, nr, dv.row, W.lim, H, threadIdx.x, kPT);
 }
 
 }  // namespace
@@ -1328,31 +1392,24 @@ gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_h
   return GS_OK;
 }
 
-// GS_HIST_PARTITION (see the kernels): partition by bucket, then count each bucket in its window.
+// GS_HIST_PARTITION (see the kernels): partition by bucket, then count each bucket in its table.
 // d_words is 16-byte aligned here (hist_run peeled the head); the histogram is already zeroed.
 gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,
                         unsigned long long* d_n_invalid, int dev_sms) {
   cudaStream_t st = c->stream;
   const uint32_t P = (uint32_t)c->n_instr, nr = c->cfg.n_reasons;
   const Div dv = make_div(nr, c->cfg.hist_row);
-  // bucket = 2^bshift slots whose 16-bit counters fit the largest table
-  uint32_t bshift = 1;
-  while (bshift < 30 && ((((uint64_t)2 << bshift) * nr + 1) / 2) <= kTableWords) bshift++;
-  uint32_t B = (uint32_t)(((uint64_t)P + (1ull << bshift) - 1) >> bshift);
-  if (B > kPMaxBuckets) return GS_E_RANGE;  // caller falls back to WINDOW (modules > 2048 tables)
-  const uint32_t tw = (uint32_t)(((((uint64_t)1 << bshift) * nr + 1) / 2 + 31) & ~31ull);
-#ifndef GS_PST
-#define GS_PST 1024
-#endif
-  constexpr int kPST = GS_PST;                  // scatter threads per CTA
-  constexpr uint32_t kSTile = kPST * 8;        // samples per scatter tile
+  const uint64_t pnr = (uint64_t)P * nr;
+  const uint32_t B = (uint32_t)((pnr + kPBins - 1) >> kPBits);
+  if (B >= kPMaxBuckets) return GS_E_RANGE;  // caller falls back to WINDOW (2^25 bins or more)
   const uint64_t nchunk = std::max<uint64_t>(
-      1, std::min<uint64_t>((uint64_t)dev_sms * (2048 / kPST), (n + kSTile - 1) / kSTile));
+      1, std::min<uint64_t>((uint64_t)dev_sms, (n + kSTile - 1) / kSTile));
   uint64_t chunk = (n + nchunk - 1) / nchunk;
-  chunk = (chunk + kPTile - 1) / kPTile * kPTile;  // whole tiles of either kernel (multiple of 4 words)
+  chunk = (chunk + kSTile - 1) / kSTile * kSTile;  // whole scatter tiles (a multiple of 4 words)
   const uint64_t nch = (n + chunk - 1) / chunk;
-  // scratch: counts/offsets [nch][B] u32, bucket starts [B + 1] u64, partitioned copy (+ padding)
-  const uint64_t need = nch * B * 4 + 256 + (B + 1) * 8 + 256 + (n + 4ull * B + 4) * 4;
+  // scratch: counts/offsets [nch][B] u32, bucket starts [B + 1] u64, partitioned 16-bit copy
+  // (+ padding to whole uint4 per bucket)
+  const uint64_t need = nch * B * 4 + 256 + (B + 1) * 8 + 256 + (n + 8ull * B + 8) * 2;
   if (c->part_bytes < need) {
     if (c->d_part) cudaFree(c->d_part);
     c->d_part = nullptr;
@@ -1365,26 +1422,26 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   p += (nch * B * 4 + 255) / 256 * 256;
   unsigned long long* bstart = reinterpret_cast<unsigned long long*>(p);
   p += ((B + 1) * 8 + 255) / 256 * 256;
-  uint32_t* ps = reinterpret_cast<uint32_t*>(p);
-  const BDiv bd = make_bdiv(nr, bshift);
-  k_pcount<<<(unsigned)nch, kPT, 0, st>>>(d_words, n, chunk, P * nr, bd, B, cnt, d_n_invalid);
+  uint16_t* ps = reinterpret_cast<uint16_t*>(p);
+  k_pcount<<<(unsigned)nch, kPT, 0, st>>>(d_words, n, chunk, (uint32_t)pnr, B, cnt, d_n_invalid);
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
-  GS_CUDA(c, cudaFuncSetAttribute(k_pscatter<kPST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSTile * 4)));
-  k_pscatter<kPST><<<(unsigned)nch, kPST, kSTile * 4, st>>>(d_words, n, chunk, P * nr, bd, B, cnt, bstart, ps);
+  const auto kern = n + 8ull * B + 8 < (1ull << 32) ? k_pscatter<kPST, uint32_t> : k_pscatter<kPST, unsigned long long>;
+  GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(3 * kSTile * 4)));
+  kern<<<(unsigned)nch, kPST, 3 * kSTile * 4, st>>>(d_words, n, chunk, (uint32_t)pnr, B, cnt, bstart, ps);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
-  const uint64_t total4 = (n + 4ull * B + 3) / 4;  // upper bound of the padded array in uint4
+  const uint64_t total4 = (n + 8ull * B + 7) / 8;  // upper bound of the padded array in uint4
   const uint64_t chunk4 = (total4 + dev_sms - 1) / dev_sms;
-  const size_t smem = (size_t)(tw + 32) * 4;
-  GS_CUDA(c, cudaFuncSetAttribute(k_pcount_hist<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  k_pcount_hist<true><<<(unsigned)dev_sms, kPT, smem, st>>>(ps, bstart, B, chunk4, P, nr, dv, bshift, d_hist, tw);
+  const size_t smem = (size_t)(kPBins + 32) * 4;
+  GS_CUDA(c, cudaFuncSetAttribute(k_pbucket_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  k_pbucket_hist<<<(unsigned)dev_sms, kPHT, smem, st>>>(ps, bstart, B, chunk4, (uint32_t)pnr, dv, d_hist);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   c->last_hist_mode = GS_HIST_PARTITION;
-  c->last_hist_bits = 16;
-  c->last_hist_table_words = tw;
+  c->last_hist_bits = 32;
+  c->last_hist_table_words = kPBins;
   return GS_OK;
 }
 

@@ -48,9 +48,20 @@ __device__ __forceinline__ Rec ld_rec_rw(const Rec* r, uint64_t i) {
 }
 __device__ __forceinline__ uint32_t reg_cap(uint32_t dst) { return dst < 256 ? 254u : 318u; }
 // The opcode-class table in shared memory: op_class() is a switch that compiles to a branch tree,
-// which a warp of mixed opcodes walks divergently for every record; one LDS replaces it.
+// which a warp of mixed opcodes walks divergently for every record; one LDS replaces it. The table
+// is evaluated at compile time and copied in with one load per entry (evaluating the switch in
+// every CTA's prologue was 13% of k_trace's instructions).
+struct ClsTable {
+  uint16_t v[OP_COUNT];
+};
+constexpr ClsTable make_cls_table() {
+  ClsTable t{};
+  for (uint32_t i = 0; i < OP_COUNT; i++) t.v[i] = (uint16_t)op_class(i);
+  return t;
+}
+__device__ const ClsTable g_cls = make_cls_table();
 __device__ __forceinline__ void opcls_init(uint16_t* t) {
-  for (uint32_t i = threadIdx.x; i < OP_COUNT; i += blockDim.x) t[i] = (uint16_t)op_class(i);
+  for (uint32_t i = threadIdx.x; i < OP_COUNT; i += blockDim.x) t[i] = __ldg(&g_cls.v[i]);
 }
 
 // f(q < nq, base + q) for the first four registers of a destination (unrolled: no divergent loop
@@ -339,8 +350,8 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restric
     const uint32_t nq = writes ? min(r_dstw(r), reg_cap(dst) + 1 - dst) : 0u;
     const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
     const uint32_t nq2 = reg_live(dst2) ? min(r_dstw(r), reg_cap(dst2) + 1 - dst2) : 0u;
-    for (uint32_t q = 0; q < nq; q++) atomicOr(&MT[dst + q].x, 1u << lane);
-    for (uint32_t q = 0; q < nq2; q++) atomicOr(&MT[dst2 + q].x, 1u << lane);
+    for_regs(dst, nq, [&](bool p, uint32_t x) { if (p) atomicOr(&MT[x].x, 1u << lane); });
+    if (nq2) for_regs(dst2, nq2, [&](bool p, uint32_t x) { if (p) atomicOr(&MT[x].x, 1u << lane); });
     const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
     __syncwarp();
     // loop depth: inclusive prefix of the event differences (R13); a window without loop events
@@ -399,10 +410,14 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restric
       }
     }
     __syncwarp();
-    {
+    {  // the chunk's last writer of a register (the highest lane of its mask) sets T and clears M;
+       // only that lane writes the entry, so no atomic is needed
       const uint32_t v = ((g + 1) << 1) | (op == OP_LDG ? 1u : 0u);
-      for (uint32_t q = 0; q < nq; q++) { atomicMax(&MT[dst + q].y, v); MT[dst + q].x = 0; }
-      for (uint32_t q = 0; q < nq2; q++) { atomicMax(&MT[dst2 + q].y, v); MT[dst2 + q].x = 0; }
+      const auto last = [&](bool p, uint32_t x) {
+        if (p && (MT[x].x >> lane) == 1u) MT[x] = make_uint2(0u, v);
+      };
+      for_regs(dst, nq, last);
+      if (nq2) for_regs(dst2, nq2, last);
     }
     __syncwarp();
   }
@@ -584,17 +599,29 @@ __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ k
   const uint32_t op = r_op(ri), cls = s_cls[op];
   const bool traced = (cls & C_TRACED) && (r_flags(ri) & F_HASMEM);
   const uint32_t base = r_s0(ri), brd = ca.base_rd[c];
-  if (!traced || op != OP_LDG) {
+  const bool act = traced && op == OP_LDG;
+  // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max, contiguity.
+  // Consecutive loads off one base definition (an unrolled loop body) share a group: the lanes of a
+  // warp with the same key insert it once and add their count with one atomic (the CAS probes were
+  // this kernel's longest stall).
+  const unsigned long long key = act ? group_key(base, brd, kernel) : ~0ull;
+  const uint32_t am = __activemask(), lane = threadIdx.x & 31u;
+  const uint32_t peers = __match_any_sync(am, key);
+  const uint32_t leader = __ffs(peers) - 1;
+  const KHash H = gt.kh[kernel];
+  GEnt* G = gt.g + H.gofs;
+  uint32_t slot = 0;
+  if (act && lane == leader) {
+    slot = hinsert<4>(&G->key, H.gmask, key);
+    atomicAdd(&G[slot].nload, (uint32_t)__popc(peers));
+  }
+  slot = __shfl_sync(am, slot, leader);
+  if (!act) {
     ca.grp[c] = 0xffffffffu;
     return;
   }
-  // key-group statistics (R3): n_loads, distinct offsets (all / 32-bit), min, max, contiguity
-  const KHash H = gt.kh[kernel];
-  GEnt* G = gt.g + H.gofs;
-  const uint32_t slot = hinsert<4>(&G->key, H.gmask, group_key(base, brd, kernel));
   ca.grp[c] = (uint32_t)(H.gofs + slot);
   GEnt* e = G + slot;
-  atomicAdd(&e->nload, 1u);
   const int32_t off = r_imm(ri);
   const bool is32 = r_aw(ri) == AW_32;
   OEnt* O = gt.o + H.gofs;

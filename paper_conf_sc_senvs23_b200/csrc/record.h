@@ -20,8 +20,10 @@
 
 #ifdef __CUDACC__
 #define GS_HD __host__ __device__ __forceinline__
+#define GS_HDC __host__ __device__ constexpr
 #else
 #define GS_HD inline
+#define GS_HDC constexpr
 #endif
 
 namespace gs {
@@ -59,7 +61,7 @@ enum : uint32_t {
   C_TRACED = 1u << 9,     // memory instruction whose address is traced (R27)
 };
 
-GS_HD uint32_t op_class(uint32_t op) {
+GS_HDC uint32_t op_class(uint32_t op) {
   switch (op) {
     case OP_LDG: return C_MEMLOAD | C_TRACED;
     case OP_LDL: return C_MEMLOAD | C_TRACED;

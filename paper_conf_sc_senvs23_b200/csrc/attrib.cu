@@ -913,14 +913,16 @@ __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, u
                                                int32_t* __restrict__ zero_h, uint64_t zero_n) {
   __shared__ unsigned long long pre[kPlanProbes];
   __shared__ unsigned long long wsum[32];
-  // the histogram's zeroing (instead of a separate memset node): every CTA zeroes a grid-strided
-  // share with 128-bit stores; CTA 0 then plans (zero_h is 16-byte aligned, zero_n words)
-  if (zero_h) {
+  // the histogram's zeroing (instead of a separate memset node): CTAs 1.. zero grid-strided shares
+  // with 128-bit stores while CTA 0 plans (zeroing, then planning, in CTA 0 put the plan on the
+  // critical path: C4 attribution 0.760 -> 0.753 ms); zero_h is 16-byte aligned, zero_n words
+  if (zero_h && (blockIdx.x != 0 || gridDim.x == 1)) {
+    const uint32_t zc = gridDim.x > 1 ? blockIdx.x - 1 : 0u, nzc = gridDim.x > 1 ? gridDim.x - 1 : 1u;
     uint4* h4 = reinterpret_cast<uint4*>(zero_h);
     const uint64_t n4w = zero_n / 4;
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n4w; i += (uint64_t)gridDim.x * blockDim.x)
+    for (uint64_t i = zc * (uint64_t)blockDim.x + threadIdx.x; i < n4w; i += (uint64_t)nzc * blockDim.x)
       h4[i] = make_uint4(0, 0, 0, 0);
-    if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (zero_n & 3)) zero_h[n4w * 4 + threadIdx.x] = 0;
+    if (zc == nzc - 1 && threadIdx.x < (zero_n & 3)) zero_h[n4w * 4 + threadIdx.x] = 0;
   }
   if (blockIdx.x != 0) return;
   const uint64_t n4 = n / 4;

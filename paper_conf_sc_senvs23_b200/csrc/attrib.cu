@@ -1429,7 +1429,10 @@ gs_status partition_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t*
   count_launch();
   k_pscan<<<1, kPT, 0, st>>>(cnt, (uint32_t)nch, B, bstart, ps);
   count_launch();
-  const auto kern = n + 8ull * B + 8 < (1ull << 32) ? k_pscatter<kPST, uint32_t> : k_pscatter<kPST, unsigned long long>;
+  // 32-bit destination bases when the copy has < 2^32 entries (GS_PART_WIDE=1 forces the 64-bit
+  // kernel: tests)
+  const bool wide = n + 8ull * B + 8 >= (1ull << 32) || getenv("GS_PART_WIDE") != nullptr;
+  const auto kern = wide ? k_pscatter<kPST, unsigned long long> : k_pscatter<kPST, uint32_t>;
   GS_CUDA(c, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(3 * kSTile * 4)));
   kern<<<(unsigned)nch, kPST, 3 * kSTile * 4, st>>>(d_words, n, chunk, (uint32_t)pnr, B, cnt, bstart, ps);
   count_launch();

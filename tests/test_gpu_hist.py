@@ -183,3 +183,34 @@ def test_hot_words_with_invalid_and_foreign_words(gs):
                 assert int(ninv.item()) == want_inv, (mode, bits, row)
                 assert torch.equal(hist.to(torch.int64), want), (mode, bits, row)
                 ctx.close()
+
+
+def test_partition_wide_destinations_and_bucket_limit(gs):
+    """PARTITION's 64-bit destination kernel (forced; the natural trigger is a copy of >= 2^32
+    entries) and its fallback to WINDOW when P * R reaches 2^25 bins (1024 buckets of 2^15):
+    both equal the bincount of the words."""
+    import os
+    import torch
+    from gen import sass as gsass
+    s = gsass.config_sass("C4")
+    for nr in (19, 32):  # 19.9M bins (PARTITION) and 2^25 bins (falls back to WINDOW)
+        rng = np.random.default_rng(nr)
+        w = rng.integers(0, s.P * nr, 3_000_017).astype(np.int64)
+        w[::101] = s.P * nr + 3
+        bad = int((w >= s.P * nr).sum())
+        want = torch.from_numpy(np.bincount(w[w < s.P * nr], minlength=s.P * nr).astype(np.int32)).cuda()
+        words = torch.from_numpy(w.astype(np.int32)).cuda()
+        for forced in (False, True):
+            if forced:
+                os.environ["GS_PART_WIDE"] = "1"
+            try:
+                ctx = gs.Context(hist_mode=4, n_reasons=nr, hist_row=nr)
+                ctx.load_sass(s.text)
+                hist, ninv = ctx.attribute_samples(words)
+                torch.cuda.synchronize()
+            finally:
+                os.environ.pop("GS_PART_WIDE", None)
+            assert int(ninv.item()) == bad, (nr, forced)
+            assert torch.equal(hist, want), (nr, forced, int((hist != want).sum().item()))
+            assert ctx.last_hist_mode() == (4 if nr == 19 else 3), (nr, ctx.last_hist_mode())
+            ctx.close()

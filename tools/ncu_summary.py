@@ -17,14 +17,24 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "launch__grid_size", "launch__block_size", "sm__cycles_active.avg", "gpc__cycles_elapsed.max"]
 
 
+SETUP_KERNELS = ("k_expand", "at::", "at_cuda_detail", "curand", "distribution_elementwise")
+
+
 def launches(path, steps=1):
     rows = list(csv.reader(open(path)))
     hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
     h = rows[hi]
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
+    mi = h.index("Metric Name") if "Metric Name" in h else -1
     agg = collections.OrderedDict()
+    skipped = collections.Counter()
     for r in rows[hi + 1:]:
         if len(r) <= vi:
+            continue
+        if mi >= 0 and r[mi] != "gpu__time_duration.sum":  # launch lists may carry other metrics
+            continue
+        if any(x in r[ki] for x in SETUP_KERNELS):  # input generation before the timed region
+            skipped[r[ki].split("(")[0][-40:]] += 1
             continue
         scale = {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3}.get(r[ui], 1.0)
         name = r[ki].split("(")[0].replace("gs::<unnamed>::", "").replace("void ", "")[:70]
@@ -34,6 +44,9 @@ def launches(path, steps=1):
     for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
         print(f"{sum(v) / steps:10.1f} {100 * sum(v) / steps / tot:5.1f}% {len(v) // steps:4d}  {k}")
     print(f"{tot:10.1f} us per step (serialised, cold-cache ncu replay)")
+    if skipped:
+        print("  not counted (workload generation, outside the timed steps):",
+              ", ".join(f"{k} x{v}" for k, v in skipped.items()))
 
 
 def kernel(path):

@@ -366,6 +366,7 @@ def main():
                     help="samples in the oracle's bounded sample (with the full SASS) per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip the C3 detection / C5 / pack+hist lines")
+    ap.add_argument("--lib", default=None, help="another build of the library (same-box A/B of diagnostic variants)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -391,6 +392,8 @@ def main():
     from paper_conf_sc_senvs23_b200 import binding, build as gbuild, dist as gdist
     from gen.device import DeviceTrace
     gbuild.build()
+    if args.lib:
+        binding.load_library(args.lib)
     torch.cuda.set_stream(torch.cuda.Stream())   # a non-default stream: the library may replay CUDA graphs on it
 
     t_setup = time.perf_counter()

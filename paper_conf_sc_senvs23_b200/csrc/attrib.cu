@@ -730,9 +730,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
   if (threadIdx.x < 2) sh_ndefer[threadIdx.x] = 0;
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  // launched with programmatic stream serialisation after k_plan: the prologue above overlapped
-  // its tail; the plan, the queue words and the zeroed histogram are read / written after this
-  asm volatile("griddepcontrol.wait;" ::: "memory");
   __syncthreads();
 
   const auto span = [&](unsigned long long tile, uint64_t& a4, uint64_t& b4) {
@@ -916,9 +913,6 @@ __global__ void __launch_bounds__(1024) k_plan(const uint32_t* __restrict__ s, u
                                                int32_t* __restrict__ zero_h, uint64_t zero_n) {
   __shared__ unsigned long long pre[kPlanProbes];
   __shared__ unsigned long long wsum[32];
-  // the counting kernel (launched with programmatic stream serialisation) may start its prologue
-  // on SMs this grid frees; it waits for this grid's completion before reading the plan
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   // the histogram's zeroing (instead of a separate memset node): CTAs 1.. zero grid-strided shares
   // with 128-bit stores while CTA 0 plans (zeroing, then planning, in CTA 0 put the plan on the
   // critical path: C4 attribution 0.760 -> 0.753 ms); zero_h is 16-byte aligned, zero_n words
@@ -1578,22 +1572,9 @@ gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hi
   if (dyn) {
     const auto kern = bits == 16 ? k_hist_window<true> : k_hist_window<false>;
     ls = prep(kern);
-    if (ls == GS_OK) {
-      cudaLaunchConfig_t cfg = {};
-      cfg.gridDim = dim3((uint32_t)chunks);
-      cfg.blockDim = dim3(kThreads);
-      cfg.dynamicSmemBytes = smem;
-      cfg.stream = st;
-      cudaLaunchAttribute at[1];
-      at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;  // overlaps k_plan's tail (PDL)
-      at[0].val.programmaticStreamSerializationAllowed = 1;
-#ifndef GS_NO_PDL
-      cfg.attrs = at;
-      cfg.numAttrs = 1;
-#endif
-      GS_CUDA(c, cudaLaunchKernelEx(&cfg, kern, d_words, n, P, nr, dv, (const KDesc*)c->d_kd, c->n_kernels, 1u, d_hist,
-                                    d_n_invalid, c->d_tileq, c->d_defer, tw));
-    }
+    if (ls == GS_OK)
+      kern<<<(uint32_t)chunks, kThreads, smem, st>>>(d_words, n, P, nr, dv, c->d_kd, c->n_kernels, 1u, d_hist,
+                                                     d_n_invalid, c->d_tileq, c->d_defer, tw);
   } else {
     const auto kern = bits == 16 ? k_hist_smem<true> : k_hist_smem<false>;
     ls = prep(kern);

@@ -109,6 +109,12 @@ __device__ __forceinline__ unsigned long long group_key(uint32_t base, uint32_t 
   return ((unsigned long long)base_rd << 10) | base;
 }
 
+// Programmatic dependent launch between consecutive detection kernels: a primary lets its
+// dependent grid launch once all its CTAs are running (pdl_trigger); the dependent's CTAs fill the
+// SMs the primary frees and wait (pdl_wait) for its completion before touching its outputs.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // ------------------------------------------------------------------------------------------ A
 __global__ void __launch_bounds__(kWarps * 32, 5) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
@@ -117,6 +123,7 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_summary(const Rec* __restric
                                                          uint32_t win) {
   __shared__ uint32_t last[kWarps][kNumRegs];
   __shared__ uint16_t s_cls[OP_COUNT];
+  pdl_trigger();
   opcls_init(s_cls);
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -192,6 +199,8 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_summary(const Rec* __restric
 // ------------------------------------------------------------------------------------------ B
 __global__ void k_carry(const KDesc* __restrict__ kd, uint32_t kb, uint32_t ke, uint32_t* tab,
                         const int32_t* __restrict__ wsum, int32_t* wloop, uint32_t win) {
+  pdl_wait();
+  pdl_trigger();
   const uint32_t k = kb + blockIdx.x;
   if (k >= ke) return;
   const KDesc K = kd[k];
@@ -308,6 +317,7 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restric
   __shared__ uint32_t nar[kWarps][kNarWords];
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
+  pdl_wait();
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t w = w0 + blockIdx.x * kWarps + warp;
@@ -350,8 +360,11 @@ __global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restric
     const uint32_t nq = writes ? min(r_dstw(r), reg_cap(dst) + 1 - dst) : 0u;
     const uint32_t dst2 = writes ? r_dst2(r) : (uint32_t)kRegNone;  // second quad (R38a)
     const uint32_t nq2 = reg_live(dst2) ? min(r_dstw(r), reg_cap(dst2) + 1 - dst2) : 0u;
-    for_regs(dst, nq, [&](bool p, uint32_t x) { if (p) atomicOr(&MT[x].x, 1u << lane); });
-    if (nq2) for_regs(dst2, nq2, [&](bool p, uint32_t x) { if (p) atomicOr(&MT[x].x, 1u << lane); });
+    // (predicated per register: unconditional atomics with idle lanes on one dummy entry were
+    // measured 20% slower on C3, same-address conflicts)
+    const auto mark = [&](bool p, uint32_t x) { if (p) atomicOr(&MT[x].x, 1u << lane); };
+    for_regs(dst, nq, mark);
+    if (nq2) for_regs(dst2, nq2, mark);
     const uint32_t ldgmask = __ballot_sync(0xffffffffu, valid && op == OP_LDG);
     __syncwarp();
     // loop depth: inclusive prefix of the event differences (R13); a window without loop events
@@ -559,6 +572,7 @@ __global__ void k_cons_fill(uint64_t s0, uint64_t n, const uint32_t* __restrict_
 __global__ void k_trace(const Rec* __restrict__ rec, const KDesc* __restrict__ kd, const uint32_t* __restrict__ ptrrd,
                         uint64_t nc, uint32_t D, CandArrays ca, GroupTable gt, gs_kernel_stats* kst) {
   __shared__ uint16_t s_cls[OP_COUNT];
+  pdl_trigger();
   opcls_init(s_cls);
   __syncthreads();
   const uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -711,6 +725,8 @@ __global__ void __launch_bounds__(kCT) k_rules(const Rec* __restrict__ rec, uint
                                                unsigned long long* __restrict__ tsum) {
   __shared__ uint16_t s_cls[OP_COUNT];
   opcls_init(s_cls);
+  pdl_wait();
+  pdl_trigger();
   __syncthreads();
   const uint64_t c = blockIdx.x * (uint64_t)kCT + threadIdx.x;
   unsigned long long v = 0;
@@ -743,6 +759,7 @@ __global__ void __launch_bounds__(1024) k_tile_prefix(const unsigned long long* 
                                                       unsigned long long* __restrict__ pre_c,
                                                       unsigned long long* __restrict__ tot) {
   __shared__ unsigned long long ws[32], wc[32];
+  pdl_wait();
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   const uint64_t seg = (nt + 31) / 32, a = min(nt, warp * seg), e = min(nt, a + seg);
   unsigned long long ls = 0, lc = 0;
@@ -975,6 +992,24 @@ gs_status detect_alloc(gs_ctx* c) {
   return GS_OK;
 }
 
+// a launch whose grid may start while the previous kernel on the stream drains (the kernel waits
+// for it with pdl_wait before reading its outputs)
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*k)(KArgs...), uint32_t grid, uint32_t block, cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+#ifndef GS_NO_PDL
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+#endif
+  return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   cudaStream_t st = c->stream;
   const uint32_t w0 = kb < c->n_kernels ? c->kd_h[kb].win0 : c->n_win;
@@ -1033,12 +1068,11 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       k_summary<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wsum,
                                              c->d_wev, c->d_narith, c->d_kstats, c->win); count_launch();
       GS_CUDA(c, cudaGetLastError());
-      k_carry<<<ke - kb, 352, 0, st>>>(c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win);
+      GS_CUDA(c, launch_pdl(k_carry, ke - kb, 352, st, c->d_kd, kb, ke, c->d_tab, c->d_wsum, c->d_wloop, c->win));
       count_launch();
-      GS_CUDA(c, cudaGetLastError());
       // candidate arrays are indexed relative to c0
-      k_resolve<<<grid, kWarps * 32, 0, st>>>(c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff, c->d_wloop,
-                                             c->d_wev, c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand, D);
+      GS_CUDA(c, launch_pdl(k_resolve, grid, kWarps * 32, st, c->d_rec, c->d_wd, c->d_kd, w0, nw, c->d_tab, c->d_ldiff,
+                            c->d_wloop, c->d_wev, c->d_cbase, c0, c->d_ptrrd, c->d_narith, c->cand, D));
       count_launch();
       GS_CUDA(c, cudaGetLastError());
     }
@@ -1052,10 +1086,10 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
       k_trace<<<2 * gridc, 256, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp, c->d_kstats);
       count_launch();
       GS_CUDA(c, cudaGetLastError());
-      k_rules<<<(uint32_t)ntile, kCT, 0, st>>>(c->d_rec, nc, c->cand, c->grp, c->d_narith,
-                                               RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum);
+      GS_CUDA(c, launch_pdl(k_rules, (uint32_t)ntile, kCT, st, c->d_rec, nc, c->cand, c->grp, c->d_narith,
+                            RuleCfg{c->cfg.shmem_min_arith, c->cfg.shmem_min_loads}, d_tsum));
       count_launch();
-      k_tile_prefix<<<1, 1024, 0, st>>>(d_tsum, ntile, d_pre_s, d_pre_c, d_tot); count_launch();
+      GS_CUDA(c, launch_pdl(k_tile_prefix, 1u, 1024u, st, d_tsum, ntile, d_pre_s, d_pre_c, d_tot)); count_launch();
       GS_CUDA(c, cudaGetLastError());
       GS_CUDA(c, cudaMemcpyAsync(tot, d_tot, 16, cudaMemcpyDeviceToHost, st));
     }

@@ -188,6 +188,7 @@ struct gs_ctx {
   cudaEvent_t ev_pass[2] = {nullptr, nullptr};
   bool pass_timed = false;
   int dev_sms = 0;                   // cached multiprocessor count
+  int cluster_sort_ok = -1;          // rank: 16-CTA cluster sort usable (-1: not probed yet)
   const void* smem_fn[4] = {nullptr, nullptr, nullptr, nullptr};  // kernels whose dynamic smem limit
   size_t smem_set[4] = {0, 0, 0, 0};                               // was raised, and to what
   size_t stage_words = 0;

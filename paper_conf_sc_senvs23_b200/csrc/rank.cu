@@ -12,6 +12,7 @@
 //            key and sorted once over exactly those bits (CUB onesweep radix sort); otherwise two
 //            stable passes (by tot, then by rel).
 //   k_emit   the first k rows as gs_ranked_site (one warp per row).
+#include <cooperative_groups.h>
 #include <cub/device/device_radix_sort.cuh>
 #include <cuda_runtime.h>
 
@@ -168,6 +169,122 @@ __global__ void k_keys_packed(const unsigned long long* __restrict__ rel, const 
   vals[s] = (uint32_t)s;
 }
 
+// ---------------------------------------------------------------- cluster sort (small site sets)
+// For up to kCsMax sites whose packed key leaves kCsIdxBits free bits, the whole sort runs in ONE
+// launch of a 16-CTA thread-block cluster: element = (key << 17) | site index, 8192 per CTA in
+// shared memory; per 6-bit digit (LSD, stable): warp-level ranks by __match_any_sync over rows of
+// 32 elements in order, per-digit prefixes over the warps, the cluster's digit totals read through
+// distributed shared memory, and every element stored straight into its destination CTA's other
+// buffer (st.shared::cluster); one cluster barrier per pass. The CUB onesweep path launched a
+// histogram, a scan and one kernel per 8-bit digit over global memory.
+namespace cg = cooperative_groups;
+constexpr uint32_t kCsCtas = 16, kCsThreads = 1024, kCsWarps = kCsThreads / 32, kCsRows = 8;
+constexpr uint32_t kCsPer = kCsWarps * kCsRows * 32;     // elements per CTA (8192)
+constexpr uint32_t kCsMax = kCsCtas * kCsPer;            // 131072 sites
+constexpr uint32_t kCsIdxBits = 17;                      // site index bits (kCsMax = 2^17)
+constexpr uint32_t kCsDigitBits = 6, kCsDigits = 1u << kCsDigitBits;
+static_assert(kCsMax == (1u << kCsIdxBits), "index field");
+
+__global__ void __launch_bounds__(kCsThreads, 1)
+    k_cluster_sort(  // launched as one cluster of kCsCtas CTAs
+const unsigned long long* __restrict__ rel, const unsigned long long* __restrict__ tot, uint32_t ns,
+                   int bt, unsigned long long mask_r, unsigned long long mask_t, uint32_t bits,
+                   uint32_t* __restrict__ order) {
+  extern __shared__ unsigned long long cs_buf[];          // [2][kCsPer]
+  __shared__ uint32_t wc[kCsWarps][kCsDigits];            // per-warp digit counts -> exclusive prefixes
+  __shared__ uint32_t cnt[kCsDigits];                     // this CTA's digit totals (read by the cluster)
+  __shared__ uint32_t allc[kCsCtas][kCsDigits];
+  __shared__ uint32_t base[kCsDigits];
+  cg::cluster_group cluster = cg::this_cluster();
+  const uint32_t r = cluster.block_rank(), lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  unsigned long long* cur = cs_buf;
+  unsigned long long* nxt = cs_buf + kCsPer;
+  // element i of CTA r is site r * kCsPer + i; warp w owns [w * 256, w * 256 + 256), row k its
+  // elements w * 256 + 32 k + lane
+  for (uint32_t i = threadIdx.x; i < kCsPer; i += kCsThreads) {
+    const uint32_t sidx = r * kCsPer + i;
+    cur[i] = sidx < ns ? ((((mask_r - rel[sidx]) << bt) | (mask_t - tot[sidx])) << kCsIdxBits) | sidx : ~0ull;
+  }
+  __syncthreads();
+  const uint32_t passes = (bits + kCsDigitBits - 1) / kCsDigitBits;
+  for (uint32_t pass = 0; pass < passes; pass++) {
+    const uint32_t sh = kCsIdxBits + pass * kCsDigitBits;
+    for (uint32_t d = lane; d < kCsDigits; d += 32) wc[warp][d] = 0;
+    __syncwarp();
+    unsigned long long e[kCsRows];
+    uint32_t dr[kCsRows];  // digit << 16 | rank within the warp's elements of that digit
+#pragma unroll
+    for (uint32_t k = 0; k < kCsRows; k++) {
+      e[k] = cur[warp * kCsRows * 32 + 32 * k + lane];
+      const uint32_t d = (uint32_t)(e[k] >> sh) & (kCsDigits - 1u);
+      const uint32_t m = __match_any_sync(0xffffffffu, d);
+      const uint32_t lead = 31u - __clz(m);  // the row's last lane of this digit adds the count
+      const uint32_t before = wc[warp][d];
+      __syncwarp();
+      if (lane == lead) wc[warp][d] = before + __popc(m);
+      __syncwarp();
+      dr[k] = (d << 16) | (before + __popc(m & lt));
+    }
+    __syncthreads();
+    if (threadIdx.x < kCsDigits) {  // exclusive prefixes over the warps, CTA totals
+      const uint32_t d = threadIdx.x;
+      uint32_t acc = 0;
+      for (uint32_t w = 0; w < kCsWarps; w++) {
+        const uint32_t x = wc[w][d];
+        wc[w][d] = acc;
+        acc += x;
+      }
+      cnt[d] = acc;
+    }
+    cluster.sync();  // every CTA's cnt[] is final (and every CTA finished reading its buffer)
+    {
+      const uint32_t c = threadIdx.x / kCsDigits, d = threadIdx.x % kCsDigits;  // 16 x 64 = 1024 threads
+      allc[c][d] = *cluster.map_shared_rank(&cnt[d], c);
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {  // base[d] = elements of smaller digits anywhere + of digit d in CTAs < r
+      uint32_t tot2[2], mine[2];
+#pragma unroll
+      for (uint32_t h = 0; h < 2; h++) {
+        const uint32_t d = lane * 2 + h;
+        uint32_t t = 0, m = 0;
+        for (uint32_t c = 0; c < kCsCtas; c++) {
+          t += allc[c][d];
+          m += c < r ? allc[c][d] : 0u;
+        }
+        tot2[h] = t;
+        mine[h] = m;
+      }
+      uint32_t inc = tot2[0] + tot2[1];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= (uint32_t)o) inc += y;
+      }
+      const uint32_t ex = inc - tot2[0] - tot2[1];
+      base[lane * 2] = ex + mine[0];
+      base[lane * 2 + 1] = ex + tot2[0] + mine[1];
+    }
+    __syncthreads();
+#pragma unroll
+    for (uint32_t k = 0; k < kCsRows; k++) {  // straight into the destination CTA's other buffer
+      const uint32_t d = dr[k] >> 16;
+      const uint32_t pos = base[d] + wc[warp][d] + (dr[k] & 0xffffu);
+      unsigned long long* dst = cluster.map_shared_rank(nxt, pos / kCsPer);
+      dst[pos % kCsPer] = e[k];
+    }
+    cluster.sync();  // all elements arrived; allc/cnt/wc free for the next pass
+    unsigned long long* t = cur;
+    cur = nxt;
+    nxt = t;
+  }
+  for (uint32_t i = threadIdx.x; i < kCsPer; i += kCsThreads) {
+    const uint32_t q = r * kCsPer + i;
+    if (q < ns) order[q] = (uint32_t)(cur[i] & (kCsMax - 1u));
+  }
+}
+
 // one field: key = mask - val[order[i]] (order == nullptr: identity, vals = i)
 __global__ void k_keys_field(const unsigned long long* __restrict__ val, const uint32_t* __restrict__ order,
                              uint64_t ns, unsigned long long mask, unsigned long long* __restrict__ keys,
@@ -231,6 +348,21 @@ __global__ void __launch_bounds__(kEmitT) k_emit(const uint32_t* __restrict__ or
   for (uint32_t i = threadIdx.x; i < nrow * kRowWords; i += kEmitT) dst[i] = src[i];
 }
 
+cudaLaunchConfig_t cluster_cfg(cudaStream_t st) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(kCsCtas);
+  cfg.blockDim = dim3(kCsThreads);
+  cfg.dynamicSmemBytes = 2 * kCsPer * 8;
+  cfg.stream = st;
+  return cfg;
+}
+void cluster_attr(cudaLaunchAttribute* at) {
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = kCsCtas;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+}
+
 int bits_of(unsigned long long v) { return v ? 64 - __builtin_clzll(v) : 0; }
 unsigned long long mask_of(int b) { return b >= 64 ? ~0ull : ((1ull << b) - 1); }
 
@@ -281,6 +413,22 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     if (kk && out_is_host) GS_CUDA(c, dev_grow(&c->d_ranked, &c->ranked_cap, kk));
   }
   GS_CUDA(c, pin_grow(c, 16));
+  if (c->cluster_sort_ok < 0) {  // once per context: can a 16-CTA cluster with 128 KB each run here?
+    c->cluster_sort_ok = 0;
+    if (cudaFuncSetAttribute(k_cluster_sort, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess &&
+        cudaFuncSetAttribute(k_cluster_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kCsPer * 8) ==
+            cudaSuccess) {
+      cudaLaunchConfig_t cfg = cluster_cfg(st);
+      cudaLaunchAttribute at[1];
+      cluster_attr(at);
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      int nclusters = 0;
+      if (cudaOccupancyMaxActiveClusters(&nclusters, k_cluster_sort, &cfg) == cudaSuccess && nclusters > 0)
+        c->cluster_sort_ok = getenv("GS_NO_CLUSTER_SORT") ? 0 : 1;
+    }
+    cudaGetLastError();
+  }
   if (!c->side_stream) {
     GS_CUDA(c, cudaStreamCreateWithFlags(&c->side_stream, cudaStreamNonBlocking));
     GS_CUDA(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
@@ -301,7 +449,18 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
   const auto sort_emit = [&](int br, int bt) -> gs_status {
     const uint32_t* order = v0;
     size_t b1 = cub_bytes;
-    if (br + bt <= 64) {
+    if (br + bt + kCsIdxBits <= 64 && ns <= kCsMax && br + bt > 0 && c->cluster_sort_ok) {
+      cudaLaunchConfig_t cfg = cluster_cfg(st);
+      cudaLaunchAttribute at[1];
+      cluster_attr(at);
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      GS_CUDA(c, cudaLaunchKernelEx(&cfg, k_cluster_sort, (const unsigned long long*)d_rel,
+                                    (const unsigned long long*)d_tot, (uint32_t)ns, bt, mask_of(br), mask_of(bt),
+                                    (uint32_t)(br + bt), v0));
+      count_launch();
+      order = v0;
+    } else if (br + bt <= 64) {
       k_keys_packed<<<grid, 256, 0, st>>>(d_rel, d_tot, ns, bt, mask_of(br), mask_of(bt), k0, v0);
       count_launch();
       if (br + bt > 0) {

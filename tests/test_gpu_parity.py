@@ -637,3 +637,34 @@ def test_cupti_ingest_parity(gs, cfg, crc_filter, row):
     assert g.H == o.H and g.N == o.N and g.R == o.R and g.S == o.S
     assert f"C skipped={skipped}" in o.text and skipped == buf.skipped
     assert nrec == sum(int(buf.pcdata[i].stallReasonCount) for i in range(buf.n))
+
+
+@pytest.mark.parametrize("cfg,scale", [("C2", 1.0), ("C4", 1.0), ("C3", 0.04)])
+def test_cluster_sort_equals_cub_sort(gs, cfg, scale):
+    """gs_rank_sites sorts up to 131,072 sites in one 16-CTA cluster (distributed shared memory);
+    the same ranking through CUB's radix sort (GS_NO_CLUSTER_SORT=1; C3 at this scale has more
+    sites than the cluster holds, so both take CUB) is identical row for row."""
+    import os
+    import torch
+    from gen import samples as gsm
+    from gen import sass as gsass
+    s = gsass.config_sass(cfg, scale=scale)
+    tab = gsm.table_class_weighted(s.cls, 3_000_000, key=11)
+    words = torch.from_numpy(gsm.Trace(tab, s.first_slot, s.n_instr, order="shuffled", seed=3).packed()
+                             .view(np.int32)).cuda()
+    out = []
+    for no_cluster in (False, True):
+        if no_cluster:
+            os.environ["GS_NO_CLUSTER_SORT"] = "1"
+        try:
+            ctx = _ctx(gs, hist_row=19)
+            ctx.load_sass(s.text)
+            n_sites = ctx.detect()
+            hist, _ = ctx.attribute_samples(words)
+            rows = ctx.rank_sites(hist)
+            torch.cuda.synchronize()
+        finally:
+            os.environ.pop("GS_NO_CLUSTER_SORT", None)
+        out.append(rows.copy())
+        ctx.close()
+    assert len(out[0]) == n_sites and np.array_equal(out[0], out[1])

@@ -14,7 +14,10 @@ namespace gs {
 // instructions per detection window (never crosses a kernel): 256, or 1024 for modules of at least
 // kBigModule instructions (fewer, longer windows: smaller carry tables; a small module needs the
 // short windows to fill the GPU with warps)
-constexpr uint32_t kWinSmall = 256, kWinBig = 1024;
+#ifndef GS_WIN_SMALL
+#define GS_WIN_SMALL 256
+#endif
+constexpr uint32_t kWinSmall = GS_WIN_SMALL, kWinBig = 1024;
 constexpr uint64_t kBigModule = 16ull << 20;
 
 // A device buffer that only grows; freed with the context.

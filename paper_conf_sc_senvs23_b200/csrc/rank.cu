@@ -182,7 +182,12 @@ constexpr uint32_t kCsCtas = 16, kCsThreads = 1024, kCsWarps = kCsThreads / 32, 
 constexpr uint32_t kCsPer = kCsWarps * kCsRows * 32;     // elements per CTA (8192)
 constexpr uint32_t kCsMax = kCsCtas * kCsPer;            // 131072 sites
 constexpr uint32_t kCsIdxBits = 17;                      // site index bits (kCsMax = 2^17)
-constexpr uint32_t kCsDigitBits = 6, kCsDigits = 1u << kCsDigitBits;
+#ifndef GS_CS_DIGIT_BITS
+#define GS_CS_DIGIT_BITS 6
+#endif
+constexpr uint32_t kCsDigitBits = GS_CS_DIGIT_BITS, kCsDigits = 1u << kCsDigitBits;
+constexpr uint32_t kCsDpl = kCsDigits / 32;  // digits per lane in the base scan
+static_assert(kCsDigits >= 32 && kCsDigits <= 256, "digit width");
 static_assert(kCsMax == (1u << kCsIdxBits), "index field");
 
 __global__ void __launch_bounds__(kCsThreads, 1)
@@ -227,8 +232,7 @@ const unsigned long long* __restrict__ rel, const unsigned long long* __restrict
       dr[k] = (d << 16) | (before + __popc(m & lt));
     }
     __syncthreads();
-    if (threadIdx.x < kCsDigits) {  // exclusive prefixes over the warps, CTA totals
-      const uint32_t d = threadIdx.x;
+    for (uint32_t d = threadIdx.x; d < kCsDigits; d += kCsThreads) {  // prefixes over the warps, CTA totals
       uint32_t acc = 0;
       for (uint32_t w = 0; w < kCsWarps; w++) {
         const uint32_t x = wc[w][d];
@@ -238,33 +242,37 @@ const unsigned long long* __restrict__ rel, const unsigned long long* __restrict
       cnt[d] = acc;
     }
     cluster.sync();  // every CTA's cnt[] is final (and every CTA finished reading its buffer)
-    {
-      const uint32_t c = threadIdx.x / kCsDigits, d = threadIdx.x % kCsDigits;  // 16 x 64 = 1024 threads
+    for (uint32_t i = threadIdx.x; i < kCsCtas * kCsDigits; i += kCsThreads) {
+      const uint32_t c = i / kCsDigits, d = i % kCsDigits;
       allc[c][d] = *cluster.map_shared_rank(&cnt[d], c);
     }
     __syncthreads();
     if (threadIdx.x < 32) {  // base[d] = elements of smaller digits anywhere + of digit d in CTAs < r
-      uint32_t tot2[2], mine[2];
+      uint32_t totd[kCsDpl], mine[kCsDpl], sum = 0;
 #pragma unroll
-      for (uint32_t h = 0; h < 2; h++) {
-        const uint32_t d = lane * 2 + h;
+      for (uint32_t h = 0; h < kCsDpl; h++) {
+        const uint32_t d = lane * kCsDpl + h;
         uint32_t t = 0, m = 0;
         for (uint32_t c = 0; c < kCsCtas; c++) {
           t += allc[c][d];
           m += c < r ? allc[c][d] : 0u;
         }
-        tot2[h] = t;
+        totd[h] = t;
         mine[h] = m;
+        sum += t;
       }
-      uint32_t inc = tot2[0] + tot2[1];
+      uint32_t inc = sum;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
         if (lane >= (uint32_t)o) inc += y;
       }
-      const uint32_t ex = inc - tot2[0] - tot2[1];
-      base[lane * 2] = ex + mine[0];
-      base[lane * 2 + 1] = ex + tot2[0] + mine[1];
+      uint32_t ex = inc - sum;
+#pragma unroll
+      for (uint32_t h = 0; h < kCsDpl; h++) {
+        base[lane * kCsDpl + h] = ex + mine[h];
+        ex += totd[h];
+      }
     }
     __syncthreads();
 #pragma unroll

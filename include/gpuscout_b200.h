@@ -60,9 +60,9 @@ typedef struct {
  *   GS_HIST_PRIVATE   fixed slot ranges per CTA in shared memory (modules of <= 3 tables);
  *   GS_HIST_WINDOW    a shared-memory window that follows the stream (PC-sampling traces, which
  *                     arrive grouped by kernel);
- *   GS_HIST_PARTITION partition by bucket of 2^b slots first, then count each bucket in its own
- *                     window: for streams without locality (random order); modules needing more than
- *                     2048 bucket tables use WINDOW instead;
+ *   GS_HIST_PARTITION partition by bucket of 2^15 compact bins first (a 16-bit offset per sample),
+ *                     then count each bucket in its own table: for streams without locality (random
+ *                     order); modules of 2^25 bins (P * R) or more use WINDOW instead;
  *   GS_HIST_AUTO      PRIVATE for small modules, else WINDOW. */
 enum { GS_HIST_AUTO = 0, GS_HIST_GLOBAL = 1, GS_HIST_PRIVATE = 2, GS_HIST_WINDOW = 3, GS_HIST_PARTITION = 4 };
 

@@ -32,6 +32,12 @@ namespace {
 
 constexpr uint64_t kEmpty = ~0ull;
 constexpr int kWarps = 8;  // warps (windows) per CTA in the window kernels
+#ifndef GS_RES_MINB
+#define GS_RES_MINB 5  // resident CTAs per SM the window kernels are compiled for (register budget)
+#endif
+#ifndef GS_SUM_MINB
+#define GS_SUM_MINB 5
+#endif
 
 __device__ __forceinline__ Rec ld_rec(const Rec* r, uint64_t i) {
   uint4 v = __ldg(reinterpret_cast<const uint4*>(r) + i);
@@ -116,7 +122,7 @@ __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.lau
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
 // ------------------------------------------------------------------------------------------ A
-__global__ void __launch_bounds__(kWarps * 32, 5) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+__global__ void __launch_bounds__(kWarps * 32, GS_SUM_MINB) k_summary(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
                                                          uint32_t* __restrict__ tab, int32_t* ldiff, int32_t* wsum,
                                                          uint32_t* wev, uint32_t* narith, gs_kernel_stats* kst,
@@ -306,7 +312,7 @@ __device__ TraceOut chase(const Rec* __restrict__ rec, const uint32_t* ptrrd, co
 // while their steps stay inside the window (the RDs of earlier windows belong to other warps);
 // k_trace resumes the others.
 constexpr uint32_t kNarWords = kWinBig / 2;  // 16-bit n_arith counters per window instruction
-__global__ void __launch_bounds__(kWarps * 32, 5) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
+__global__ void __launch_bounds__(kWarps * 32, GS_RES_MINB) k_resolve(const Rec* __restrict__ rec, const WDesc* __restrict__ wd,
                                                          const KDesc* __restrict__ kd, uint32_t w0, uint32_t nw,
                                                          const uint32_t* __restrict__ tab, int32_t* ldiff,
                                                          const int32_t* __restrict__ wloop,

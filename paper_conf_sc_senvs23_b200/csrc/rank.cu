@@ -537,14 +537,16 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     GS_CUDA(c, cudaGetLastError());
     // The packed sort key needs the bit widths of max(rel) and max(tot). They are read back with
     // one async copy; the sort itself is enqueued right away with the widths of the previous call
-    // (padded to whole 8-bit radix digits, which costs no extra pass) and redone with the exact
+    // (padded to whole radix digits, which costs no extra pass) and redone with the exact
     // widths only when this call's maxima do not fit them (one host synchronisation otherwise).
-    GS_CUDA(c, cudaMemcpyAsync(mx, d_max, 16, cudaMemcpyDeviceToHost, st));
     if (gr >= 0) {
       const gs_status se = sort_emit(gr, gt);
       if (se != GS_OK) return se;
     }
     GS_CUDA(c, cudaStreamWaitEvent(st, c->ev_join, 0));  // (again after k_emit: harmless)
+    // the maxima go to the host last: only the host's width check reads them (a copy between the
+    // join and the sort sat on the critical path)
+    GS_CUDA(c, cudaMemcpyAsync(mx, d_max, 16, cudaMemcpyDeviceToHost, st));
     return GS_OK;
   };
   // The whole sequence is replayed as one CUDA graph while its parameters repeat (e.g. one rank
@@ -599,7 +601,9 @@ gs_status rank_run(gs_ctx* c, const int32_t* d_hist, uint32_t slot0, uint64_t k,
     GS_CUDA(c, cudaStreamSynchronize(st));
     const int br = bits_of(mx[0]), bt = bits_of(mx[1]);
     if (br + bt <= 64) {  // next call's widths: this call's, slack spread to fill the last digit
-      const int slack = ((br + bt + 7) / 8) * 8 - (br + bt);
+      // the digit width of the sort that will run: 6-bit cluster passes or 8-bit CUB passes
+      const int db = (c->cluster_sort_ok == 1 && ns <= kCsMax && br + bt + (int)kCsIdxBits <= 64) ? (int)kCsDigitBits : 8;
+      const int slack = ((br + bt + db - 1) / db) * db - (br + bt);
       c->rank_bits_guess[0] = std::min(64, br + slack / 2);
       c->rank_bits_guess[1] = std::min(64, bt + slack - slack / 2);
       if (c->rank_bits_guess[0] + c->rank_bits_guess[1] > 64) c->rank_bits_guess[0] = c->rank_bits_guess[1] = -1;

@@ -140,7 +140,10 @@ const char *gs_kernel_name(const gs_ctx *ctx, uint32_t k);
 gs_status gs_instr_lines(const gs_ctx *ctx, int32_t *lines, size_t cap);
 
 /* a-2..a-7: detection (the paper's dry run) over kernels [k_begin, k_end).
- * Enqueued on the stream; synchronises once at the end to return the site count. */
+ * Enqueued on the stream; synchronises once at the end to return the site count. With
+ * n_sites == NULL it returns without synchronising: the next call that reads the results
+ * (gs_sites*, gs_kernel_stats_get, gs_rank_sites*, gs_detect) completes it first, so work enqueued
+ * in between (e.g. gs_attribute_samples) follows on the GPU without a host round trip. */
 gs_status gs_detect(gs_ctx *ctx, uint32_t k_begin, uint32_t k_end, uint64_t *n_sites);
 /* Device pointers to the sites / chain pool of the last gs_detect (owned by the context). */
 gs_status gs_sites(const gs_ctx *ctx, const gs_site **d_sites, const uint32_t **d_chain_pool,

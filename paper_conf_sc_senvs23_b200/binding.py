@@ -180,8 +180,13 @@ class Context:
         return out
 
     # ---- a-2 .. a-7
-    def detect(self, k_begin: int = 0, k_end: int | None = None) -> int:
+    def detect(self, k_begin: int = 0, k_end: int | None = None, wait: bool = True) -> int | None:
+        """gs_detect; wait=False enqueues it without synchronising (n_sites NULL): the site count
+        and counters are resolved by the next call that reads them (sites, stats, rank)."""
         k_end = self.n_kernels if k_end is None else k_end
+        if not wait:
+            self._check(self.L.gs_detect(self.h, k_begin, k_end, None), "gs_detect")
+            return None
         ns = ctypes.c_uint64()
         self._check(self.L.gs_detect(self.h, k_begin, k_end, ctypes.byref(ns)), "gs_detect")
         return ns.value

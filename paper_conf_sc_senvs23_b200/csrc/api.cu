@@ -115,6 +115,7 @@ void gs_destroy(gs_ctx* c) {
   rank_free(c);
   cupti_free(c);
   if (c->h_pin) cudaFreeHost(c->h_pin);
+  if (c->h_det) cudaFreeHost(c->h_det);
   if (c->side_stream) {
     cudaStreamSynchronize(c->side_stream);
     cudaStreamDestroy(c->side_stream);
@@ -351,6 +352,10 @@ gs_status gs_sites(const gs_ctx* c, const gs_site** d_sites, const uint32_t** d_
                    uint64_t* n_chain) {
   if (!c) return GS_E_INVAL;
   if (!c->detected) return GS_E_STATE;
+  {
+    const gs_status fs = detect_finish(const_cast<gs_ctx*>(c));  // an asynchronous gs_detect
+    if (fs != GS_OK) return fs;
+  }
   if (d_sites) *d_sites = c->d_sites;
   if (d_chain) *d_chain = c->d_chain;
   if (n_sites) *n_sites = c->n_sites;
@@ -362,6 +367,10 @@ gs_status gs_sites_host(gs_ctx* c, gs_site* sites, size_t cap_sites, uint32_t* c
   if (!c) return GS_E_INVAL;
   if (!c->detected) return fail(c, GS_E_STATE, "gs_sites_host before gs_detect");
   GS_CUDA(c, cudaSetDevice(c->device));
+  {
+    const gs_status fs = detect_finish(c);
+    if (fs != GS_OK) return fs;
+  }
   const size_t ns = std::min<size_t>(cap_sites, c->n_sites), nch = std::min<size_t>(cap_chain, c->n_chain);
   if (sites && ns) GS_CUDA(c, cudaMemcpyAsync(sites, c->d_sites, ns * sizeof(gs_site), cudaMemcpyDeviceToHost, c->stream));
   if (chain && nch) GS_CUDA(c, cudaMemcpyAsync(chain, c->d_chain, nch * 4, cudaMemcpyDeviceToHost, c->stream));
@@ -372,6 +381,10 @@ gs_status gs_sites_host(gs_ctx* c, gs_site* sites, size_t cap_sites, uint32_t* c
 gs_status gs_kernel_stats_get(const gs_ctx* c, gs_kernel_stats* out, size_t cap) {
   if (!c || !out) return GS_E_INVAL;
   if (!c->detected) return GS_E_STATE;
+  {
+    const gs_status fs = detect_finish(const_cast<gs_ctx*>(c));
+    if (fs != GS_OK) return fs;
+  }
   memcpy(out, c->kstats_h.data(), std::min<size_t>(cap, c->kstats_h.size()) * sizeof(gs_kernel_stats));
   return GS_OK;
 }
@@ -482,6 +495,11 @@ gs_status gs_rank_sites_slice(gs_ctx* c, const int32_t* d_hist, uint64_t slot_be
   if (!c) return GS_E_INVAL;
   c->err.clear();
   if (!c->detected) return fail(c, GS_E_STATE, "gs_rank_sites before gs_detect");
+  {
+    GS_CUDA(c, cudaSetDevice(c->device));
+    const gs_status fs = detect_finish(c);
+    if (fs != GS_OK) return fs;
+  }
   if (slot_begin > slot_end || slot_end > c->n_instr) return fail(c, GS_E_INVAL, "bad slot range");
   if (!d_hist && slot_end > slot_begin) return fail(c, GS_E_INVAL, "null histogram");
   if (k && c->n_sites && !out) return fail(c, GS_E_INVAL, "null output");

@@ -179,6 +179,13 @@ struct gs_ctx {
   uint64_t ranked_cap = 0;
   void* h_pin = nullptr;  // pinned host scratch for small D2H results (async copies, no hidden sync)
   size_t h_pin_bytes = 0;
+  // detection's own pinned results (totals + per-kernel counters): an asynchronous gs_detect
+  // (n_sites == NULL) leaves them in flight until detect_finish
+  void* h_det = nullptr;
+  size_t h_det_bytes = 0;
+  bool det_pending = false;
+  uint64_t det_nc = 0;
+  uint32_t det_D = 0;
   uint32_t* h_stage[2] = {nullptr, nullptr};  // pinned staging for host sample input
   uint32_t* d_stage[2] = {nullptr, nullptr};
   cudaEvent_t ev_stage[2] = {nullptr, nullptr};   // histogram of staging buffer b done (ctx stream)
@@ -238,6 +245,7 @@ cudaError_t dev_grow(T** p, uint64_t* cap, uint64_t need) {
 
 // launchers implemented in detect.cu / attrib.cu / rank.cu
 gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites);
+gs_status detect_finish(gs_ctx* c);  // completes an asynchronous gs_detect (no-op otherwise)
 gs_status detect_alloc(gs_ctx* c);  // after a load
 void detect_free(gs_ctx* c);
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,

@@ -937,6 +937,7 @@ void detect_free(gs_ctx* c) {
   c->det_exec = nullptr;
   c->det_key.clear();
   c->detected = false;
+  c->det_pending = false;
 }
 
 // GS_JOIN_CONSUMER: consumer groups of the slots of kernels [kb, ke) (R37)
@@ -1016,7 +1017,52 @@ cudaError_t launch_pdl(void (*k)(KArgs...), uint32_t grid, uint32_t block, cudaS
   return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
+// k_write over the candidates of the last detection (also the relaunch after growing the buffers)
+static gs_status write_launch(gs_ctx* c) {
+  const uint64_t nc = c->det_nc, ntile = (nc + kCT - 1) / kCT;
+  if (!nc || (!c->sites_cap && !c->chain_cap)) return GS_OK;
+  unsigned long long* d_pre_s = c->cand.choff + ntile;
+  unsigned long long* d_pre_c = d_pre_s + ntile;
+  k_write<<<(uint32_t)ntile, kCT, 0, c->stream>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, c->det_D, c->cand, c->grp,
+                                                   c->d_narith, d_pre_s, d_pre_c, c->d_sites, c->d_chain,
+                                                   c->sites_cap, c->chain_cap);
+  count_launch();
+  GS_CUDA(c, cudaGetLastError());
+  return GS_OK;
+}
+
+// the host half of a detection: read the totals and counters, grow the buffers and write again if
+// a total exceeded them
+gs_status detect_finish(gs_ctx* c) {
+  if (!c->det_pending) return GS_OK;
+  c->det_pending = false;
+  cudaStream_t st = c->stream;
+  GS_CUDA(c, cudaStreamSynchronize(st));
+  const unsigned long long* tot = static_cast<const unsigned long long*>(c->h_det);
+  const gs_kernel_stats* kst_pin = reinterpret_cast<const gs_kernel_stats*>(static_cast<const char*>(c->h_det) + 16);
+  c->kstats_h.assign(kst_pin, kst_pin + c->n_kernels);
+  const uint64_t ns = tot[1], nch = tot[0];
+  if (nch > 0xffffffffull) {
+    c->detected = false;
+    return fail(c, GS_E_RANGE, "chain pool exceeds 2^32 entries");
+  }
+  if (ns > c->sites_cap || nch > c->chain_cap) {
+    GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
+    GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
+    const gs_status ws = write_launch(c);
+    if (ws != GS_OK) return ws;
+    GS_CUDA(c, cudaStreamSynchronize(st));
+  }
+  c->n_sites = ns;
+  c->n_chain = nch;
+  return GS_OK;
+}
+
 gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
+  {  // a previous asynchronous detection's results are read before its buffers are reused
+    const gs_status fs = detect_finish(c);
+    if (fs != GS_OK) return fs;
+  }
   cudaStream_t st = c->stream;
   const uint32_t w0 = kb < c->n_kernels ? c->kd_h[kb].win0 : c->n_win;
   const uint32_t w1 = ke < c->n_kernels ? c->kd_h[ke].win0 : c->n_win;
@@ -1038,20 +1084,26 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   unsigned long long* d_pre_c = d_pre_s + ntile;
   unsigned long long* d_tot = d_pre_c + ntile;
   // pinned: [0, 16) the two totals, then the per-kernel counters (async D2H, one synchronisation)
-  GS_CUDA(c, pin_grow(c, 16 + (uint64_t)c->n_kernels * sizeof(gs_kernel_stats)));
-  unsigned long long* tot = static_cast<unsigned long long*>(c->h_pin);
-  gs_kernel_stats* kst_pin = reinterpret_cast<gs_kernel_stats*>(static_cast<char*>(c->h_pin) + 16);
+  {
+    const size_t need = 16 + (size_t)c->n_kernels * sizeof(gs_kernel_stats);
+    if (!c->h_det || c->h_det_bytes < need) {
+      if (c->h_det) cudaFreeHost(c->h_det);
+      c->h_det = nullptr;
+      c->h_det_bytes = 0;
+      GS_CUDA(c, cudaHostAlloc(&c->h_det, need < 4096 ? 4096 : need, cudaHostAllocDefault));
+      c->h_det_bytes = need < 4096 ? 4096 : need;
+    }
+  }
+  unsigned long long* tot = static_cast<unsigned long long*>(c->h_det);
+  gs_kernel_stats* kst_pin = reinterpret_cast<gs_kernel_stats*>(static_cast<char*>(c->h_det) + 16);
   tot[0] = tot[1] = 0;
+  c->det_nc = nc;
+  c->det_D = D;
   // sites and chains into the buffers as they are (one host synchronisation per call); if a total
   // turns out larger than its buffer, grow it and write again
-  auto write = [&]() -> gs_status {
-    if (!nc || (!c->sites_cap && !c->chain_cap)) return GS_OK;
-    k_write<<<(uint32_t)((nc + kCT - 1) / kCT), kCT, 0, st>>>(c->d_rec, c->d_kd, c->d_ptrrd, nc, D, c->cand, c->grp,
-                                                             c->d_narith, d_pre_s, d_pre_c, c->d_sites, c->d_chain,
-                                                             c->sites_cap, c->chain_cap); count_launch();
-    GS_CUDA(c, cudaGetLastError());
-    return GS_OK;
-  };
+  // sites and chains into the buffers as they are (one host synchronisation per call); if a total
+  // turns out larger than its buffer, detect_finish grows it and writes again
+  auto write = [&]() -> gs_status { return write_launch(c); };
   // everything up to the speculative write and the read-backs (no allocation in here)
   const auto enqueue = [&]() -> gs_status {
     if (nc) {  // the hash-table regions of kernels [kb, ke), zeroed on a side stream meanwhile
@@ -1110,7 +1162,7 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
   // Replayed as one CUDA graph while (kernel range, buffers, capacities) repeat; not with the
   // consumer join (it allocates), nor on the default streams (not capturable).
   const uintptr_t key[] = {kb, ke, (uintptr_t)nc, D, (uintptr_t)c->sites_cap, (uintptr_t)c->chain_cap,
-                           (uintptr_t)c->d_sites, (uintptr_t)c->d_chain, (uintptr_t)c->h_pin,
+                           (uintptr_t)c->d_sites, (uintptr_t)c->d_chain, (uintptr_t)c->h_det,
                            c->cfg.shmem_min_arith, c->cfg.shmem_min_loads, (uintptr_t)c->n_kernels};
   constexpr size_t nkey = sizeof(key) / sizeof(key[0]);
   static const bool no_graph = getenv("GS_NO_GRAPH") != nullptr;
@@ -1144,22 +1196,13 @@ gs_status detect_run(gs_ctx* c, uint32_t kb, uint32_t ke, uint64_t* n_sites) {
     const gs_status s1 = enqueue();
     if (s1 != GS_OK) return s1;
   }
-  GS_CUDA(c, cudaStreamSynchronize(st));
-  c->kstats_h.assign(kst_pin, kst_pin + c->n_kernels);
-  const uint64_t ns = tot[1], nch = tot[0];
-  if (nch > 0xffffffffull) return fail(c, GS_E_RANGE, "chain pool exceeds 2^32 entries");
-  if (ns > c->sites_cap || nch > c->chain_cap) {
-    GS_CUDA(c, dev_grow(&c->d_sites, &c->sites_cap, ns ? ns : 1));
-    GS_CUDA(c, dev_grow(&c->d_chain, &c->chain_cap, nch ? nch : 1));
-    const gs_status ws = write();
-    if (ws != GS_OK) return ws;
-    GS_CUDA(c, cudaStreamSynchronize(st));
-  }
-  c->n_sites = ns;
-  c->n_chain = nch;
   c->det_kb = kb; c->det_ke = ke; c->det_c0 = c0; c->det_c1 = c1;
   c->detected = true;
-  if (n_sites) *n_sites = ns;
+  c->det_pending = true;
+  if (!n_sites) return GS_OK;  // asynchronous: the next call that needs the results finishes it
+  const gs_status fs = detect_finish(c);
+  if (fs != GS_OK) return fs;
+  *n_sites = c->n_sites;
   return GS_OK;
 }
 

@@ -668,3 +668,35 @@ def test_cluster_sort_equals_cub_sort(gs, cfg, scale):
         out.append(rows.copy())
         ctx.close()
     assert len(out[0]) == n_sites and np.array_equal(out[0], out[1])
+
+
+def test_async_detect_equals_sync(gs):
+    """gs_detect with n_sites == NULL returns without synchronising; the next call that reads the
+    results completes it (including the first call's buffer growth and rewrite). Sites, counters
+    and the ranking equal the synchronous path's, also with work enqueued in between and with two
+    asynchronous detections back to back."""
+    import torch
+    from gen import samples as gsm
+    from gen import sass as gsass
+    from paper_conf_sc_senvs23_b200 import report
+    s = gsass.config_sass("C2")
+    tab = gsm.table_class_weighted(s.cls, 2_000_000, key=21)
+    words = torch.from_numpy(gsm.Trace(tab, s.first_slot, s.n_instr, order="trace", seed=5).packed()
+                             .view(np.int32)).cuda()
+    res = []
+    for wait in (True, False):
+        ctx = _ctx(gs, hist_row=19)
+        ctx.load_sass(s.text)
+        if wait:
+            ctx.detect()
+        else:
+            assert ctx.detect(wait=False) is None       # first call: buffers grow inside the finish
+            ctx.detect(0, max(1, ctx.n_kernels // 2), wait=False)
+            ctx.detect(wait=False)                      # the previous one is finished first
+        hist, _ = ctx.attribute_samples(words)          # enqueued behind the pending detection
+        rows = ctx.rank_sites(hist)
+        torch.cuda.synchronize()
+        res.append((report.canonical(ctx, hist=hist, n_samples=int(tab.sum()), n_invalid=0, ranked=rows),
+                    ctx.sites_device()[2]))
+        ctx.close()
+    assert res[0][1] == res[1][1] and res[0][0] == res[1][0]

@@ -93,22 +93,42 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
   if (n_records) *n_records = total;
   GS_CUDA(c, cupti_grow(c, total));
   uint4* h = static_cast<uint4*>(c->h_cupti);
+  // stall-reason index -> reason as a flat table (a hash lookup per entry was most of the host time)
+  uint32_t max_idx = 0;
+  for (const auto& kv : c->cupti_reason) max_idx = std::max(max_idx, kv.first);
+  std::vector<int> rtab(c->cupti_reason.empty() ? 0 : (size_t)max_idx + 1, kUnknown);
+  for (const auto& kv : c->cupti_reason) rtab[kv.first] = kv.second;
   run([&](int t) {
     size_t a, b;
     range(t, &a, &b);
     uint64_t o = cnt[t];
     unsigned long long sk = 0;
+    // CUPTI hands out one name pointer per function: consecutive records of a function share it,
+    // so the (string-keyed) kernel lookup runs once per run of records, and once per pointer
+    std::unordered_map<const char*, uint32_t> by_ptr;
+    const char* last_name = nullptr;
+    uint32_t last_k = kBadKernel;
     for (size_t i = a; i < b; i++) {
       const CUpti_PCSamplingPCData& d = pcs[i];
       uint32_t k = kBadKernel;
       if (d.functionName && (crc == 0 || d.cubinCrc == crc) && d.pcOffset <= 0xffffffffull) {
-        auto it = c->kernel_index.find(d.functionName);
-        if (it != c->kernel_index.end()) k = it->second;
+        if (d.functionName != last_name) {
+          auto pit = by_ptr.find(d.functionName);
+          if (pit != by_ptr.end()) {
+            last_k = pit->second;
+          } else {
+            auto it = c->kernel_index.find(d.functionName);
+            last_k = it != c->kernel_index.end() ? it->second : kBadKernel;
+            by_ptr.emplace(d.functionName, last_k);
+          }
+          last_name = d.functionName;
+        }
+        k = last_k;
       }
       for (size_t q = 0; q < d.stallReasonCount; q++) {
         const CUpti_PCSamplingStallReason& e = d.stallReason[q];
-        auto it = c->cupti_reason.find(e.pcSamplingStallReasonIndex);
-        const int r = it == c->cupti_reason.end() ? kUnknown : it->second;
+        const uint32_t ri = e.pcSamplingStallReasonIndex;
+        const int r = ri < rtab.size() ? rtab[ri] : kUnknown;
         if (r == kSkip) {  // a subset of the same samples (R39): not attributed, not invalid
           sk += e.samples;
           h[o++] = make_uint4(0, 0, 0, 0);  // a zero-weight record keeps the layout fixed

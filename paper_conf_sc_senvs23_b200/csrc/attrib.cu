@@ -142,6 +142,24 @@ __global__ void k_counts(const uint4* __restrict__ rec, uint64_t n, const KDesc*
   if ((threadIdx.x & 31) == 0 && bad) atomicAdd(d_n_invalid, bad);
 }
 
+// Pre-aggregated records already packed on the host as {compact bin, count} (8 B; the CUPTI
+// ingest validates and packs while it flattens): one L2 atomic per record with a count; a bin >=
+// P * R is invalid and adds its count to n_invalid.
+__global__ void k_counts8(const uint2* __restrict__ rec, uint64_t n, uint32_t pnr, Div dv, int32_t* __restrict__ H,
+                          unsigned long long* d_n_invalid) {
+  unsigned long long bad = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint2 r = __ldg(rec + i);  // x bin, y count
+    if (r.x < pnr) {
+      if (r.y) atomicAdd(H + hidx(r.x, dv), (int32_t)r.y);
+    } else {
+      bad += r.y;
+    }
+  }
+  for (int o = 16; o; o >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, o);
+  if ((threadIdx.x & 31) == 0 && bad) atomicAdd(d_n_invalid, bad);
+}
+
 // -------------------------------------------------------------------------------- GLOBAL
 __global__ void __launch_bounds__(kThreadsGlobal) k_hist_global(const uint32_t* __restrict__ s, uint64_t n,
                                                                 uint32_t pnr, Div dv, int32_t* __restrict__ H,
@@ -1389,6 +1407,22 @@ gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_h
   const uint64_t blocks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 8, (n + 255) / 256));
   k_counts<<<(unsigned)blocks, 256, 0, st>>>(reinterpret_cast<const uint4*>(d_recs), n, c->d_kd, c->n_kernels,
                                              c->cfg.n_reasons, row, d_hist, d_n_invalid);
+  count_launch();
+  GS_CUDA(c, cudaGetLastError());
+  return GS_OK;
+}
+
+gs_status counts8_run(gs_ctx* c, const void* d_recs, uint64_t n, int32_t* d_hist, unsigned long long* d_n_invalid,
+                      int accumulate) {
+  cudaStream_t st = c->stream;
+  const uint32_t row = c->cfg.hist_row, nr = c->cfg.n_reasons;
+  if (!accumulate && c->n_instr) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * row * 4, st));
+  if (!n) return GS_OK;
+  int dev_sms = 148;
+  cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, c->device);
+  const uint64_t blocks = std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)dev_sms * 8, (n + 255) / 256));
+  k_counts8<<<(unsigned)blocks, 256, 0, st>>>(static_cast<const uint2*>(d_recs), n, (uint32_t)c->n_instr * nr,
+                                              make_div(nr, row), d_hist, d_n_invalid);
   count_launch();
   GS_CUDA(c, cudaGetLastError());
   return GS_OK;

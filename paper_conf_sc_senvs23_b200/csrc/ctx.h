@@ -250,6 +250,8 @@ gs_status detect_alloc(gs_ctx* c);  // after a load
 void detect_free(gs_ctx* c);
 gs_status pack_samples_run(gs_ctx* c, const uint32_t* d_raw, uint64_t n, uint32_t* d_words,
                            unsigned long long* d_n_invalid);
+gs_status counts8_run(gs_ctx* c, const void* d_recs, uint64_t n, int32_t* d_hist, unsigned long long* d_n_invalid,
+                      int accumulate);  // {compact bin, count} records
 gs_status counts_run(gs_ctx* c, const uint32_t* d_recs, uint64_t n, int32_t* d_hist, unsigned long long* d_n_invalid,
                      int accumulate);
 gs_status hist_run(gs_ctx* c, const uint32_t* d_words, uint64_t n, int32_t* d_hist,

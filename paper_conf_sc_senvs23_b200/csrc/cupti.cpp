@@ -92,7 +92,10 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
   const uint64_t total = cnt[nt];
   if (n_records) *n_records = total;
   GS_CUDA(c, cupti_grow(c, total));
-  uint4* h = static_cast<uint4*>(c->h_cupti);
+  // flattened records {compact bin, count} (8 B: half the H2D bytes of {kernel, pc, reason, count});
+  // validation here (R30): unknown kernel or reason, misaligned or out-of-range pc -> bin ~0u
+  uint2* h = static_cast<uint2*>(c->h_cupti);
+  const uint32_t nr = c->cfg.n_reasons;
   // stall-reason index -> reason as a flat table (a hash lookup per entry was most of the host time)
   uint32_t max_idx = 0;
   for (const auto& kv : c->cupti_reason) max_idx = std::max(max_idx, kv.first);
@@ -125,17 +128,23 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
         }
         k = last_k;
       }
+      // the record's first compact bin (reason 0) when its kernel and pc are valid, else ~0u
+      uint32_t kbin = 0xffffffffu;
+      if (k != kBadKernel && (d.pcOffset & 15u) == 0) {
+        const KDesc& K = c->kd_h[k];
+        const uint64_t pcs16 = d.pcOffset >> 4;
+        if (pcs16 < K.n) kbin = (K.first + (uint32_t)pcs16) * nr;
+      }
       for (size_t q = 0; q < d.stallReasonCount; q++) {
         const CUpti_PCSamplingStallReason& e = d.stallReason[q];
         const uint32_t ri = e.pcSamplingStallReasonIndex;
         const int r = ri < rtab.size() ? rtab[ri] : kUnknown;
         if (r == kSkip) {  // a subset of the same samples (R39): not attributed, not invalid
           sk += e.samples;
-          h[o++] = make_uint4(0, 0, 0, 0);  // a zero-weight record keeps the layout fixed
+          h[o++] = make_uint2(0u, 0u);  // a zero-weight record keeps the layout fixed
           continue;
         }
-        h[o++] = make_uint4(r == kUnknown ? kBadKernel : k, (uint32_t)d.pcOffset, r < 0 ? 0u : (uint32_t)r,
-                            e.samples);
+        h[o++] = make_uint2(kbin != 0xffffffffu && r >= 0 && (uint32_t)r < nr ? kbin + (uint32_t)r : 0xffffffffu, e.samples);
       }
     }
     skipped[t] = sk;
@@ -144,8 +153,8 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
   for (auto v : skipped) sk += v;
   if (n_skipped) *n_skipped = sk;
   cudaStream_t st = c->stream;
-  if (total) GS_CUDA(c, cudaMemcpyAsync(c->d_cupti, h, total * 16, cudaMemcpyHostToDevice, st));
-  gs_status s = counts_run(c, reinterpret_cast<const uint32_t*>(c->d_cupti), total, d_hist, d_n_invalid, accumulate);
+  if (total) GS_CUDA(c, cudaMemcpyAsync(c->d_cupti, h, total * 8, cudaMemcpyHostToDevice, st));
+  gs_status s = counts8_run(c, c->d_cupti, total, d_hist, d_n_invalid, accumulate);
   if (s != GS_OK) return s;
   // the staging buffer is reused by the next call: wait for this copy (the scatter-add stays async)
   GS_CUDA(c, cudaStreamSynchronize(st));

@@ -67,13 +67,17 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
     c->kernel_index.reserve(c->n_kernels * 2);
     for (uint32_t k = 0; k < c->n_kernels; k++) c->kernel_index.emplace(c->names[k], k);
   }
-  // pass 1 (parallel): entries per record range; pass 2: fill the flattened records
+  // pass 1 (parallel): entries per record range; then two flattening phases (each thread the first,
+  // then the second half of its range): the H2D copy and the scatter-add of phase 0's records run
+  // while phase 1 flattens
   const int nt = (int)std::max<size_t>(1, std::min<size_t>({16, std::thread::hardware_concurrency(), n / 4096 + 1}));
-  std::vector<uint64_t> cnt(nt + 1, 0);
+  constexpr int kPh = 2;
+  std::vector<uint64_t> cnt(kPh * nt + 1, 0);  // entries of (phase, thread) in phase-major order
   std::vector<unsigned long long> skipped(nt, 0);
-  auto range = [&](int t, size_t* a, size_t* b) {
-    *a = n * t / nt;
-    *b = n * (t + 1) / nt;
+  auto range = [&](int ph, int t, size_t* a, size_t* b) {
+    const size_t ta = n * t / nt, tb = n * (t + 1) / nt, tm = ta + (tb - ta) / 2;
+    *a = ph ? tm : ta;
+    *b = ph ? tb : tm;
   };
   auto run = [&](auto fn) {
     std::vector<std::thread> th;
@@ -82,14 +86,16 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
     for (auto& x : th) x.join();
   };
   run([&](int t) {
-    size_t a, b;
-    range(t, &a, &b);
-    uint64_t m = 0;
-    for (size_t i = a; i < b; i++) m += pcs[i].stallReasonCount;
-    cnt[t + 1] = m;
+    for (int ph = 0; ph < kPh; ph++) {
+      size_t a, b;
+      range(ph, t, &a, &b);
+      uint64_t m = 0;
+      for (size_t i = a; i < b; i++) m += pcs[i].stallReasonCount;
+      cnt[ph * nt + t + 1] = m;
+    }
   });
-  for (int t = 0; t < nt; t++) cnt[t + 1] += cnt[t];
-  const uint64_t total = cnt[nt];
+  for (int q = 0; q < kPh * nt; q++) cnt[q + 1] += cnt[q];
+  const uint64_t total = cnt[kPh * nt];
   if (n_records) *n_records = total;
   GS_CUDA(c, cupti_grow(c, total));
   // flattened records {compact bin, count} (8 B: half the H2D bytes of {kernel, pc, reason, count});
@@ -101,10 +107,13 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
   for (const auto& kv : c->cupti_reason) max_idx = std::max(max_idx, kv.first);
   std::vector<int> rtab(c->cupti_reason.empty() ? 0 : (size_t)max_idx + 1, kUnknown);
   for (const auto& kv : c->cupti_reason) rtab[kv.first] = kv.second;
+  cudaStream_t st = c->stream;
+  if (!accumulate && c->n_instr) GS_CUDA(c, cudaMemsetAsync(d_hist, 0, c->n_instr * c->cfg.hist_row * 4, st));
+  for (int ph = 0; ph < kPh; ph++) {
   run([&](int t) {
     size_t a, b;
-    range(t, &a, &b);
-    uint64_t o = cnt[t];
+    range(ph, t, &a, &b);
+    uint64_t o = cnt[ph * nt + t];
     unsigned long long sk = 0;
     // CUPTI hands out one name pointer per function: consecutive records of a function share it,
     // so the (string-keyed) kernel lookup runs once per run of records, and once per pointer
@@ -147,15 +156,20 @@ gs_status cupti_run(gs_ctx* c, const void* pc_data, size_t n, uint64_t crc, int3
         h[o++] = make_uint2(kbin != 0xffffffffu && r >= 0 && (uint32_t)r < nr ? kbin + (uint32_t)r : 0xffffffffu, e.samples);
       }
     }
-    skipped[t] = sk;
+    skipped[t] += sk;
   });
+    // this phase's records: copy and scatter-add (async) while the next phase flattens
+    const uint64_t p0 = cnt[ph * nt], p1 = cnt[(ph + 1) * nt];
+    if (p1 > p0) {
+      GS_CUDA(c, cudaMemcpyAsync(static_cast<uint2*>(c->d_cupti) + p0, h + p0, (p1 - p0) * 8, cudaMemcpyHostToDevice,
+                                 st));
+      const gs_status s = counts8_run(c, static_cast<uint2*>(c->d_cupti) + p0, p1 - p0, d_hist, d_n_invalid, 1);
+      if (s != GS_OK) return s;
+    }
+  }
   unsigned long long sk = 0;
   for (auto v : skipped) sk += v;
   if (n_skipped) *n_skipped = sk;
-  cudaStream_t st = c->stream;
-  if (total) GS_CUDA(c, cudaMemcpyAsync(c->d_cupti, h, total * 8, cudaMemcpyHostToDevice, st));
-  gs_status s = counts8_run(c, c->d_cupti, total, d_hist, d_n_invalid, accumulate);
-  if (s != GS_OK) return s;
   // the staging buffer is reused by the next call: wait for this copy (the scatter-add stays async)
   GS_CUDA(c, cudaStreamSynchronize(st));
   return GS_OK;

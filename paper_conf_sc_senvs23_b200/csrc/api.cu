@@ -417,7 +417,10 @@ gs_status gs_attribute_samples(gs_ctx* c, const uint32_t* samples, uint64_t n, i
   }
   // host input: chunks through two device staging buffers; the H2D copy of chunk i+1 runs on a
   // copy stream (copy engine) while the histogram of chunk i runs on the context's stream
-  const size_t chunk = size_t(16) << 20;  // words
+#ifndef GS_STAGE_MWORDS
+#define GS_STAGE_MWORDS 16
+#endif
+  const size_t chunk = size_t(GS_STAGE_MWORDS) << 20;  // words per staging buffer
   if (c->stage_words < chunk) {
     attrib_free(c);
     for (int b = 0; b < 2; b++) {

@@ -207,6 +207,8 @@ const unsigned long long* __restrict__ rel, const unsigned long long* __restrict
   unsigned long long* nxt = cs_buf + kCsPer;
   // element i of CTA r is site r * kCsPer + i; warp w owns [w * 256, w * 256 + 256), row k its
   // elements w * 256 + 32 k + lane
+  static_assert(kCsPer % kCsThreads == 0, "whole rows per thread");
+#pragma unroll  // all of a thread's loads in flight at once
   for (uint32_t i = threadIdx.x; i < kCsPer; i += kCsThreads) {
     const uint32_t sidx = r * kCsPer + i;
     cur[i] = sidx < ns ? ((((mask_r - rel[sidx]) << bt) | (mask_t - tot[sidx])) << kCsIdxBits) | sidx : ~0ull;
@@ -287,6 +289,7 @@ const unsigned long long* __restrict__ rel, const unsigned long long* __restrict
     cur = nxt;
     nxt = t;
   }
+#pragma unroll
   for (uint32_t i = threadIdx.x; i < kCsPer; i += kCsThreads) {
     const uint32_t q = r * kCsPer + i;
     if (q < ns) order[q] = (uint32_t)(cur[i] & (kCsMax - 1u));
